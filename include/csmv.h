@@ -1,0 +1,199 @@
+/*
+ * csmv.h -- C ABI of the B200 (sm_100a) CSMV batched commit pipeline.
+ *
+ * CSMV (Nunes, Castro, Romano, IPDPS 2022; /root/reference/PAPER.md, cited
+ * P:<line>) is a multi-versioned STM for GPUs with a client-server commit:
+ * client warps run transactions over versioned boxes (VBoxes),
+ * pre-validate them inside the warp and ship each warp's update
+ * transactions as one batch to a persistent server that validates them
+ * against recently committed write-sets held in shared memory (the ATR,
+ * P:65) and hands back consecutive commit timestamps (CTS,
+ * P:101); clients then write the new versions back and
+ * advance the global timestamp GTS in commit order.
+ *
+ * "The CSMV library masks away from the programmer all the complexity
+ * associated with the management of transactions and of activating the
+ * (server) kernel": this header is that library's boundary.  The
+ * transaction bodies are the paper's two benchmarks (Bank P:177-183,
+ * MemcachedGPU P:185), selected by csmv_workload.kind and generated from a
+ * counter-based generator (docs/GENERATOR.md) inside the kernel.
+ *
+ * Conventions
+ *  - Every call is extern "C", takes plain pointers and sizes.  Functions
+ *    returning int return CSMV_OK (0) or a negative CSMV_E* code; the
+ *    message of the last error of the calling thread is csmv_last_error().
+ *  - A handle is single-threaded (not re-entrant); one handle per device.
+ *  - The library owns all device memory.  Host buffers passed in are read
+ *    during the call (the caller keeps ownership); output buffers are
+ *    caller-allocated host memory.
+ *  - There is no CPU fallback: without an sm_100a device csmv_create
+ *    returns NULL and csmv_last_error() says why.
+ */
+#ifndef CSMV_H
+#define CSMV_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CSMV_ABI_VERSION 1
+
+/* ---- error codes ---- */
+#define CSMV_OK 0
+#define CSMV_EINVAL (-1)    /* bad argument */
+#define CSMV_ENOMEM (-2)    /* device allocation failed */
+#define CSMV_ECUDA (-3)     /* CUDA runtime error / no sm_100a device */
+#define CSMV_ESTATE (-4)    /* wrong call order (e.g. run before load) */
+#define CSMV_ETIMEOUT (-5)  /* device watchdog fired (a spin loop overran) */
+#define CSMV_EOVERFLOW (-6) /* caller buffer too small / timestamp space exhausted */
+
+/* ---- workload descriptor ---- */
+#define CSMV_KIND_BANK 0u
+#define CSMV_KIND_KV 1u        /* P:185 (MemcachedGPU) */
+#define CSMV_DIST_UNIFORM 0u
+#define CSMV_DIST_ZIPF 1u
+#define CSMV_LOG_NONE 0u       /* timed runs */
+#define CSMV_LOG_DIGEST 1u     /* 32 B record per transaction */
+#define CSMV_LOG_FULL 2u       /* + every value read */
+#define CSMV_SERVER_CTA 0u     /* single-SM server (the paper's) */
+#define CSMV_SERVER_CLUSTER 1u /* thread-block-cluster server (DSMEM) */
+#define CSMV_PUBLISH_CLIENT 0u /* client advances GTS when GTS == CTS-1 */
+#define CSMV_PUBLISH_SERVER 1u /* a server warp advances GTS over finished write-backs */
+#define CSMV_ATR_HASH 0u       /* item-indexed ATR (set-associative, smem) */
+#define CSMV_ATR_LIST 1u       /* ATR as a list of write-sets, warp-striped scan */
+
+#define CSMV_DBG_NO_PREVAL 1u  /* negative control: skip client pre-validation */
+#define CSMV_DBG_NO_VALIDATE 2u/* negative control: server commits without validating */
+#define CSMV_DBG_JITTER 4u     /* random __nanosleep in client and server */
+
+typedef struct csmv_workload {
+    uint32_t kind;             /* CSMV_KIND_* */
+    uint32_t dist;             /* CSMV_DIST_* for the items an update picks */
+    uint32_t zipf_theta_milli; /* 990 = theta 0.99 */
+    uint32_t p_update_ppm;     /* update probability, parts per million */
+    uint32_t ro_period;        /* >0: tx % ro_period == ro_period-1 is read-only */
+    uint32_t ro_reads;         /* bank ROT: 0 = total sum of all accounts, L = L-item scan */
+    uint32_t amount_max;       /* bank transfer amount uniform in [1, amount_max] */
+    uint32_t kv_ways;          /* KV associativity A */
+    uint32_t kv_keys;          /* KV key space */
+    uint32_t client_warps;     /* active client warps; 0 = full grid */
+    uint32_t server;           /* CSMV_SERVER_* */
+    uint32_t cluster_size;     /* cluster server CTAs (2..16) */
+    uint32_t atr_capacity;     /* ATR entries (0 = default); rounded to the layout */
+    uint32_t atr_mode;         /* CSMV_ATR_* */
+    uint32_t publish;          /* CSMV_PUBLISH_* */
+    uint32_t log_mode;         /* CSMV_LOG_* */
+    uint32_t debug_flags;      /* CSMV_DBG_* */
+    uint32_t watchdog_ms;      /* 0 = default (20000) */
+} csmv_workload;
+
+/* ---- statistics ---- */
+#define CSMV_AB_PREVAL 0u      /* lost client pre-validation */
+#define CSMV_AB_CONFLICT 1u    /* server validation failed */
+#define CSMV_AB_EARLY 2u       /* client read a version newer than its snapshot (validation would fail) */
+#define CSMV_AB_OVERFLOW 3u    /* ATR no longer covers the snapshot (bounded ATR) */
+#define CSMV_AB_VERSION 4u     /* no version old enough */
+#define CSMV_N_ABORT 5u
+
+typedef struct csmv_stats {
+    uint64_t committed_update;
+    uint64_t committed_ro;
+    uint64_t aborts[CSMV_N_ABORT][2]; /* [reason][0 = read-only, 1 = update] */
+    uint64_t batches;          /* requests the server processed */
+    uint64_t rounds;           /* client warp rounds */
+    uint64_t gts_start;
+    uint64_t gts_final;
+    uint64_t elapsed_ns;       /* fused kernel, CUDA events */
+    uint64_t ro_checksum;      /* xor of read-only results (keeps them live) */
+    uint64_t store_bytes;      /* device bytes of the version store */
+    uint64_t store_bytes_paper;/* same items in the paper's VBox layout */
+    uint64_t server_lock_cycles; /* cycles the commit critical section was held */
+    uint64_t server_busy_cycles; /* cycles workers spent processing batches */
+    uint32_t client_warps;
+    uint32_t server_ctas;
+    uint32_t server_workers;
+    uint32_t atr_entries;
+    uint32_t sm_count;
+    uint32_t kernel_launches;  /* kernels launched by the last csmv_run */
+} csmv_stats_t;
+
+/* One record per committed transaction, indexed by transaction number
+ * (docs/GENERATOR.md section 5). cts = 0 marks a read-only transaction. */
+typedef struct csmv_log_rec {
+    uint32_t tx, snapshot, cts, attempts;
+    uint64_t read_digest, aux;
+} csmv_log_rec;
+
+typedef struct csmv csmv_t;
+
+/* Version of this ABI (CSMV_ABI_VERSION). */
+int csmv_abi_version(void);
+
+/* Create a store of n_items 4-byte items (bank accounts), each a VBox of
+ * n_versions in [1,16] versions.  Needs an sm_100a device
+ * (the current CUDA device).  NULL on error (EINVAL, ENOMEM, ECUDA). */
+csmv_t *csmv_create(uint64_t n_items, uint32_t n_versions);
+
+/* Create a MemcachedGPU store: n_slots slots of `ways` ways, with
+ * 16-byte keys, 32-byte values, per-slot LRU and per-set clocks, each a VBox
+ * of n_versions versions.  n_slots must be a multiple of ways. */
+csmv_t *csmv_create_kv(uint64_t n_slots, uint32_t ways, uint32_t n_versions);
+
+/* Bank: install init_values[0..n) (host memory) as version ts = 0 of every
+ * item and reset GTS to 0.  EINVAL if n != n_items. */
+int csmv_load(csmv_t *h, const int32_t *init_values, uint64_t n);
+
+/* KV: preload keys 0..n_keys-1 with PUT semantics (docs/GENERATOR.md
+ * section 4) as version ts = 0 and reset GTS to 0. */
+int csmv_load_kv(csmv_t *h, uint64_t n_keys);
+
+/* Run on the given CUDA stream (a cudaStream_t, e.g. torch's current
+ * stream); NULL = the legacy default stream. */
+int csmv_set_stream(csmv_t *h, void *cuda_stream);
+
+/* Run transactions 0..n_tx-1 of the workload to completion: every
+ * transaction commits exactly once, aborted attempts are retried.
+ * Blocking.  Continues from the current store and GTS.  ESTATE if not
+ * loaded; ETIMEOUT if the device watchdog fired (the handle must then be
+ * reloaded); EOVERFLOW if GTS + n_tx would exceed 2^32 - 2. */
+int csmv_run(csmv_t *h, const csmv_workload *w, uint64_t n_tx, uint64_t seed);
+
+/* Statistics of the last csmv_run. */
+int csmv_stats(const csmv_t *h, csmv_stats_t *out);
+
+/* Log of the last csmv_run (needs log_mode != NONE): n_tx records into buf
+ * (cap records).  EOVERFLOW if cap < n_tx; *n_out = records written. */
+int csmv_get_log(const csmv_t *h, csmv_log_rec *buf, uint64_t cap, uint64_t *n_out);
+
+/* FULL log values of the last run: n_tx * (*max_vals) u32 words, transaction
+ * t's reads at [t * max_vals, ...).  Pass buf = NULL to query the size. */
+int csmv_get_vals(const csmv_t *h, uint32_t *buf, uint64_t cap_words, uint32_t *max_vals);
+
+/* Bank: copy the version store out as n_items * n_versions packed slots
+ * (ts << 32) | (uint32_t)value, ts = 0xFFFFFFFF for an unused slot. */
+int csmv_dump_store(const csmv_t *h, uint64_t *rings_out, uint64_t cap);
+
+/* KV: newest value of every item: keys (n_slots*4 words), values
+ * (n_slots*8), lru (n_slots), clocks (n_slots/ways).  Any may be NULL. */
+int csmv_dump_kv(const csmv_t *h, uint32_t *keys, uint32_t *vals, uint32_t *lru,
+                 uint32_t *clocks);
+
+/* Copy transaction descriptors tx0..tx0+n-1 as the device generator sees
+ * them (6 u32 per bank tx: is_update, src, dst, amt, start, len), for the
+ * generator parity check. */
+int csmv_gen_descs(csmv_t *h, const csmv_workload *w, uint64_t seed, uint64_t tx0,
+                   uint64_t n, uint32_t *out);
+
+/* The zipf CDF table the library built for (n, theta_milli). */
+int csmv_zipf_table(uint32_t n, uint32_t theta_milli, uint64_t *out);
+
+/* Release everything; accepts NULL. */
+void csmv_destroy(csmv_t *h);
+
+/* Message of the last error on this thread ("" if none). */
+const char *csmv_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,456 @@
+// host.cu -- the C ABI of include/csmv.h: device memory, launches, stats.
+//
+// Every transaction step runs in the fused kernel (kernel.cu); the host only
+// allocates, initialises, launches and copies results.  Nothing here falls
+// back to the CPU: without an sm_100a device csmv_create fails.
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/csmv.h"
+#include "kernel.cuh"
+
+using namespace csmvd;
+
+namespace {
+
+thread_local char g_err[512] = "";
+
+int set_err(int code, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
+int set_err(int code, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof g_err, fmt, ap);
+  va_end(ap);
+  return code;
+}
+
+#define CK(call)                                                                         \
+  do {                                                                                   \
+    cudaError_t e_ = (call);                                                             \
+    if (e_ != cudaSuccess)                                                               \
+      return set_err(CSMV_ECUDA, "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, \
+                     __LINE__);                                                          \
+  } while (0)
+
+// zipf CDF (docs/GENERATOR.md section 2), built on the host in IEEE double
+std::vector<uint64_t> build_zipf(uint32_t n, uint32_t theta_milli) {
+  std::vector<uint64_t> cdf(n);
+  const double theta = (double)theta_milli / 1000.0;
+  double h = 0.0;
+  for (uint32_t r = 1; r <= n; ++r) h += std::pow((double)r, -theta);
+  double s = 0.0;
+  for (uint32_t i = 0; i < n; ++i) {
+    s += std::pow((double)(i + 1), -theta);
+    const double x = std::ldexp(s / h, 64);
+    cdf[i] = (x >= 18446744073709551616.0) ? UINT64_MAX : (uint64_t)x;
+  }
+  cdf[n - 1] = UINT64_MAX;
+  return cdf;
+}
+
+uint32_t nslot_for(uint32_t k) { return k <= 2 ? 2 : k <= 4 ? 4 : k <= 8 ? 8 : 16; }
+
+}  // namespace
+
+struct csmv {
+  int kind = CSMV_KIND_BANK;
+  uint64_t n_items = 0;
+  uint32_t K = 0, nslot = 0;
+  int device = 0, sm_count = 0;
+  cudaStream_t stream = nullptr;
+  bool loaded = false;
+
+  uint64_t* d_rings = nullptr;
+  uint32_t* d_gts = nullptr;
+  Ctl* d_ctl = nullptr;
+  DevStats* d_stats = nullptr;
+  uint32_t* d_done = nullptr;
+  // per-client-warp message slots, sized for the full grid
+  uint32_t max_cw = 0;
+  uint32_t* d_req_seq = nullptr;
+  ReqHdr* d_req_hdr = nullptr;
+  uint32_t* d_req_ids = nullptr;
+  Resp* d_resp = nullptr;
+  // logs
+  csmv_log_rec* d_log = nullptr;
+  uint64_t log_cap = 0;
+  uint32_t* d_vals = nullptr;
+  uint64_t vals_cap = 0;
+  uint64_t last_n_tx = 0;
+  uint32_t last_log_mode = 0, last_max_vals = 0;
+  // zipf table cache
+  uint64_t* d_zipf = nullptr;
+  uint32_t zipf_n = 0, zipf_theta = 0;
+
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  csmv_stats_t last{};
+};
+
+static void free_all(csmv* h) {
+  cudaFree(h->d_rings);
+  cudaFree(h->d_gts);
+  cudaFree(h->d_ctl);
+  cudaFree(h->d_stats);
+  cudaFree(h->d_done);
+  cudaFree(h->d_req_seq);
+  cudaFree(h->d_req_hdr);
+  cudaFree(h->d_req_ids);
+  cudaFree(h->d_resp);
+  cudaFree(h->d_log);
+  cudaFree(h->d_vals);
+  cudaFree(h->d_zipf);
+  if (h->ev0) cudaEventDestroy(h->ev0);
+  if (h->ev1) cudaEventDestroy(h->ev1);
+}
+
+extern "C" {
+
+int csmv_abi_version(void) { return CSMV_ABI_VERSION; }
+
+const char* csmv_last_error(void) { return g_err; }
+
+static int device_check(int* dev, int* sms) {
+  int n = 0;
+  cudaError_t e = cudaGetDeviceCount(&n);
+  if (e != cudaSuccess || n == 0)
+    return set_err(CSMV_ECUDA, "no CUDA device (%s); there is no CPU fallback",
+                   e == cudaSuccess ? "0 devices" : cudaGetErrorString(e));
+  CK(cudaGetDevice(dev));
+  cudaDeviceProp pr;
+  CK(cudaGetDeviceProperties(&pr, *dev));
+  if (pr.major != 10 || pr.minor != 0)
+    return set_err(CSMV_ECUDA, "device %s is sm_%d%d; this library is built for sm_100a only",
+                   pr.name, pr.major, pr.minor);
+  if (!pr.cooperativeLaunch) return set_err(CSMV_ECUDA, "device lacks cooperative launch");
+  *sms = pr.multiProcessorCount;
+  return CSMV_OK;
+}
+
+csmv_t* csmv_create(uint64_t n_items, uint32_t n_versions) {
+  g_err[0] = 0;
+  if (n_items < 2 || n_items >= (1ull << 31) || n_versions < 1 || n_versions > 16) {
+    set_err(CSMV_EINVAL, "csmv_create: need 2 <= n_items < 2^31 and 1 <= n_versions <= 16");
+    return nullptr;
+  }
+  int dev = 0, sms = 0;
+  if (device_check(&dev, &sms) != CSMV_OK) return nullptr;
+  csmv* h = new csmv();
+  h->kind = CSMV_KIND_BANK;
+  h->n_items = n_items;
+  h->K = n_versions;
+  h->nslot = nslot_for(n_versions);
+  h->device = dev;
+  h->sm_count = sms;
+  h->max_cw = (uint32_t)(sms - 1) * kWarps;
+  auto fail = [&](const char* what) -> csmv_t* {
+    set_err(CSMV_ENOMEM, "csmv_create: cudaMalloc %s failed (%s)", what,
+            cudaGetErrorString(cudaGetLastError()));
+    free_all(h);
+    delete h;
+    return nullptr;
+  };
+  if (cudaMalloc(&h->d_rings, n_items * h->nslot * sizeof(uint64_t)) != cudaSuccess) return fail("rings");
+  if (cudaMalloc(&h->d_gts, 64) != cudaSuccess) return fail("gts");
+  if (cudaMalloc(&h->d_ctl, sizeof(Ctl)) != cudaSuccess) return fail("ctl");
+  if (cudaMalloc(&h->d_stats, sizeof(DevStats)) != cudaSuccess) return fail("stats");
+  if (cudaMalloc(&h->d_done, sizeof(uint32_t) << kDoneLog2) != cudaSuccess) return fail("done");
+  if (cudaMalloc(&h->d_req_seq, h->max_cw * sizeof(uint32_t)) != cudaSuccess) return fail("req_seq");
+  if (cudaMalloc(&h->d_req_hdr, h->max_cw * sizeof(ReqHdr)) != cudaSuccess) return fail("req_hdr");
+  if (cudaMalloc(&h->d_req_ids, (size_t)h->max_cw * 2 * 32 * sizeof(uint32_t)) != cudaSuccess) return fail("req_ids");
+  if (cudaMalloc(&h->d_resp, h->max_cw * sizeof(Resp)) != cudaSuccess) return fail("resp");
+  cudaMemset(h->d_done, 0, sizeof(uint32_t) << kDoneLog2);
+  cudaMemset(h->d_gts, 0, 64);
+  cudaEventCreate(&h->ev0);
+  cudaEventCreate(&h->ev1);
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail("init");
+  return h;
+}
+
+csmv_t* csmv_create_kv(uint64_t, uint32_t, uint32_t) {
+  set_err(CSMV_EINVAL, "csmv_create_kv: KV store not built in this version");
+  return nullptr;
+}
+
+void csmv_destroy(csmv_t* h) {
+  if (!h) return;
+  cudaStreamSynchronize(h->stream);
+  free_all(h);
+  delete h;
+}
+
+int csmv_set_stream(csmv_t* h, void* s) {
+  if (!h) return set_err(CSMV_EINVAL, "null handle");
+  h->stream = (cudaStream_t)s;
+  return CSMV_OK;
+}
+
+int csmv_load(csmv_t* h, const int32_t* init, uint64_t n) {
+  if (!h || !init) return set_err(CSMV_EINVAL, "csmv_load: null argument");
+  if (h->kind != CSMV_KIND_BANK) return set_err(CSMV_EINVAL, "csmv_load: not a bank store");
+  if (n != h->n_items) return set_err(CSMV_EINVAL, "csmv_load: n=%llu != n_items=%llu",
+                                      (unsigned long long)n, (unsigned long long)h->n_items);
+  int32_t* d_init = nullptr;
+  CK(cudaMallocAsync((void**)&d_init, n * sizeof(int32_t), h->stream));
+  CK(cudaMemcpyAsync(d_init, init, n * sizeof(int32_t), cudaMemcpyHostToDevice, h->stream));
+  CK(launch_init_rings(h->d_rings, h->nslot, d_init, n, h->d_gts, h->stream));
+  CK(cudaFreeAsync(d_init, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  h->loaded = true;
+  return CSMV_OK;
+}
+
+int csmv_load_kv(csmv_t* h, uint64_t) {
+  if (!h) return set_err(CSMV_EINVAL, "null handle");
+  return set_err(CSMV_EINVAL, "csmv_load_kv: KV store not built in this version");
+}
+
+static int prepare_zipf(csmv* h, uint32_t n, uint32_t theta) {
+  if (h->d_zipf && h->zipf_n == n && h->zipf_theta == theta) return CSMV_OK;
+  cudaFree(h->d_zipf);
+  h->d_zipf = nullptr;
+  std::vector<uint64_t> cdf = build_zipf(n, theta);
+  CK(cudaMalloc(&h->d_zipf, n * sizeof(uint64_t)));
+  CK(cudaMemcpy(h->d_zipf, cdf.data(), n * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  h->zipf_n = n;
+  h->zipf_theta = theta;
+  return CSMV_OK;
+}
+
+static int make_gen(csmv* h, const csmv_workload* w, uint64_t seed, GenParams* g) {
+  memset(g, 0, sizeof *g);
+  g->seed = seed;
+  g->upd_thresh = ((uint64_t)w->p_update_ppm << 32) / 1000000ull;
+  g->n_items = (uint32_t)h->n_items;
+  g->ro_period = w->ro_period;
+  g->ro_reads = w->ro_reads;
+  g->amount_max = w->amount_max;
+  if (w->dist == CSMV_DIST_ZIPF) {
+    int rc = prepare_zipf(h, (uint32_t)h->n_items, w->zipf_theta_milli);
+    if (rc) return rc;
+    g->zipf_cdf = h->d_zipf;
+  } else if (w->dist != CSMV_DIST_UNIFORM) {
+    return set_err(CSMV_EINVAL, "unknown dist %u", w->dist);
+  }
+  return CSMV_OK;
+}
+
+int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
+  if (!h || !w) return set_err(CSMV_EINVAL, "csmv_run: null argument");
+  if (!h->loaded) return set_err(CSMV_ESTATE, "csmv_run: store not loaded");
+  if (w->kind != CSMV_KIND_BANK) return set_err(CSMV_EINVAL, "csmv_run: only the bank workload is built");
+  if (w->amount_max == 0) return set_err(CSMV_EINVAL, "csmv_run: amount_max must be >= 1");
+  if (w->p_update_ppm > 1000000) return set_err(CSMV_EINVAL, "csmv_run: p_update_ppm > 10^6");
+  if (w->log_mode > CSMV_LOG_FULL || w->publish > CSMV_PUBLISH_SERVER)
+    return set_err(CSMV_EINVAL, "csmv_run: bad log_mode/publish");
+  if (w->server != CSMV_SERVER_CTA) return set_err(CSMV_EINVAL, "csmv_run: cluster server not built yet");
+  if (w->atr_mode != CSMV_ATR_HASH) return set_err(CSMV_EINVAL, "csmv_run: ATR list mode not built yet");
+  if (n_tx >= (1ull << 32)) return set_err(CSMV_EINVAL, "csmv_run: n_tx must be < 2^32");
+
+  uint32_t gts0 = 0;
+  CK(cudaMemcpyAsync(&gts0, h->d_gts, 4, cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  if ((uint64_t)gts0 + n_tx >= 0xFFFFFFFEull)
+    return set_err(CSMV_EOVERFLOW, "csmv_run: timestamp space exhausted (GTS %u); reload", gts0);
+
+  KParams p;
+  memset(&p, 0, sizeof p);
+  int rc = make_gen(h, w, seed, &p.gen);
+  if (rc) return rc;
+
+  // grid: CTA 0 = server, CTAs 1..C = clients, warps spread round-robin
+  uint32_t n_cw = w->client_warps ? w->client_warps : h->max_cw;
+  if (n_cw > h->max_cw) n_cw = h->max_cw;
+  if (n_cw == 0) return set_err(CSMV_EINVAL, "csmv_run: no client warps");
+  uint32_t n_ctas = (uint32_t)h->sm_count - 1;
+  if (n_cw < n_ctas) n_ctas = n_cw;
+  const uint32_t n_workers = kWarps - 1;
+  if ((n_cw + n_workers - 1) / n_workers > 32u * kMaxPoll)
+    return set_err(CSMV_EINVAL, "csmv_run: too many client warps per server worker");
+
+  uint32_t entries = w->atr_capacity ? w->atr_capacity : 16384u;
+  uint32_t sets_log2 = 1;
+  while (((uint32_t)kWays << sets_log2) < entries && sets_log2 < 14) ++sets_log2;
+  size_t smem = server_smem_bytes(sets_log2, n_cw);
+  if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
+  int bps = 0;
+  CK(fused_occupancy(h->nslot, smem, &bps));
+  if (bps < 1) return set_err(CSMV_ECUDA, "csmv_run: fused kernel cannot be resident (smem %zu)", smem);
+
+  // logs
+  uint32_t max_vals = 0;
+  if (w->log_mode != CSMV_LOG_NONE) {
+    if (n_tx > h->log_cap) {
+      cudaFree(h->d_log);
+      h->d_log = nullptr;
+      CK(cudaMalloc(&h->d_log, n_tx * sizeof(csmv_log_rec)));
+      h->log_cap = n_tx;
+    }
+    CK(cudaMemsetAsync(h->d_log, 0, n_tx * sizeof(csmv_log_rec), h->stream));
+    if (w->log_mode == CSMV_LOG_FULL) {
+      max_vals = w->ro_reads ? w->ro_reads : (uint32_t)h->n_items;
+      if (max_vals < 2) max_vals = 2;
+      uint64_t words = n_tx * (uint64_t)max_vals;
+      if (words > h->vals_cap) {
+        cudaFree(h->d_vals);
+        h->d_vals = nullptr;
+        CK(cudaMalloc(&h->d_vals, words * sizeof(uint32_t)));
+        h->vals_cap = words;
+      }
+      CK(cudaMemsetAsync(h->d_vals, 0, words * sizeof(uint32_t), h->stream));
+    }
+  }
+
+  p.rings = h->d_rings;
+  p.n_items = (uint32_t)h->n_items;
+  p.K = h->K;
+  p.gts = h->d_gts;
+  p.ctl = h->d_ctl;
+  p.req_seq = h->d_req_seq;
+  p.req_hdr = h->d_req_hdr;
+  p.req_ids = h->d_req_ids;
+  p.resp = h->d_resp;
+  p.done_ring = h->d_done;
+  p.stats = h->d_stats;
+  p.log = h->d_log;
+  p.vals = h->d_vals;
+  p.max_vals = max_vals;
+  p.log_mode = w->log_mode;
+  p.n_tx = n_tx;
+  p.n_cw = n_cw;
+  p.n_client_ctas = n_ctas;
+  p.n_workers = n_workers;
+  p.sets_log2 = sets_log2;
+  p.publish = w->publish;
+  p.debug = w->debug_flags;
+  p.watchdog_ns = (uint64_t)(w->watchdog_ms ? w->watchdog_ms : 20000u) * 1000000ull;
+
+  CK(cudaMemsetAsync(h->d_ctl, 0, sizeof(Ctl), h->stream));
+  CK(cudaMemsetAsync(h->d_stats, 0, sizeof(DevStats), h->stream));
+  CK(cudaMemsetAsync(h->d_req_seq, 0, n_cw * sizeof(uint32_t), h->stream));
+  CK(cudaMemsetAsync(h->d_resp, 0, n_cw * sizeof(Resp), h->stream));
+  CK(cudaEventRecord(h->ev0, h->stream));
+  CK(launch_fused(p, h->nslot, 1 + n_ctas, smem, h->stream));
+  CK(cudaEventRecord(h->ev1, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+
+  Ctl ctl;
+  DevStats ds;
+  uint32_t gts1 = 0;
+  CK(cudaMemcpy(&ctl, h->d_ctl, sizeof ctl, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(&ds, h->d_stats, sizeof ds, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(&gts1, h->d_gts, 4, cudaMemcpyDeviceToHost));
+  float ms = 0.f;
+  CK(cudaEventElapsedTime(&ms, h->ev0, h->ev1));
+
+  csmv_stats_t& s = h->last;
+  memset(&s, 0, sizeof s);
+  s.committed_update = ds.committed_update;
+  s.committed_ro = ds.committed_ro;
+  for (int i = 0; i < (int)CSMV_N_ABORT; ++i)
+    for (int k = 0; k < 2; ++k) s.aborts[i][k] = ds.aborts[i][k];
+  s.batches = ds.batches;
+  s.rounds = ds.rounds;
+  s.gts_start = gts0;
+  s.gts_final = gts1;
+  s.elapsed_ns = (uint64_t)((double)ms * 1e6);
+  s.ro_checksum = ds.ro_checksum;
+  s.store_bytes = h->n_items * h->nslot * sizeof(uint64_t);
+  s.store_bytes_paper = h->n_items * (4ull + 8ull * h->K);
+  s.server_lock_cycles = ds.lock_cycles;
+  s.server_busy_cycles = ds.busy_cycles;
+  s.client_warps = n_cw;
+  s.server_ctas = 1;
+  s.server_workers = n_workers;
+  s.atr_entries = kWays << sets_log2;
+  s.sm_count = (uint32_t)h->sm_count;
+  s.kernel_launches = 1;
+  h->last_n_tx = n_tx;
+  h->last_log_mode = w->log_mode;
+  h->last_max_vals = max_vals;
+  if (ctl.error) {
+    h->loaded = false;
+    return set_err(CSMV_ETIMEOUT, "csmv_run: device watchdog fired (loop %u); store state undefined",
+                   ctl.where);
+  }
+  if (s.committed_update + s.committed_ro != n_tx || gts1 != ctl.tail_final)
+    return set_err(CSMV_ECUDA, "csmv_run: protocol error (committed %llu of %llu, gts %u, tail %u)",
+                   (unsigned long long)(s.committed_update + s.committed_ro),
+                   (unsigned long long)n_tx, gts1, ctl.tail_final);
+  return CSMV_OK;
+}
+
+int csmv_stats(const csmv_t* h, csmv_stats_t* out) {
+  if (!h || !out) return set_err(CSMV_EINVAL, "csmv_stats: null argument");
+  *out = h->last;
+  return CSMV_OK;
+}
+
+int csmv_get_log(const csmv_t* h, csmv_log_rec* buf, uint64_t cap, uint64_t* n_out) {
+  if (!h || !buf) return set_err(CSMV_EINVAL, "csmv_get_log: null argument");
+  if (h->last_log_mode == CSMV_LOG_NONE || !h->d_log)
+    return set_err(CSMV_ESTATE, "csmv_get_log: last run had no log");
+  if (cap < h->last_n_tx) return set_err(CSMV_EOVERFLOW, "csmv_get_log: cap %llu < n_tx %llu",
+                                         (unsigned long long)cap, (unsigned long long)h->last_n_tx);
+  CK(cudaMemcpy(buf, h->d_log, h->last_n_tx * sizeof(csmv_log_rec), cudaMemcpyDeviceToHost));
+  if (n_out) *n_out = h->last_n_tx;
+  return CSMV_OK;
+}
+
+int csmv_get_vals(const csmv_t* h, uint32_t* buf, uint64_t cap_words, uint32_t* max_vals) {
+  if (!h) return set_err(CSMV_EINVAL, "csmv_get_vals: null handle");
+  if (h->last_log_mode != CSMV_LOG_FULL) return set_err(CSMV_ESTATE, "csmv_get_vals: last run not FULL");
+  if (max_vals) *max_vals = h->last_max_vals;
+  if (!buf) return CSMV_OK;
+  const uint64_t words = h->last_n_tx * (uint64_t)h->last_max_vals;
+  if (cap_words < words) return set_err(CSMV_EOVERFLOW, "csmv_get_vals: buffer too small");
+  CK(cudaMemcpy(buf, h->d_vals, words * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+  return CSMV_OK;
+}
+
+int csmv_dump_store(const csmv_t* h, uint64_t* out, uint64_t cap) {
+  if (!h || !out) return set_err(CSMV_EINVAL, "csmv_dump_store: null argument");
+  if (h->kind != CSMV_KIND_BANK) return set_err(CSMV_EINVAL, "csmv_dump_store: not a bank store");
+  if (cap < h->n_items * h->K) return set_err(CSMV_EOVERFLOW, "csmv_dump_store: cap too small");
+  std::vector<uint64_t> raw(h->n_items * h->nslot);
+  CK(cudaMemcpy(raw.data(), h->d_rings, raw.size() * sizeof(uint64_t), cudaMemcpyDeviceToHost));
+  for (uint64_t i = 0; i < h->n_items; ++i)
+    for (uint32_t j = 0; j < h->K; ++j) out[i * h->K + j] = raw[i * h->nslot + j];
+  return CSMV_OK;
+}
+
+int csmv_dump_kv(const csmv_t* h, uint32_t*, uint32_t*, uint32_t*, uint32_t*) {
+  if (!h) return set_err(CSMV_EINVAL, "null handle");
+  return set_err(CSMV_EINVAL, "csmv_dump_kv: KV store not built in this version");
+}
+
+int csmv_gen_descs(csmv_t* h, const csmv_workload* w, uint64_t seed, uint64_t tx0, uint64_t n,
+                   uint32_t* out) {
+  if (!h || !w || !out) return set_err(CSMV_EINVAL, "csmv_gen_descs: null argument");
+  GenParams g;
+  int rc = make_gen(h, w, seed, &g);
+  if (rc) return rc;
+  uint32_t* d = nullptr;
+  CK(cudaMalloc(&d, n * 6 * sizeof(uint32_t) + 4));
+  cudaError_t e = launch_gen_descs(g, tx0, n, d, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess) e = cudaMemcpy(out, d, n * 6 * sizeof(uint32_t), cudaMemcpyDeviceToHost);
+  cudaFree(d);
+  if (e != cudaSuccess) return set_err(CSMV_ECUDA, "csmv_gen_descs: %s", cudaGetErrorString(e));
+  return CSMV_OK;
+}
+
+int csmv_zipf_table(uint32_t n, uint32_t theta_milli, uint64_t* out) {
+  if (!out || n == 0) return set_err(CSMV_EINVAL, "csmv_zipf_table: bad argument");
+  std::vector<uint64_t> c = build_zipf(n, theta_milli);
+  memcpy(out, c.data(), n * sizeof(uint64_t));
+  return CSMV_OK;
+}
+
+}  // extern "C"

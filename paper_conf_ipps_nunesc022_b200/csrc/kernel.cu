@@ -1,0 +1,721 @@
+// kernel.cu -- the fused persistent CSMV kernel for sm_100a.
+//
+// One cooperative grid holds both roles of the paper's client-server split
+// (P:99-105): CTA 0 is the server SM, CTAs 1..C are client SMs.  Fusing the
+// roles into one launch guarantees co-residency of a server that spins on
+// its clients (the paper launches two kernels; separate kernels deadlock when
+// a profiler serialises them).
+//
+// Client warp, one round (section III):
+//   TXBegin     s <- GTS (one acquire load per warp round)
+//   TXRead      newest version with ts <= s from the VBox ring
+//               read-only lanes finish here, no commit
+//   pre-validation of the warp's update lanes (shuffle/ballot)
+//   submit the batch (request slot + doorbell), wait for the response P:101
+//   write-back of the new versions by the client
+//   ordered GTS advance by n (CSMV_PUBLISH_CLIENT) or a done
+//   flag per CTS for the server publisher (CSMV_PUBLISH_SERVER)
+//   aborted lanes retry with a fresh snapshot next round
+//
+// Server CTA: worker warps each own a contiguous slice of client doorbells
+// (receiving and working are merged per warp); a batch is
+// validated by the whole warp (one lane per transaction, __ballot_sync /
+// __match_any_sync) against the ATR, which lives in shared memory as an
+// item-indexed set-associative table of (item, last CTS) covering every
+// commit after the watermark W_low;
+// consecutive CTS are reserved and the write-sets inserted inside one
+// shared-memory critical section.  No global atomics on the
+// commit path.
+#include <cuda_runtime.h>
+
+#include "kernel.cuh"
+#include "ptx.cuh"
+
+namespace csmvd {
+
+enum : int { ST_NONE = 0, ST_RO_OK, ST_CAND, ST_UPD_OK, ST_ABORT };
+
+// --------------------------------------------------------------------------
+// VBox read (TXRead) and write-back
+// --------------------------------------------------------------------------
+struct Sel {
+  int best;          // slot of the newest version with ts <= s, -1 if none
+  uint32_t best_ts;
+  uint32_t newest;   // largest ts present
+};
+
+template <int NS>
+__device__ __forceinline__ Sel select_version(const Ring<NS>& r, uint32_t s) {
+  Sel q{-1, 0u, 0u};
+#pragma unroll
+  for (int j = 0; j < NS; ++j) {
+    uint32_t ts = (uint32_t)(r.s[j] >> 32);
+    if (ts != kEmptyTs) {
+      q.newest = max(q.newest, ts);
+      if (ts <= s && (q.best < 0 || ts > q.best_ts)) {
+        q.best = j;
+        q.best_ts = ts;
+      }
+    }
+  }
+  return q;
+}
+
+template <int NS>
+__device__ __forceinline__ uint64_t slot_at(const Ring<NS>& r, int j) {
+  uint64_t v = r.s[0];
+#pragma unroll
+  for (int i = 1; i < NS; ++i) v = (j == i) ? r.s[i] : v;
+  return v;
+}
+
+// Replace the first unused slot, else the oldest version.  The
+// writer owns the item: the WW check orders all writers of an item
+// and the ring is unchanged since this transaction read it.
+template <int NS>
+__device__ __forceinline__ void write_back(uint64_t* ring, const Ring<NS>& r, uint32_t K,
+                                           uint32_t cts, uint32_t val) {
+  int victim = -1;
+  uint32_t vts = kEmptyTs;
+#pragma unroll
+  for (int j = 0; j < NS; ++j) {
+    uint32_t ts = (uint32_t)(r.s[j] >> 32);
+    if ((uint32_t)j < K && victim < 0 && ts == kEmptyTs) victim = j;
+  }
+  if (victim < 0) {
+    victim = 0;
+    vts = (uint32_t)(r.s[0] >> 32);
+#pragma unroll
+    for (int j = 1; j < NS; ++j) {
+      uint32_t ts = (uint32_t)(r.s[j] >> 32);
+      if ((uint32_t)j < K && ts < vts) {
+        victim = j;
+        vts = ts;
+      }
+    }
+  }
+  st_relaxed64(ring + victim, ((uint64_t)cts << 32) | val);
+}
+
+__device__ __forceinline__ bool watchdog(const KParams& p, uint64_t t0, uint32_t where) {
+  if (globaltimer() - t0 > p.watchdog_ns) {
+    if (atomicCAS(&p.ctl->error, 0u, 1u) == 0u) p.ctl->where = where;
+    return true;
+  }
+  return false;
+}
+
+// --------------------------------------------------------------------------
+// Read-only transaction: L consecutive accounts (or all)
+// --------------------------------------------------------------------------
+template <int NS>
+__device__ __forceinline__ bool rot_scan(const KParams& p, uint32_t start, uint32_t len, uint32_t s,
+                                         uint64_t tx, int64_t& sum, uint64_t& dg) {
+  constexpr int U = 4;
+  sum = 0;
+  dg = 0;
+  const uint32_t N = p.n_items;
+  uint32_t x = start;
+  for (uint32_t j = 0; j < len; j += U) {
+    Ring<NS> r[U];
+    uint32_t xs[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      xs[u] = x;
+      if (j + u < len) r[u] = ld_ring<NS>(p.rings + (size_t)x * NS);
+      x = (x + 1 == N) ? 0u : x + 1;
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (j + u >= len) break;
+      Sel q = select_version<NS>(r[u], s);
+      if (q.best < 0) return false;  // version recycled
+      uint64_t v = slot_at<NS>(r[u], q.best);
+      if (q.newest > s) {
+        // A newer version exists, so write-backs may have overwritten slots
+        // while we read.  Versions are evicted oldest first, so if the chosen
+        // slot still holds the same version, no version in (best_ts, s] was
+        // missed; otherwise the snapshot's version is gone.
+        if (ld_relaxed64(p.rings + (size_t)xs[u] * NS + q.best) != v) return false;
+      }
+      int32_t val = (int32_t)(uint32_t)v;
+      sum += val;
+      if (p.log_mode) {
+        dg += dig1(xs[u], (uint32_t)val);
+        if (p.log_mode == CSMV_LOG_FULL && j + u < p.max_vals)
+          p.vals[tx * p.max_vals + j + u] = (uint32_t)val;
+      }
+    }
+  }
+  return true;
+}
+
+// --------------------------------------------------------------------------
+// Client warp
+// --------------------------------------------------------------------------
+template <int NS>
+__device__ void client_warp(const KParams& p, uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t cw = (threadIdx.x >> 5) * p.n_client_ctas + (blockIdx.x - 1);
+  if (cw >= p.n_cw) return;
+  const uint64_t T = (uint64_t)p.n_cw * 32;
+  uint64_t cur = (uint64_t)cw * 32 + lane;  // static assignment: tx = lane + k*T
+  uint32_t att = 0;
+  uint32_t c_upd = 0, c_ro = 0, n_batches = 0, n_rounds = 0;
+  uint32_t ab[CSMV_N_ABORT][2];
+#pragma unroll
+  for (int i = 0; i < (int)CSMV_N_ABORT; ++i) ab[i][0] = ab[i][1] = 0;
+  uint64_t ro_ck = 0;
+  uint32_t round = 0;
+  uint32_t* my_ids = p.req_ids + (size_t)cw * 2 * 32;
+  const uint32_t K = p.K;
+  const uint32_t lt = lanemask_lt();
+
+  for (;;) {
+    const bool has = cur < p.n_tx;
+    if (!__any_sync(FULL, has)) break;
+    ++round;
+    ++n_rounds;
+    uint32_t s = 0, err = 0;
+    if (lane == 0) {
+      s = ld_acquire(p.gts);  // TXBegin: snapshot
+      err = ld_relaxed(&p.ctl->error);
+    }
+    s = __shfl_sync(FULL, s, 0);
+    if (__shfl_sync(FULL, err, 0)) break;
+
+    int status = ST_NONE;
+    int reason = 0;
+    BankTx d{};
+    Ring<NS> rs{}, rd{};
+    uint32_t vs = 0, vd = 0;
+    int64_t rsum = 0;
+    uint64_t rdig = 0;
+    if (has) {
+      ++att;
+      d = gen_bank(p.gen, cur);
+      if (!d.is_update) {
+        status = rot_scan<NS>(p, d.start, d.len, s, cur, rsum, rdig) ? ST_RO_OK : ST_ABORT;
+        reason = CSMV_AB_VERSION;
+      } else {
+        rs = ld_ring<NS>(p.rings + (size_t)d.src * NS);
+        rd = ld_ring<NS>(p.rings + (size_t)d.dst * NS);
+        Sel qs = select_version<NS>(rs, s), qd = select_version<NS>(rd, s);
+        if (qs.newest > s || qd.newest > s) {
+          status = ST_ABORT;  // a commit after s wrote it: validation must fail
+          reason = CSMV_AB_EARLY;
+        } else if (qs.best < 0 || qd.best < 0) {
+          status = ST_ABORT;
+          reason = CSMV_AB_VERSION;
+        } else {
+          vs = (uint32_t)slot_at<NS>(rs, qs.best);
+          vd = (uint32_t)slot_at<NS>(rd, qd.best);
+          status = ST_CAND;
+        }
+      }
+    }
+
+    // Client-side pre-validation: greedy in lane order, a lane is
+    // dropped if it shares an item with an earlier kept lane (RS = WS).
+    const uint32_t cand = __ballot_sync(FULL, status == ST_CAND);
+    uint32_t kept = cand;
+    if (!(p.debug & CSMV_DBG_NO_PREVAL)) {
+      kept = 0;
+      uint32_t rem = cand;
+      while (rem) {
+        const int i = __ffs(rem) - 1;
+        const uint32_t a = __shfl_sync(FULL, d.src, i), b = __shfl_sync(FULL, d.dst, i);
+        kept |= 1u << i;
+        const bool conf = ((rem >> lane) & 1u) && lane > (uint32_t)i &&
+                          (d.src == a || d.src == b || d.dst == a || d.dst == b);
+        rem &= ~__ballot_sync(FULL, conf) & ~(1u << i);
+      }
+    }
+    const bool mine = (kept >> lane) & 1u;
+    if (status == ST_CAND && !mine) {
+      status = ST_ABORT;
+      reason = CSMV_AB_PREVAL;
+    }
+
+    uint32_t cts = 0, ns = 0, nd = 0;
+    if (kept) {
+      // Batch submit: ids, header, then the doorbell.
+      if (mine) {
+        my_ids[lane] = d.src | kWriteBit;
+        my_ids[32 + lane] = d.dst | kWriteBit;
+      }
+      if (lane == 0) {
+        p.req_hdr[cw].snapshot = s;
+        p.req_hdr[cw].mask = kept;
+        ++n_batches;
+      }
+      __syncwarp();
+      fence_gpu();
+      uint32_t base = 0, cmask = 0, omask = 0;
+      if (lane == 0) {
+        st_relaxed(&p.req_seq[cw], round);
+        uint32_t it = 0;
+        bool ok = true;
+        while (ld_relaxed(&p.resp[cw].seq) != round) {
+          if ((++it & 255u) == 0 && (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1))) {
+            ok = false;
+            break;
+          }
+          __nanosleep(64);
+        }
+        fence_gpu();  // acquire: response payload after its seq
+        if (ok) {
+          base = ld_relaxed(&p.resp[cw].cts_base);
+          cmask = ld_relaxed(&p.resp[cw].commit_mask);
+          omask = ld_relaxed(&p.resp[cw].overflow_mask);
+        }
+      }
+      base = __shfl_sync(FULL, base, 0);
+      cmask = __shfl_sync(FULL, cmask, 0);
+      omask = __shfl_sync(FULL, omask, 0);
+      if (mine) {
+        if ((cmask >> lane) & 1u) {
+          // Client-side write-back with CTS = base + rank.
+          cts = base + __popc(cmask & lt);
+          ns = vs - (uint32_t)d.amt;
+          nd = vd + (uint32_t)d.amt;
+          write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
+          write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
+          status = ST_UPD_OK;
+        } else {
+          status = ST_ABORT;
+          reason = ((omask >> lane) & 1u) ? CSMV_AB_OVERFLOW : CSMV_AB_CONFLICT;
+        }
+      }
+      const uint32_t n = __popc(cmask);
+      if (n) {
+        if (p.publish == CSMV_PUBLISH_CLIENT) {
+          // Advance GTS by n once every earlier commit is visible:
+          // spin until GTS == first CTS - 1 ("GTS 1" = GTS+1).
+          __syncwarp();
+          fence_gpu();
+          if (lane == 0) {
+            uint32_t it = 0;
+            while (ld_relaxed(p.gts) != base - 1) {
+              if ((++it & 255u) == 0 &&
+                  (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 2))) break;
+              __nanosleep(32);
+            }
+            st_release(p.gts, base + n - 1);  // release also orders the write-backs
+          }
+        } else if (status == ST_UPD_OK) {
+          st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
+        }
+      }
+    }
+
+    if (status == ST_RO_OK || status == ST_UPD_OK) {
+      if (p.log_mode) {
+        csmv_log_rec rec;
+        rec.tx = (uint32_t)cur;
+        rec.snapshot = s;
+        rec.cts = cts;
+        rec.attempts = att;
+        if (status == ST_RO_OK) {
+          rec.read_digest = rdig;
+          rec.aux = (uint64_t)rsum;
+        } else {
+          rec.read_digest = dig1(d.src, vs) + dig1(d.dst, vd);
+          rec.aux = dig1(d.src, ns) + dig1(d.dst, nd);
+          if (p.log_mode == CSMV_LOG_FULL && p.max_vals >= 2) {
+            p.vals[cur * p.max_vals] = vs;
+            p.vals[cur * p.max_vals + 1] = vd;
+          }
+        }
+        p.log[cur] = rec;
+      }
+      if (status == ST_RO_OK) {
+        ++c_ro;
+        ro_ck ^= (uint64_t)rsum;
+      } else {
+        ++c_upd;
+      }
+      cur += T;
+      att = 0;
+    } else if (status == ST_ABORT) {
+#pragma unroll
+      for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
+        if (reason == i) ++ab[i][d.is_update ? 1 : 0];
+      }
+    }
+  }
+
+  // flush per-warp counters once (no global atomics on the commit path)
+  const uint32_t s_upd = __reduce_add_sync(FULL, c_upd), s_ro = __reduce_add_sync(FULL, c_ro);
+  uint32_t s_ab[CSMV_N_ABORT][2];
+#pragma unroll
+  for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
+    s_ab[i][0] = __reduce_add_sync(FULL, ab[i][0]);
+    s_ab[i][1] = __reduce_add_sync(FULL, ab[i][1]);
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) ro_ck ^= __shfl_xor_sync(FULL, ro_ck, o);
+  if (lane == 0) {
+    atomicAdd(&p.stats->committed_update, (unsigned long long)s_upd);
+    atomicAdd(&p.stats->committed_ro, (unsigned long long)s_ro);
+    for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
+      if (s_ab[i][0]) atomicAdd(&p.stats->aborts[i][0], (unsigned long long)s_ab[i][0]);
+      if (s_ab[i][1]) atomicAdd(&p.stats->aborts[i][1], (unsigned long long)s_ab[i][1]);
+    }
+    atomicAdd(&p.stats->rounds, (unsigned long long)n_rounds);
+    atomicXor(&p.stats->ro_checksum, (unsigned long long)ro_ck);
+    __threadfence();
+    atomicAdd(&p.ctl->done_warps, 1u);
+  }
+  (void)n_batches;
+}
+
+// --------------------------------------------------------------------------
+// Server CTA
+// --------------------------------------------------------------------------
+struct SrvShared {
+  uint32_t tail;         // last CTS assigned (the CTS counter)
+  uint32_t wlow;         // every commit with CTS > wlow is in the ATR
+  uint32_t next_ticket;  // ticket lock around validate+reserve+insert
+  uint32_t now_serving;
+  uint32_t gts_seen;     // publisher progress seen by workers (back-pressure)
+};
+
+__device__ __forceinline__ uint32_t atr_set(uint32_t key, uint32_t sets_log2) {
+  return (key * 0x9E3779B1u) >> (32 - sets_log2);
+}
+
+// conflict iff some ATR entry for `key` has CTS > s
+__device__ __forceinline__ bool atr_conflict(const uint64_t* htab, uint32_t sets_log2, uint32_t key,
+                                             uint32_t s) {
+  const ulonglong2* e = reinterpret_cast<const ulonglong2*>(htab + (size_t)atr_set(key, sets_log2) * kWays);
+  bool c = false;
+#pragma unroll
+  for (int j = 0; j < (int)kWays / 2; ++j) {
+    ulonglong2 v = e[j];
+    c |= ((uint32_t)v.x == key && (uint32_t)(v.x >> 32) > s);
+    c |= ((uint32_t)v.y == key && (uint32_t)(v.y >> 32) > s);
+  }
+  return c;
+}
+
+// Insert (key, cts) for every lane with `active`; lanes whose keys map to
+// the same set are serialised with __match_any_sync.  A full set evicts its
+// oldest entry and raises W_low to that entry's CTS.
+__device__ __forceinline__ void atr_insert(uint64_t* htab, uint32_t sets_log2, SrvShared* sh,
+                                           uint32_t key, uint32_t cts, bool active) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t set = atr_set(key, sets_log2);
+  bool pending = active;
+  for (;;) {
+    const uint32_t act = __ballot_sync(0xFFFFFFFFu, pending);
+    if (!act) break;
+    if (pending) {
+      const uint32_t peers = __match_any_sync(act, set);
+      if (lane == (uint32_t)(__ffs(peers) - 1)) {
+        uint64_t* e = htab + (size_t)set * kWays;
+        int hit = -1, vic = 0;
+        uint32_t vmin = 0xFFFFFFFFu;
+#pragma unroll
+        for (int j = 0; j < (int)kWays; ++j) {
+          uint64_t v = e[j];
+          uint32_t c = (uint32_t)(v >> 32);
+          if ((uint32_t)v == key) hit = j;
+          if (c < vmin) {
+            vmin = c;
+            vic = j;
+          }
+        }
+        if (hit >= 0) {
+          vic = hit;
+        } else if (vmin > *(volatile uint32_t*)&sh->wlow) {
+          atomicMax(&sh->wlow, vmin);  // evicting a live entry (bounded ATR)
+        }
+        e[vic] = ((uint64_t)cts << 32) | key;
+        pending = false;
+      }
+    }
+    __syncwarp();
+  }
+}
+
+__device__ void server_worker(const KParams& p, uint64_t* htab, uint32_t* last_seen, SrvShared* sh,
+                              uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t per = (p.n_cw + p.n_workers - 1) / p.n_workers;
+  const uint32_t base = warp * per;
+  const uint32_t end = min(base + per, p.n_cw);
+  const uint32_t lt = lanemask_lt();
+  const uint32_t dmask = (1u << kDoneLog2) - 1;
+  unsigned long long busy = 0, locked = 0, batches = 0;
+  uint32_t spins = 0;
+  for (;;) {
+    // Receive: one coalesced sweep over this warp's doorbells.
+    uint32_t seq[kMaxPoll];
+    uint32_t pend[kMaxPoll];
+#pragma unroll
+    for (int k = 0; k < kMaxPoll; ++k) {
+      const uint32_t w = base + k * 32 + lane;
+      seq[k] = (w < end) ? ld_relaxed(p.req_seq + w) : 0u;
+    }
+    bool any = false;
+#pragma unroll
+    for (int k = 0; k < kMaxPoll; ++k) {
+      const uint32_t w = base + k * 32 + lane;
+      pend[k] = __ballot_sync(FULL, w < end && seq[k] != last_seen[w]);
+      any |= pend[k] != 0;
+    }
+    if (!any) {
+      if ((++spins & 63u) == 0) {
+        uint32_t dw = 0, er = 0;
+        if (lane == 0) {
+          dw = ld_relaxed(&p.ctl->done_warps);
+          er = ld_relaxed(&p.ctl->error);
+          if (!er && dw < p.n_cw && watchdog(p, t_begin, 3)) er = 1;
+        }
+        dw = __shfl_sync(FULL, dw, 0);
+        er = __shfl_sync(FULL, er, 0);
+        if (dw >= p.n_cw || er) break;
+      }
+      continue;
+    }
+    fence_gpu();  // acquire: doorbells seen before payload loads
+#pragma unroll
+    for (int k = 0; k < kMaxPoll; ++k) {
+      uint32_t pm = pend[k];
+      while (pm) {
+        const int i = __ffs(pm) - 1;
+        pm &= pm - 1;
+        const uint32_t cw = base + k * 32 + i;
+        const uint32_t sq = __shfl_sync(FULL, seq[k], i);
+        const long long t0 = clock64();
+        // Load the batch: header broadcast + one id row per RS u WS entry.
+        const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
+        const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
+        const bool mine = (mask >> lane) & 1u;
+        uint32_t id0 = 0, id1 = 0;
+        if (mine) {
+          id0 = ld_relaxed(p.req_ids + (size_t)cw * 64 + lane) & ~kWriteBit;
+          id1 = ld_relaxed(p.req_ids + (size_t)cw * 64 + 32 + lane) & ~kWriteBit;
+        }
+        // ---- critical section: validate, reserve CTS, insert
+        uint32_t ticket = 0;
+        if (lane == 0) {
+          ticket = atomicAdd(&sh->next_ticket, 1u);
+          while (*(volatile uint32_t*)&sh->now_serving != ticket) __nanosleep(20);
+        }
+        __syncwarp();
+        __threadfence_block();
+        const long long t1 = clock64();
+        const uint32_t t0c = *(volatile uint32_t*)&sh->tail;
+        const uint32_t wl = *(volatile uint32_t*)&sh->wlow;
+        const bool ovf = mine && s < wl;
+        bool conflict = false;
+        if (mine && !ovf && !(p.debug & CSMV_DBG_NO_VALIDATE))
+          conflict = atr_conflict(htab, p.sets_log2, id0, s) || atr_conflict(htab, p.sets_log2, id1, s);
+        const bool commit = mine && !ovf && !conflict;
+        const uint32_t cm = __ballot_sync(FULL, commit);
+        const uint32_t n = __popc(cm);
+        const uint32_t cts = t0c + 1 + __popc(cm & lt);
+        if (p.publish == CSMV_PUBLISH_SERVER && n) {
+          // done ring back-pressure: CTS c may reuse slot c & dmask only once
+          // GTS >= c - 2^20
+          if (lane == 0) {
+            uint32_t it = 0;
+            while (t0c + n > sh->gts_seen + dmask) {
+              sh->gts_seen = ld_relaxed(p.gts);
+              if ((++it & 255u) == 0 && watchdog(p, t_begin, 4)) break;
+            }
+          }
+          __syncwarp();
+        }
+        atr_insert(htab, p.sets_log2, sh, id0, cts, commit);
+        atr_insert(htab, p.sets_log2, sh, id1, cts, commit);
+        __syncwarp();
+        __threadfence_block();
+        if (lane == 0) {
+          sh->tail = t0c + n;
+          __threadfence_block();
+          *(volatile uint32_t*)&sh->now_serving = ticket + 1;
+        }
+        const long long t2 = clock64();
+        // ---- respond
+        const uint32_t om = __ballot_sync(FULL, ovf);
+        if (lane == 0) {
+          st_relaxed(&p.resp[cw].cts_base, t0c + 1);
+          st_relaxed(&p.resp[cw].commit_mask, cm);
+          st_relaxed(&p.resp[cw].overflow_mask, om);
+          st_release(&p.resp[cw].seq, sq);
+          last_seen[cw] = sq;
+        }
+        __syncwarp();
+        busy += (unsigned long long)(t2 - t0);
+        locked += (unsigned long long)(t2 - t1);
+        ++batches;
+      }
+    }
+  }
+  if (lane == 0) {
+    atomicAdd(&p.stats->batches, batches);
+    atomicAdd(&p.stats->busy_cycles, busy);
+    atomicAdd(&p.stats->lock_cycles, locked);
+  }
+}
+
+// CSMV_PUBLISH_SERVER: advance GTS over the prefix of CTS whose write-backs
+// are done.  Same invariant as P:116 (GTS = c only once every commit <= c
+// has written back), without a client-side serial chain.
+__device__ void server_publisher(const KParams& p, SrvShared* sh, uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t dmask = (1u << kDoneLog2) - 1;
+  uint32_t g = *(volatile uint32_t*)&sh->tail;
+  uint32_t spins = 0;
+  for (;;) {
+    uint32_t v[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) v[k] = ld_relaxed(p.done_ring + ((g + 1 + k * 32 + lane) & dmask));
+    uint32_t adv = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const uint32_t bad = __ballot_sync(FULL, v[k] != g + 1 + k * 32 + lane);
+      if (adv == (uint32_t)k * 32) adv += bad ? (uint32_t)(__ffs(bad) - 1) : 32u;
+    }
+    if (adv) {
+      fence_gpu();
+      g += adv;
+      if (lane == 0) st_release(p.gts, g);
+      continue;
+    }
+    if ((++spins & 63u) == 0) {
+      uint32_t dw = 0, er = 0;
+      if (lane == 0) {
+        dw = ld_relaxed(&p.ctl->done_warps);
+        er = ld_relaxed(&p.ctl->error);
+        if (!er && watchdog(p, t_begin, 5)) er = 1;
+      }
+      dw = __shfl_sync(FULL, dw, 0);
+      er = __shfl_sync(FULL, er, 0);
+      if (er) break;
+      if (dw >= p.n_cw && g == *(volatile uint32_t*)&sh->tail) break;
+    }
+  }
+}
+
+__device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
+  uint64_t* htab = reinterpret_cast<uint64_t*>(smem);
+  const uint32_t n_entries = kWays << p.sets_log2;
+  uint32_t* last_seen = reinterpret_cast<uint32_t*>(htab + n_entries);
+  const uint32_t ls_words = (p.n_cw + 31) / 32 * 32;
+  SrvShared* sh = reinterpret_cast<SrvShared*>(last_seen + ls_words);
+  for (uint32_t i = threadIdx.x; i < n_entries; i += blockDim.x) htab[i] = 0xFFFFFFFFull;  // cts 0, no key
+  for (uint32_t i = threadIdx.x; i < ls_words; i += blockDim.x) last_seen[i] = 0;
+  if (threadIdx.x == 0) {
+    const uint32_t g0 = *p.gts;
+    sh->tail = g0;
+    sh->wlow = g0;
+    sh->next_ticket = 0;
+    sh->now_serving = 0;
+    sh->gts_seen = g0;
+  }
+  __syncthreads();
+  const uint32_t warp = threadIdx.x >> 5;
+  if (warp < p.n_workers) {
+    server_worker(p, htab, last_seen, sh, t_begin);
+  } else if (warp == p.n_workers && p.publish == CSMV_PUBLISH_SERVER) {
+    server_publisher(p, sh, t_begin);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) p.ctl->tail_final = sh->tail;
+}
+
+template <int NS>
+__global__ void __launch_bounds__(kBlock, 1) csmv_fused(const KParams p) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const uint64_t t_begin = globaltimer();
+  if (blockIdx.x == 0) server_cta(p, smem, t_begin);
+  else client_warp<NS>(p, t_begin);
+}
+
+template <int NS>
+__global__ void init_rings(uint64_t* rings, const int32_t* init, uint64_t n, uint32_t* gts) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i == 0) *gts = 0;
+  if (i >= n) return;
+  Ring<NS> r;
+#pragma unroll
+  for (int j = 0; j < NS; ++j) r.s[j] = (uint64_t)kEmptyTs << 32;
+  r.s[0] = (uint64_t)(uint32_t)init[i];
+  *reinterpret_cast<Ring<NS>*>(rings + i * NS) = r;
+}
+
+__global__ void gen_descs_kernel(GenParams g, uint64_t tx0, uint64_t n, uint32_t* out) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  BankTx d = gen_bank(g, tx0 + i);
+  uint32_t* o = out + i * 6;
+  o[0] = d.is_update;
+  o[1] = d.src;
+  o[2] = d.dst;
+  o[3] = (uint32_t)d.amt;
+  o[4] = d.start;
+  o[5] = d.len;
+}
+
+template <int NS>
+static cudaError_t launch_ns(const KParams& p, uint32_t grid, size_t smem, cudaStream_t st) {
+  cudaError_t e = cudaFuncSetAttribute(csmv_fused<NS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  void* args[] = {(void*)&p};
+  return cudaLaunchCooperativeKernel((const void*)csmv_fused<NS>, dim3(grid), dim3(kBlock), args, smem, st);
+}
+
+cudaError_t launch_fused(const KParams& p, uint32_t nslot, uint32_t grid, size_t smem, cudaStream_t st) {
+  switch (nslot) {
+    case 2: return launch_ns<2>(p, grid, smem, st);
+    case 4: return launch_ns<4>(p, grid, smem, st);
+    case 8: return launch_ns<8>(p, grid, smem, st);
+    case 16: return launch_ns<16>(p, grid, smem, st);
+  }
+  return cudaErrorInvalidValue;
+}
+
+template <int NS>
+static cudaError_t occ_ns(size_t smem, int* b) {
+  cudaError_t e = cudaFuncSetAttribute(csmv_fused<NS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(b, csmv_fused<NS>, kBlock, smem);
+}
+
+cudaError_t fused_occupancy(uint32_t nslot, size_t smem, int* b) {
+  switch (nslot) {
+    case 2: return occ_ns<2>(smem, b);
+    case 4: return occ_ns<4>(smem, b);
+    case 8: return occ_ns<8>(smem, b);
+    case 16: return occ_ns<16>(smem, b);
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_init_rings(uint64_t* rings, uint32_t nslot, const int32_t* init, uint64_t n,
+                              uint32_t* gts, cudaStream_t st) {
+  const uint32_t blocks = (uint32_t)((n + 255) / 256) + 1;
+  switch (nslot) {
+    case 2: init_rings<2><<<blocks, 256, 0, st>>>(rings, init, n, gts); break;
+    case 4: init_rings<4><<<blocks, 256, 0, st>>>(rings, init, n, gts); break;
+    case 8: init_rings<8><<<blocks, 256, 0, st>>>(rings, init, n, gts); break;
+    case 16: init_rings<16><<<blocks, 256, 0, st>>>(rings, init, n, gts); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_gen_descs(GenParams g, uint64_t tx0, uint64_t n, uint32_t* out, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  gen_descs_kernel<<<(uint32_t)((n + 255) / 256), 256, 0, st>>>(g, tx0, n, out);
+  return cudaGetLastError();
+}
+
+}  // namespace csmvd

@@ -1,0 +1,99 @@
+// kernel.cuh -- device-side data layout shared by host.cu and kernel.cu.
+//
+// HBM layout (one handle):
+//   rings     u64[n_items][NSLOT]   packed (ts << 32 | value) versions; NSLOT
+//                                   = K rounded up to 2/4/8/16 so a VBox is one
+//                                   aligned record (32 B = one sector at K = 4)
+//   gts       u32                   the global timestamp GTS
+//   req_seq   u32[n_cw]             per client warp request doorbell
+//   req_hdr   {snapshot, mask}[n_cw]
+//   req_ids   u32[n_cw][MAXID][32]  lane-major item ids of RS u WS (bit 31 =
+//                                   also in WS); coalesced 128 B rows
+//   resp      {cts_base, commit_mask, overflow_mask, seq}[n_cw]
+//   done_ring u32[2^20]             CSMV_PUBLISH_SERVER: done[cts & mask] = cts
+//                                   after the write-back of cts
+//   log       csmv_log_rec[n_tx]    parity runs only
+#pragma once
+#include <cstdint>
+
+#include "../../include/csmv.h"
+#include "gen.cuh"
+
+namespace csmvd {
+
+constexpr uint32_t kEmptyTs = 0xFFFFFFFFu;
+constexpr uint32_t kWriteBit = 0x80000000u;
+constexpr int kBlock = 512;            // threads per CTA (16 warps)
+constexpr int kWarps = kBlock / 32;
+constexpr int kMaxPoll = 8;            // doorbell words per worker lane (<= 256 warps/worker)
+constexpr uint32_t kDoneLog2 = 20;     // done ring entries (CSMV_PUBLISH_SERVER)
+constexpr uint32_t kWays = 8;          // ATR hash associativity (64 B per set)
+
+struct Ctl {
+  uint32_t error;       // 0 ok, 1 watchdog, 2 protocol
+  uint32_t done_warps;  // client warps that finished
+  uint32_t tail_final;  // server: last CTS assigned
+  uint32_t where;       // which spin loop fired the watchdog
+};
+
+struct ReqHdr {
+  uint32_t snapshot;
+  uint32_t mask;
+};
+
+struct Resp {
+  uint32_t cts_base;
+  uint32_t commit_mask;
+  uint32_t overflow_mask;
+  uint32_t seq;
+};
+
+struct DevStats {
+  unsigned long long committed_update, committed_ro;
+  unsigned long long aborts[CSMV_N_ABORT][2];
+  unsigned long long batches, rounds;
+  unsigned long long ro_checksum;
+  unsigned long long lock_cycles, busy_cycles;
+};
+
+struct KParams {
+  uint64_t* rings;
+  uint32_t n_items;
+  uint32_t K;
+  uint32_t* gts;
+  Ctl* ctl;
+  uint32_t* req_seq;
+  ReqHdr* req_hdr;
+  uint32_t* req_ids;
+  Resp* resp;
+  uint32_t* done_ring;
+  DevStats* stats;
+  csmv_log_rec* log;
+  uint32_t* vals;
+  uint32_t max_vals;
+  uint32_t log_mode;
+  GenParams gen;
+  uint64_t n_tx;
+  uint32_t n_cw;           // active client warps
+  uint32_t n_client_ctas;  // CTAs 1..n_client_ctas host clients
+  uint32_t n_workers;      // server worker warps
+  uint32_t sets_log2;      // ATR hash sets
+  uint32_t publish;
+  uint32_t debug;
+  uint64_t watchdog_ns;
+};
+
+// smem the server CTA needs (every CTA of the fused grid gets the same)
+inline size_t server_smem_bytes(uint32_t sets_log2, uint32_t n_cw) {
+  return ((size_t)kWays * 8u << sets_log2) + (((size_t)n_cw + 31) / 32 * 32) * 4 + 64;
+}
+
+// host-callable launchers (kernel.cu)
+cudaError_t launch_fused(const KParams& p, uint32_t nslot, uint32_t grid, size_t smem,
+                         cudaStream_t st);
+cudaError_t launch_init_rings(uint64_t* rings, uint32_t nslot, const int32_t* init, uint64_t n,
+                              uint32_t* gts, cudaStream_t st);
+cudaError_t launch_gen_descs(GenParams g, uint64_t tx0, uint64_t n, uint32_t* out, cudaStream_t st);
+cudaError_t fused_occupancy(uint32_t nslot, size_t smem, int* blocks_per_sm);
+
+}  // namespace csmvd

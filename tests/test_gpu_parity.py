@@ -1,0 +1,176 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle,
+element by element -- every committed transaction's snapshot, CTS, attempts,
+read digest and written values, every value a FULL log records, the final
+version rings, and the claimed counters."""
+import numpy as np
+import pytest
+
+import oracle
+from tests import _ref as R
+
+pytestmark = pytest.mark.gpu
+
+csmv = pytest.importorskip("paper_conf_ipps_nunesc022_b200.csmv")
+from paper_conf_ipps_nunesc022_b200 import workloads as W  # noqa: E402
+
+
+def oracle_cfg(cfg):
+    w = cfg.workload
+    return oracle.bank_cfg(cfg.n_items, cfg.n_versions, dist=w.dist,
+                           zipf_theta_milli=w.zipf_theta_milli, p_update_ppm=w.p_update_ppm,
+                           ro_period=w.ro_period, ro_reads=w.ro_reads, amount_max=w.amount_max)
+
+
+def run_gpu(cfg, init=None):
+    init = cfg.init_values() if init is None else init
+    with csmv.Store(cfg.n_items, cfg.n_versions) as st:
+        st.load(init)
+        stats = st.run(cfg.workload, cfg.n_tx, cfg.seed)
+        log = st.log(cfg.n_tx) if cfg.workload.log_mode else None
+        vals = st.vals() if cfg.workload.log_mode == csmv.LOG_FULL else (None, 0)
+        rings = st.dump()
+    return stats, log, vals, rings
+
+
+def check(cfg, init=None, expect_ok=True):
+    init = cfg.init_values() if init is None else init
+    stats, log, (vals, mv), rings = run_gpu(cfg, init)
+    ocfg = oracle_cfg(cfg)
+    descs = oracle.bank_gen(ocfg, cfg.seed, cfg.n_tx)
+    rep = oracle.bank_check(ocfg, init, descs, log, vals=vals, max_vals=mv, rings=rings,
+                            claims=dict(committed_update=stats["committed_update"],
+                                        committed_ro=stats["committed_ro"],
+                                        gts_final=stats["gts_final"],
+                                        total_aborts=stats["total_aborts"]))
+    if expect_ok:
+        assert rep["ok"], (cfg.name, rep, stats)
+    return rep, stats, log, rings, descs
+
+
+def closed_form(cfg, descs, init):
+    upd = descs["is_update"] == 1
+    final = init.astype(np.int64).copy()
+    np.add.at(final, descs["src"][upd], -descs["amt"][upd].astype(np.int64))
+    np.add.at(final, descs["dst"][upd], descs["amt"][upd].astype(np.int64))
+    return final.astype(np.int32)
+
+
+def newest(rings, n, k):
+    rr = rings.reshape(n, k)
+    ts = (rr >> np.uint64(32)).astype(np.int64)
+    ts[ts == R.EMPTY] = -1
+    return (rr[np.arange(n), ts.argmax(axis=1)] & np.uint64(0xFFFFFFFF)).astype(np.uint32).view(np.int32)
+
+
+@pytest.mark.parametrize("publish", [csmv.PUBLISH_CLIENT, csmv.PUBLISH_SERVER])
+def test_c1_full_parity(publish):
+    cfg = W.c1(publish=publish)
+    rep, stats, log, rings, descs = check(cfg)
+    init = cfg.init_values()
+    assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions), closed_form(cfg, descs, init))  # P1
+    assert np.all(log["aux"][descs["is_update"] == 0].view(np.int64) == 1024 * 1000)  # P2
+    assert stats["gts_final"] == 10000 and stats["committed_ro"] == 1111           # P3
+    assert sum(stats["aborts"][r]["ro"] for r in ("preval", "conflict", "early", "overflow")) == 0
+
+
+@pytest.mark.parametrize("k", [1, 2, 4, 8, 16])
+def test_one_warp_is_deterministic(k):
+    """with one client warp the oracle predicts every snapshot,
+    CTS, attempt count and ring exactly."""
+    cfg = W.c1(client_warps=1, n_versions=k, n_tx=3000, log_mode=csmv.LOG_FULL)
+    stats, log, (vals, mv), rings = run_gpu(cfg)
+    ocfg = oracle_cfg(cfg)
+    descs = oracle.bank_gen(ocfg, cfg.seed, cfg.n_tx)
+    plog, pvals, prings, pst = oracle.bank_predict(ocfg, cfg.init_values(), descs, 32, max_vals=mv)
+    bad = np.nonzero(log != plog)[0]
+    assert len(bad) == 0, (bad[:5], log[bad[:5]], plog[bad[:5]])
+    assert np.array_equal(vals, pvals)
+    assert np.array_equal(rings, prings)
+    assert stats["aborts"]["preval"]["update"] == pst["aborts_preval"]
+    assert stats["total_aborts"] == pst["aborts_preval"]
+    assert stats["batches"] == pst["batches"] and stats["rounds"] == pst["rounds"]
+
+
+@pytest.mark.parametrize("publish", [csmv.PUBLISH_CLIENT, csmv.PUBLISH_SERVER])
+def test_c2_shrunk_parity(publish):
+    cfg = W.c2(n_items=1 << 16, n_tx=1 << 18, publish=publish)
+    rep, stats, log, rings, descs = check(cfg)
+    assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions),
+                          closed_form(cfg, descs, cfg.init_values()))
+
+
+def test_c3_shrunk_parity():
+    cfg = W.c3(n_tx=1 << 18)
+    rep, stats, log, rings, descs = check(cfg)
+    assert stats["aborts"]["conflict"]["ro"] == 0 and stats["aborts"]["early"]["ro"] == 0  # P6/Q7
+
+
+def test_version_misses_k1():
+    """K = 1 under contention: read-only transactions restart only with
+    VERSION_MISS, and parity still holds."""
+    cfg = W.c3(n_versions=1, n_tx=1 << 16)
+    rep, stats, *_ = check(cfg)
+    assert stats["aborts"]["version"]["ro"] > 0
+    assert stats["aborts"]["conflict"]["ro"] == 0
+
+
+def test_tiny_atr_overflow():
+    """A tiny ATR forces evictions: spurious aborts appear only with the
+    labelled OVERFLOW reason and never let a conflicting commit through."""
+    cfg = W.c2(n_items=1 << 12, n_tx=1 << 17, atr_capacity=16)
+    rep, stats, *_ = check(cfg)
+    assert stats["aborts"]["overflow"]["update"] > 0
+
+
+def test_read_only_workload():
+    """P5: p_update = 0 leaves the store unchanged; zero aborts and no batches."""
+    cfg = W.c2(n_items=1 << 14, n_tx=1 << 16, p_update_ppm=0)
+    rep, stats, log, rings, _ = check(cfg)
+    assert stats["total_aborts"] == 0 and stats["batches"] == 0 and stats["gts_final"] == 0
+    assert np.all((rings.reshape(-1, cfg.n_versions)[:, 0] >> np.uint64(32)) == 0)
+
+
+def test_empty_run():
+    cfg = W.c2(n_items=1 << 10, n_tx=0)
+    stats, *_ = run_gpu(cfg)
+    assert stats["committed"] == 0 and stats["gts_final"] == 0
+
+
+def test_update_only_high_contention():
+    cfg = W.c2(n_items=64, n_tx=1 << 15, p_update_ppm=1_000_000, client_warps=64)
+    rep, stats, *_ = check(cfg)
+    assert stats["aborts"]["preval"]["update"] > 0
+
+
+def test_no_validate_is_caught():
+    """Negative control: a server that skips validation produces
+    a history the oracle rejects."""
+    cfg = W.c2(n_items=128, n_tx=1 << 15, p_update_ppm=900_000, client_warps=64,
+               debug_flags=csmv.DBG_NO_VALIDATE)
+    rep, *_ = check(cfg, expect_ok=False)
+    assert not rep["ok"]
+
+
+def test_generator_parity():
+    """the device generator equals the oracle's regenerated
+    descriptors, and the zipf tables are byte-equal."""
+    for cfg in (W.c1(), W.c2(n_items=1 << 20), W.c3()):
+        ocfg = oracle_cfg(cfg)
+        od = oracle.bank_gen(ocfg, 77, 50_000, tx0=123)
+        with csmv.Store(cfg.n_items, cfg.n_versions) as st:
+            gd = st.gen_descs(cfg.workload, 77, 50_000, tx0=123)
+        for j, f in enumerate(("is_update", "src", "dst", "amt", "start", "len")):
+            assert np.array_equal(gd[:, j], od[f].astype(np.uint32)), f
+    for n, th in ((4096, 990), (1 << 22, 990), (1000, 500)):
+        assert np.array_equal(csmv.zipf_table(n, th), oracle.zipf_cdf(n, th))
+
+
+def test_runs_continue_from_store():
+    """Two runs back to back continue the store and GTS."""
+    cfg = W.c2(n_items=1 << 12, n_tx=1 << 14, log_mode=csmv.LOG_NONE)
+    with csmv.Store(cfg.n_items, cfg.n_versions) as st:
+        st.load(cfg.init_values())
+        s1 = st.run(cfg.workload, cfg.n_tx, 1)
+        s2 = st.run(cfg.workload, cfg.n_tx, 2)
+        assert s2["gts_start"] == s1["gts_final"]
+        assert s2["gts_final"] == s1["gts_final"] + s2["committed_update"]
