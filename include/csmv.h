@@ -79,9 +79,12 @@ typedef struct csmv_workload {
     uint32_t client_warps;     /* active client warps; 0 = full grid */
     uint32_t server;           /* CSMV_SERVER_* */
     uint32_t cluster_size;     /* cluster server CTAs (2..16) */
+    uint32_t server_workers;   /* worker warps per server CTA (0 = default) */
     uint32_t atr_capacity;     /* ATR entries (0 = default); rounded to the layout */
     uint32_t atr_mode;         /* CSMV_ATR_* */
     uint32_t publish;          /* CSMV_PUBLISH_* */
+    uint32_t ro_streak;        /* 0: one transaction per lane per round (paper); R: a lane runs up to
+                                  R read-only transactions per round until it holds an update */
     uint32_t log_mode;         /* CSMV_LOG_* */
     uint32_t debug_flags;      /* CSMV_DBG_* */
     uint32_t watchdog_ms;      /* 0 = default (20000) */
@@ -109,6 +112,7 @@ typedef struct csmv_stats {
     uint64_t store_bytes_paper;/* same items in the paper's VBox layout */
     uint64_t server_lock_cycles; /* cycles the commit critical section was held */
     uint64_t server_busy_cycles; /* cycles workers spent processing batches */
+    uint64_t server_phase_cycles[8]; /* worker: queue wait, payload load, lock wait, critical section, respond */
     uint32_t client_warps;
     uint32_t server_ctas;
     uint32_t server_workers;

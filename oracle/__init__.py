@@ -39,7 +39,8 @@ class BankCfg(C.Structure):
     _fields_ = [("n_items", C.c_uint32), ("n_versions", C.c_uint32),
                 ("dist", C.c_uint32), ("zipf_theta_milli", C.c_uint32),
                 ("p_update_ppm", C.c_uint32), ("ro_period", C.c_uint32),
-                ("ro_reads", C.c_uint32), ("amount_max", C.c_uint32)]
+                ("ro_reads", C.c_uint32), ("amount_max", C.c_uint32),
+                ("ro_streak", C.c_uint32)]
 
 
 class Report(C.Structure):
@@ -133,9 +134,10 @@ def zipf_cdf(n: int, theta_milli: int) -> np.ndarray:
 
 
 def bank_cfg(n_items, n_versions=4, dist=DIST_UNIFORM, zipf_theta_milli=990,
-             p_update_ppm=500000, ro_period=0, ro_reads=64, amount_max=100) -> BankCfg:
+             p_update_ppm=500000, ro_period=0, ro_reads=64, amount_max=100,
+             ro_streak=0) -> BankCfg:
     return BankCfg(n_items, n_versions, dist, zipf_theta_milli, p_update_ppm,
-                   ro_period, ro_reads, amount_max)
+                   ro_period, ro_reads, amount_max, ro_streak)
 
 
 def bank_gen(cfg: BankCfg, seed: int, n_tx: int, tx0: int = 0) -> np.ndarray:

@@ -338,7 +338,9 @@ out:
  * Per round:
  *   1. s <- GTS (begin; one snapshot per warp round);
  *   2. each lane executes its transaction at s; read-only ones finish
- *      (P:69);
+ *      (P:69).  With ro_streak = R > 0 a lane keeps running its next
+ *      read-only transactions (at most R per round) until it holds an update;
+ *      with ro_streak = 0 it runs exactly one transaction per round;
  *   3. client-side pre-validation: update lanes in lane order, a
  *      lane is dropped if it conflicts with an earlier kept lane
  *      (SURVEY Q5); dropped lanes abort;
@@ -376,24 +378,33 @@ int or_bank_predict(const or_bank_cfg *c, const int32_t *init, uint64_t n_tx,
         uint32_t s = gts;                                   /* step 1 */
         int cand[32] = {0};
         for (uint32_t l = 0; l < L; l++) {                  /* step 2 */
-            if (cur[l] >= n_tx) continue;
-            uint64_t t = cur[l];
-            const or_bank_desc *T = &d[t];
-            att[l]++;
-            if (T->is_update) { cand[l] = 1; continue; }
-            int64_t sum = 0;
-            uint64_t dg = 0;
-            for (uint32_t j = 0; j < T->len; j++) {
-                uint32_t x = (T->start + j) % N;
-                if (vals && j < max_vals) vals[t * (uint64_t)max_vals + j] = (uint32_t)state[x];
-                sum += state[x];
-                dg += dig1(x, (uint32_t)state[x]);
+            uint32_t n_ro = 0;
+            while (cur[l] < n_tx) {
+                uint64_t t = cur[l];
+                const or_bank_desc *T = &d[t];
+                if (T->is_update) {
+                    if (!c->ro_streak && n_ro) break;  /* one tx per round */
+                    att[l]++;
+                    cand[l] = 1;
+                    break;
+                }
+                if (c->ro_streak ? n_ro >= c->ro_streak : n_ro >= 1) break;
+                att[l]++;
+                n_ro++;
+                int64_t sum = 0;
+                uint64_t dg = 0;
+                for (uint32_t j = 0; j < T->len; j++) {
+                    uint32_t x = (T->start + j) % N;
+                    if (vals && j < max_vals) vals[t * (uint64_t)max_vals + j] = (uint32_t)state[x];
+                    sum += state[x];
+                    dg += dig1(x, (uint32_t)state[x]);
+                }
+                log[t].tx = (uint32_t)t; log[t].snapshot = s; log[t].cts = 0;
+                log[t].attempts = att[l]; log[t].read_digest = dg; log[t].aux = (uint64_t)sum;
+                st->committed_ro++;
+                att[l] = 0;
+                cur[l] += L;
             }
-            log[t].tx = (uint32_t)t; log[t].snapshot = s; log[t].cts = 0;
-            log[t].attempts = att[l]; log[t].read_digest = dg; log[t].aux = (uint64_t)sum;
-            st->committed_ro++;
-            att[l] = 0;
-            cur[l] += L;
         }
         int kept[32] = {0};                                 /* step 3 */
         int nk = 0;

@@ -56,6 +56,9 @@ typedef struct {
     uint32_t ro_period;        /* >0: tx % p == p-1 is read-only (C1) */
     uint32_t ro_reads;         /* 0: total-sum ROT; L: L-item scan */
     uint32_t amount_max;       /* amount uniform in [1, amount_max] */
+    uint32_t ro_streak;        /* predictor: 0 = one tx per lane per round; R = a lane
+                                  runs up to R read-only txs per round until it
+                                  holds an update (csmv_workload.ro_streak) */
 } or_bank_cfg;
 
 typedef struct {

@@ -38,8 +38,8 @@ class CsmvError(RuntimeError):
 class _Workload(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in (
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
-        "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size",
-        "atr_capacity", "atr_mode", "publish", "log_mode", "debug_flags", "watchdog_ms")]
+        "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers",
+        "atr_capacity", "atr_mode", "publish", "ro_streak", "log_mode", "debug_flags", "watchdog_ms")]
 
 
 class _Stats(C.Structure):
@@ -49,6 +49,7 @@ class _Stats(C.Structure):
                 ("elapsed_ns", C.c_uint64), ("ro_checksum", C.c_uint64),
                 ("store_bytes", C.c_uint64), ("store_bytes_paper", C.c_uint64),
                 ("server_lock_cycles", C.c_uint64), ("server_busy_cycles", C.c_uint64),
+                ("server_phase_cycles", C.c_uint64 * 8),
                 ("client_warps", C.c_uint32), ("server_ctas", C.c_uint32),
                 ("server_workers", C.c_uint32), ("atr_entries", C.c_uint32),
                 ("sm_count", C.c_uint32), ("kernel_launches", C.c_uint32)]
@@ -69,9 +70,11 @@ class Workload:
     client_warps: int = 0
     server: int = SERVER_CTA
     cluster_size: int = 16
+    server_workers: int = 0
     atr_capacity: int = 0
     atr_mode: int = ATR_HASH
     publish: int = PUBLISH_CLIENT
+    ro_streak: int = 0
     log_mode: int = LOG_NONE
     debug_flags: int = 0
     watchdog_ms: int = 0
@@ -126,7 +129,9 @@ def _ptr(a: np.ndarray):
 
 
 def stats_dict(s: _Stats) -> dict:
-    d = {f: getattr(s, f) for f, _ in _Stats._fields_ if f != "aborts"}
+    d = {f: getattr(s, f) for f, _ in _Stats._fields_ if f not in ("aborts", "server_phase_cycles")}
+    d["server_phase_cycles"] = dict(zip(("queue", "load", "lock_wait", "critical", "respond", "cs_validate", "cs_insert0", "cs_insert1"),
+                                        list(s.server_phase_cycles)))
     d["aborts"] = {ABORT_REASONS[i]: {"ro": s.aborts[i][0], "update": s.aborts[i][1]}
                    for i in range(5)}
     d["total_aborts"] = sum(s.aborts[i][k] for i in range(5) for k in range(2))

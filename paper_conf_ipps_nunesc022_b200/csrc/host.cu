@@ -68,6 +68,7 @@ struct csmv {
   bool loaded = false;
 
   uint64_t* d_rings = nullptr;
+  uint32_t* d_lastw = nullptr;
   uint32_t* d_gts = nullptr;
   Ctl* d_ctl = nullptr;
   DevStats* d_stats = nullptr;
@@ -95,6 +96,7 @@ struct csmv {
 
 static void free_all(csmv* h) {
   cudaFree(h->d_rings);
+  cudaFree(h->d_lastw);
   cudaFree(h->d_gts);
   cudaFree(h->d_ctl);
   cudaFree(h->d_stats);
@@ -157,6 +159,7 @@ csmv_t* csmv_create(uint64_t n_items, uint32_t n_versions) {
     return nullptr;
   };
   if (cudaMalloc(&h->d_rings, n_items * h->nslot * sizeof(uint64_t)) != cudaSuccess) return fail("rings");
+  if (cudaMalloc(&h->d_lastw, n_items * sizeof(uint32_t)) != cudaSuccess) return fail("lastw");
   if (cudaMalloc(&h->d_gts, 64) != cudaSuccess) return fail("gts");
   if (cudaMalloc(&h->d_ctl, sizeof(Ctl)) != cudaSuccess) return fail("ctl");
   if (cudaMalloc(&h->d_stats, sizeof(DevStats)) != cudaSuccess) return fail("stats");
@@ -200,6 +203,7 @@ int csmv_load(csmv_t* h, const int32_t* init, uint64_t n) {
   CK(cudaMallocAsync((void**)&d_init, n * sizeof(int32_t), h->stream));
   CK(cudaMemcpyAsync(d_init, init, n * sizeof(int32_t), cudaMemcpyHostToDevice, h->stream));
   CK(launch_init_rings(h->d_rings, h->nslot, d_init, n, h->d_gts, h->stream));
+  CK(cudaMemsetAsync(h->d_lastw, 0, n * sizeof(uint32_t), h->stream));
   CK(cudaFreeAsync(d_init, h->stream));
   CK(cudaStreamSynchronize(h->stream));
   h->loaded = true;
@@ -270,14 +274,15 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (n_cw == 0) return set_err(CSMV_EINVAL, "csmv_run: no client warps");
   uint32_t n_ctas = (uint32_t)h->sm_count - 1;
   if (n_cw < n_ctas) n_ctas = n_cw;
-  const uint32_t n_workers = kWarps - 1;
-  if ((n_cw + n_workers - 1) / n_workers > 32u * kMaxPoll)
-    return set_err(CSMV_EINVAL, "csmv_run: too many client warps per server worker");
+  // server CTA: warp 0 receiver, warps 1..n_workers workers, last warp publisher
+  uint32_t n_workers = w->server_workers ? w->server_workers : 4u;
+  if (n_workers > kWarps - 2) n_workers = kWarps - 2;
 
+  // recent-commit table: 2 entries per bucket (default 16384 entries, 128 KB)
   uint32_t entries = w->atr_capacity ? w->atr_capacity : 16384u;
-  uint32_t sets_log2 = 1;
-  while (((uint32_t)kWays << sets_log2) < entries && sets_log2 < 14) ++sets_log2;
-  size_t smem = server_smem_bytes(sets_log2, n_cw);
+  uint32_t rt_log2 = 1;
+  while ((2u << rt_log2) < entries && rt_log2 < 13) ++rt_log2;
+  size_t smem = server_smem_bytes(rt_log2, n_cw);
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
   int bps = 0;
   CK(fused_occupancy(h->nslot, smem, &bps));
@@ -286,10 +291,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   // logs
   uint32_t max_vals = 0;
   if (w->log_mode != CSMV_LOG_NONE) {
-    if (n_tx > h->log_cap) {
+    if (n_tx > h->log_cap || !h->d_log) {
       cudaFree(h->d_log);
       h->d_log = nullptr;
-      CK(cudaMalloc(&h->d_log, n_tx * sizeof(csmv_log_rec)));
+      CK(cudaMalloc(&h->d_log, (n_tx ? n_tx : 1) * sizeof(csmv_log_rec)));
       h->log_cap = n_tx;
     }
     CK(cudaMemsetAsync(h->d_log, 0, n_tx * sizeof(csmv_log_rec), h->stream));
@@ -326,8 +331,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.n_cw = n_cw;
   p.n_client_ctas = n_ctas;
   p.n_workers = n_workers;
-  p.sets_log2 = sets_log2;
+  p.rt_log2 = rt_log2;
+  p.lastw = h->d_lastw;
   p.publish = w->publish;
+  p.ro_streak = w->ro_streak;
   p.debug = w->debug_flags;
   p.watchdog_ns = (uint64_t)(w->watchdog_ms ? w->watchdog_ms : 20000u) * 1000000ull;
 
@@ -365,10 +372,11 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   s.store_bytes_paper = h->n_items * (4ull + 8ull * h->K);
   s.server_lock_cycles = ds.lock_cycles;
   s.server_busy_cycles = ds.busy_cycles;
+  for (int i = 0; i < 8; ++i) s.server_phase_cycles[i] = ds.phase[i];
   s.client_warps = n_cw;
   s.server_ctas = 1;
   s.server_workers = n_workers;
-  s.atr_entries = kWays << sets_log2;
+  s.atr_entries = 2u << rt_log2;
   s.sm_count = (uint32_t)h->sm_count;
   s.kernel_launches = 1;
   h->last_n_tx = n_tx;

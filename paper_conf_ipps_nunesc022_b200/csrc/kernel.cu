@@ -97,6 +97,13 @@ __device__ __forceinline__ void write_back(uint64_t* ring, const Ring<NS>& r, ui
   st_relaxed64(ring + victim, ((uint64_t)cts << 32) | val);
 }
 
+// one relaxed load by lane 0, broadcast: keeps spin loops warp-uniform
+__device__ __forceinline__ uint32_t warp_ld_relaxed(const uint32_t* p) {
+  uint32_t v = 0;
+  if ((threadIdx.x & 31) == 0) v = ld_relaxed(p);
+  return __shfl_sync(0xFFFFFFFFu, v, 0);
+}
+
 __device__ __forceinline__ bool watchdog(const KParams& p, uint64_t t0, uint32_t where) {
   if (globaltimer() - t0 > p.watchdog_ns) {
     if (atomicCAS(&p.ctl->error, 0u, 1u) == 0u) p.ctl->where = where;
@@ -153,6 +160,33 @@ __device__ __forceinline__ bool rot_scan(const KParams& p, uint32_t start, uint3
 // --------------------------------------------------------------------------
 // Client warp
 // --------------------------------------------------------------------------
+struct ClientCounters {
+  uint32_t c_upd = 0, c_ro = 0, n_rounds = 0;
+  uint32_t ab[CSMV_N_ABORT][2];
+  uint64_t ro_ck = 0;
+  __device__ ClientCounters() {
+#pragma unroll
+    for (int i = 0; i < (int)CSMV_N_ABORT; ++i) ab[i][0] = ab[i][1] = 0;
+  }
+  __device__ __forceinline__ void abort(int reason, bool upd) {
+#pragma unroll
+    for (int i = 0; i < (int)CSMV_N_ABORT; ++i)
+      if (reason == i) ++ab[i][upd ? 1 : 0];
+  }
+};
+
+__device__ __forceinline__ void log_commit(const KParams& p, uint64_t tx, uint32_t s, uint32_t cts,
+                                           uint32_t att, uint64_t rdig, uint64_t aux) {
+  csmv_log_rec rec;
+  rec.tx = (uint32_t)tx;
+  rec.snapshot = s;
+  rec.cts = cts;
+  rec.attempts = att;
+  rec.read_digest = rdig;
+  rec.aux = aux;
+  p.log[tx] = rec;
+}
+
 template <int NS>
 __device__ void client_warp(const KParams& p, uint64_t t_begin) {
   const uint32_t FULL = 0xFFFFFFFFu;
@@ -162,21 +196,21 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
   const uint64_t T = (uint64_t)p.n_cw * 32;
   uint64_t cur = (uint64_t)cw * 32 + lane;  // static assignment: tx = lane + k*T
   uint32_t att = 0;
-  uint32_t c_upd = 0, c_ro = 0, n_batches = 0, n_rounds = 0;
-  uint32_t ab[CSMV_N_ABORT][2];
-#pragma unroll
-  for (int i = 0; i < (int)CSMV_N_ABORT; ++i) ab[i][0] = ab[i][1] = 0;
-  uint64_t ro_ck = 0;
+  ClientCounters cc;
   uint32_t round = 0;
   uint32_t* my_ids = p.req_ids + (size_t)cw * 2 * 32;
   const uint32_t K = p.K;
   const uint32_t lt = lanemask_lt();
+  // ro_streak = 0: each lane runs one transaction per round (the paper's
+  // one-transaction-per-thread model).  ro_streak = R > 0: a lane runs up to
+  // R read-only transactions at the round's snapshot until it holds an
+  // update, so batches carry more updates.
+  const uint32_t streak = p.ro_streak;
 
   for (;;) {
-    const bool has = cur < p.n_tx;
-    if (!__any_sync(FULL, has)) break;
+    if (!__any_sync(FULL, cur < p.n_tx)) break;
     ++round;
-    ++n_rounds;
+    ++cc.n_rounds;
     uint32_t s = 0, err = 0;
     if (lane == 0) {
       s = ld_acquire(p.gts);  // TXBegin: snapshot
@@ -186,34 +220,48 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
     if (__shfl_sync(FULL, err, 0)) break;
 
     int status = ST_NONE;
-    int reason = 0;
     BankTx d{};
     Ring<NS> rs{}, rd{};
     uint32_t vs = 0, vd = 0;
-    int64_t rsum = 0;
-    uint64_t rdig = 0;
-    if (has) {
-      ++att;
+    uint32_t n_ro = 0;
+    while (cur < p.n_tx) {
       d = gen_bank(p.gen, cur);
       if (!d.is_update) {
-        status = rot_scan<NS>(p, d.start, d.len, s, cur, rsum, rdig) ? ST_RO_OK : ST_ABORT;
-        reason = CSMV_AB_VERSION;
-      } else {
-        rs = ld_ring<NS>(p.rings + (size_t)d.src * NS);
-        rd = ld_ring<NS>(p.rings + (size_t)d.dst * NS);
-        Sel qs = select_version<NS>(rs, s), qd = select_version<NS>(rd, s);
-        if (qs.newest > s || qd.newest > s) {
-          status = ST_ABORT;  // a commit after s wrote it: validation must fail
-          reason = CSMV_AB_EARLY;
-        } else if (qs.best < 0 || qd.best < 0) {
+        // Read-only transaction: reads at s, no read-set, no commit.
+        if (streak ? n_ro >= streak : n_ro >= 1) break;
+        ++att;
+        ++n_ro;
+        int64_t rsum;
+        uint64_t rdig;
+        if (!rot_scan<NS>(p, d.start, d.len, s, cur, rsum, rdig)) {
+          cc.abort(CSMV_AB_VERSION, false);  // retried next round
           status = ST_ABORT;
-          reason = CSMV_AB_VERSION;
-        } else {
-          vs = (uint32_t)slot_at<NS>(rs, qs.best);
-          vd = (uint32_t)slot_at<NS>(rd, qd.best);
-          status = ST_CAND;
+          break;
         }
+        if (p.log_mode) log_commit(p, cur, s, 0, att, rdig, (uint64_t)rsum);
+        ++cc.c_ro;
+        cc.ro_ck ^= (uint64_t)rsum;
+        cur += T;
+        att = 0;
+        continue;
       }
+      if (!streak && n_ro) break;  // paper mode: one transaction per round
+      ++att;
+      rs = ld_ring<NS>(p.rings + (size_t)d.src * NS);
+      rd = ld_ring<NS>(p.rings + (size_t)d.dst * NS);
+      const Sel qs = select_version<NS>(rs, s), qd = select_version<NS>(rd, s);
+      if (qs.newest > s || qd.newest > s) {
+        cc.abort(CSMV_AB_EARLY, true);  // a commit after s wrote it: validation must fail
+        status = ST_ABORT;
+      } else if (qs.best < 0 || qd.best < 0) {
+        cc.abort(CSMV_AB_VERSION, true);
+        status = ST_ABORT;
+      } else {
+        vs = (uint32_t)slot_at<NS>(rs, qs.best);
+        vd = (uint32_t)slot_at<NS>(rd, qd.best);
+        status = ST_CAND;
+      }
+      break;
     }
 
     // Client-side pre-validation: greedy in lane order, a lane is
@@ -233,127 +281,99 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
       }
     }
     const bool mine = (kept >> lane) & 1u;
-    if (status == ST_CAND && !mine) {
-      status = ST_ABORT;
-      reason = CSMV_AB_PREVAL;
-    }
+    if (status == ST_CAND && !mine) cc.abort(CSMV_AB_PREVAL, true);
+    if (!kept) continue;
 
-    uint32_t cts = 0, ns = 0, nd = 0;
-    if (kept) {
-      // Batch submit: ids, header, then the doorbell.
-      if (mine) {
-        my_ids[lane] = d.src | kWriteBit;
-        my_ids[32 + lane] = d.dst | kWriteBit;
-      }
-      if (lane == 0) {
-        p.req_hdr[cw].snapshot = s;
-        p.req_hdr[cw].mask = kept;
-        ++n_batches;
-      }
-      __syncwarp();
-      fence_gpu();
-      uint32_t base = 0, cmask = 0, omask = 0;
-      if (lane == 0) {
-        st_relaxed(&p.req_seq[cw], round);
-        uint32_t it = 0;
-        bool ok = true;
-        while (ld_relaxed(&p.resp[cw].seq) != round) {
-          if ((++it & 255u) == 0 && (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1))) {
+    // Batch submit: ids, header, then the doorbell.
+    if (mine) {
+      my_ids[lane] = d.src | kWriteBit;
+      my_ids[32 + lane] = d.dst | kWriteBit;
+    }
+    if (lane == 0) {
+      p.req_hdr[cw].snapshot = s;
+      p.req_hdr[cw].mask = kept;
+    }
+    __syncwarp();
+    fence_gpu();
+    uint32_t base = 0, cmask = 0, omask = 0;
+    if (lane == 0) st_relaxed(&p.req_seq[cw], round);
+    {
+      // convergent wait on the response
+      uint32_t it = 0;
+      bool ok = true;
+      while (warp_ld_relaxed(&p.resp[cw].seq) != round) {
+        if ((++it & 255u) == 0) {
+          uint32_t bad = 0;
+          if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);
+          if (__shfl_sync(FULL, bad, 0)) {
             ok = false;
             break;
           }
-          __nanosleep(64);
         }
-        fence_gpu();  // acquire: response payload after its seq
-        if (ok) {
-          base = ld_relaxed(&p.resp[cw].cts_base);
-          cmask = ld_relaxed(&p.resp[cw].commit_mask);
-          omask = ld_relaxed(&p.resp[cw].overflow_mask);
-        }
+        __nanosleep(64);
       }
-      base = __shfl_sync(FULL, base, 0);
-      cmask = __shfl_sync(FULL, cmask, 0);
-      omask = __shfl_sync(FULL, omask, 0);
-      if (mine) {
-        if ((cmask >> lane) & 1u) {
-          // Client-side write-back with CTS = base + rank.
-          cts = base + __popc(cmask & lt);
-          ns = vs - (uint32_t)d.amt;
-          nd = vd + (uint32_t)d.amt;
-          write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
-          write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
-          status = ST_UPD_OK;
-        } else {
-          status = ST_ABORT;
-          reason = ((omask >> lane) & 1u) ? CSMV_AB_OVERFLOW : CSMV_AB_CONFLICT;
-        }
-      }
-      const uint32_t n = __popc(cmask);
-      if (n) {
-        if (p.publish == CSMV_PUBLISH_CLIENT) {
-          // Advance GTS by n once every earlier commit is visible:
-          // spin until GTS == first CTS - 1 ("GTS 1" = GTS+1).
-          __syncwarp();
-          fence_gpu();
-          if (lane == 0) {
-            uint32_t it = 0;
-            while (ld_relaxed(p.gts) != base - 1) {
-              if ((++it & 255u) == 0 &&
-                  (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 2))) break;
-              __nanosleep(32);
-            }
-            st_release(p.gts, base + n - 1);  // release also orders the write-backs
-          }
-        } else if (status == ST_UPD_OK) {
-          st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
-        }
+      fence_gpu();  // acquire: response payload after its seq
+      if (ok) {
+        base = ld_relaxed(&p.resp[cw].cts_base);
+        cmask = ld_relaxed(&p.resp[cw].commit_mask);
+        omask = ld_relaxed(&p.resp[cw].overflow_mask);
       }
     }
-
-    if (status == ST_RO_OK || status == ST_UPD_OK) {
-      if (p.log_mode) {
-        csmv_log_rec rec;
-        rec.tx = (uint32_t)cur;
-        rec.snapshot = s;
-        rec.cts = cts;
-        rec.attempts = att;
-        if (status == ST_RO_OK) {
-          rec.read_digest = rdig;
-          rec.aux = (uint64_t)rsum;
-        } else {
-          rec.read_digest = dig1(d.src, vs) + dig1(d.dst, vd);
-          rec.aux = dig1(d.src, ns) + dig1(d.dst, nd);
+    uint32_t cts = 0;
+    if (mine) {
+      if ((cmask >> lane) & 1u) {
+        // Client-side write-back with CTS = base + rank.
+        cts = base + __popc(cmask & lt);
+        const uint32_t ns = vs - (uint32_t)d.amt, nd = vd + (uint32_t)d.amt;
+        write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
+        write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
+        if (p.log_mode) {
+          log_commit(p, cur, s, cts, att, dig1(d.src, vs) + dig1(d.dst, vd),
+                     dig1(d.src, ns) + dig1(d.dst, nd));
           if (p.log_mode == CSMV_LOG_FULL && p.max_vals >= 2) {
             p.vals[cur * p.max_vals] = vs;
             p.vals[cur * p.max_vals + 1] = vd;
           }
         }
-        p.log[cur] = rec;
-      }
-      if (status == ST_RO_OK) {
-        ++c_ro;
-        ro_ck ^= (uint64_t)rsum;
+        ++cc.c_upd;
+        cur += T;
+        att = 0;
       } else {
-        ++c_upd;
+        cc.abort(((omask >> lane) & 1u) ? CSMV_AB_OVERFLOW : CSMV_AB_CONFLICT, true);
       }
-      cur += T;
-      att = 0;
-    } else if (status == ST_ABORT) {
-#pragma unroll
-      for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
-        if (reason == i) ++ab[i][d.is_update ? 1 : 0];
+    }
+    const uint32_t n = __popc(cmask);
+    if (n) {
+      if (p.publish == CSMV_PUBLISH_CLIENT) {
+        // Advance GTS by n once every earlier commit is visible:
+        // spin until GTS == first CTS - 1 ("GTS 1" = GTS+1).
+        __syncwarp();
+        fence_gpu();
+        uint32_t it = 0;
+        while (warp_ld_relaxed(p.gts) != base - 1) {
+          if ((++it & 255u) == 0) {
+            uint32_t bad = 0;
+            if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 2);
+            if (__shfl_sync(FULL, bad, 0)) break;
+          }
+          __nanosleep(32);
+        }
+        if (lane == 0) st_release(p.gts, base + n - 1);  // release also orders the write-backs
+      } else if (cts) {
+        st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
       }
     }
   }
 
   // flush per-warp counters once (no global atomics on the commit path)
-  const uint32_t s_upd = __reduce_add_sync(FULL, c_upd), s_ro = __reduce_add_sync(FULL, c_ro);
+  const uint32_t s_upd = __reduce_add_sync(FULL, cc.c_upd), s_ro = __reduce_add_sync(FULL, cc.c_ro);
   uint32_t s_ab[CSMV_N_ABORT][2];
 #pragma unroll
   for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
-    s_ab[i][0] = __reduce_add_sync(FULL, ab[i][0]);
-    s_ab[i][1] = __reduce_add_sync(FULL, ab[i][1]);
+    s_ab[i][0] = __reduce_add_sync(FULL, cc.ab[i][0]);
+    s_ab[i][1] = __reduce_add_sync(FULL, cc.ab[i][1]);
   }
+  uint64_t ro_ck = cc.ro_ck;
 #pragma unroll
   for (int o = 16; o; o >>= 1) ro_ck ^= __shfl_xor_sync(FULL, ro_ck, o);
   if (lane == 0) {
@@ -363,12 +383,11 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
       if (s_ab[i][0]) atomicAdd(&p.stats->aborts[i][0], (unsigned long long)s_ab[i][0]);
       if (s_ab[i][1]) atomicAdd(&p.stats->aborts[i][1], (unsigned long long)s_ab[i][1]);
     }
-    atomicAdd(&p.stats->rounds, (unsigned long long)n_rounds);
+    atomicAdd(&p.stats->rounds, (unsigned long long)cc.n_rounds);
     atomicXor(&p.stats->ro_checksum, (unsigned long long)ro_ck);
     __threadfence();
     atomicAdd(&p.ctl->done_warps, 1u);
   }
-  (void)n_batches;
 }
 
 // --------------------------------------------------------------------------
@@ -376,188 +395,279 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
 // --------------------------------------------------------------------------
 struct SrvShared {
   uint32_t tail;         // last CTS assigned (the CTS counter)
-  uint32_t wlow;         // every commit with CTS > wlow is in the ATR
   uint32_t next_ticket;  // ticket lock around validate+reserve+insert
   uint32_t now_serving;
   uint32_t gts_seen;     // publisher progress seen by workers (back-pressure)
+  uint32_t q_head;       // next dispatch-queue slot a worker claims
+  uint32_t exit;         // receiver: all clients finished
 };
 
-__device__ __forceinline__ uint32_t atr_set(uint32_t key, uint32_t sets_log2) {
-  return (key * 0x9E3779B1u) >> (32 - sets_log2);
+// ---------------------------------------------------------------------------
+// The ATR, item-indexed and split in two levels:
+//  * lastw[x] in HBM: CTS of the last commit that wrote x -- the exact
+//    record of every committed write-set, all history;
+//  * rt in shared memory: 2-way buckets of (cts << 32 | item) holding the
+//    latest writes, so that commits made after a worker prefetched lastw
+//    (CTS > e_pre) are seen with on-chip latency.
+// Validation of x for snapshot s (P:75 read-set, P:115 write-set):
+//    conflict  iff  lastw[x] (as of e_pre) > s  or  rt has (x, c) with c > s;
+//    unknown   iff  x is not in its bucket and both entries have CTS > e_pre
+//                   (an eviction may have hidden a write of x) -> OVERFLOW.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t rt_bucket(uint32_t key, uint32_t rt_log2) {
+  return (key * 0x9E3779B1u) >> (32 - rt_log2);
 }
 
-// conflict iff some ATR entry for `key` has CTS > s
-__device__ __forceinline__ bool atr_conflict(const uint64_t* htab, uint32_t sets_log2, uint32_t key,
-                                             uint32_t s) {
-  const ulonglong2* e = reinterpret_cast<const ulonglong2*>(htab + (size_t)atr_set(key, sets_log2) * kWays);
-  bool c = false;
-#pragma unroll
-  for (int j = 0; j < (int)kWays / 2; ++j) {
-    ulonglong2 v = e[j];
-    c |= ((uint32_t)v.x == key && (uint32_t)(v.x >> 32) > s);
-    c |= ((uint32_t)v.y == key && (uint32_t)(v.y >> 32) > s);
-  }
-  return c;
+struct RtProbe {
+  ulonglong2 b;  // the bucket
+  bool conflict;
+  bool unknown;
+};
+
+__device__ __forceinline__ RtProbe rt_probe(const uint64_t* rt, uint32_t bucket, uint32_t key, uint32_t s,
+                                            uint32_t e_pre, uint32_t lastw) {
+  RtProbe r;
+  r.b = reinterpret_cast<const ulonglong2*>(rt)[bucket];
+  const uint32_t k0 = (uint32_t)r.b.x, k1 = (uint32_t)r.b.y;
+  const uint32_t c0 = (uint32_t)(r.b.x >> 32), c1 = (uint32_t)(r.b.y >> 32);
+  const bool f0 = k0 == key, f1 = k1 == key;
+  r.conflict = lastw > s || (f0 && c0 > s) || (f1 && c1 > s);
+  r.unknown = !f0 && !f1 && min(c0, c1) > e_pre;
+  return r;
 }
 
-// Insert (key, cts) for every lane with `active`; lanes whose keys map to
-// the same set are serialised with __match_any_sync.  A full set evicts its
-// oldest entry and raises W_low to that entry's CTS.
-__device__ __forceinline__ void atr_insert(uint64_t* htab, uint32_t sets_log2, SrvShared* sh,
-                                           uint32_t key, uint32_t cts, bool active) {
-  const uint32_t lane = threadIdx.x & 31;
-  const uint32_t set = atr_set(key, sets_log2);
-  bool pending = active;
-  for (;;) {
-    const uint32_t act = __ballot_sync(0xFFFFFFFFu, pending);
-    if (!act) break;
-    if (pending) {
-      const uint32_t peers = __match_any_sync(act, set);
-      if (lane == (uint32_t)(__ffs(peers) - 1)) {
-        uint64_t* e = htab + (size_t)set * kWays;
-        int hit = -1, vic = 0;
-        uint32_t vmin = 0xFFFFFFFFu;
-#pragma unroll
-        for (int j = 0; j < (int)kWays; ++j) {
-          uint64_t v = e[j];
-          uint32_t c = (uint32_t)(v >> 32);
-          if ((uint32_t)v == key) hit = j;
-          if (c < vmin) {
-            vmin = c;
-            vic = j;
-          }
-        }
-        if (hit >= 0) {
-          vic = hit;
-        } else if (vmin > *(volatile uint32_t*)&sh->wlow) {
-          atomicMax(&sh->wlow, vmin);  // evicting a live entry (bounded ATR)
-        }
-        e[vic] = ((uint64_t)cts << 32) | key;
-        pending = false;
+// Record (key0, cts) and (key1, cts) for every lane with `active`: each
+// replaces the entry of the same key, else the older way of its bucket.
+// Lanes write in parallel and verify after a __syncwarp; two writers of the
+// same way leave one winner and the loser retries on the re-read bucket.
+// Entries are only ever evicted by newer batches (or by lanes of the same
+// batch, whose CTS lie between the same two tail values), which is what
+// makes the `unknown` rule of rt_probe sufficient.
+__device__ __forceinline__ int rt_way(ulonglong2 b, uint32_t key) {
+  if ((uint32_t)b.x == key) return 0;
+  if ((uint32_t)b.y == key) return 1;
+  return ((uint32_t)(b.y >> 32) < (uint32_t)(b.x >> 32)) ? 1 : 0;
+}
+
+__device__ __forceinline__ void rt_insert2(uint64_t* rt, uint32_t bk0, uint32_t key0, ulonglong2 b0,
+                                           uint32_t bk1, uint32_t key1, ulonglong2 b1, uint32_t cts,
+                                           bool active) {
+  const uint64_t m0 = ((uint64_t)cts << 32) | key0, m1 = ((uint64_t)cts << 32) | key1;
+  const ulonglong2* rb = reinterpret_cast<const ulonglong2*>(rt);
+  bool p0 = active, p1 = active;
+  bool first = true;
+  while (__any_sync(0xFFFFFFFFu, p0 || p1)) {
+    int w0 = 0, w1 = 0;
+    if (p0 || p1) {
+      if (!first) {
+        b0 = rb[bk0];
+        b1 = rb[bk1];
       }
+      if (p0) w0 = rt_way(b0, key0);
+      if (p1) {
+        w1 = rt_way(b1, key1);
+        if (p0 && bk1 == bk0 && w1 == w0) w1 ^= 1;  // both keys of one lane share a bucket
+      }
+      if (p0) rt[2 * (size_t)bk0 + w0] = m0;
+      if (p1) rt[2 * (size_t)bk1 + w1] = m1;
     }
+    __syncwarp();
+    if (p0 && rt[2 * (size_t)bk0 + w0] == m0) p0 = false;
+    if (p1 && rt[2 * (size_t)bk1 + w1] == m1) p1 = false;
+    first = false;
     __syncwarp();
   }
 }
 
-__device__ void server_worker(const KParams& p, uint64_t* htab, uint32_t* last_seen, SrvShared* sh,
-                              uint64_t t_begin) {
+// Receiver warp: sweeps every client doorbell with coalesced loads
+// and dispatches new requests to the workers through a shared-memory queue
+// (entry = lap << 32 | client warp; a worker that claimed slot i waits for
+// lap i / QN + 1).  At most one request per client warp is outstanding, so
+// QN >= n_cw slots never wrap onto an unconsumed entry.
+__device__ void server_receiver(const KParams& p, uint32_t* last_seen, uint64_t* queue, uint32_t qn_log2,
+                                SrvShared* sh, uint64_t t_begin) {
   const uint32_t FULL = 0xFFFFFFFFu;
-  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint32_t per = (p.n_cw + p.n_workers - 1) / p.n_workers;
-  const uint32_t base = warp * per;
-  const uint32_t end = min(base + per, p.n_cw);
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t rows = (p.n_cw + 31) / 32;
   const uint32_t lt = lanemask_lt();
-  const uint32_t dmask = (1u << kDoneLog2) - 1;
-  unsigned long long busy = 0, locked = 0, batches = 0;
-  uint32_t spins = 0;
+  const uint32_t qmask = (1u << qn_log2) - 1;
+  uint32_t tail = 0;  // next queue slot to fill
+  uint32_t idle = 0;
   for (;;) {
-    // Receive: one coalesced sweep over this warp's doorbells.
-    uint32_t seq[kMaxPoll];
-    uint32_t pend[kMaxPoll];
+    bool found = false;
+    for (uint32_t r0 = 0; r0 < rows; r0 += 8) {
+      uint32_t seq[8];
 #pragma unroll
-    for (int k = 0; k < kMaxPoll; ++k) {
-      const uint32_t w = base + k * 32 + lane;
-      seq[k] = (w < end) ? ld_relaxed(p.req_seq + w) : 0u;
-    }
-    bool any = false;
-#pragma unroll
-    for (int k = 0; k < kMaxPoll; ++k) {
-      const uint32_t w = base + k * 32 + lane;
-      pend[k] = __ballot_sync(FULL, w < end && seq[k] != last_seen[w]);
-      any |= pend[k] != 0;
-    }
-    if (!any) {
-      if ((++spins & 63u) == 0) {
-        uint32_t dw = 0, er = 0;
-        if (lane == 0) {
-          dw = ld_relaxed(&p.ctl->done_warps);
-          er = ld_relaxed(&p.ctl->error);
-          if (!er && dw < p.n_cw && watchdog(p, t_begin, 3)) er = 1;
-        }
-        dw = __shfl_sync(FULL, dw, 0);
-        er = __shfl_sync(FULL, er, 0);
-        if (dw >= p.n_cw || er) break;
+      for (int k = 0; k < 8; ++k) {
+        const uint32_t w = (r0 + k) * 32 + lane;
+        seq[k] = (r0 + k < rows && w < p.n_cw) ? ld_relaxed(p.req_seq + w) : 0u;
       }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const uint32_t w = (r0 + k) * 32 + lane;
+        const bool pend = r0 + k < rows && w < p.n_cw && seq[k] != last_seen[w];
+        const uint32_t pm = __ballot_sync(FULL, pend);
+        if (pm) {
+          found = true;
+          if (pend) {
+            const uint32_t pos = tail + __popc(pm & lt);
+            last_seen[w] = seq[k];
+            *(volatile uint64_t*)&queue[pos & qmask] = ((uint64_t)((pos >> qn_log2) + 1) << 32) | w;
+          }
+          tail += __popc(pm);
+        }
+      }
+    }
+    if (found) {
+      idle = 0;
       continue;
     }
-    fence_gpu();  // acquire: doorbells seen before payload loads
-#pragma unroll
-    for (int k = 0; k < kMaxPoll; ++k) {
-      uint32_t pm = pend[k];
-      while (pm) {
-        const int i = __ffs(pm) - 1;
-        pm &= pm - 1;
-        const uint32_t cw = base + k * 32 + i;
-        const uint32_t sq = __shfl_sync(FULL, seq[k], i);
-        const long long t0 = clock64();
-        // Load the batch: header broadcast + one id row per RS u WS entry.
-        const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
-        const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
-        const bool mine = (mask >> lane) & 1u;
-        uint32_t id0 = 0, id1 = 0;
-        if (mine) {
-          id0 = ld_relaxed(p.req_ids + (size_t)cw * 64 + lane) & ~kWriteBit;
-          id1 = ld_relaxed(p.req_ids + (size_t)cw * 64 + 32 + lane) & ~kWriteBit;
-        }
-        // ---- critical section: validate, reserve CTS, insert
-        uint32_t ticket = 0;
-        if (lane == 0) {
-          ticket = atomicAdd(&sh->next_ticket, 1u);
-          while (*(volatile uint32_t*)&sh->now_serving != ticket) __nanosleep(20);
-        }
-        __syncwarp();
-        __threadfence_block();
-        const long long t1 = clock64();
-        const uint32_t t0c = *(volatile uint32_t*)&sh->tail;
-        const uint32_t wl = *(volatile uint32_t*)&sh->wlow;
-        const bool ovf = mine && s < wl;
-        bool conflict = false;
-        if (mine && !ovf && !(p.debug & CSMV_DBG_NO_VALIDATE))
-          conflict = atr_conflict(htab, p.sets_log2, id0, s) || atr_conflict(htab, p.sets_log2, id1, s);
-        const bool commit = mine && !ovf && !conflict;
-        const uint32_t cm = __ballot_sync(FULL, commit);
-        const uint32_t n = __popc(cm);
-        const uint32_t cts = t0c + 1 + __popc(cm & lt);
-        if (p.publish == CSMV_PUBLISH_SERVER && n) {
-          // done ring back-pressure: CTS c may reuse slot c & dmask only once
-          // GTS >= c - 2^20
-          if (lane == 0) {
-            uint32_t it = 0;
-            while (t0c + n > sh->gts_seen + dmask) {
-              sh->gts_seen = ld_relaxed(p.gts);
-              if ((++it & 255u) == 0 && watchdog(p, t_begin, 4)) break;
-            }
-          }
-          __syncwarp();
-        }
-        atr_insert(htab, p.sets_log2, sh, id0, cts, commit);
-        atr_insert(htab, p.sets_log2, sh, id1, cts, commit);
-        __syncwarp();
-        __threadfence_block();
-        if (lane == 0) {
-          sh->tail = t0c + n;
-          __threadfence_block();
-          *(volatile uint32_t*)&sh->now_serving = ticket + 1;
-        }
-        const long long t2 = clock64();
-        // ---- respond
-        const uint32_t om = __ballot_sync(FULL, ovf);
-        if (lane == 0) {
-          st_relaxed(&p.resp[cw].cts_base, t0c + 1);
-          st_relaxed(&p.resp[cw].commit_mask, cm);
-          st_relaxed(&p.resp[cw].overflow_mask, om);
-          st_release(&p.resp[cw].seq, sq);
-          last_seen[cw] = sq;
-        }
-        __syncwarp();
-        busy += (unsigned long long)(t2 - t0);
-        locked += (unsigned long long)(t2 - t1);
-        ++batches;
+    if ((++idle & 15u) == 0) {
+      uint32_t dw = 0, er = 0;
+      if (lane == 0) {
+        dw = ld_relaxed(&p.ctl->done_warps);
+        er = ld_relaxed(&p.ctl->error);
+        if (!er && dw < p.n_cw && watchdog(p, t_begin, 3)) er = 1;
+      }
+      dw = __shfl_sync(FULL, dw, 0);
+      er = __shfl_sync(FULL, er, 0);
+      if (dw >= p.n_cw || er) {
+        if (lane == 0) *(volatile uint32_t*)&sh->exit = 1;
+        return;
       }
     }
   }
+}
+
+__device__ void server_worker(const KParams& p, uint64_t* rt, uint64_t* queue, uint32_t qn_log2,
+                              SrvShared* sh, uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t lt = lanemask_lt();
+  const uint32_t qmask = (1u << qn_log2) - 1;
+  const uint32_t dmask = (1u << kDoneLog2) - 1;
+  unsigned long long busy = 0, locked = 0, batches = 0;
+  unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  for (;;) {
+    const long long tq = clock64();
+    // Claim the next dispatched request.
+    uint32_t slot = 0;
+    if (lane == 0) slot = atomicAdd(&sh->q_head, 1u);
+    slot = __shfl_sync(FULL, slot, 0);
+    const uint32_t lap = (slot >> qn_log2) + 1;
+    // Convergent wait (every lane polls the same word: one broadcast LDS).
+    uint64_t ent;
+    bool quit = false;
+    for (;;) {
+      ent = *(volatile uint64_t*)&queue[slot & qmask];
+      if ((uint32_t)(ent >> 32) == lap) break;
+      if (*(volatile uint32_t*)&sh->exit) {
+        quit = true;
+        break;
+      }
+      __nanosleep(64);
+    }
+    if (quit) break;
+    const uint32_t cw = (uint32_t)ent;
+    const long long t0 = clock64();
+    // Load the batch: doorbell (acquire pattern), header, one id row per
+    // RS u WS entry (coalesced 128 B), then prefetch lastw of every item.
+    const uint32_t sq = ld_relaxed(p.req_seq + cw);
+    fence_gpu();
+    const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
+    const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
+    const bool mine = (mask >> lane) & 1u;
+    uint32_t id0 = 0, id1 = 0;
+    if (mine) {
+      id0 = ld_relaxed(p.req_ids + (size_t)cw * 64 + lane) & ~kWriteBit;
+      id1 = ld_relaxed(p.req_ids + (size_t)cw * 64 + 32 + lane) & ~kWriteBit;
+    }
+    const uint32_t e_pre = *(volatile uint32_t*)&sh->tail;  // lastw covers every CTS <= e_pre
+    fence_cta();
+    uint32_t lw0 = 0, lw1 = 0;
+    if (mine) {
+      lw0 = ld_relaxed(p.lastw + id0);
+      lw1 = ld_relaxed(p.lastw + id1);
+    }
+    const uint32_t b0 = rt_bucket(id0, p.rt_log2), b1 = rt_bucket(id1, p.rt_log2);
+    // The payload must have arrived before the lock is taken: a warp vote on
+    // values derived from it makes the loads complete here, not inside the
+    // critical section.
+    if (__ballot_sync(FULL, (b0 ^ b1 ^ lw0 ^ lw1 ^ s) == 0xFFFFFFFFu) == 0xFFFFFFFFu) __nanosleep(1);
+    const long long tl = clock64();
+    // ---- critical section: validate, reserve CTS, record
+    uint32_t ticket = 0;
+    if (lane == 0) ticket = atomicAdd(&sh->next_ticket, 1u);
+    ticket = __shfl_sync(FULL, ticket, 0);
+    while (*(volatile uint32_t*)&sh->now_serving != ticket) __nanosleep(16);
+    __syncwarp();
+    fence_cta();
+    const long long t1 = clock64();
+    const uint32_t t0c = *(volatile uint32_t*)&sh->tail;
+    RtProbe q0{}, q1{};
+    if (mine) {
+      q0 = rt_probe(rt, b0, id0, s, e_pre, lw0);
+      q1 = rt_probe(rt, b1, id1, s, e_pre, lw1);
+    }
+    bool ovf = mine && (q0.unknown || q1.unknown);
+    bool conflict = mine && (q0.conflict || q1.conflict);
+    if (p.debug & CSMV_DBG_NO_VALIDATE) ovf = conflict = false;
+    const bool commit = mine && !ovf && !conflict;
+    const uint32_t cm = __ballot_sync(FULL, commit);
+    const uint32_t n = __popc(cm);
+    const uint32_t cts = t0c + 1 + __popc(cm & lt);
+    const long long ta = clock64();
+    if (p.publish == CSMV_PUBLISH_SERVER && n) {
+      // done-ring back-pressure: CTS c may reuse slot c & dmask only once
+      // GTS >= c - 2^20
+      if (lane == 0) {
+        uint32_t it = 0;
+        while (t0c + n > sh->gts_seen + dmask) {
+          sh->gts_seen = ld_relaxed(p.gts);
+          if ((++it & 255u) == 0 && watchdog(p, t_begin, 4)) break;
+        }
+      }
+      __syncwarp();
+    }
+    if (commit) {
+      st_relaxed(p.lastw + id0, cts);
+      st_relaxed(p.lastw + id1, cts);
+    }
+    const long long tb = clock64();
+    rt_insert2(rt, b0, id0, q0.b, b1, id1, q1.b, cts, commit);
+    const long long tc = clock64();
+    __syncwarp();
+    fence_cta();
+    if (lane == 0) {
+      sh->tail = t0c + n;
+      fence_cta();
+      *(volatile uint32_t*)&sh->now_serving = ticket + 1;
+    }
+    const long long t2 = clock64();
+    // ---- respond
+    const uint32_t om = __ballot_sync(FULL, ovf);
+    if (lane == 0) {
+      st_relaxed(&p.resp[cw].cts_base, t0c + 1);
+      st_relaxed(&p.resp[cw].commit_mask, cm);
+      st_relaxed(&p.resp[cw].overflow_mask, om);
+      st_release(&p.resp[cw].seq, sq);
+    }
+    __syncwarp();
+    const long long t3 = clock64();
+    busy += (unsigned long long)(t3 - t0);
+    locked += (unsigned long long)(t2 - t1);
+    ph[0] += (unsigned long long)(t0 - tq);
+    ph[1] += (unsigned long long)(tl - t0);
+    ph[2] += (unsigned long long)(t1 - tl);
+    ph[3] += (unsigned long long)(t2 - t1);
+    ph[4] += (unsigned long long)(t3 - t2);
+    ph[5] += (unsigned long long)(ta - t1);
+    ph[6] += (unsigned long long)(tb - ta);
+    ph[7] += (unsigned long long)(tc - tb);
+    ++batches;
+  }
   if (lane == 0) {
+    for (int i = 0; i < 8; ++i) atomicAdd(&p.stats->phase[i], ph[i]);
     atomicAdd(&p.stats->batches, batches);
     atomicAdd(&p.stats->busy_cycles, busy);
     atomicAdd(&p.stats->lock_cycles, locked);
@@ -605,26 +715,32 @@ __device__ void server_publisher(const KParams& p, SrvShared* sh, uint64_t t_beg
 }
 
 __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
-  uint64_t* htab = reinterpret_cast<uint64_t*>(smem);
-  const uint32_t n_entries = kWays << p.sets_log2;
-  uint32_t* last_seen = reinterpret_cast<uint32_t*>(htab + n_entries);
+  uint64_t* rt = reinterpret_cast<uint64_t*>(smem);
+  const uint32_t rt_words = 2u << p.rt_log2;
+  const uint32_t qn_log2 = queue_log2(p.n_cw);
+  uint64_t* queue = rt + rt_words;
+  uint32_t* last_seen = reinterpret_cast<uint32_t*>(queue + (1u << qn_log2));
   const uint32_t ls_words = (p.n_cw + 31) / 32 * 32;
   SrvShared* sh = reinterpret_cast<SrvShared*>(last_seen + ls_words);
-  for (uint32_t i = threadIdx.x; i < n_entries; i += blockDim.x) htab[i] = 0xFFFFFFFFull;  // cts 0, no key
+  for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) rt[i] = 0xFFFFFFFFull;  // cts 0, no item
+  for (uint32_t i = threadIdx.x; i < (1u << qn_log2); i += blockDim.x) queue[i] = 0;
   for (uint32_t i = threadIdx.x; i < ls_words; i += blockDim.x) last_seen[i] = 0;
   if (threadIdx.x == 0) {
     const uint32_t g0 = *p.gts;
     sh->tail = g0;
-    sh->wlow = g0;
     sh->next_ticket = 0;
     sh->now_serving = 0;
     sh->gts_seen = g0;
+    sh->q_head = 0;
+    sh->exit = 0;
   }
   __syncthreads();
   const uint32_t warp = threadIdx.x >> 5;
-  if (warp < p.n_workers) {
-    server_worker(p, htab, last_seen, sh, t_begin);
-  } else if (warp == p.n_workers && p.publish == CSMV_PUBLISH_SERVER) {
+  if (warp == 0) {
+    server_receiver(p, last_seen, queue, qn_log2, sh, t_begin);
+  } else if (warp <= p.n_workers) {
+    server_worker(p, rt, queue, qn_log2, sh, t_begin);
+  } else if (warp == p.n_workers + 1 && p.publish == CSMV_PUBLISH_SERVER) {
     server_publisher(p, sh, t_begin);
   }
   __syncthreads();

@@ -12,6 +12,8 @@
 //   resp      {cts_base, commit_mask, overflow_mask, seq}[n_cw]
 //   done_ring u32[2^20]             CSMV_PUBLISH_SERVER: done[cts & mask] = cts
 //                                   after the write-back of cts
+//   lastw     u32[n_items]          CTS of the last commit that wrote the item
+//                                   (server-private level of the ATR)
 //   log       csmv_log_rec[n_tx]    parity runs only
 #pragma once
 #include <cstdint>
@@ -25,9 +27,7 @@ constexpr uint32_t kEmptyTs = 0xFFFFFFFFu;
 constexpr uint32_t kWriteBit = 0x80000000u;
 constexpr int kBlock = 512;            // threads per CTA (16 warps)
 constexpr int kWarps = kBlock / 32;
-constexpr int kMaxPoll = 8;            // doorbell words per worker lane (<= 256 warps/worker)
 constexpr uint32_t kDoneLog2 = 20;     // done ring entries (CSMV_PUBLISH_SERVER)
-constexpr uint32_t kWays = 8;          // ATR hash associativity (64 B per set)
 
 struct Ctl {
   uint32_t error;       // 0 ok, 1 watchdog, 2 protocol
@@ -54,6 +54,7 @@ struct DevStats {
   unsigned long long batches, rounds;
   unsigned long long ro_checksum;
   unsigned long long lock_cycles, busy_cycles;
+  unsigned long long phase[8];  // server worker: queue wait, load, lock wait, critical, respond
 };
 
 struct KParams {
@@ -77,15 +78,26 @@ struct KParams {
   uint32_t n_cw;           // active client warps
   uint32_t n_client_ctas;  // CTAs 1..n_client_ctas host clients
   uint32_t n_workers;      // server worker warps
-  uint32_t sets_log2;      // ATR hash sets
+  uint32_t rt_log2;        // recent-commit table buckets (2 ways, 16 B each)
+  uint32_t* lastw;         // per-item CTS of the last committed write
   uint32_t publish;
+  uint32_t ro_streak;      // read-only transactions a lane may run per round (0 = one tx per round)
   uint32_t debug;
   uint64_t watchdog_ns;
 };
 
-// smem the server CTA needs (every CTA of the fused grid gets the same)
-inline size_t server_smem_bytes(uint32_t sets_log2, uint32_t n_cw) {
-  return ((size_t)kWays * 8u << sets_log2) + (((size_t)n_cw + 31) / 32 * 32) * 4 + 64;
+// dispatch queue slots: a power of two >= n_cw
+__host__ __device__ inline uint32_t queue_log2(uint32_t n_cw) {
+  uint32_t l = 5;
+  while ((1u << l) < n_cw) ++l;
+  return l;
+}
+
+// smem the server CTA needs (every CTA of the fused grid gets the same):
+// recent-commit table, dispatch queue, receiver's last-seen doorbells, control words
+inline size_t server_smem_bytes(uint32_t rt_log2, uint32_t n_cw) {
+  return ((size_t)16 << rt_log2) + ((size_t)8 << queue_log2(n_cw)) +
+         (((size_t)n_cw + 31) / 32 * 32) * 4 + 64;
 }
 
 // host-callable launchers (kernel.cu)

@@ -18,7 +18,8 @@ def oracle_cfg(cfg):
     w = cfg.workload
     return oracle.bank_cfg(cfg.n_items, cfg.n_versions, dist=w.dist,
                            zipf_theta_milli=w.zipf_theta_milli, p_update_ppm=w.p_update_ppm,
-                           ro_period=w.ro_period, ro_reads=w.ro_reads, amount_max=w.amount_max)
+                           ro_period=w.ro_period, ro_reads=w.ro_reads, amount_max=w.amount_max,
+                           ro_streak=w.ro_streak)
 
 
 def run_gpu(cfg, init=None):
@@ -73,11 +74,13 @@ def test_c1_full_parity(publish):
     assert sum(stats["aborts"][r]["ro"] for r in ("preval", "conflict", "early", "overflow")) == 0
 
 
-@pytest.mark.parametrize("k", [1, 2, 4, 8, 16])
-def test_one_warp_is_deterministic(k):
+@pytest.mark.parametrize("k,streak,ro_reads", [(1, 0, 0), (2, 0, 0), (4, 0, 0), (8, 0, 0), (16, 0, 0),
+                                               (4, 4, 0), (4, 8, 16), (2, 1, 16)])
+def test_one_warp_is_deterministic(k, streak, ro_reads):
     """with one client warp the oracle predicts every snapshot,
     CTS, attempt count and ring exactly."""
-    cfg = W.c1(client_warps=1, n_versions=k, n_tx=3000, log_mode=csmv.LOG_FULL)
+    cfg = W.c1(client_warps=1, n_versions=k, n_tx=3000, log_mode=csmv.LOG_FULL,
+               ro_streak=streak, ro_reads=ro_reads)
     stats, log, (vals, mv), rings = run_gpu(cfg)
     ocfg = oracle_cfg(cfg)
     descs = oracle.bank_gen(ocfg, cfg.seed, cfg.n_tx)
@@ -91,16 +94,19 @@ def test_one_warp_is_deterministic(k):
     assert stats["batches"] == pst["batches"] and stats["rounds"] == pst["rounds"]
 
 
-@pytest.mark.parametrize("publish", [csmv.PUBLISH_CLIENT, csmv.PUBLISH_SERVER])
-def test_c2_shrunk_parity(publish):
-    cfg = W.c2(n_items=1 << 16, n_tx=1 << 18, publish=publish)
+@pytest.mark.parametrize("publish,streak,workers", [(csmv.PUBLISH_CLIENT, 0, 4), (csmv.PUBLISH_SERVER, 0, 8),
+                                                   (csmv.PUBLISH_SERVER, 8, 8), (csmv.PUBLISH_CLIENT, 8, 2)])
+def test_c2_shrunk_parity(publish, streak, workers):
+    cfg = W.c2(n_items=1 << 16, n_tx=1 << 18, publish=publish, ro_streak=streak,
+               server_workers=workers)
     rep, stats, log, rings, descs = check(cfg)
     assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions),
                           closed_form(cfg, descs, cfg.init_values()))
 
 
-def test_c3_shrunk_parity():
-    cfg = W.c3(n_tx=1 << 18)
+@pytest.mark.parametrize("streak", [0, 8])
+def test_c3_shrunk_parity(streak):
+    cfg = W.c3(n_tx=1 << 18, ro_streak=streak, client_warps=256)
     rep, stats, log, rings, descs = check(cfg)
     assert stats["aborts"]["conflict"]["ro"] == 0 and stats["aborts"]["early"]["ro"] == 0  # P6/Q7
 

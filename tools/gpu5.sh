@@ -1,0 +1,2 @@
+python -c "import __graft_entry__ as g; g.build()"
+for cw in 16 64; do timeout 120 python tools/probe.py C2 n_tx=2097152 client_warps=$cw publish=1 reps=1; done
