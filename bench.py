@@ -1,0 +1,338 @@
+#!/usr/bin/env python
+"""Benchmark: committed transactions/s and abort rate of the CSMV batched
+commit pipeline (BASELINE.json metric) on the config it is quoted on,
+configs[1] = C2: bank, 1M accounts, K=4 versions, full-GPU client grid, 50%
+update, uniform access, read-only = 64-read scans.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+A step is one csmv_run over n_tx = 2^24 freshly generated transactions
+(every one commits exactly once; aborted attempts are retried inside the
+step).  The store and GTS persist across steps.  L2 is flushed (a 512 MiB
+write) before every timed step.  N > 1 runs one process per GPU under
+torchrun as independent key-range-partitioned instances (no cross-GPU
+transactions; NCCL only reduces statistics), scaling "weak"-ish: the job's
+n_tx and accounts are split across ranks.
+
+--impl reference times the CPU oracle (the deterministic 1-warp schedule of
+oracle/, single-threaded C) on bounded samples of the same workload: the
+tier's reference arm is the oracle, there is no GPU reference to install.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "committed tx/sec and abort rate at 1 B200 (+partitioned 2/4/8)"
+UNIT = "tx/s"
+
+# tuned launch configuration of the C2 workload
+TUNED = dict(client_warps_per_sm=2, server_workers=8, ro_streak=8, publish=1)
+
+# algorithmic bytes (paper VBox layout P:289): a read moves the
+# VBox head, the visited version's ts and the value (4+4+4); a write-back the
+# same; a request 4 B per RS and per WS id, a response 4 B per tx and a batch
+# header 16 B per 32 transactions.
+BYTES_READ = 12.0
+BYTES_WRITE = 12.0
+BYTES_TRANSFER = 2 * BYTES_READ + 2 * BYTES_WRITE + 4 * 4 + 4 + 16 / 32   # 68.5
+
+
+def algorithmic_bytes(stats: dict, ro_reads: int, n_items: int) -> float:
+    L = ro_reads if ro_reads else n_items
+    return stats["committed_update"] * BYTES_TRANSFER + stats["committed_ro"] * BYTES_READ * L
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def traffic_per_launch():
+    """dram bytes per launch of csmv_fused from the committed ncu capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        d = json.load(f)
+    return d.get("c2_bench", {}).get("dram_bytes_per_launch")
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.proc = None
+        self.path = None
+
+    def __enter__(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except (FileNotFoundError, OSError):
+            self.proc = None
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.path or not os.path.exists(self.path):
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm, smax, reasons = [], None, set()
+        names = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")
+        for line in open(self.path):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax = float(f[2])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        os.unlink(self.path)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": smax,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def oracle_sample_rate(cfg, budget_s: float, chunk: int, tx_start: int = 0):
+    """CPU oracle (1-warp deterministic schedule, single thread) on bounded
+    chunks of the workload; returns (tx/s, txs, seconds)."""
+    import numpy as np
+
+    import oracle
+
+    w = cfg.workload
+    ocfg = oracle.bank_cfg(cfg.n_items, cfg.n_versions, dist=w.dist, zipf_theta_milli=w.zipf_theta_milli,
+                           p_update_ppm=w.p_update_ppm, ro_period=w.ro_period, ro_reads=w.ro_reads,
+                           amount_max=w.amount_max, ro_streak=w.ro_streak)
+    init = np.full(cfg.n_items, 1000, dtype=np.int32)
+    done, spent, tx0 = 0, 0.0, tx_start
+    while True:
+        descs = oracle.bank_gen(ocfg, cfg.seed, chunk, tx0=tx0)
+        t = time.perf_counter()
+        oracle.bank_predict(ocfg, init, descs, 32)
+        spent += time.perf_counter() - t
+        done += chunk
+        tx0 += chunk
+        if spent >= budget_s:
+            break
+    return done / spent, done, spent
+
+
+def make_cfg(args, world: int, rank: int):
+    from paper_conf_ipps_nunesc022_b200 import partition, workloads
+    cfg = workloads.c2()
+    n_tx = args.n_tx or cfg.n_tx
+    cfg = cfg.with_(n_tx=n_tx, log_mode=0, ro_streak=TUNED["ro_streak"], publish=TUNED["publish"],
+                    server_workers=TUNED["server_workers"])
+    part = partition.partition(cfg.n_items, n_tx, cfg.seed, rank, world)
+    return cfg, partition.local_config(cfg, part), part
+
+
+def bench_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    cfg, _, _ = make_cfg(args, 1, 0)
+    chunk = 1 << 18
+    for i in range(args.warmup):
+        oracle_sample_rate(cfg, 0.0, chunk, tx_start=i * chunk)
+    rates, total_tx, total_s = [], 0, 0.0
+    for i in range(args.steps):
+        r, n, s = oracle_sample_rate(cfg, 0.0, chunk, tx_start=(args.warmup + i) * chunk)
+        rates.append(r)
+        total_tx += n
+        total_s += s
+    value = total_tx / total_s
+    sample = f"{args.steps} chunks of {chunk} consecutive C2 transactions (1M accounts, 50% update)"
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total_s / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+            "data": "synthetic", "config": {"workload": "C2", "n_items": cfg.n_items,
+                                            "n_versions": cfg.n_versions, "sample": sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def bench_ours(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_nunesc022_b200 import csmv, partition
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    cfg, lcfg, part = make_cfg(args, world, rank)
+    props = torch.cuda.get_device_properties(dev)
+    n_cw = args.client_warps or TUNED["client_warps_per_sm"] * (props.multi_processor_count - 1)
+    lcfg = lcfg.with_(client_warps=n_cw)
+    w = lcfg.workload
+
+    stream = torch.cuda.current_stream()
+    store = csmv.Store(lcfg.n_items, lcfg.n_versions)
+    store.set_stream(stream.cuda_stream)
+    init = np.full(lcfg.n_items, 1000, dtype=np.int32)
+    store.load(init)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    for i in range(args.warmup):
+        store.run(w, lcfg.n_tx, lcfg.seed + 1000 + i)
+
+    barrier()
+    torch.cuda.synchronize()
+    steps = []
+    with Clocks(dev.index) as clk:
+        for i in range(args.steps):
+            flush.zero_()                                   # L2 flush, outside the events
+            ev0 = torch.cuda.Event(enable_timing=True)
+            ev1 = torch.cuda.Event(enable_timing=True)
+            ev0.record(stream)
+            st = store.run(w, lcfg.n_tx, lcfg.seed + i)
+            ev1.record(stream)
+            steps.append((ev0, ev1, st))
+        torch.cuda.synchronize()
+    barrier()
+    step_ms = [a.elapsed_time(b) for a, b, _ in steps]
+    kern_ns = [s["elapsed_ns"] for _, _, s in steps]
+    agg = {k: sum(s[k] for _, _, s in steps) for k in ("committed", "committed_update", "committed_ro",
+                                                        "total_aborts", "batches", "rounds")}
+    agg["elapsed_ns"] = int(sum(step_ms) * 1e6)
+    red = partition.reduce_stats(agg, device=dev if world > 1 else None)
+    total_ms_max = red["elapsed_ns"] / 1e6
+    value = red["committed"] / (total_ms_max * 1e-3)
+
+    # roofline of the dominant (only) kernel, csmv_fused
+    algo = sum(algorithmic_bytes(s, w.ro_reads, lcfg.n_items) for _, _, s in steps) / len(steps)
+    kmean = sum(kern_ns) / len(kern_ns)
+    achieved = algo / (kmean * 1e-9) / 1e9
+    peak, peak_kind = peaks()
+    traffic = traffic_per_launch()
+    last = steps[-1][2]
+    # serial commit chain: batches/s against the critical section's own bound
+    cs_cycles = last["server_phase_cycles"]["critical"] / max(1, last["batches"])
+
+    # end to end through the public API with host buffers: load (H2D of the
+    # initial balances), run, stats (D2H)
+    e2e_steps = max(1, min(3, args.steps))
+    init_pinned = torch.from_numpy(init).pin_memory()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    e2e_committed = 0
+    for i in range(e2e_steps):
+        store.load(init_pinned.numpy())
+        s = store.run(w, lcfg.n_tx, lcfg.seed + 500 + i)
+        e2e_committed += s["committed"]
+    torch.cuda.synchronize()
+    e2e_s = time.perf_counter() - t0
+    e2e_red = partition.reduce_stats({"committed_update": 0, "committed_ro": 0, "batches": 0, "rounds": 0,
+                                      "total_aborts": 0, "committed": e2e_committed,
+                                      "elapsed_ns": int(e2e_s * 1e9)}, device=dev if world > 1 else None)
+    e2e_value = e2e_red["committed"] / (e2e_red["elapsed_ns"] * 1e-9)
+    store.close()
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return 0
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        r, n, s = oracle_sample_rate(cfg, args.cpu_budget, 1 << 18)
+        cpu = {"value": r, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"{n} consecutive C2 transactions ({s:.1f} s, 1M accounts, 1-warp schedule)"}
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": total_ms_max / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "abort_rate": red["abort_rate"],
+        "config": {"workload": "C2: bank, 1M accounts, K=4, 50% update, uniform, 64-read ROT scans",
+                   "n_items": cfg.n_items, "n_versions": cfg.n_versions, "n_tx_per_step": cfg.n_tx,
+                   "client_warps_per_gpu": n_cw, "server_workers": w.server_workers,
+                   "ro_streak": w.ro_streak, "publish": ["client", "server"][w.publish],
+                   "parallelism": "partitioned" if world > 1 else "single-gpu",
+                   "multi_gpu": "independent key-range partitions, no cross-GPU transactions, NCCL stats only",
+                   "l2": "flushed (512 MiB write) before every timed step"},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                     "kernel": "csmv_fused", "algorithmic_bytes_per_launch": algo,
+                     "note": "latency/serialisation-bound: see serial_chain"},
+        "serial_chain": {"batches_per_s": red["batches"] / (total_ms_max * 1e-3),
+                         "critical_section_cycles_per_batch": cs_cycles,
+                         "updates_per_batch": red["committed_update"] / max(1, red["batches"])},
+        "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(init.nbytes),
+                "d2h_bytes_per_step": 400},
+        "gpu_launches": args.steps * int(last["kernel_launches"]),
+        "clocks": clk.summary(),
+        "kernel_ms_per_step": statistics.mean(kern_ns) / 1e6,
+        "aborts": last["aborts"],
+    }
+    if cpu:
+        line["cpu_baseline"] = cpu
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser(description=__doc__.split("\n")[0])
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
+    ap.add_argument("--n-tx", type=int, default=0)
+    ap.add_argument("--client-warps", type=int, default=0)
+    ap.add_argument("--cpu-budget", type=float, default=10.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return bench_reference(args)
+    return bench_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())
