@@ -37,7 +37,7 @@ METRIC = "committed tx/sec and abort rate at 1 B200 (+partitioned 2/4/8)"
 UNIT = "tx/s"
 
 # tuned launch configuration of the C2 workload
-TUNED = dict(client_warps_per_sm=2, server_workers=8, ro_streak=8, publish=1)
+TUNED = dict(client_warps_per_sm=2, server_workers=6, server_combine=4, ro_streak=8, publish=1)
 
 # algorithmic bytes (paper VBox layout P:289): a read moves the
 # VBox head, the visited version's ts and the value (4+4+4); a write-back the
@@ -155,7 +155,7 @@ def make_cfg(args, world: int, rank: int):
     cfg = workloads.c2()
     n_tx = args.n_tx or cfg.n_tx
     cfg = cfg.with_(n_tx=n_tx, log_mode=0, ro_streak=TUNED["ro_streak"], publish=TUNED["publish"],
-                    server_workers=TUNED["server_workers"])
+                    server_workers=TUNED["server_workers"], server_combine=TUNED["server_combine"])
     part = partition.partition(cfg.n_items, n_tx, cfg.seed, rank, world)
     return cfg, partition.local_config(cfg, part), part
 
@@ -292,6 +292,7 @@ def bench_ours(args):
         "config": {"workload": "C2: bank, 1M accounts, K=4, 50% update, uniform, 64-read ROT scans",
                    "n_items": cfg.n_items, "n_versions": cfg.n_versions, "n_tx_per_step": cfg.n_tx,
                    "client_warps_per_gpu": n_cw, "server_workers": w.server_workers,
+                   "server_combine": w.server_combine,
                    "ro_streak": w.ro_streak, "publish": ["client", "server"][w.publish],
                    "parallelism": "partitioned" if world > 1 else "single-gpu",
                    "multi_gpu": "independent key-range partitions, no cross-GPU transactions, NCCL stats only",

@@ -80,6 +80,7 @@ typedef struct csmv_workload {
     uint32_t server;           /* CSMV_SERVER_* */
     uint32_t cluster_size;     /* cluster server CTAs (2..16) */
     uint32_t server_workers;   /* worker warps per server CTA (0 = default) */
+    uint32_t server_combine;   /* batches a worker commits per critical section (1..4; 0 = 1) */
     uint32_t atr_capacity;     /* ATR entries (0 = default); rounded to the layout */
     uint32_t atr_mode;         /* CSMV_ATR_* */
     uint32_t publish;          /* CSMV_PUBLISH_* */
@@ -103,6 +104,7 @@ typedef struct csmv_stats {
     uint64_t committed_ro;
     uint64_t aborts[CSMV_N_ABORT][2]; /* [reason][0 = read-only, 1 = update] */
     uint64_t batches;          /* requests the server processed */
+    uint64_t server_groups;    /* critical sections (each commits 1..4 batches) */
     uint64_t rounds;           /* client warp rounds */
     uint64_t gts_start;
     uint64_t gts_final;

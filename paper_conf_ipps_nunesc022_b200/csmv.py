@@ -38,13 +38,14 @@ class CsmvError(RuntimeError):
 class _Workload(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in (
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
-        "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers",
+        "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers", "server_combine",
         "atr_capacity", "atr_mode", "publish", "ro_streak", "log_mode", "debug_flags", "watchdog_ms")]
 
 
 class _Stats(C.Structure):
     _fields_ = [("committed_update", C.c_uint64), ("committed_ro", C.c_uint64),
                 ("aborts", (C.c_uint64 * 2) * 5), ("batches", C.c_uint64),
+                ("server_groups", C.c_uint64),
                 ("rounds", C.c_uint64), ("gts_start", C.c_uint64), ("gts_final", C.c_uint64),
                 ("elapsed_ns", C.c_uint64), ("ro_checksum", C.c_uint64),
                 ("store_bytes", C.c_uint64), ("store_bytes_paper", C.c_uint64),
@@ -71,6 +72,7 @@ class Workload:
     server: int = SERVER_CTA
     cluster_size: int = 16
     server_workers: int = 0
+    server_combine: int = 0
     atr_capacity: int = 0
     atr_mode: int = ATR_HASH
     publish: int = PUBLISH_CLIENT

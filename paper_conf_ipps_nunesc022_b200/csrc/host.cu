@@ -278,10 +278,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   uint32_t n_workers = w->server_workers ? w->server_workers : 4u;
   if (n_workers > kWarps - 2) n_workers = kWarps - 2;
 
-  // recent-commit table: 2 entries per bucket (default 16384 entries, 128 KB)
+  // recent-commit table: 4 entries per bucket (default 16384 entries, 144 KB)
   uint32_t entries = w->atr_capacity ? w->atr_capacity : 16384u;
   uint32_t rt_log2 = 1;
-  while ((2u << rt_log2) < entries && rt_log2 < 13) ++rt_log2;
+  while ((4u << rt_log2) < entries && rt_log2 < 12) ++rt_log2;
   size_t smem = server_smem_bytes(rt_log2, n_cw);
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
   int bps = 0;
@@ -335,6 +335,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.lastw = h->d_lastw;
   p.publish = w->publish;
   p.ro_streak = w->ro_streak;
+  p.combine = w->server_combine ? w->server_combine : 1u;
   p.debug = w->debug_flags;
   p.watchdog_ns = (uint64_t)(w->watchdog_ms ? w->watchdog_ms : 20000u) * 1000000ull;
 
@@ -363,6 +364,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   for (int i = 0; i < (int)CSMV_N_ABORT; ++i)
     for (int k = 0; k < 2; ++k) s.aborts[i][k] = ds.aborts[i][k];
   s.batches = ds.batches;
+  s.server_groups = ds.groups;
   s.rounds = ds.rounds;
   s.gts_start = gts0;
   s.gts_final = gts1;
@@ -376,7 +378,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   s.client_warps = n_cw;
   s.server_ctas = 1;
   s.server_workers = n_workers;
-  s.atr_entries = 2u << rt_log2;
+  s.atr_entries = 4u << rt_log2;
   s.sm_count = (uint32_t)h->sm_count;
   s.kernel_launches = 1;
   h->last_n_tx = n_tx;

@@ -406,77 +406,65 @@ struct SrvShared {
 // The ATR, item-indexed and split in two levels:
 //  * lastw[x] in HBM: CTS of the last commit that wrote x -- the exact
 //    record of every committed write-set, all history;
-//  * rt in shared memory: 2-way buckets of (cts << 32 | item) holding the
-//    latest writes, so that commits made after a worker prefetched lastw
-//    (CTS > e_pre) are seen with on-chip latency.
-// Validation of x for snapshot s (P:75 read-set, P:115 write-set):
-//    conflict  iff  lastw[x] (as of e_pre) > s  or  rt has (x, c) with c > s;
-//    unknown   iff  x is not in its bucket and both entries have CTS > e_pre
-//                   (an eviction may have hidden a write of x) -> OVERFLOW.
+//  * rt in shared memory: 4-way buckets of (cts << 32 | item) holding recent
+//    writes plus, per bucket, evmax = the largest CTS ever evicted from it,
+//    so that commits made after a worker prefetched lastw (CTS > e_pre) are
+//    seen with on-chip latency.
+// Invariant: if the latest write c of item y (bucket b) is not in b, then
+// evmax[b] >= c (entries leave a bucket only through atomicExch, and the
+// evictor records the evicted CTS with atomicMax).
+// Validation of x for snapshot s (P:75 read-set, P:115 write-set), s <= e_pre:
+//    conflict  iff  lastw[x] (as of e_pre) > s  or  some way holds (x, c), c > s
+//    unknown   iff  not conflict and evmax[b] > e_pre -> abort, reason OVERFLOW
 // ---------------------------------------------------------------------------
+constexpr int kRtWays = 4;
+
 __device__ __forceinline__ uint32_t rt_bucket(uint32_t key, uint32_t rt_log2) {
   return (key * 0x9E3779B1u) >> (32 - rt_log2);
 }
 
 struct RtProbe {
-  ulonglong2 b;  // the bucket
+  int way;        // way to overwrite: the way holding x, else the oldest
   bool conflict;
   bool unknown;
 };
 
-__device__ __forceinline__ RtProbe rt_probe(const uint64_t* rt, uint32_t bucket, uint32_t key, uint32_t s,
-                                            uint32_t e_pre, uint32_t lastw) {
+__device__ __forceinline__ RtProbe rt_probe(const uint64_t* rt, const uint32_t* evmax, uint32_t bucket,
+                                            uint32_t key, uint32_t s, uint32_t e_pre, uint32_t lastw) {
+  const ulonglong2* e = reinterpret_cast<const ulonglong2*>(rt + (size_t)bucket * kRtWays);
+  const ulonglong2 a = e[0], b = e[1];
+  const uint32_t ev = evmax[bucket];
+  const uint64_t w[4] = {a.x, a.y, b.x, b.y};
   RtProbe r;
-  r.b = reinterpret_cast<const ulonglong2*>(rt)[bucket];
-  const uint32_t k0 = (uint32_t)r.b.x, k1 = (uint32_t)r.b.y;
-  const uint32_t c0 = (uint32_t)(r.b.x >> 32), c1 = (uint32_t)(r.b.y >> 32);
-  const bool f0 = k0 == key, f1 = k1 == key;
-  r.conflict = lastw > s || (f0 && c0 > s) || (f1 && c1 > s);
-  r.unknown = !f0 && !f1 && min(c0, c1) > e_pre;
+  r.conflict = lastw > s;
+  int hit = -1, old = 0;
+  uint32_t oldc = 0xFFFFFFFFu;
+#pragma unroll
+  for (int i = 0; i < kRtWays; ++i) {
+    const uint32_t k = (uint32_t)w[i], c = (uint32_t)(w[i] >> 32);
+    if (k == key) {
+      hit = i;
+      r.conflict |= c > s;
+    }
+    if (c < oldc) {
+      oldc = c;
+      old = i;
+    }
+  }
+  r.unknown = !r.conflict && ev > e_pre;
+  r.way = hit >= 0 ? hit : old;
   return r;
 }
 
-// Record (key0, cts) and (key1, cts) for every lane with `active`: each
-// replaces the entry of the same key, else the older way of its bucket.
-// Lanes write in parallel and verify after a __syncwarp; two writers of the
-// same way leave one winner and the loser retries on the re-read bucket.
-// Entries are only ever evicted by newer batches (or by lanes of the same
-// batch, whose CTS lie between the same two tail values), which is what
-// makes the `unknown` rule of rt_probe sufficient.
-__device__ __forceinline__ int rt_way(ulonglong2 b, uint32_t key) {
-  if ((uint32_t)b.x == key) return 0;
-  if ((uint32_t)b.y == key) return 1;
-  return ((uint32_t)(b.y >> 32) < (uint32_t)(b.x >> 32)) ? 1 : 0;
-}
-
-__device__ __forceinline__ void rt_insert2(uint64_t* rt, uint32_t bk0, uint32_t key0, ulonglong2 b0,
-                                           uint32_t bk1, uint32_t key1, ulonglong2 b1, uint32_t cts,
-                                           bool active) {
-  const uint64_t m0 = ((uint64_t)cts << 32) | key0, m1 = ((uint64_t)cts << 32) | key1;
-  const ulonglong2* rb = reinterpret_cast<const ulonglong2*>(rt);
-  bool p0 = active, p1 = active;
-  bool first = true;
-  while (__any_sync(0xFFFFFFFFu, p0 || p1)) {
-    int w0 = 0, w1 = 0;
-    if (p0 || p1) {
-      if (!first) {
-        b0 = rb[bk0];
-        b1 = rb[bk1];
-      }
-      if (p0) w0 = rt_way(b0, key0);
-      if (p1) {
-        w1 = rt_way(b1, key1);
-        if (p0 && bk1 == bk0 && w1 == w0) w1 ^= 1;  // both keys of one lane share a bucket
-      }
-      if (p0) rt[2 * (size_t)bk0 + w0] = m0;
-      if (p1) rt[2 * (size_t)bk1 + w1] = m1;
-    }
-    __syncwarp();
-    if (p0 && rt[2 * (size_t)bk0 + w0] == m0) p0 = false;
-    if (p1 && rt[2 * (size_t)bk1 + w1] == m1) p1 = false;
-    first = false;
-    __syncwarp();
-  }
+// Record (key, cts) into `way` of its bucket; an evicted entry of another
+// key raises evmax.  Exchanges by several lanes on one slot are serialised
+// by the hardware and each evictor sees the value it replaced.
+__device__ __forceinline__ void rt_record(uint64_t* rt, uint32_t* evmax, uint32_t bucket, int way,
+                                          uint32_t key, uint32_t cts) {
+  const unsigned long long old =
+      atomicExch(reinterpret_cast<unsigned long long*>(rt + (size_t)bucket * kRtWays + way),
+                 ((unsigned long long)cts << 32) | key);
+  if ((uint32_t)old != key && (uint32_t)(old >> 32) != 0u) atomicMax(evmax + bucket, (uint32_t)(old >> 32));
 }
 
 // Receiver warp: sweeps every client doorbell with coalesced loads
@@ -539,28 +527,35 @@ __device__ void server_receiver(const KParams& p, uint32_t* last_seen, uint64_t*
   }
 }
 
-__device__ void server_worker(const KParams& p, uint64_t* rt, uint64_t* queue, uint32_t qn_log2,
-                              SrvShared* sh, uint64_t t_begin) {
+// Server worker warp.  Claims up to kMaxCombine dispatched batches (the
+// first blocking, the rest only if already queued), loads them outside the
+// lock, and commits them inside ONE critical section, one after another in
+// queue order -- exactly as if each had its own critical section: batch j
+// is validated after batch j-1's write-set was recorded, and receives the
+// next consecutive CTS range.
+__device__ void server_worker(const KParams& p, uint64_t* rt, uint32_t* evmax, uint64_t* queue,
+                              uint32_t qn_log2, SrvShared* sh, uint64_t t_begin) {
+  constexpr int M = kMaxCombine;
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t lt = lanemask_lt();
   const uint32_t qmask = (1u << qn_log2) - 1;
   const uint32_t dmask = (1u << kDoneLog2) - 1;
-  unsigned long long busy = 0, locked = 0, batches = 0;
+  const uint32_t m_max = p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine);
+  unsigned long long busy = 0, locked = 0, batches = 0, groups = 0;
   unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   for (;;) {
     const long long tq = clock64();
-    // Claim the next dispatched request.
+    // ---- claim: first request blocking
     uint32_t slot = 0;
     if (lane == 0) slot = atomicAdd(&sh->q_head, 1u);
     slot = __shfl_sync(FULL, slot, 0);
-    const uint32_t lap = (slot >> qn_log2) + 1;
-    // Convergent wait (every lane polls the same word: one broadcast LDS).
+    uint32_t cwv[M];
     uint64_t ent;
     bool quit = false;
     for (;;) {
       ent = *(volatile uint64_t*)&queue[slot & qmask];
-      if ((uint32_t)(ent >> 32) == lap) break;
+      if ((uint32_t)(ent >> 32) == (slot >> qn_log2) + 1) break;
       if (*(volatile uint32_t*)&sh->exit) {
         quit = true;
         break;
@@ -568,32 +563,62 @@ __device__ void server_worker(const KParams& p, uint64_t* rt, uint64_t* queue, u
       __nanosleep(64);
     }
     if (quit) break;
-    const uint32_t cw = (uint32_t)ent;
+    cwv[0] = (uint32_t)ent;
+    // ---- combine: grab further requests that are already queued
+    uint32_t m = 1;
+#pragma unroll
+    for (int j = 1; j < M; ++j) {
+      uint32_t got = 0xFFFFFFFFu;
+      if (m == (uint32_t)j && m < m_max && lane == 0) {
+        const uint32_t h = *(volatile uint32_t*)&sh->q_head;
+        const uint64_t e = *(volatile uint64_t*)&queue[h & qmask];
+        if ((uint32_t)(e >> 32) == (h >> qn_log2) + 1 && atomicCAS(&sh->q_head, h, h + 1) == h) got = (uint32_t)e;
+      }
+      got = __shfl_sync(FULL, got, 0);
+      cwv[j] = got;
+      if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
+    }
     const long long t0 = clock64();
-    // Load the batch: doorbell (acquire pattern), header, one id row per
-    // RS u WS entry (coalesced 128 B), then prefetch lastw of every item.
-    const uint32_t sq = ld_relaxed(p.req_seq + cw);
+    // ---- load the batches: doorbell (acquire pattern), header, ids
+    uint32_t sq[M], sn[M], msk[M], id0[M], id1[M];
+#pragma unroll
+    for (int j = 0; j < M; ++j) sq[j] = (j < (int)m) ? ld_relaxed(p.req_seq + cwv[j]) : 0u;
     fence_gpu();
-    const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
-    const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
-    const bool mine = (mask >> lane) & 1u;
-    uint32_t id0 = 0, id1 = 0;
-    if (mine) {
-      id0 = ld_relaxed(p.req_ids + (size_t)cw * 64 + lane) & ~kWriteBit;
-      id1 = ld_relaxed(p.req_ids + (size_t)cw * 64 + 32 + lane) & ~kWriteBit;
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      sn[j] = msk[j] = id0[j] = id1[j] = 0;
+      if (j < (int)m) {
+        sn[j] = ld_relaxed(&p.req_hdr[cwv[j]].snapshot);
+        msk[j] = ld_relaxed(&p.req_hdr[cwv[j]].mask);
+      }
+    }
+    bool mine[M];
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      mine[j] = (msk[j] >> lane) & 1u;
+      if (mine[j]) {
+        id0[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + lane) & ~kWriteBit;
+        id1[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + 32 + lane) & ~kWriteBit;
+      }
     }
     const uint32_t e_pre = *(volatile uint32_t*)&sh->tail;  // lastw covers every CTS <= e_pre
     fence_cta();
-    uint32_t lw0 = 0, lw1 = 0;
-    if (mine) {
-      lw0 = ld_relaxed(p.lastw + id0);
-      lw1 = ld_relaxed(p.lastw + id1);
+    uint32_t lw0[M], lw1[M], bk0[M], bk1[M];
+    uint32_t xor_all = e_pre;
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      lw0[j] = lw1[j] = 0;
+      if (mine[j]) {
+        lw0[j] = ld_relaxed(p.lastw + id0[j]);
+        lw1[j] = ld_relaxed(p.lastw + id1[j]);
+      }
+      bk0[j] = rt_bucket(id0[j], p.rt_log2);
+      bk1[j] = rt_bucket(id1[j], p.rt_log2);
+      xor_all ^= bk0[j] ^ bk1[j] ^ lw0[j] ^ lw1[j] ^ sn[j];
     }
-    const uint32_t b0 = rt_bucket(id0, p.rt_log2), b1 = rt_bucket(id1, p.rt_log2);
     // The payload must have arrived before the lock is taken: a warp vote on
-    // values derived from it makes the loads complete here, not inside the
-    // critical section.
-    if (__ballot_sync(FULL, (b0 ^ b1 ^ lw0 ^ lw1 ^ s) == 0xFFFFFFFFu) == 0xFFFFFFFFu) __nanosleep(1);
+    // values derived from it makes the loads complete here.
+    if (__ballot_sync(FULL, xor_all == 0x12345679u) == FULL) __nanosleep(1);
     const long long tl = clock64();
     // ---- critical section: validate, reserve CTS, record
     uint32_t ticket = 0;
@@ -604,53 +629,70 @@ __device__ void server_worker(const KParams& p, uint64_t* rt, uint64_t* queue, u
     fence_cta();
     const long long t1 = clock64();
     const uint32_t t0c = *(volatile uint32_t*)&sh->tail;
-    RtProbe q0{}, q1{};
-    if (mine) {
-      q0 = rt_probe(rt, b0, id0, s, e_pre, lw0);
-      q1 = rt_probe(rt, b1, id1, s, e_pre, lw1);
+    uint32_t t = t0c;
+    uint32_t cm[M], om[M], base[M];
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      cm[j] = om[j] = 0;
+      base[j] = t + 1;
+      if (j >= (int)m) continue;
+      RtProbe q0{0, false, false}, q1{0, false, false};
+      if (mine[j]) {
+        q0 = rt_probe(rt, evmax, bk0[j], id0[j], sn[j], e_pre, lw0[j]);
+        q1 = rt_probe(rt, evmax, bk1[j], id1[j], sn[j], e_pre, lw1[j]);
+        if (bk1[j] == bk0[j] && q1.way == q0.way) q1.way = (q1.way + 1) & (kRtWays - 1);
+      }
+      bool ovf = mine[j] && (q0.unknown || q1.unknown);
+      bool conflict = mine[j] && (q0.conflict || q1.conflict);
+      if (p.debug & CSMV_DBG_NO_VALIDATE) ovf = conflict = false;
+      const bool commit = mine[j] && !ovf && !conflict;
+      cm[j] = __ballot_sync(FULL, commit);
+      om[j] = __ballot_sync(FULL, ovf);
+      const uint32_t c = t + 1 + __popc(cm[j] & lt);
+      t += __popc(cm[j]);
+      if (commit) {
+        p.lastw[id0[j]] = c;
+        p.lastw[id1[j]] = c;
+        rt_record(rt, evmax, bk0[j], q0.way, id0[j], c);
+        rt_record(rt, evmax, bk1[j], q1.way, id1[j], c);
+      }
+      __syncwarp();  // batch j's records precede batch j+1's probes
     }
-    bool ovf = mine && (q0.unknown || q1.unknown);
-    bool conflict = mine && (q0.conflict || q1.conflict);
-    if (p.debug & CSMV_DBG_NO_VALIDATE) ovf = conflict = false;
-    const bool commit = mine && !ovf && !conflict;
-    const uint32_t cm = __ballot_sync(FULL, commit);
-    const uint32_t n = __popc(cm);
-    const uint32_t cts = t0c + 1 + __popc(cm & lt);
     const long long ta = clock64();
-    if (p.publish == CSMV_PUBLISH_SERVER && n) {
+    if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) {
       // done-ring back-pressure: CTS c may reuse slot c & dmask only once
       // GTS >= c - 2^20
       if (lane == 0) {
         uint32_t it = 0;
-        while (t0c + n > sh->gts_seen + dmask) {
+        while (t > sh->gts_seen + dmask) {
           sh->gts_seen = ld_relaxed(p.gts);
           if ((++it & 255u) == 0 && watchdog(p, t_begin, 4)) break;
         }
       }
       __syncwarp();
     }
-    if (commit) {
-      st_relaxed(p.lastw + id0, cts);
-      st_relaxed(p.lastw + id1, cts);
-    }
-    const long long tb = clock64();
-    rt_insert2(rt, b0, id0, q0.b, b1, id1, q1.b, cts, commit);
-    const long long tc = clock64();
-    __syncwarp();
     fence_cta();
     if (lane == 0) {
-      sh->tail = t0c + n;
+      sh->tail = t;
       fence_cta();
       *(volatile uint32_t*)&sh->now_serving = ticket + 1;
     }
     const long long t2 = clock64();
-    // ---- respond
-    const uint32_t om = __ballot_sync(FULL, ovf);
+    // ---- respond: one fence, then the payloads and sequence words
     if (lane == 0) {
-      st_relaxed(&p.resp[cw].cts_base, t0c + 1);
-      st_relaxed(&p.resp[cw].commit_mask, cm);
-      st_relaxed(&p.resp[cw].overflow_mask, om);
-      st_release(&p.resp[cw].seq, sq);
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        if (j >= (int)m) break;
+        st_relaxed(&p.resp[cwv[j]].cts_base, base[j]);
+        st_relaxed(&p.resp[cwv[j]].commit_mask, cm[j]);
+        st_relaxed(&p.resp[cwv[j]].overflow_mask, om[j]);
+      }
+      fence_gpu();
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        if (j >= (int)m) break;
+        st_relaxed(&p.resp[cwv[j]].seq, sq[j]);
+      }
     }
     __syncwarp();
     const long long t3 = clock64();
@@ -662,13 +704,13 @@ __device__ void server_worker(const KParams& p, uint64_t* rt, uint64_t* queue, u
     ph[3] += (unsigned long long)(t2 - t1);
     ph[4] += (unsigned long long)(t3 - t2);
     ph[5] += (unsigned long long)(ta - t1);
-    ph[6] += (unsigned long long)(tb - ta);
-    ph[7] += (unsigned long long)(tc - tb);
-    ++batches;
+    batches += m;
+    ++groups;
   }
   if (lane == 0) {
     for (int i = 0; i < 8; ++i) atomicAdd(&p.stats->phase[i], ph[i]);
     atomicAdd(&p.stats->batches, batches);
+    atomicAdd(&p.stats->groups, groups);
     atomicAdd(&p.stats->busy_cycles, busy);
     atomicAdd(&p.stats->lock_cycles, locked);
   }
@@ -716,13 +758,15 @@ __device__ void server_publisher(const KParams& p, SrvShared* sh, uint64_t t_beg
 
 __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   uint64_t* rt = reinterpret_cast<uint64_t*>(smem);
-  const uint32_t rt_words = 2u << p.rt_log2;
+  const uint32_t rt_words = (uint32_t)kRtWays << p.rt_log2;
   const uint32_t qn_log2 = queue_log2(p.n_cw);
   uint64_t* queue = rt + rt_words;
-  uint32_t* last_seen = reinterpret_cast<uint32_t*>(queue + (1u << qn_log2));
+  uint32_t* evmax = reinterpret_cast<uint32_t*>(queue + (1u << qn_log2));
+  uint32_t* last_seen = evmax + (1u << p.rt_log2);
   const uint32_t ls_words = (p.n_cw + 31) / 32 * 32;
   SrvShared* sh = reinterpret_cast<SrvShared*>(last_seen + ls_words);
   for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) rt[i] = 0xFFFFFFFFull;  // cts 0, no item
+  for (uint32_t i = threadIdx.x; i < (1u << p.rt_log2); i += blockDim.x) evmax[i] = 0;
   for (uint32_t i = threadIdx.x; i < (1u << qn_log2); i += blockDim.x) queue[i] = 0;
   for (uint32_t i = threadIdx.x; i < ls_words; i += blockDim.x) last_seen[i] = 0;
   if (threadIdx.x == 0) {
@@ -739,7 +783,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   if (warp == 0) {
     server_receiver(p, last_seen, queue, qn_log2, sh, t_begin);
   } else if (warp <= p.n_workers) {
-    server_worker(p, rt, queue, qn_log2, sh, t_begin);
+    server_worker(p, rt, evmax, queue, qn_log2, sh, t_begin);
   } else if (warp == p.n_workers + 1 && p.publish == CSMV_PUBLISH_SERVER) {
     server_publisher(p, sh, t_begin);
   }

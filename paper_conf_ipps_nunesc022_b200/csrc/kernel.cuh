@@ -25,9 +25,10 @@ namespace csmvd {
 
 constexpr uint32_t kEmptyTs = 0xFFFFFFFFu;
 constexpr uint32_t kWriteBit = 0x80000000u;
-constexpr int kBlock = 512;            // threads per CTA (16 warps)
+constexpr int kBlock = 256;            // threads per CTA (8 warps)
 constexpr int kWarps = kBlock / 32;
 constexpr uint32_t kDoneLog2 = 20;     // done ring entries (CSMV_PUBLISH_SERVER)
+constexpr int kMaxCombine = 4;         // batches a server worker commits per critical section
 
 struct Ctl {
   uint32_t error;       // 0 ok, 1 watchdog, 2 protocol
@@ -51,7 +52,7 @@ struct Resp {
 struct DevStats {
   unsigned long long committed_update, committed_ro;
   unsigned long long aborts[CSMV_N_ABORT][2];
-  unsigned long long batches, rounds;
+  unsigned long long batches, rounds, groups;
   unsigned long long ro_checksum;
   unsigned long long lock_cycles, busy_cycles;
   unsigned long long phase[8];  // server worker: queue wait, load, lock wait, critical, respond
@@ -78,10 +79,11 @@ struct KParams {
   uint32_t n_cw;           // active client warps
   uint32_t n_client_ctas;  // CTAs 1..n_client_ctas host clients
   uint32_t n_workers;      // server worker warps
-  uint32_t rt_log2;        // recent-commit table buckets (2 ways, 16 B each)
+  uint32_t rt_log2;        // recent-commit table buckets (4 ways, 32 B each, + evmax)
   uint32_t* lastw;         // per-item CTS of the last committed write
   uint32_t publish;
   uint32_t ro_streak;      // read-only transactions a lane may run per round (0 = one tx per round)
+  uint32_t combine;        // batches per critical section (1..kMaxCombine)
   uint32_t debug;
   uint64_t watchdog_ns;
 };
@@ -96,7 +98,7 @@ __host__ __device__ inline uint32_t queue_log2(uint32_t n_cw) {
 // smem the server CTA needs (every CTA of the fused grid gets the same):
 // recent-commit table, dispatch queue, receiver's last-seen doorbells, control words
 inline size_t server_smem_bytes(uint32_t rt_log2, uint32_t n_cw) {
-  return ((size_t)16 << rt_log2) + ((size_t)8 << queue_log2(n_cw)) +
+  return ((size_t)(32 + 4) << rt_log2) + ((size_t)8 << queue_log2(n_cw)) +
          (((size_t)n_cw + 31) / 32 * 32) * 4 + 64;
 }
 

@@ -94,11 +94,12 @@ def test_one_warp_is_deterministic(k, streak, ro_reads):
     assert stats["batches"] == pst["batches"] and stats["rounds"] == pst["rounds"]
 
 
-@pytest.mark.parametrize("publish,streak,workers", [(csmv.PUBLISH_CLIENT, 0, 4), (csmv.PUBLISH_SERVER, 0, 8),
-                                                   (csmv.PUBLISH_SERVER, 8, 8), (csmv.PUBLISH_CLIENT, 8, 2)])
-def test_c2_shrunk_parity(publish, streak, workers):
+@pytest.mark.parametrize("publish,streak,workers,combine", [
+    (csmv.PUBLISH_CLIENT, 0, 4, 1), (csmv.PUBLISH_SERVER, 0, 6, 1), (csmv.PUBLISH_SERVER, 8, 6, 4),
+    (csmv.PUBLISH_CLIENT, 8, 2, 2), (csmv.PUBLISH_SERVER, 8, 6, 3)])
+def test_c2_shrunk_parity(publish, streak, workers, combine):
     cfg = W.c2(n_items=1 << 16, n_tx=1 << 18, publish=publish, ro_streak=streak,
-               server_workers=workers)
+               server_workers=workers, server_combine=combine, client_warps=512)
     rep, stats, log, rings, descs = check(cfg)
     assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions),
                           closed_form(cfg, descs, cfg.init_values()))
@@ -106,7 +107,7 @@ def test_c2_shrunk_parity(publish, streak, workers):
 
 @pytest.mark.parametrize("streak", [0, 8])
 def test_c3_shrunk_parity(streak):
-    cfg = W.c3(n_tx=1 << 18, ro_streak=streak, client_warps=256)
+    cfg = W.c3(n_tx=1 << 18, ro_streak=streak, client_warps=256, server_combine=4, server_workers=6)
     rep, stats, log, rings, descs = check(cfg)
     assert stats["aborts"]["conflict"]["ro"] == 0 and stats["aborts"]["early"]["ro"] == 0  # P6/Q7
 
@@ -120,10 +121,11 @@ def test_version_misses_k1():
     assert stats["aborts"]["conflict"]["ro"] == 0
 
 
-def test_tiny_atr_overflow():
+@pytest.mark.parametrize("combine", [1, 4])
+def test_tiny_atr_overflow(combine):
     """A tiny ATR forces evictions: spurious aborts appear only with the
     labelled OVERFLOW reason and never let a conflicting commit through."""
-    cfg = W.c2(n_items=1 << 12, n_tx=1 << 17, atr_capacity=16)
+    cfg = W.c2(n_items=1 << 12, n_tx=1 << 17, atr_capacity=16, server_combine=combine, client_warps=256)
     rep, stats, *_ = check(cfg)
     assert stats["aborts"]["overflow"]["update"] > 0
 
@@ -142,8 +144,9 @@ def test_empty_run():
     assert stats["committed"] == 0 and stats["gts_final"] == 0
 
 
-def test_update_only_high_contention():
-    cfg = W.c2(n_items=64, n_tx=1 << 15, p_update_ppm=1_000_000, client_warps=64)
+@pytest.mark.parametrize("combine", [1, 4])
+def test_update_only_high_contention(combine):
+    cfg = W.c2(n_items=64, n_tx=1 << 15, p_update_ppm=1_000_000, client_warps=64, server_combine=combine)
     rep, stats, *_ = check(cfg)
     assert stats["aborts"]["preval"]["update"] > 0
 

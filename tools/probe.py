@@ -30,7 +30,7 @@ def main(argv):
                                      "batches", "rounds", "elapsed_ns", "client_warps",
                                      "server_lock_cycles", "server_busy_cycles", "wall_s")}
             b = max(1, s["batches"])
-            out["phase_per_batch"] = {k: v // b for k, v in s["server_phase_cycles"].items()}
+            out["phase_per_batch"] = {k: v // max(1, s["server_groups"]) for k, v in s["server_phase_cycles"].items()}
             out["aborts"] = {k: v for k, v in s["aborts"].items() if v["ro"] or v["update"]}
             out["cfg"] = dict(name=name, **kw)
             print(json.dumps(out), flush=True)
