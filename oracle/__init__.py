@@ -20,6 +20,7 @@ import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SRC = os.path.join(HERE, "oracle.c")
+SRC_KV = os.path.join(HERE, "oracle_kv.c")
 HDR = os.path.join(HERE, "oracle.h")
 LIB = os.path.join(HERE, "liboracle.so")
 
@@ -71,13 +72,46 @@ class PredStats(C.Structure):
         return {f: getattr(self, f) for f, _ in self._fields_}
 
 
+class KvCfg(C.Structure):
+    _fields_ = [(n, C.c_uint32) for n in ("n_slots", "ways", "n_keys", "n_versions", "dist",
+                                         "zipf_theta_milli", "p_update_ppm", "ro_streak")]
+
+
+class KvState(C.Structure):
+    _fields_ = [("keys", C.c_void_p), ("vals", C.c_void_p), ("lru", C.c_void_p),
+                ("clocks", C.c_void_p)]
+
+
+KV_DESC_DTYPE = np.dtype([("is_update", "<u4"), ("key", "<u4"), ("val", "<u4", (8,))])
+
+
+class KvStore:
+    """numpy-backed or_kv_state (keys S x 4, vals S x 8, lru S, clocks S/A)."""
+
+    def __init__(self, n_slots, ways):
+        self.keys = np.zeros((n_slots, 4), dtype=np.uint32)
+        self.vals = np.zeros((n_slots, 8), dtype=np.uint32)
+        self.lru = np.zeros(n_slots, dtype=np.uint32)
+        self.clocks = np.zeros(n_slots // ways, dtype=np.uint32)
+
+    def c(self) -> KvState:
+        return KvState(self.keys.ctypes.data, self.vals.ctypes.data, self.lru.ctypes.data,
+                       self.clocks.ctypes.data)
+
+    def copy(self):
+        o = KvStore.__new__(KvStore)
+        o.keys, o.vals, o.lru, o.clocks = (self.keys.copy(), self.vals.copy(), self.lru.copy(),
+                                           self.clocks.copy())
+        return o
+
+
 def build(force: bool = False) -> str:
     """Compile liboracle.so with gcc (plain C99)."""
     stale = force or not os.path.exists(LIB) or any(
-        os.path.getmtime(p) > os.path.getmtime(LIB) for p in (SRC, HDR))
+        os.path.getmtime(p) > os.path.getmtime(LIB) for p in (SRC, SRC_KV, HDR))
     if stale:
         subprocess.check_call(["gcc", "-O2", "-std=c99", "-Wall", "-Wextra", "-fPIC",
-                               "-shared", "-o", LIB, SRC, "-lm"])
+                               "-shared", "-o", LIB, SRC, SRC_KV, "-lm"])
     return LIB
 
 
@@ -106,6 +140,15 @@ def lib():
                                       vp, C.POINTER(PredStats)]
         L.or_vbox_bytes.restype = u64
         L.or_vbox_bytes.argtypes = [u64, u32, u32]
+        L.or_kv_key16.argtypes = [u32, vp]
+        L.or_kv_set.restype = u32
+        L.or_kv_set.argtypes = [u32, u32]
+        L.or_kv_gen.argtypes = [C.POINTER(KvCfg), u64, u64, u64, vp, vp]
+        L.or_kv_preload.argtypes = [C.POINTER(KvCfg), C.POINTER(KvState)]
+        L.or_kv_check.argtypes = [C.POINTER(KvCfg), C.POINTER(KvState), u64, vp, vp,
+                                  C.POINTER(KvState), C.POINTER(Claims), C.POINTER(Report)]
+        L.or_kv_predict.argtypes = [C.POINTER(KvCfg), C.POINTER(KvState), u64, vp, u32, vp,
+                                    C.POINTER(KvState), C.POINTER(PredStats)]
         _lib = L
     return _lib
 
@@ -195,3 +238,65 @@ def pack(ts: int, val: int) -> int:
 def unpack(slot: int):
     ts, v = slot >> 32, slot & 0xFFFFFFFF
     return ts, v - (1 << 32) if v >= (1 << 31) else v
+
+
+def kv_cfg(n_slots, ways=16, n_keys=None, n_versions=4, dist=DIST_ZIPF, zipf_theta_milli=990,
+           p_update_ppm=10_000, ro_streak=0) -> KvCfg:
+    return KvCfg(n_slots, ways, n_slots if n_keys is None else n_keys, n_versions, dist,
+                 zipf_theta_milli, p_update_ppm, ro_streak)
+
+
+def key16(k: int) -> np.ndarray:
+    out = np.zeros(4, dtype=np.uint32)
+    lib().or_kv_key16(k, _ptr(out))
+    return out
+
+
+def kv_set(k: int, n_sets: int) -> int:
+    return lib().or_kv_set(k, n_sets)
+
+
+def kv_gen(cfg: KvCfg, seed: int, n_tx: int, tx0: int = 0) -> np.ndarray:
+    out = np.zeros(n_tx, dtype=KV_DESC_DTYPE)
+    cdf = zipf_cdf(cfg.n_keys, cfg.zipf_theta_milli) if cfg.dist == DIST_ZIPF else None
+    rc = lib().or_kv_gen(C.byref(cfg), seed, tx0, n_tx, _ptr(cdf), _ptr(out))
+    assert rc == 0, rc
+    return out
+
+
+def kv_preload(cfg: KvCfg) -> KvStore:
+    st = KvStore(cfg.n_slots, cfg.ways)
+    cs = st.c()
+    rc = lib().or_kv_preload(C.byref(cfg), C.byref(cs))
+    assert rc == 0, rc
+    return st
+
+
+def kv_check(cfg: KvCfg, init: KvStore, descs, log, final: KvStore | None = None,
+             claims: dict | None = None) -> dict:
+    descs = np.ascontiguousarray(descs, dtype=KV_DESC_DTYPE)
+    log = np.ascontiguousarray(log, dtype=LOG_DTYPE)
+    ci = init.c()
+    cf = final.c() if final is not None else None
+    cl = None
+    if claims is not None:
+        cl = Claims(claims["committed_update"], claims["committed_ro"], claims["gts_final"],
+                    claims["total_aborts"])
+    rep = Report()
+    lib().or_kv_check(C.byref(cfg), C.byref(ci), len(descs), _ptr(descs), _ptr(log),
+                      C.byref(cf) if cf is not None else None,
+                      C.byref(cl) if cl is not None else None, C.byref(rep))
+    return rep.as_dict()
+
+
+def kv_predict(cfg: KvCfg, init: KvStore, descs, n_lanes=32):
+    descs = np.ascontiguousarray(descs, dtype=KV_DESC_DTYPE)
+    n = len(descs)
+    log = np.zeros(n, dtype=LOG_DTYPE)
+    out = KvStore(cfg.n_slots, cfg.ways)
+    ci, co = init.c(), out.c()
+    st = PredStats()
+    rc = lib().or_kv_predict(C.byref(cfg), C.byref(ci), n, _ptr(descs), n_lanes, _ptr(log),
+                             C.byref(co), C.byref(st))
+    assert rc == 0, rc
+    return log, out, st.as_dict()

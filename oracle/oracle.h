@@ -133,6 +133,49 @@ int or_bank_predict(const or_bank_cfg *cfg, const int32_t *init, uint64_t n_tx,
  * (P:289). */
 uint64_t or_vbox_bytes(uint64_t n_items, uint32_t value_bytes, uint32_t k);
 
+
+/* ---- KV workload: MemcachedGPU, docs/GENERATOR.md section 4 ---- */
+typedef struct {
+    uint32_t n_slots;          /* S */
+    uint32_t ways;             /* A (S % A == 0) */
+    uint32_t n_keys;           /* key space */
+    uint32_t n_versions;       /* K */
+    uint32_t dist, zipf_theta_milli;
+    uint32_t p_update_ppm;     /* PUT probability */
+    uint32_t ro_streak;        /* predictor, as in or_bank_cfg */
+} or_kv_cfg;
+
+typedef struct {
+    uint32_t is_update;        /* 1 = PUT, 0 = GET */
+    uint32_t key;              /* key index k */
+    uint32_t val[8];           /* PUT value words */
+} or_kv_desc;
+
+/* Current value of every KV item (newest version). */
+typedef struct {
+    uint32_t *keys;    /* S * 4 words: key of slot i */
+    uint32_t *vals;    /* S * 8 words: value of slot i */
+    uint32_t *lru;     /* S: LRU stamp of slot i */
+    uint32_t *clocks;  /* S / A: clock of set t */
+} or_kv_state;
+
+void or_kv_key16(uint32_t k, uint32_t out[4]);
+uint32_t or_kv_set(uint32_t k, uint32_t n_sets);
+int or_kv_gen(const or_kv_cfg *cfg, uint64_t seed, uint64_t tx0, uint64_t n,
+              const uint64_t *zipf_cdf, or_kv_desc *out);
+/* Preload keys 0..n_keys-1 with PUT semantics (docs/GENERATOR.md 4). */
+int or_kv_preload(const or_kv_cfg *cfg, or_kv_state *st);
+/* Replaying checker: as or_bank_check, over the KV store; final_state (may
+ * be NULL) is the implementation's newest value of every item. */
+int or_kv_check(const or_kv_cfg *cfg, const or_kv_state *init, uint64_t n_tx,
+                const or_kv_desc *d, const or_log_rec *log,
+                const or_kv_state *final_state, const or_claims *claims,
+                or_report *rep);
+/* Deterministic 1-warp schedule; st_out receives the final store. */
+int or_kv_predict(const or_kv_cfg *cfg, const or_kv_state *init, uint64_t n_tx,
+                  const or_kv_desc *d, uint32_t n_lanes, or_log_rec *log_out,
+                  or_kv_state *st_out, or_pred_stats *st);
+
 #ifdef __cplusplus
 }
 #endif

@@ -19,7 +19,7 @@ BANK_DESC_DTYPE = np.dtype([("is_update", "<u4"), ("src", "<u4"), ("dst", "<u4")
 
 
 def mix64(x: int) -> int:
-    z = (x + GOLDEN) & M64
+    z = (int(x) + GOLDEN) & M64
     z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & M64
     z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & M64
     return z ^ (z >> 31)
