@@ -218,3 +218,33 @@ def zipf_table(n: int, theta_milli: int) -> np.ndarray:
     out = np.zeros(n, dtype=np.uint64)
     _check(lib().csmv_zipf_table(n, theta_milli, _ptr(out)))
     return out
+
+
+class KvStore(Store):
+    """A MemcachedGPU store (csmv_create_kv): n_slots slots, `ways` ways."""
+
+    def __init__(self, n_slots: int, ways: int = 16, n_versions: int = 4):
+        h = lib().csmv_create_kv(n_slots, ways, n_versions)
+        if not h:
+            raise CsmvError(ECUDA, lib().csmv_last_error().decode())
+        self.h = h
+        self.n_slots, self.ways, self.n_versions = n_slots, ways, n_versions
+        self.n_items = 3 * n_slots + n_slots // ways
+
+    def load(self, n_keys: int):
+        _check(lib().csmv_load_kv(self.h, n_keys))
+
+    def dump(self):
+        S, T = self.n_slots, self.n_slots // self.ways
+        keys = np.zeros((S, 4), dtype=np.uint32)
+        vals = np.zeros((S, 8), dtype=np.uint32)
+        lru = np.zeros(S, dtype=np.uint32)
+        clocks = np.zeros(T, dtype=np.uint32)
+        _check(lib().csmv_dump_kv(self.h, _ptr(keys), _ptr(vals), _ptr(lru), _ptr(clocks)))
+        return keys, vals, lru, clocks
+
+    def gen_descs(self, w: Workload, seed: int, n: int, tx0: int = 0) -> np.ndarray:
+        out = np.zeros(n * 10, dtype=np.uint32)
+        wc = w.to_c()
+        _check(lib().csmv_gen_descs(self.h, C.byref(wc), seed, tx0, n, _ptr(out)))
+        return out.reshape(n, 10)

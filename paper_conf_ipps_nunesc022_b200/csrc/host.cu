@@ -2,7 +2,9 @@
 //
 // Every transaction step runs in the fused kernel (kernel.cu); the host only
 // allocates, initialises, launches and copies results.  Nothing here falls
-// back to the CPU: without an sm_100a device csmv_create fails.
+// back to the CPU: without an sm_100a device csmv_create fails.  The one
+// host-side computation is the KV preload (setup, not timed): keys
+// 0..n_keys-1 inserted serially with PUT semantics (docs/GENERATOR.md 4).
 #include <cuda_runtime.h>
 
 #include <cmath>
@@ -31,12 +33,11 @@ int set_err(int code, const char* fmt, ...) {
   return code;
 }
 
-#define CK(call)                                                                         \
-  do {                                                                                   \
-    cudaError_t e_ = (call);                                                             \
-    if (e_ != cudaSuccess)                                                               \
-      return set_err(CSMV_ECUDA, "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, \
-                     __LINE__);                                                          \
+#define CK(call)                                                                                 \
+  do {                                                                                           \
+    cudaError_t e_ = (call);                                                                     \
+    if (e_ != cudaSuccess)                                                                       \
+      return set_err(CSMV_ECUDA, "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
   } while (0)
 
 // zipf CDF (docs/GENERATOR.md section 2), built on the host in IEEE double
@@ -57,27 +58,34 @@ std::vector<uint64_t> build_zipf(uint32_t n, uint32_t theta_milli) {
 
 uint32_t nslot_for(uint32_t k) { return k <= 2 ? 2 : k <= 4 ? 4 : k <= 8 ? 8 : 16; }
 
+uint64_t umulhi(uint64_t a, uint64_t b) { return (uint64_t)(((unsigned __int128)a * b) >> 64); }
+
 }  // namespace
 
 struct csmv {
   int kind = CSMV_KIND_BANK;
-  uint64_t n_items = 0;
+  uint64_t n_items = 0;  // bank: accounts; KV: all items (3S + T)
   uint32_t K = 0, nslot = 0;
   int device = 0, sm_count = 0;
   cudaStream_t stream = nullptr;
   bool loaded = false;
-
+  // bank store
   uint64_t* d_rings = nullptr;
+  // KV store
+  uint32_t kv_S = 0, kv_A = 0, kv_T = 0, kv_keys = 0;
+  uint64_t *d_key = nullptr, *d_val = nullptr, *d_lru = nullptr, *d_clk = nullptr;
+  // shared
   uint32_t* d_lastw = nullptr;
   uint32_t* d_gts = nullptr;
   Ctl* d_ctl = nullptr;
   DevStats* d_stats = nullptr;
   uint32_t* d_done = nullptr;
   // per-client-warp message slots, sized for the full grid
-  uint32_t max_cw = 0;
+  uint32_t max_cw = 0, maxid = 2;
   uint32_t* d_req_seq = nullptr;
   ReqHdr* d_req_hdr = nullptr;
   uint32_t* d_req_ids = nullptr;
+  uint32_t* d_req_cnt = nullptr;
   Resp* d_resp = nullptr;
   // logs
   csmv_log_rec* d_log = nullptr;
@@ -95,19 +103,10 @@ struct csmv {
 };
 
 static void free_all(csmv* h) {
-  cudaFree(h->d_rings);
-  cudaFree(h->d_lastw);
-  cudaFree(h->d_gts);
-  cudaFree(h->d_ctl);
-  cudaFree(h->d_stats);
-  cudaFree(h->d_done);
-  cudaFree(h->d_req_seq);
-  cudaFree(h->d_req_hdr);
-  cudaFree(h->d_req_ids);
-  cudaFree(h->d_resp);
-  cudaFree(h->d_log);
-  cudaFree(h->d_vals);
-  cudaFree(h->d_zipf);
+  void* ps[] = {h->d_rings, h->d_key, h->d_val, h->d_lru, h->d_clk, h->d_lastw, h->d_gts, h->d_ctl,
+                h->d_stats, h->d_done, h->d_req_seq, h->d_req_hdr, h->d_req_ids, h->d_req_cnt,
+                h->d_resp, h->d_log, h->d_vals, h->d_zipf};
+  for (void* q : ps) cudaFree(q);
   if (h->ev0) cudaEventDestroy(h->ev0);
   if (h->ev1) cudaEventDestroy(h->ev1);
 }
@@ -128,11 +127,39 @@ static int device_check(int* dev, int* sms) {
   cudaDeviceProp pr;
   CK(cudaGetDeviceProperties(&pr, *dev));
   if (pr.major != 10 || pr.minor != 0)
-    return set_err(CSMV_ECUDA, "device %s is sm_%d%d; this library is built for sm_100a only",
-                   pr.name, pr.major, pr.minor);
+    return set_err(CSMV_ECUDA, "device %s is sm_%d%d; this library is built for sm_100a only", pr.name,
+                   pr.major, pr.minor);
   if (!pr.cooperativeLaunch) return set_err(CSMV_ECUDA, "device lacks cooperative launch");
   *sms = pr.multiProcessorCount;
   return CSMV_OK;
+}
+
+// allocations common to both store kinds
+static bool alloc_common(csmv* h) {
+  h->max_cw = (uint32_t)(h->sm_count - 1) * kWarps;
+  if (cudaMalloc(&h->d_lastw, h->n_items * sizeof(uint32_t)) != cudaSuccess) return false;
+  if (cudaMalloc(&h->d_gts, 64) != cudaSuccess) return false;
+  if (cudaMalloc(&h->d_ctl, sizeof(Ctl)) != cudaSuccess) return false;
+  if (cudaMalloc(&h->d_stats, sizeof(DevStats)) != cudaSuccess) return false;
+  if (cudaMalloc(&h->d_done, sizeof(uint32_t) << kDoneLog2) != cudaSuccess) return false;
+  if (cudaMalloc(&h->d_req_seq, h->max_cw * sizeof(uint32_t)) != cudaSuccess) return false;
+  if (cudaMalloc(&h->d_req_hdr, h->max_cw * sizeof(ReqHdr)) != cudaSuccess) return false;
+  if (cudaMalloc(&h->d_req_ids, (size_t)h->max_cw * h->maxid * 32 * sizeof(uint32_t)) != cudaSuccess) return false;
+  if (cudaMalloc(&h->d_req_cnt, (size_t)h->max_cw * 32 * sizeof(uint32_t)) != cudaSuccess) return false;
+  if (cudaMalloc(&h->d_resp, h->max_cw * sizeof(Resp)) != cudaSuccess) return false;
+  cudaMemset(h->d_done, 0, sizeof(uint32_t) << kDoneLog2);
+  cudaMemset(h->d_gts, 0, 64);
+  cudaMemset(h->d_lastw, 0, h->n_items * sizeof(uint32_t));
+  cudaEventCreate(&h->ev0);
+  cudaEventCreate(&h->ev1);
+  return cudaDeviceSynchronize() == cudaSuccess;
+}
+
+static csmv_t* create_fail(csmv* h, const char* what) {
+  set_err(CSMV_ENOMEM, "csmv_create: allocation of %s failed (%s)", what, cudaGetErrorString(cudaGetLastError()));
+  free_all(h);
+  delete h;
+  return nullptr;
 }
 
 csmv_t* csmv_create(uint64_t n_items, uint32_t n_versions) {
@@ -150,35 +177,40 @@ csmv_t* csmv_create(uint64_t n_items, uint32_t n_versions) {
   h->nslot = nslot_for(n_versions);
   h->device = dev;
   h->sm_count = sms;
-  h->max_cw = (uint32_t)(sms - 1) * kWarps;
-  auto fail = [&](const char* what) -> csmv_t* {
-    set_err(CSMV_ENOMEM, "csmv_create: cudaMalloc %s failed (%s)", what,
-            cudaGetErrorString(cudaGetLastError()));
-    free_all(h);
-    delete h;
-    return nullptr;
-  };
-  if (cudaMalloc(&h->d_rings, n_items * h->nslot * sizeof(uint64_t)) != cudaSuccess) return fail("rings");
-  if (cudaMalloc(&h->d_lastw, n_items * sizeof(uint32_t)) != cudaSuccess) return fail("lastw");
-  if (cudaMalloc(&h->d_gts, 64) != cudaSuccess) return fail("gts");
-  if (cudaMalloc(&h->d_ctl, sizeof(Ctl)) != cudaSuccess) return fail("ctl");
-  if (cudaMalloc(&h->d_stats, sizeof(DevStats)) != cudaSuccess) return fail("stats");
-  if (cudaMalloc(&h->d_done, sizeof(uint32_t) << kDoneLog2) != cudaSuccess) return fail("done");
-  if (cudaMalloc(&h->d_req_seq, h->max_cw * sizeof(uint32_t)) != cudaSuccess) return fail("req_seq");
-  if (cudaMalloc(&h->d_req_hdr, h->max_cw * sizeof(ReqHdr)) != cudaSuccess) return fail("req_hdr");
-  if (cudaMalloc(&h->d_req_ids, (size_t)h->max_cw * 2 * 32 * sizeof(uint32_t)) != cudaSuccess) return fail("req_ids");
-  if (cudaMalloc(&h->d_resp, h->max_cw * sizeof(Resp)) != cudaSuccess) return fail("resp");
-  cudaMemset(h->d_done, 0, sizeof(uint32_t) << kDoneLog2);
-  cudaMemset(h->d_gts, 0, 64);
-  cudaEventCreate(&h->ev0);
-  cudaEventCreate(&h->ev1);
-  if (cudaDeviceSynchronize() != cudaSuccess) return fail("init");
+  h->maxid = 2;
+  if (cudaMalloc(&h->d_rings, n_items * h->nslot * sizeof(uint64_t)) != cudaSuccess) return create_fail(h, "rings");
+  if (!alloc_common(h)) return create_fail(h, "control buffers");
   return h;
 }
 
-csmv_t* csmv_create_kv(uint64_t, uint32_t, uint32_t) {
-  set_err(CSMV_EINVAL, "csmv_create_kv: KV store not built in this version");
-  return nullptr;
+csmv_t* csmv_create_kv(uint64_t n_slots, uint32_t ways, uint32_t n_versions) {
+  g_err[0] = 0;
+  if (ways < 1 || ways > kKvMaxWays || n_slots < ways || n_slots % ways || n_slots >= (1ull << 29) ||
+      n_versions < 1 || n_versions > 16) {
+    set_err(CSMV_EINVAL, "csmv_create_kv: need 1 <= ways <= %u, n_slots a multiple of ways below 2^29, "
+                         "1 <= n_versions <= 16", kKvMaxWays);
+    return nullptr;
+  }
+  int dev = 0, sms = 0;
+  if (device_check(&dev, &sms) != CSMV_OK) return nullptr;
+  csmv* h = new csmv();
+  h->kind = CSMV_KIND_KV;
+  h->kv_S = (uint32_t)n_slots;
+  h->kv_A = ways;
+  h->kv_T = (uint32_t)(n_slots / ways);
+  h->n_items = 3ull * h->kv_S + h->kv_T;
+  h->K = n_versions;
+  h->nslot = nslot_for(n_versions);
+  h->device = dev;
+  h->sm_count = sms;
+  h->maxid = kKvMaxId;
+  const size_t S = h->kv_S, T = h->kv_T, NS = h->nslot;
+  if (cudaMalloc(&h->d_key, S * NS * 4 * 8) != cudaSuccess) return create_fail(h, "key rings");
+  if (cudaMalloc(&h->d_val, S * NS * 8 * 8) != cudaSuccess) return create_fail(h, "value rings");
+  if (cudaMalloc(&h->d_lru, S * NS * 8) != cudaSuccess) return create_fail(h, "LRU rings");
+  if (cudaMalloc(&h->d_clk, T * NS * 8) != cudaSuccess) return create_fail(h, "clock rings");
+  if (!alloc_common(h)) return create_fail(h, "control buffers");
+  return h;
 }
 
 void csmv_destroy(csmv_t* h) {
@@ -197,8 +229,9 @@ int csmv_set_stream(csmv_t* h, void* s) {
 int csmv_load(csmv_t* h, const int32_t* init, uint64_t n) {
   if (!h || !init) return set_err(CSMV_EINVAL, "csmv_load: null argument");
   if (h->kind != CSMV_KIND_BANK) return set_err(CSMV_EINVAL, "csmv_load: not a bank store");
-  if (n != h->n_items) return set_err(CSMV_EINVAL, "csmv_load: n=%llu != n_items=%llu",
-                                      (unsigned long long)n, (unsigned long long)h->n_items);
+  if (n != h->n_items)
+    return set_err(CSMV_EINVAL, "csmv_load: n=%llu != n_items=%llu", (unsigned long long)n,
+                   (unsigned long long)h->n_items);
   int32_t* d_init = nullptr;
   CK(cudaMallocAsync((void**)&d_init, n * sizeof(int32_t), h->stream));
   CK(cudaMemcpyAsync(d_init, init, n * sizeof(int32_t), cudaMemcpyHostToDevice, h->stream));
@@ -210,9 +243,71 @@ int csmv_load(csmv_t* h, const int32_t* init, uint64_t n) {
   return CSMV_OK;
 }
 
-int csmv_load_kv(csmv_t* h, uint64_t) {
-  if (!h) return set_err(CSMV_EINVAL, "null handle");
-  return set_err(CSMV_EINVAL, "csmv_load_kv: KV store not built in this version");
+static KParams kv_params(const csmv* h) {
+  KParams p;
+  memset(&p, 0, sizeof p);
+  p.kind = CSMV_KIND_KV;
+  p.K = h->K;
+  p.gts = h->d_gts;
+  p.kv_S = h->kv_S;
+  p.kv_A = h->kv_A;
+  p.kv_T = h->kv_T;
+  p.kv_key = h->d_key;
+  p.kv_val = h->d_val;
+  p.kv_lru = h->d_lru;
+  p.kv_clk = h->d_clk;
+  return p;
+}
+
+int csmv_load_kv(csmv_t* h, uint64_t n_keys) {
+  if (!h) return set_err(CSMV_EINVAL, "csmv_load_kv: null handle");
+  if (h->kind != CSMV_KIND_KV) return set_err(CSMV_EINVAL, "csmv_load_kv: not a KV store");
+  if (n_keys == 0 || n_keys >= (1ull << 32)) return set_err(CSMV_EINVAL, "csmv_load_kv: bad n_keys");
+  const uint32_t S = h->kv_S, A = h->kv_A, T = h->kv_T;
+  std::vector<uint32_t> keys((size_t)S * 4, 0), vals((size_t)S * 8, 0), lru(S, 0), clocks(T, 0);
+  // PUT semantics per key, in key order (docs/GENERATOR.md 4)
+  for (uint64_t k = 0; k < n_keys; ++k) {
+    const uint64_t a = mix64(k), b = mix64(k ^ 0x5555555555555555ull);
+    const uint32_t kk[4] = {(uint32_t)a, (uint32_t)(a >> 32), (uint32_t)b, (uint32_t)(b >> 32)};
+    const uint32_t t = (uint32_t)umulhi(mix64(k ^ 0xA5A5A5A5A5A5A5A5ull), T);
+    uint32_t victim = UINT32_MAX;
+    for (uint32_t w = 0; w < A && victim == UINT32_MAX; ++w) {
+      const uint32_t* q = &keys[((size_t)t * A + w) * 4];
+      if ((q[0] == kk[0] && q[1] == kk[1] && q[2] == kk[2] && q[3] == kk[3]) || !(q[0] | q[1] | q[2] | q[3]))
+        victim = t * A + w;
+    }
+    if (victim == UINT32_MAX) {
+      victim = t * A;
+      for (uint32_t w = 1; w < A; ++w)
+        if (lru[t * A + w] < lru[victim]) victim = t * A + w;
+    }
+    const uint32_t c = clocks[t] + 1;
+    memcpy(&keys[(size_t)victim * 4], kk, 16);
+    for (uint32_t j = 0; j < 4; ++j) {
+      const uint64_t x = mix64(((k << 2) | j) ^ 0x3C3C3C3C3C3C3C3Cull);
+      vals[(size_t)victim * 8 + 2 * j] = (uint32_t)x;
+      vals[(size_t)victim * 8 + 2 * j + 1] = (uint32_t)(x >> 32);
+    }
+    lru[victim] = c;
+    clocks[t] = c;
+  }
+  uint32_t* d = nullptr;
+  const size_t words = (size_t)S * 13 + T;
+  CK(cudaMalloc(&d, words * 4));
+  cudaError_t e = cudaMemcpy(d, keys.data(), (size_t)S * 16, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d + (size_t)S * 4, vals.data(), (size_t)S * 32, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d + (size_t)S * 12, lru.data(), (size_t)S * 4, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d + (size_t)S * 13, clocks.data(), (size_t)T * 4, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess)
+    e = launch_init_kv(kv_params(h), h->nslot, d, d + (size_t)S * 4, d + (size_t)S * 12, d + (size_t)S * 13,
+                       h->stream);
+  if (e == cudaSuccess) e = cudaMemsetAsync(h->d_lastw, 0, h->n_items * 4, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  cudaFree(d);
+  if (e != cudaSuccess) return set_err(CSMV_ECUDA, "csmv_load_kv: %s", cudaGetErrorString(e));
+  h->kv_keys = (uint32_t)n_keys;
+  h->loaded = true;
+  return CSMV_OK;
 }
 
 static int prepare_zipf(csmv* h, uint32_t n, uint32_t theta) {
@@ -231,12 +326,17 @@ static int make_gen(csmv* h, const csmv_workload* w, uint64_t seed, GenParams* g
   memset(g, 0, sizeof *g);
   g->seed = seed;
   g->upd_thresh = ((uint64_t)w->p_update_ppm << 32) / 1000000ull;
-  g->n_items = (uint32_t)h->n_items;
   g->ro_period = w->ro_period;
   g->ro_reads = w->ro_reads;
   g->amount_max = w->amount_max;
+  if (h->kind == CSMV_KIND_KV) {
+    g->n_items = w->kv_keys ? w->kv_keys : h->kv_S;  // picks range over the key space
+    g->ro_period = 0;
+  } else {
+    g->n_items = (uint32_t)h->n_items;
+  }
   if (w->dist == CSMV_DIST_ZIPF) {
-    int rc = prepare_zipf(h, (uint32_t)h->n_items, w->zipf_theta_milli);
+    int rc = prepare_zipf(h, g->n_items, w->zipf_theta_milli);
     if (rc) return rc;
     g->zipf_cdf = h->d_zipf;
   } else if (w->dist != CSMV_DIST_UNIFORM) {
@@ -248,8 +348,12 @@ static int make_gen(csmv* h, const csmv_workload* w, uint64_t seed, GenParams* g
 int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (!h || !w) return set_err(CSMV_EINVAL, "csmv_run: null argument");
   if (!h->loaded) return set_err(CSMV_ESTATE, "csmv_run: store not loaded");
-  if (w->kind != CSMV_KIND_BANK) return set_err(CSMV_EINVAL, "csmv_run: only the bank workload is built");
-  if (w->amount_max == 0) return set_err(CSMV_EINVAL, "csmv_run: amount_max must be >= 1");
+  if (w->kind != (uint32_t)h->kind) return set_err(CSMV_EINVAL, "csmv_run: workload kind does not match the store");
+  if (h->kind == CSMV_KIND_BANK && w->amount_max == 0) return set_err(CSMV_EINVAL, "csmv_run: amount_max must be >= 1");
+  if (h->kind == CSMV_KIND_KV && w->log_mode == CSMV_LOG_FULL)
+    return set_err(CSMV_EINVAL, "csmv_run: the KV workload logs digests only (use CSMV_LOG_DIGEST)");
+  if (h->kind == CSMV_KIND_KV && w->kv_ways && w->kv_ways != h->kv_A)
+    return set_err(CSMV_EINVAL, "csmv_run: kv_ways %u does not match the store's %u", w->kv_ways, h->kv_A);
   if (w->p_update_ppm > 1000000) return set_err(CSMV_EINVAL, "csmv_run: p_update_ppm > 10^6");
   if (w->log_mode > CSMV_LOG_FULL || w->publish > CSMV_PUBLISH_SERVER)
     return set_err(CSMV_EINVAL, "csmv_run: bad log_mode/publish");
@@ -283,9 +387,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   uint32_t rt_log2 = 1;
   while ((4u << rt_log2) < entries && rt_log2 < 12) ++rt_log2;
   size_t smem = server_smem_bytes(rt_log2, n_cw);
+  if (h->kind == CSMV_KIND_KV && smem < kv_client_smem_bytes()) smem = kv_client_smem_bytes();
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
   int bps = 0;
-  CK(fused_occupancy(h->nslot, smem, &bps));
+  CK(fused_occupancy(h->nslot, (uint32_t)h->kind, smem, &bps));
   if (bps < 1) return set_err(CSMV_ECUDA, "csmv_run: fused kernel cannot be resident (smem %zu)", smem);
 
   // logs
@@ -301,17 +406,25 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
     if (w->log_mode == CSMV_LOG_FULL) {
       max_vals = w->ro_reads ? w->ro_reads : (uint32_t)h->n_items;
       if (max_vals < 2) max_vals = 2;
-      uint64_t words = n_tx * (uint64_t)max_vals;
-      if (words > h->vals_cap) {
+      const uint64_t words = n_tx * (uint64_t)max_vals;
+      if (words > h->vals_cap || !h->d_vals) {
         cudaFree(h->d_vals);
         h->d_vals = nullptr;
-        CK(cudaMalloc(&h->d_vals, words * sizeof(uint32_t)));
+        CK(cudaMalloc(&h->d_vals, (words ? words : 1) * sizeof(uint32_t)));
         h->vals_cap = words;
       }
       CK(cudaMemsetAsync(h->d_vals, 0, words * sizeof(uint32_t), h->stream));
     }
   }
 
+  if (h->kind == CSMV_KIND_KV) {
+    p = [&] {
+      KParams q = kv_params(h);
+      q.gen = p.gen;
+      return q;
+    }();
+  }
+  p.kind = (uint32_t)h->kind;
   p.rings = h->d_rings;
   p.n_items = (uint32_t)h->n_items;
   p.K = h->K;
@@ -320,6 +433,8 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.req_seq = h->d_req_seq;
   p.req_hdr = h->d_req_hdr;
   p.req_ids = h->d_req_ids;
+  p.req_cnt = h->d_req_cnt;
+  p.maxid = h->maxid;
   p.resp = h->d_resp;
   p.done_ring = h->d_done;
   p.stats = h->d_stats;
@@ -370,8 +485,14 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   s.gts_final = gts1;
   s.elapsed_ns = (uint64_t)((double)ms * 1e6);
   s.ro_checksum = ds.ro_checksum;
-  s.store_bytes = h->n_items * h->nslot * sizeof(uint64_t);
-  s.store_bytes_paper = h->n_items * (4ull + 8ull * h->K);
+  if (h->kind == CSMV_KIND_KV) {
+    s.store_bytes = (uint64_t)h->kv_S * h->nslot * (32 + 64 + 8) + (uint64_t)h->kv_T * h->nslot * 8;
+    s.store_bytes_paper = (uint64_t)h->kv_S * ((4 + 20ull * h->K) + (4 + 36ull * h->K) + (4 + 8ull * h->K)) +
+                          (uint64_t)h->kv_T * (4 + 8ull * h->K);
+  } else {
+    s.store_bytes = h->n_items * h->nslot * sizeof(uint64_t);
+    s.store_bytes_paper = h->n_items * (4ull + 8ull * h->K);
+  }
   s.server_lock_cycles = ds.lock_cycles;
   s.server_busy_cycles = ds.busy_cycles;
   for (int i = 0; i < 8; ++i) s.server_phase_cycles[i] = ds.phase[i];
@@ -386,13 +507,12 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   h->last_max_vals = max_vals;
   if (ctl.error) {
     h->loaded = false;
-    return set_err(CSMV_ETIMEOUT, "csmv_run: device watchdog fired (loop %u); store state undefined",
-                   ctl.where);
+    return set_err(CSMV_ETIMEOUT, "csmv_run: device watchdog fired (loop %u); store state undefined", ctl.where);
   }
   if (s.committed_update + s.committed_ro != n_tx || gts1 != ctl.tail_final)
     return set_err(CSMV_ECUDA, "csmv_run: protocol error (committed %llu of %llu, gts %u, tail %u)",
-                   (unsigned long long)(s.committed_update + s.committed_ro),
-                   (unsigned long long)n_tx, gts1, ctl.tail_final);
+                   (unsigned long long)(s.committed_update + s.committed_ro), (unsigned long long)n_tx, gts1,
+                   ctl.tail_final);
   return CSMV_OK;
 }
 
@@ -404,10 +524,10 @@ int csmv_stats(const csmv_t* h, csmv_stats_t* out) {
 
 int csmv_get_log(const csmv_t* h, csmv_log_rec* buf, uint64_t cap, uint64_t* n_out) {
   if (!h || !buf) return set_err(CSMV_EINVAL, "csmv_get_log: null argument");
-  if (h->last_log_mode == CSMV_LOG_NONE || !h->d_log)
-    return set_err(CSMV_ESTATE, "csmv_get_log: last run had no log");
-  if (cap < h->last_n_tx) return set_err(CSMV_EOVERFLOW, "csmv_get_log: cap %llu < n_tx %llu",
-                                         (unsigned long long)cap, (unsigned long long)h->last_n_tx);
+  if (h->last_log_mode == CSMV_LOG_NONE || !h->d_log) return set_err(CSMV_ESTATE, "csmv_get_log: last run had no log");
+  if (cap < h->last_n_tx)
+    return set_err(CSMV_EOVERFLOW, "csmv_get_log: cap %llu < n_tx %llu", (unsigned long long)cap,
+                   (unsigned long long)h->last_n_tx);
   CK(cudaMemcpy(buf, h->d_log, h->last_n_tx * sizeof(csmv_log_rec), cudaMemcpyDeviceToHost));
   if (n_out) *n_out = h->last_n_tx;
   return CSMV_OK;
@@ -435,22 +555,36 @@ int csmv_dump_store(const csmv_t* h, uint64_t* out, uint64_t cap) {
   return CSMV_OK;
 }
 
-int csmv_dump_kv(const csmv_t* h, uint32_t*, uint32_t*, uint32_t*, uint32_t*) {
-  if (!h) return set_err(CSMV_EINVAL, "null handle");
-  return set_err(CSMV_EINVAL, "csmv_dump_kv: KV store not built in this version");
+int csmv_dump_kv(const csmv_t* h, uint32_t* keys, uint32_t* vals, uint32_t* lru, uint32_t* clocks) {
+  if (!h) return set_err(CSMV_EINVAL, "csmv_dump_kv: null handle");
+  if (h->kind != CSMV_KIND_KV) return set_err(CSMV_EINVAL, "csmv_dump_kv: not a KV store");
+  if (!h->loaded) return set_err(CSMV_ESTATE, "csmv_dump_kv: store not loaded");
+  const size_t S = h->kv_S, T = h->kv_T;
+  uint32_t* d = nullptr;
+  CK(cudaMalloc(&d, (S * 13 + T) * 4));
+  cudaError_t e = launch_kv_newest(kv_params(h), h->nslot, d, d + S * 4, d + S * 12, d + S * 13, h->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  if (e == cudaSuccess && keys) e = cudaMemcpy(keys, d, S * 16, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && vals) e = cudaMemcpy(vals, d + S * 4, S * 32, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && lru) e = cudaMemcpy(lru, d + S * 12, S * 4, cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && clocks) e = cudaMemcpy(clocks, d + S * 13, T * 4, cudaMemcpyDeviceToHost);
+  cudaFree(d);
+  if (e != cudaSuccess) return set_err(CSMV_ECUDA, "csmv_dump_kv: %s", cudaGetErrorString(e));
+  return CSMV_OK;
 }
 
-int csmv_gen_descs(csmv_t* h, const csmv_workload* w, uint64_t seed, uint64_t tx0, uint64_t n,
-                   uint32_t* out) {
+int csmv_gen_descs(csmv_t* h, const csmv_workload* w, uint64_t seed, uint64_t tx0, uint64_t n, uint32_t* out) {
   if (!h || !w || !out) return set_err(CSMV_EINVAL, "csmv_gen_descs: null argument");
   GenParams g;
   int rc = make_gen(h, w, seed, &g);
   if (rc) return rc;
+  const uint32_t per = h->kind == CSMV_KIND_KV ? 10 : 6;
   uint32_t* d = nullptr;
-  CK(cudaMalloc(&d, n * 6 * sizeof(uint32_t) + 4));
-  cudaError_t e = launch_gen_descs(g, tx0, n, d, h->stream);
+  CK(cudaMalloc(&d, n * per * sizeof(uint32_t) + 4));
+  cudaError_t e = h->kind == CSMV_KIND_KV ? launch_gen_kv_descs(g, tx0, n, d, h->stream)
+                                          : launch_gen_descs(g, tx0, n, d, h->stream);
   if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
-  if (e == cudaSuccess) e = cudaMemcpy(out, d, n * 6 * sizeof(uint32_t), cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess) e = cudaMemcpy(out, d, n * per * sizeof(uint32_t), cudaMemcpyDeviceToHost);
   cudaFree(d);
   if (e != cudaSuccess) return set_err(CSMV_ECUDA, "csmv_gen_descs: %s", cudaGetErrorString(e));
   return CSMV_OK;

@@ -187,6 +187,34 @@ __device__ __forceinline__ void log_commit(const KParams& p, uint64_t tx, uint32
   p.log[tx] = rec;
 }
 
+// flush per-warp counters once (no global atomics on the commit path)
+__device__ __forceinline__ void client_flush(const KParams& p, const ClientCounters& cc) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t s_upd = __reduce_add_sync(FULL, cc.c_upd), s_ro = __reduce_add_sync(FULL, cc.c_ro);
+  uint32_t s_ab[CSMV_N_ABORT][2];
+#pragma unroll
+  for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
+    s_ab[i][0] = __reduce_add_sync(FULL, cc.ab[i][0]);
+    s_ab[i][1] = __reduce_add_sync(FULL, cc.ab[i][1]);
+  }
+  uint64_t ro_ck = cc.ro_ck;
+#pragma unroll
+  for (int o = 16; o; o >>= 1) ro_ck ^= __shfl_xor_sync(FULL, ro_ck, o);
+  if (lane == 0) {
+    atomicAdd(&p.stats->committed_update, (unsigned long long)s_upd);
+    atomicAdd(&p.stats->committed_ro, (unsigned long long)s_ro);
+    for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
+      if (s_ab[i][0]) atomicAdd(&p.stats->aborts[i][0], (unsigned long long)s_ab[i][0]);
+      if (s_ab[i][1]) atomicAdd(&p.stats->aborts[i][1], (unsigned long long)s_ab[i][1]);
+    }
+    atomicAdd(&p.stats->rounds, (unsigned long long)cc.n_rounds);
+    atomicXor(&p.stats->ro_checksum, (unsigned long long)ro_ck);
+    __threadfence();
+    atomicAdd(&p.ctl->done_warps, 1u);
+  }
+}
+
 template <int NS>
 __device__ void client_warp(const KParams& p, uint64_t t_begin) {
   const uint32_t FULL = 0xFFFFFFFFu;
@@ -365,29 +393,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
     }
   }
 
-  // flush per-warp counters once (no global atomics on the commit path)
-  const uint32_t s_upd = __reduce_add_sync(FULL, cc.c_upd), s_ro = __reduce_add_sync(FULL, cc.c_ro);
-  uint32_t s_ab[CSMV_N_ABORT][2];
-#pragma unroll
-  for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
-    s_ab[i][0] = __reduce_add_sync(FULL, cc.ab[i][0]);
-    s_ab[i][1] = __reduce_add_sync(FULL, cc.ab[i][1]);
-  }
-  uint64_t ro_ck = cc.ro_ck;
-#pragma unroll
-  for (int o = 16; o; o >>= 1) ro_ck ^= __shfl_xor_sync(FULL, ro_ck, o);
-  if (lane == 0) {
-    atomicAdd(&p.stats->committed_update, (unsigned long long)s_upd);
-    atomicAdd(&p.stats->committed_ro, (unsigned long long)s_ro);
-    for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
-      if (s_ab[i][0]) atomicAdd(&p.stats->aborts[i][0], (unsigned long long)s_ab[i][0]);
-      if (s_ab[i][1]) atomicAdd(&p.stats->aborts[i][1], (unsigned long long)s_ab[i][1]);
-    }
-    atomicAdd(&p.stats->rounds, (unsigned long long)cc.n_rounds);
-    atomicXor(&p.stats->ro_checksum, (unsigned long long)ro_ck);
-    __threadfence();
-    atomicAdd(&p.ctl->done_warps, 1u);
-  }
+  client_flush(p, cc);
 }
 
 // --------------------------------------------------------------------------
@@ -756,6 +762,14 @@ __device__ void server_publisher(const KParams& p, SrvShared* sh, uint64_t t_beg
   }
 }
 
+}  // namespace csmvd
+
+#include "kv.cuh"
+#include "kv_kernels.cuh"
+
+namespace csmvd {
+
+template <int KIND>
 __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   uint64_t* rt = reinterpret_cast<uint64_t*>(smem);
   const uint32_t rt_words = (uint32_t)kRtWays << p.rt_log2;
@@ -783,7 +797,8 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   if (warp == 0) {
     server_receiver(p, last_seen, queue, qn_log2, sh, t_begin);
   } else if (warp <= p.n_workers) {
-    server_worker(p, rt, evmax, queue, qn_log2, sh, t_begin);
+    if constexpr (KIND == CSMV_KIND_KV) server_worker_generic(p, queue, qn_log2, sh, t_begin);
+    else server_worker(p, rt, evmax, queue, qn_log2, sh, t_begin);
   } else if (warp == p.n_workers + 1 && p.publish == CSMV_PUBLISH_SERVER) {
     server_publisher(p, sh, t_begin);
   }
@@ -791,11 +806,12 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   if (threadIdx.x == 0) p.ctl->tail_final = sh->tail;
 }
 
-template <int NS>
+template <int NS, int KIND>
 __global__ void __launch_bounds__(kBlock, 1) csmv_fused(const KParams p) {
   extern __shared__ __align__(16) uint8_t smem[];
   const uint64_t t_begin = globaltimer();
-  if (blockIdx.x == 0) server_cta(p, smem, t_begin);
+  if (blockIdx.x == 0) server_cta<KIND>(p, smem, t_begin);
+  else if constexpr (KIND == CSMV_KIND_KV) client_warp_kv<NS>(p, t_begin, reinterpret_cast<uint32_t*>(smem));
   else client_warp<NS>(p, t_begin);
 }
 
@@ -824,39 +840,88 @@ __global__ void gen_descs_kernel(GenParams g, uint64_t tx0, uint64_t n, uint32_t
   o[5] = d.len;
 }
 
-template <int NS>
+template <int NS, int KIND>
 static cudaError_t launch_ns(const KParams& p, uint32_t grid, size_t smem, cudaStream_t st) {
-  cudaError_t e = cudaFuncSetAttribute(csmv_fused<NS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e =
+      cudaFuncSetAttribute(csmv_fused<NS, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   void* args[] = {(void*)&p};
-  return cudaLaunchCooperativeKernel((const void*)csmv_fused<NS>, dim3(grid), dim3(kBlock), args, smem, st);
+  return cudaLaunchCooperativeKernel((const void*)csmv_fused<NS, KIND>, dim3(grid), dim3(kBlock), args, smem, st);
+}
+
+template <int KIND>
+static cudaError_t launch_kind(const KParams& p, uint32_t nslot, uint32_t grid, size_t smem, cudaStream_t st) {
+  switch (nslot) {
+    case 2: return launch_ns<2, KIND>(p, grid, smem, st);
+    case 4: return launch_ns<4, KIND>(p, grid, smem, st);
+    case 8: return launch_ns<8, KIND>(p, grid, smem, st);
+    case 16: return launch_ns<16, KIND>(p, grid, smem, st);
+  }
+  return cudaErrorInvalidValue;
 }
 
 cudaError_t launch_fused(const KParams& p, uint32_t nslot, uint32_t grid, size_t smem, cudaStream_t st) {
-  switch (nslot) {
-    case 2: return launch_ns<2>(p, grid, smem, st);
-    case 4: return launch_ns<4>(p, grid, smem, st);
-    case 8: return launch_ns<8>(p, grid, smem, st);
-    case 16: return launch_ns<16>(p, grid, smem, st);
-  }
-  return cudaErrorInvalidValue;
+  if (p.kind == CSMV_KIND_KV) return launch_kind<CSMV_KIND_KV>(p, nslot, grid, smem, st);
+  return launch_kind<CSMV_KIND_BANK>(p, nslot, grid, smem, st);
 }
 
-template <int NS>
+template <int NS, int KIND>
 static cudaError_t occ_ns(size_t smem, int* b) {
-  cudaError_t e = cudaFuncSetAttribute(csmv_fused<NS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e =
+      cudaFuncSetAttribute(csmv_fused<NS, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(b, csmv_fused<NS>, kBlock, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(b, csmv_fused<NS, KIND>, kBlock, smem);
 }
 
-cudaError_t fused_occupancy(uint32_t nslot, size_t smem, int* b) {
+cudaError_t fused_occupancy(uint32_t nslot, uint32_t kind, size_t smem, int* b) {
+  if (kind == CSMV_KIND_KV) {
+    switch (nslot) {
+      case 2: return occ_ns<2, CSMV_KIND_KV>(smem, b);
+      case 4: return occ_ns<4, CSMV_KIND_KV>(smem, b);
+      case 8: return occ_ns<8, CSMV_KIND_KV>(smem, b);
+      case 16: return occ_ns<16, CSMV_KIND_KV>(smem, b);
+    }
+    return cudaErrorInvalidValue;
+  }
   switch (nslot) {
-    case 2: return occ_ns<2>(smem, b);
-    case 4: return occ_ns<4>(smem, b);
-    case 8: return occ_ns<8>(smem, b);
-    case 16: return occ_ns<16>(smem, b);
+    case 2: return occ_ns<2, CSMV_KIND_BANK>(smem, b);
+    case 4: return occ_ns<4, CSMV_KIND_BANK>(smem, b);
+    case 8: return occ_ns<8, CSMV_KIND_BANK>(smem, b);
+    case 16: return occ_ns<16, CSMV_KIND_BANK>(smem, b);
   }
   return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_init_kv(const KParams& p, uint32_t nslot, const uint32_t* keys, const uint32_t* vals,
+                           const uint32_t* lru, const uint32_t* clocks, cudaStream_t st) {
+  const uint32_t blocks = (uint32_t)((p.kv_S + 255) / 256);
+  switch (nslot) {
+    case 2: init_kv_rings<2><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
+    case 4: init_kv_rings<4><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
+    case 8: init_kv_rings<8><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
+    case 16: init_kv_rings<16><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_kv_newest(const KParams& p, uint32_t nslot, uint32_t* keys, uint32_t* vals, uint32_t* lru,
+                             uint32_t* clocks, cudaStream_t st) {
+  const uint32_t blocks = (uint32_t)((p.kv_S + 255) / 256);
+  switch (nslot) {
+    case 2: kv_newest<2><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
+    case 4: kv_newest<4><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
+    case 8: kv_newest<8><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
+    case 16: kv_newest<16><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_gen_kv_descs(GenParams g, uint64_t tx0, uint64_t n, uint32_t* out, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  gen_kv_descs_kernel<<<(uint32_t)((n + 255) / 256), 256, 0, st>>>(g, tx0, n, out);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_init_rings(uint64_t* rings, uint32_t nslot, const int32_t* init, uint64_t n,

@@ -86,7 +86,23 @@ struct KParams {
   uint32_t combine;        // batches per critical section (1..kMaxCombine)
   uint32_t debug;
   uint64_t watchdog_ns;
+  // KV workload (kind == CSMV_KIND_KV)
+  uint32_t kind;
+  uint32_t kv_S, kv_A, kv_T;  // slots, ways, sets
+  uint64_t* kv_key;           // u64[S][NS][4]
+  uint64_t* kv_val;           // u64[S][NS][8]
+  uint64_t* kv_lru;           // u64[S][NS]
+  uint64_t* kv_clk;           // u64[T][NS]
+  uint32_t* req_cnt;          // ids per lane [n_cw][32] (generic requests)
+  uint32_t maxid;             // id rows per request slot
 };
+
+constexpr uint32_t kKvMaxWays = 16;               // KV ways supported by the device path
+constexpr uint32_t kKvMaxRs = 2 * kKvMaxWays + 1;  // keys + LRU stamps + clock
+constexpr uint32_t kKvMaxId = 2 * kKvMaxWays + 2;  // RS u WS
+
+// client smem scratch per warp (KV read/write sets of its update lanes)
+inline size_t kv_client_smem_bytes() { return (size_t)kWarps * 32 * (kKvMaxRs + 4 + 1) * 4; }
 
 // dispatch queue slots: a power of two >= n_cw
 __host__ __device__ inline uint32_t queue_log2(uint32_t n_cw) {
@@ -108,6 +124,11 @@ cudaError_t launch_fused(const KParams& p, uint32_t nslot, uint32_t grid, size_t
 cudaError_t launch_init_rings(uint64_t* rings, uint32_t nslot, const int32_t* init, uint64_t n,
                               uint32_t* gts, cudaStream_t st);
 cudaError_t launch_gen_descs(GenParams g, uint64_t tx0, uint64_t n, uint32_t* out, cudaStream_t st);
-cudaError_t fused_occupancy(uint32_t nslot, size_t smem, int* blocks_per_sm);
+cudaError_t fused_occupancy(uint32_t nslot, uint32_t kind, size_t smem, int* blocks_per_sm);
+cudaError_t launch_init_kv(const KParams& p, uint32_t nslot, const uint32_t* keys, const uint32_t* vals,
+                           const uint32_t* lru, const uint32_t* clocks, cudaStream_t st);
+cudaError_t launch_kv_newest(const KParams& p, uint32_t nslot, uint32_t* keys, uint32_t* vals, uint32_t* lru,
+                             uint32_t* clocks, cudaStream_t st);
+cudaError_t launch_gen_kv_descs(GenParams g, uint64_t tx0, uint64_t n, uint32_t* out, cudaStream_t st);
 
 }  // namespace csmvd

@@ -1,0 +1,152 @@
+// kv.cuh -- MemcachedGPU workload on the CSMV pipeline.
+//
+// The store is an A-way set-associative cache of S slots (T = S/A sets).
+// Every key (16 B), value (32 B), per-slot LRU stamp and per-set clock is a
+// versioned item (VBox) with K versions:
+//   key ring   u64[S][NS][4]   value ring u64[S][NS][8]
+//   lru ring   u64[S][NS]      clock ring u64[T][NS]
+// A version of a multi-word item stores every 4-byte word as (ts << 32 |
+// word): a reader accepts a version only if all its words carry the same ts,
+// so a version being recycled by a concurrent write-back is detected without
+// fences (a torn read shows two timestamps).  Item ids (docs/GENERATOR.md 4):
+// key i, value S+i, LRU 2S+i, clock 3S+t.
+#pragma once
+#include "kernel.cuh"
+#include "ptx.cuh"
+
+namespace csmvd {
+
+enum : int { RD_OK = 0, RD_MISS = 1, RD_NEWER = 2 };
+
+__device__ __forceinline__ void kv_key16(uint32_t k, uint32_t (&out)[4]) {
+  const uint64_t a = mix64((uint64_t)k), b = mix64((uint64_t)k ^ 0x5555555555555555ull);
+  out[0] = (uint32_t)a;
+  out[1] = (uint32_t)(a >> 32);
+  out[2] = (uint32_t)b;
+  out[3] = (uint32_t)(b >> 32);
+}
+
+__device__ __forceinline__ uint32_t kv_set(uint32_t k, uint32_t T) {
+  return (uint32_t)uniform(mix64((uint64_t)k ^ 0xA5A5A5A5A5A5A5A5ull), T);
+}
+
+struct KvTx {
+  uint32_t is_update;
+  uint32_t key;
+  uint32_t val[8];
+};
+
+__device__ __forceinline__ KvTx gen_kv(const GenParams& g, uint64_t tx) {
+  KvTx d;
+  d.is_update = (draw(g.seed, tx, 0) >> 32) < g.upd_thresh;
+  d.key = gen_pick(g, draw(g.seed, tx, 1));
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const uint64_t v = d.is_update ? draw(g.seed, tx, 4 + j) : 0ull;
+    d.val[2 * j] = (uint32_t)v;
+    d.val[2 * j + 1] = (uint32_t)(v >> 32);
+  }
+  return d;
+}
+
+__device__ __forceinline__ uint64_t dig_word(uint32_t item, uint32_t w, uint32_t word) {
+  return mix64(((uint64_t)item << 35) ^ ((uint64_t)w << 32) ^ (uint64_t)word);
+}
+
+// Read a W-word item at snapshot s.  rot: a read-only transaction (a newer
+// version is fine); otherwise any version newer than s means
+// validation must fail (RD_NEWER).
+template <int NS, int W>
+__device__ __forceinline__ int kv_read_mw(const uint64_t* ring, uint32_t K, uint32_t s, bool rot,
+                                          uint32_t (&out)[W]) {
+  uint32_t ts[NS];
+#pragma unroll
+  for (int j = 0; j < NS; ++j) ts[j] = ((uint32_t)j < K) ? (uint32_t)(ld_relaxed64(ring + j * W) >> 32) : kEmptyTs;
+  int cand = -1;
+  uint32_t cts = 0, newest = 0;
+#pragma unroll
+  for (int j = 0; j < NS; ++j) {
+    if (ts[j] == kEmptyTs) continue;
+    newest = max(newest, ts[j]);
+    if (ts[j] <= s && (cand < 0 || ts[j] > cts)) {
+      cand = j;
+      cts = ts[j];
+    }
+  }
+  if (!rot && newest > s) return RD_NEWER;
+  if (cand < 0) return RD_MISS;
+  // the payload read is the re-check: every word still tagged cts means the
+  // version was intact after the scan (oldest-first recycling)
+  if constexpr (W == 1) {
+    const uint64_t v = ld_relaxed64(ring + cand);
+    if ((uint32_t)(v >> 32) != cts) return rot ? RD_MISS : RD_NEWER;
+    out[0] = (uint32_t)v;
+  } else {
+    const Ring<W> r = ld_ring<W>(ring + cand * W);
+#pragma unroll
+    for (int w = 0; w < W; ++w) {
+      if ((uint32_t)(r.s[w] >> 32) != cts) return rot ? RD_MISS : RD_NEWER;
+      out[w] = (uint32_t)r.s[w];
+    }
+  }
+  return RD_OK;
+}
+
+// Install version (cts, data) over the first unused slot, else the oldest
+// (P:291).  The writer owns the item (WW check).
+template <int NS, int W>
+__device__ __forceinline__ void kv_write_mw(uint64_t* ring, uint32_t K, uint32_t cts, const uint32_t (&data)[W]) {
+  uint32_t ts[NS];
+#pragma unroll
+  for (int j = 0; j < NS; ++j) ts[j] = ((uint32_t)j < K) ? (uint32_t)(ld_relaxed64(ring + j * W) >> 32) : 0u;
+  int victim = -1;
+#pragma unroll
+  for (int j = 0; j < NS; ++j)
+    if ((uint32_t)j < K && victim < 0 && ts[j] == kEmptyTs) victim = j;
+  if (victim < 0) {
+    victim = 0;
+    uint32_t vts = ts[0];
+#pragma unroll
+    for (int j = 1; j < NS; ++j)
+      if ((uint32_t)j < K && ts[j] < vts) {
+        victim = j;
+        vts = ts[j];
+      }
+  }
+  uint64_t* dst = ring + victim * W;
+#pragma unroll
+  for (int w = 0; w < W; w += 4) {
+    if (W - w >= 4) {
+      asm volatile("st.relaxed.gpu.global.v4.u64 [%0], {%1,%2,%3,%4};" ::"l"(dst + w),
+                   "l"(((uint64_t)cts << 32) | data[w]), "l"(((uint64_t)cts << 32) | data[w + 1]),
+                   "l"(((uint64_t)cts << 32) | data[w + 2]), "l"(((uint64_t)cts << 32) | data[w + 3])
+                   : "memory");
+    } else {
+      st_relaxed64(dst + w, ((uint64_t)cts << 32) | data[w]);
+    }
+  }
+}
+
+// Single-word item (LRU stamp, set clock): only update transactions read them.
+template <int NS>
+__device__ __forceinline__ int kv_read_1(const uint64_t* ring, uint32_t K, uint32_t s, uint32_t& out) {
+  uint32_t o[1];
+  const int r = kv_read_mw<NS, 1>(ring, K, s, false, o);
+  out = o[0];
+  return r;
+}
+
+template <int NS>
+__device__ __forceinline__ void kv_write_1(uint64_t* ring, uint32_t K, uint32_t cts, uint32_t v) {
+  const uint32_t d[1] = {v};
+  kv_write_mw<NS, 1>(ring, K, cts, d);
+}
+
+struct KvRings {
+  uint64_t* key;
+  uint64_t* val;
+  uint64_t* lru;
+  uint64_t* clk;
+};
+
+}  // namespace csmvd

@@ -61,10 +61,13 @@ def c3(**kw) -> Config:
 
 def c4(**kw) -> Config:
     """MemcachedGPU-style KV: 4M slots / 4M keys, 16 ways (Q16, Q27), 99% GET,
-    zipf 0.99 keys, 16 B keys, 32 B values, K=4."""
+    zipf 0.99 keys, 16 B keys, 32 B values, K=4.  n_items = slots."""
     w = Workload(kind=KIND_KV, dist=DIST_ZIPF, zipf_theta_milli=990, p_update_ppm=10_000,
                  kv_ways=16, kv_keys=1 << 22, client_warps=0, log_mode=LOG_DIGEST)
-    return Config("C4", 1 << 22, 4, w, 1 << 24, 1, kv_slots=1 << 22).with_(**kw)
+    cfg = Config("C4", 1 << 22, 4, w, 1 << 24, 1, kv_slots=1 << 22).with_(**kw)
+    if "n_items" in kw and "kv_keys" not in kw:   # shrunk configs: key space = slots
+        cfg = cfg.with_(kv_keys=cfg.n_items)
+    return cfg
 
 
 C5_UPDATE = (100_000, 300_000, 500_000, 700_000, 900_000)          # Q28

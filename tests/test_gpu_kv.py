@@ -1,0 +1,97 @@
+"""GPU parity of the MemcachedGPU workload (C4) against the CPU
+oracle: preload, every GET's and PUT's digests, snapshots and CTS, the
+final store, the counters; the 1-warp deterministic schedule exactly."""
+import numpy as np
+import pytest
+
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+csmv = pytest.importorskip("paper_conf_ipps_nunesc022_b200.csmv")
+from paper_conf_ipps_nunesc022_b200 import workloads as W  # noqa: E402
+
+
+def ocfg_of(cfg):
+    w = cfg.workload
+    return oracle.kv_cfg(cfg.n_items, w.kv_ways, n_keys=w.kv_keys, n_versions=cfg.n_versions,
+                         dist=w.dist, zipf_theta_milli=w.zipf_theta_milli, p_update_ppm=w.p_update_ppm,
+                         ro_streak=w.ro_streak)
+
+
+def as_state(dump, S, A):
+    st = oracle.KvStore(S, A)
+    st.keys[:], st.vals[:], st.lru[:], st.clocks[:] = dump
+    return st
+
+
+def run(cfg):
+    w = cfg.workload
+    with csmv.KvStore(cfg.n_items, w.kv_ways, cfg.n_versions) as st:
+        st.load(w.kv_keys)
+        pre = st.dump()
+        stats = st.run(w, cfg.n_tx, cfg.seed)
+        log = st.log(cfg.n_tx) if w.log_mode else None
+        fin = st.dump()
+    return pre, stats, log, fin
+
+
+@pytest.mark.parametrize("S,A", [(1 << 12, 16), (1 << 10, 4)])
+def test_preload_parity(S, A):
+    cfg = W.c4(n_items=S, kv_ways=A, n_tx=0)
+    pre, *_ = run(cfg)
+    ref = oracle.kv_preload(ocfg_of(cfg))
+    for a, b in zip(pre, (ref.keys, ref.vals, ref.lru, ref.clocks)):
+        assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("p_update,streak,k", [(10_000, 0, 4), (10_000, 8, 4), (200_000, 4, 4),
+                                               (500_000, 0, 2), (50_000, 8, 8)])
+def test_kv_parity(p_update, streak, k):
+    cfg = W.c4(n_items=1 << 14, n_tx=1 << 17, p_update_ppm=p_update, ro_streak=streak, n_versions=k,
+               client_warps=256, server_workers=6)
+    pre, stats, log, fin = run(cfg)
+    oc = ocfg_of(cfg)
+    init = oracle.kv_preload(oc)
+    d = oracle.kv_gen(oc, cfg.seed, cfg.n_tx)
+    rep = oracle.kv_check(oc, init, d, log, final=as_state(fin, cfg.n_items, cfg.workload.kv_ways),
+                          claims=dict(committed_update=stats["committed_update"],
+                                      committed_ro=stats["committed_ro"], gts_final=stats["gts_final"],
+                                      total_aborts=stats["total_aborts"]))
+    assert rep["ok"], (rep, stats)
+    assert stats["committed_update"] == int(d["is_update"].sum())
+
+
+@pytest.mark.parametrize("streak", [0, 4])
+def test_kv_one_warp_deterministic(streak):
+    cfg = W.c4(n_items=1 << 11, kv_ways=8, n_tx=4000, p_update_ppm=300_000, client_warps=1,
+               ro_streak=streak)
+    pre, stats, log, fin = run(cfg)
+    oc = ocfg_of(cfg)
+    init = oracle.kv_preload(oc)
+    d = oracle.kv_gen(oc, cfg.seed, cfg.n_tx)
+    plog, pfin, ps = oracle.kv_predict(oc, init, d, 32)
+    bad = np.nonzero(log != plog)[0]
+    assert len(bad) == 0, (bad[:5], log[bad[:5]], plog[bad[:5]])
+    for a, b in zip(fin, (pfin.keys, pfin.vals, pfin.lru, pfin.clocks)):
+        assert np.array_equal(a, b)
+    assert stats["total_aborts"] == ps["aborts_preval"] and stats["batches"] == ps["batches"]
+
+
+def test_kv_generator_parity():
+    cfg = W.c4()
+    oc = ocfg_of(cfg)
+    od = oracle.kv_gen(oc, 99, 20_000, tx0=5)
+    with csmv.KvStore(1 << 10, 16, 4) as st:
+        gd = st.gen_descs(cfg.workload, 99, 20_000, tx0=5)
+    assert np.array_equal(gd[:, 0], od["is_update"]) and np.array_equal(gd[:, 1], od["key"])
+    assert np.array_equal(gd[:, 2:], od["val"])
+
+
+def test_kv_no_validate_is_caught():
+    cfg = W.c4(n_items=1 << 8, kv_ways=4, n_tx=1 << 14, p_update_ppm=600_000, client_warps=64,
+               debug_flags=csmv.DBG_NO_VALIDATE, dist=0)
+    pre, stats, log, fin = run(cfg)
+    oc = ocfg_of(cfg)
+    rep = oracle.kv_check(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), log)
+    assert not rep["ok"]
