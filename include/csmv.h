@@ -85,7 +85,9 @@ typedef struct csmv_workload {
     uint32_t atr_mode;         /* CSMV_ATR_* */
     uint32_t publish;          /* CSMV_PUBLISH_* */
     uint32_t ro_streak;        /* 0: one transaction per lane per round (paper); R: a lane runs up to
-                                  R read-only transactions per round until it holds an update */
+                                  R read-only transactions per round, ahead of a pending update */
+    uint32_t backoff_max;      /* 0: an aborted update retries every round (paper); B: an
+                                  update rejected by the server sits out up to B rounds */
     uint32_t log_mode;         /* CSMV_LOG_* */
     uint32_t debug_flags;      /* CSMV_DBG_* */
     uint32_t watchdog_ms;      /* 0 = default (20000) */

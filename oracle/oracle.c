@@ -337,10 +337,12 @@ out:
  * ... in order, retrying an aborted one in the next round.
  * Per round:
  *   1. s <- GTS (begin; one snapshot per warp round);
- *   2. each lane executes its transaction at s; read-only ones finish
- *      (P:69).  With ro_streak = R > 0 a lane keeps running its next
- *      read-only transactions (at most R per round) until it holds an update;
- *      with ro_streak = 0 it runs exactly one transaction per round;
+ *   2. (a) a lane whose current transaction is an update reads it at s;
+ *      (b) a lane whose current transaction is read-only runs it at s and
+ *      finishes -- with ro_streak = R > 0 it keeps running its
+ *      next read-only transactions (at most R per round) and stops at its
+ *      next update, which waits for the next round; with ro_streak = 0 it
+ *      runs exactly one transaction per round;
  *   3. client-side pre-validation: update lanes in lane order, a
  *      lane is dropped if it conflicts with an earlier kept lane
  *      (SURVEY Q5); dropped lanes abort;
@@ -366,30 +368,37 @@ int or_bank_predict(const or_bank_cfg *c, const int32_t *init, uint64_t n_tx,
         state[x] = init[x];
         vbox_init(&ring[(size_t)x * K], K, init[x]);
     }
-    uint64_t cur[32];
-    uint32_t att[32];
-    for (uint32_t l = 0; l < L; l++) { cur[l] = l; att[l] = 0; }
+    /* lane state: pending update cu (NONE = UINT64_MAX) and read cursor cr */
+    uint64_t cu[32], cr[32];
+    uint32_t att_u[32], att_r[32];
+    for (uint32_t l = 0; l < L; l++) { cu[l] = UINT64_MAX; cr[l] = l; att_u[l] = att_r[l] = 0; }
     uint32_t gts = 0;
     for (;;) {
         int any = 0;
-        for (uint32_t l = 0; l < L; l++) any |= cur[l] < n_tx;
+        for (uint32_t l = 0; l < L; l++) any |= cu[l] != UINT64_MAX || cr[l] < n_tx;
         if (!any) break;
         st->rounds++;
         uint32_t s = gts;                                   /* step 1 */
         int cand[32] = {0};
-        for (uint32_t l = 0; l < L; l++) {                  /* step 2 */
+        for (uint32_t l = 0; l < L; l++) {                  /* step 2a */
+            if (cu[l] == UINT64_MAX && cr[l] < n_tx && d[cr[l]].is_update) {
+                cu[l] = cr[l];
+                cr[l] += L;
+            }
+            if (cu[l] != UINT64_MAX) {
+                att_u[l]++;
+                cand[l] = 1;
+            }
+        }
+        for (uint32_t l = 0; l < L; l++) {                  /* step 2b */
+            if (!c->ro_streak && cu[l] != UINT64_MAX) continue;
             uint32_t n_ro = 0;
-            while (cur[l] < n_tx) {
-                uint64_t t = cur[l];
+            while (cr[l] < n_tx) {
+                uint64_t t = cr[l];
                 const or_bank_desc *T = &d[t];
-                if (T->is_update) {
-                    if (!c->ro_streak && n_ro) break;  /* one tx per round */
-                    att[l]++;
-                    cand[l] = 1;
-                    break;
-                }
+                if (T->is_update) break;  /* adopted in a later round */
                 if (c->ro_streak ? n_ro >= c->ro_streak : n_ro >= 1) break;
-                att[l]++;
+                att_r[l]++;
                 n_ro++;
                 int64_t sum = 0;
                 uint64_t dg = 0;
@@ -400,21 +409,21 @@ int or_bank_predict(const or_bank_cfg *c, const int32_t *init, uint64_t n_tx,
                     dg += dig1(x, (uint32_t)state[x]);
                 }
                 log[t].tx = (uint32_t)t; log[t].snapshot = s; log[t].cts = 0;
-                log[t].attempts = att[l]; log[t].read_digest = dg; log[t].aux = (uint64_t)sum;
+                log[t].attempts = att_r[l]; log[t].read_digest = dg; log[t].aux = (uint64_t)sum;
                 st->committed_ro++;
-                att[l] = 0;
-                cur[l] += L;
+                att_r[l] = 0;
+                cr[l] += L;
             }
         }
         int kept[32] = {0};                                 /* step 3 */
         int nk = 0;
         for (uint32_t j = 0; j < L; j++) {
             if (!cand[j]) continue;
-            const or_bank_desc *B = &d[cur[j]];
+            const or_bank_desc *B = &d[cu[j]];
             int conflict = 0;
             for (uint32_t i = 0; i < j && !conflict; i++) {
                 if (!kept[i]) continue;
-                const or_bank_desc *A = &d[cur[i]];
+                const or_bank_desc *A = &d[cu[i]];
                 /* RS = WS = {src, dst}: any shared item is a conflict */
                 conflict = A->src == B->src || A->src == B->dst ||
                            A->dst == B->src || A->dst == B->dst;
@@ -427,7 +436,7 @@ int or_bank_predict(const or_bank_cfg *c, const int32_t *init, uint64_t n_tx,
         uint32_t rank = 0;                                  /* steps 4-5 */
         for (uint32_t l = 0; l < L; l++) {
             if (!kept[l]) continue;
-            uint64_t t = cur[l];
+            uint64_t t = cu[l];
             const or_bank_desc *T = &d[t];
             uint32_t cts = s + 1 + rank++;
             int32_t vs = state[T->src], vd = state[T->dst];
@@ -438,7 +447,7 @@ int or_bank_predict(const or_bank_cfg *c, const int32_t *init, uint64_t n_tx,
             uint32_t ns = (uint32_t)vs - (uint32_t)T->amt;
             uint32_t nd = (uint32_t)vd + (uint32_t)T->amt;
             log[t].tx = (uint32_t)t; log[t].snapshot = s; log[t].cts = cts;
-            log[t].attempts = att[l];
+            log[t].attempts = att_u[l];
             log[t].read_digest = dig1(T->src, (uint32_t)vs) + dig1(T->dst, (uint32_t)vd);
             log[t].aux = dig1(T->src, ns) + dig1(T->dst, nd);
             state[T->src] = (int32_t)ns;
@@ -446,8 +455,8 @@ int or_bank_predict(const or_bank_cfg *c, const int32_t *init, uint64_t n_tx,
             vbox_install(&ring[(size_t)T->src * K], K, cts, ns);
             vbox_install(&ring[(size_t)T->dst * K], K, cts, nd);
             st->committed_update++;
-            att[l] = 0;
-            cur[l] += L;
+            att_u[l] = 0;
+            cu[l] = UINT64_MAX;
         }
         gts = s + (uint32_t)nk;                             /* P:130 */
     }

@@ -370,37 +370,47 @@ int or_kv_predict(const or_kv_cfg *c, const or_kv_state *init, uint64_t n_tx, co
     kv_effect *eff = (kv_effect *)malloc(32 * sizeof(kv_effect));
     if (!state_alloc(&g, &st) || !eff) { free(eff); state_free(&st); return OR_E_ARGS; }
     state_copy(&g, &st, init);
-    uint64_t cur[32];
-    uint32_t att[32];
-    for (uint32_t l = 0; l < L; l++) { cur[l] = l; att[l] = 0; }
+    /* lane state as or_bank_predict: pending PUT cu, read cursor cr */
+    uint64_t cu[32], cr[32];
+    uint32_t att_u[32], att_r[32];
+    for (uint32_t l = 0; l < L; l++) { cu[l] = UINT64_MAX; cr[l] = l; att_u[l] = att_r[l] = 0; }
+    kv_effect *eg = &eff[L < 32 ? L : 31];  /* scratch for GETs */
+    kv_effect get_tmp;
+    if (L == 32) eg = &get_tmp;
     uint32_t gts = 0;
     for (;;) {
         int any = 0;
-        for (uint32_t l = 0; l < L; l++) any |= cur[l] < n_tx;
+        for (uint32_t l = 0; l < L; l++) any |= cu[l] != UINT64_MAX || cr[l] < n_tx;
         if (!any) break;
         ps->rounds++;
         uint32_t s = gts;
         int cand[32] = {0};
-        for (uint32_t l = 0; l < L; l++) {
+        for (uint32_t l = 0; l < L; l++) {  /* pending PUTs read at s */
+            if (cu[l] == UINT64_MAX && cr[l] < n_tx && d[cr[l]].is_update) {
+                cu[l] = cr[l];
+                cr[l] += L;
+            }
+            if (cu[l] != UINT64_MAX) {
+                att_u[l]++;
+                cand[l] = 1;
+                kv_put(&g, &st, d[cu[l]].key, d[cu[l]].val, 0, &eff[l]);
+            }
+        }
+        for (uint32_t l = 0; l < L; l++) {  /* GETs at s */
+            if (!c->ro_streak && cu[l] != UINT64_MAX) continue;
             uint32_t n_ro = 0;
-            while (cur[l] < n_tx) {
-                uint64_t t = cur[l];
-                if (d[t].is_update) {
-                    if (!c->ro_streak && n_ro) break;
-                    att[l]++;
-                    cand[l] = 1;
-                    kv_put(&g, &st, d[t].key, d[t].val, 0, &eff[l]);  /* reads at s */
-                    break;
-                }
+            while (cr[l] < n_tx) {
+                uint64_t t = cr[l];
+                if (d[t].is_update) break;
                 if (c->ro_streak ? n_ro >= c->ro_streak : n_ro >= 1) break;
-                att[l]++;
+                att_r[l]++;
                 n_ro++;
-                kv_get(&g, &st, d[t].key, &eff[l]);
-                log[t].tx = (uint32_t)t; log[t].snapshot = s; log[t].cts = 0; log[t].attempts = att[l];
-                log[t].read_digest = eff[l].read_digest; log[t].aux = eff[l].aux;
+                kv_get(&g, &st, d[t].key, eg);
+                log[t].tx = (uint32_t)t; log[t].snapshot = s; log[t].cts = 0; log[t].attempts = att_r[l];
+                log[t].read_digest = eg->read_digest; log[t].aux = eg->aux;
                 ps->committed_ro++;
-                att[l] = 0;
-                cur[l] += L;
+                att_r[l] = 0;
+                cr[l] += L;
             }
         }
         int kept[32] = {0};
@@ -418,15 +428,15 @@ int or_kv_predict(const or_kv_cfg *c, const or_kv_state *init, uint64_t n_tx, co
         uint32_t rank = 0;
         for (uint32_t l = 0; l < L; l++) {
             if (!kept[l]) continue;
-            uint64_t t = cur[l];
+            uint64_t t = cu[l];
             uint32_t cts = s + 1 + rank++;
             /* pairwise conflict-free: each kept PUT reads what it read at s */
             kv_put(&g, &st, d[t].key, d[t].val, 1, &eff[l]);
-            log[t].tx = (uint32_t)t; log[t].snapshot = s; log[t].cts = cts; log[t].attempts = att[l];
+            log[t].tx = (uint32_t)t; log[t].snapshot = s; log[t].cts = cts; log[t].attempts = att_u[l];
             log[t].read_digest = eff[l].read_digest; log[t].aux = eff[l].aux;
             ps->committed_update++;
-            att[l] = 0;
-            cur[l] += L;
+            att_u[l] = 0;
+            cu[l] = UINT64_MAX;
         }
         gts = s + (uint32_t)nk;
     }

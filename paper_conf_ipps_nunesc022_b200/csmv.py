@@ -39,7 +39,7 @@ class _Workload(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in (
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
         "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers", "server_combine",
-        "atr_capacity", "atr_mode", "publish", "ro_streak", "log_mode", "debug_flags", "watchdog_ms")]
+        "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms")]
 
 
 class _Stats(C.Structure):
@@ -77,6 +77,7 @@ class Workload:
     atr_mode: int = ATR_HASH
     publish: int = PUBLISH_CLIENT
     ro_streak: int = 0
+    backoff_max: int = 0
     log_mode: int = LOG_NONE
     debug_flags: int = 0
     watchdog_ms: int = 0

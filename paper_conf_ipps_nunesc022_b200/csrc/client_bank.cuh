@@ -1,0 +1,215 @@
+// client_bank.cuh -- the client warp of the Bank workload.
+// Included by kernel.cu after the shared client helpers.
+//
+// Lane state: at most one pending update transaction `cu` and a read cursor
+// `cr` over the lane's own transactions (static assignment: lane l of client
+// warp w runs tx (32w + l) + k*T).  A round (one snapshot s):
+//   A  TXBegin s <- GTS; the pending update (adopting the next transaction if
+//      it is an update) reads its items at s;
+//   B  client-side pre-validation and the batch submit;
+//   C  read-only transactions at s while the batch is at the server
+//      (P:69): ro_streak = 0 -> one transaction per lane per round (the
+//      paper's model: only lanes without a pending update run one); R > 0 ->
+//      up to R of them, running ahead of a pending update, stopping at the
+//      next update;
+//   D  the response, client write-back, GTS advance.
+// An update rejected by the server may sit out `backoff` rounds
+// (backoff_max > 0); its lane keeps running read-only transactions.
+#pragma once
+
+namespace csmvd {
+
+constexpr uint64_t kNoTx = ~0ull;
+
+template <int NS>
+__device__ void client_warp(const KParams& p, uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t cw = (threadIdx.x >> 5) * p.n_client_ctas + (blockIdx.x - 1);
+  if (cw >= p.n_cw) return;
+  const uint64_t T = (uint64_t)p.n_cw * 32;
+  uint64_t cu = kNoTx;                       // pending update
+  uint64_t cr = (uint64_t)cw * 32 + lane;    // read cursor
+  uint32_t att_u = 0, att_r = 0, hold = 0, n_srv_ab = 0;
+  ClientCounters cc;
+  uint32_t round = 0;
+  uint32_t* my_ids = p.req_ids + (size_t)cw * 2 * 32;
+  const uint32_t K = p.K;
+  const uint32_t lt = lanemask_lt();
+  const uint32_t streak = p.ro_streak;
+
+  for (;;) {
+    if (!__any_sync(FULL, cu != kNoTx || cr < p.n_tx)) break;
+    ++round;
+    ++cc.n_rounds;
+    uint32_t s = 0, err = 0;
+    if (lane == 0) {
+      s = ld_acquire(p.gts);  // TXBegin: snapshot
+      err = ld_relaxed(&p.ctl->error);
+    }
+    s = __shfl_sync(FULL, s, 0);
+    if (__shfl_sync(FULL, err, 0)) break;
+
+    // ---- A: the pending update reads at s
+    int status = ST_NONE;
+    BankTx d{};
+    Ring<NS> rs{}, rd{};
+    uint32_t vs = 0, vd = 0;
+    if (cu == kNoTx && cr < p.n_tx && gen_is_update(p.gen, cr)) {
+      cu = cr;
+      cr += T;
+    }
+    if (cu != kNoTx) {
+      if (hold) {
+        --hold;
+        status = ST_ABORT;  // sitting out (backoff)
+      } else {
+        d = gen_bank(p.gen, cu);
+        ++att_u;
+        rs = ld_ring<NS>(p.rings + (size_t)d.src * NS);
+        rd = ld_ring<NS>(p.rings + (size_t)d.dst * NS);
+        const Sel qs = select_version<NS>(rs, s), qd = select_version<NS>(rd, s);
+        if (qs.newest > s || qd.newest > s) {
+          cc.abort(CSMV_AB_EARLY, true);  // a commit after s wrote it: validation must fail
+          status = ST_ABORT;
+          if (p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
+        } else if (qs.best < 0 || qd.best < 0) {
+          cc.abort(CSMV_AB_VERSION, true);
+          status = ST_ABORT;
+        } else {
+          vs = (uint32_t)slot_at<NS>(rs, qs.best);
+          vd = (uint32_t)slot_at<NS>(rd, qd.best);
+          status = ST_CAND;
+        }
+      }
+    }
+
+    // ---- B: pre-validation, greedy in lane order (RS = WS = {src, dst})
+    const uint32_t cand = __ballot_sync(FULL, status == ST_CAND);
+    uint32_t kept = cand;
+    if (!(p.debug & CSMV_DBG_NO_PREVAL)) {
+      kept = 0;
+      uint32_t rem = cand;
+      while (rem) {
+        const int i = __ffs(rem) - 1;
+        const uint32_t a = __shfl_sync(FULL, d.src, i), b = __shfl_sync(FULL, d.dst, i);
+        kept |= 1u << i;
+        const bool conf = ((rem >> lane) & 1u) && lane > (uint32_t)i &&
+                          (d.src == a || d.src == b || d.dst == a || d.dst == b);
+        rem &= ~__ballot_sync(FULL, conf) & ~(1u << i);
+      }
+    }
+    const bool mine = (kept >> lane) & 1u;
+    if (status == ST_CAND && !mine) cc.abort(CSMV_AB_PREVAL, true);
+    if (kept) {
+      if (mine) {
+        my_ids[lane] = d.src | kWriteBit;
+        my_ids[32 + lane] = d.dst | kWriteBit;
+      }
+      if (lane == 0) {
+        p.req_hdr[cw].snapshot = s;
+        p.req_hdr[cw].mask = kept;
+      }
+      __syncwarp();
+      fence_gpu();
+      if (lane == 0) st_relaxed(&p.req_seq[cw], round);
+    }
+
+    // ---- C: read-only transactions at s
+    if (streak || cu == kNoTx) {
+      uint32_t n_ro = 0;
+      while (cr < p.n_tx) {
+        const BankTx r = gen_bank(p.gen, cr);
+        if (r.is_update) break;
+        if (streak ? n_ro >= streak : n_ro >= 1) break;
+        ++att_r;
+        ++n_ro;
+        int64_t rsum;
+        uint64_t rdig;
+        if (!rot_scan<NS>(p, r.start, r.len, s, cr, rsum, rdig)) {
+          cc.abort(CSMV_AB_VERSION, false);  // retried next round
+          break;
+        }
+        if (p.log_mode) log_commit(p, cr, s, 0, att_r, rdig, (uint64_t)rsum);
+        ++cc.c_ro;
+        cc.ro_ck ^= (uint64_t)rsum;
+        cr += T;
+        att_r = 0;
+      }
+    }
+    if (!kept) continue;
+
+    // ---- D: the server's answer, write-back, GTS
+    uint32_t base = 0, cmask = 0, omask = 0;
+    {
+      uint32_t it = 0;
+      bool ok = true;
+      while (warp_ld_relaxed(&p.resp[cw].seq) != round) {
+        if ((++it & 255u) == 0) {
+          uint32_t bad = 0;
+          if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);
+          if (__shfl_sync(FULL, bad, 0)) {
+            ok = false;
+            break;
+          }
+        }
+        __nanosleep(64);
+      }
+      fence_gpu();  // acquire: response payload after its seq
+      if (ok) {
+        base = ld_relaxed(&p.resp[cw].cts_base);
+        cmask = ld_relaxed(&p.resp[cw].commit_mask);
+        omask = ld_relaxed(&p.resp[cw].overflow_mask);
+      }
+    }
+    uint32_t cts = 0;
+    if (mine) {
+      if ((cmask >> lane) & 1u) {
+        // Client-side write-back with CTS = base + rank.
+        cts = base + __popc(cmask & lt);
+        const uint32_t ns = vs - (uint32_t)d.amt, nd = vd + (uint32_t)d.amt;
+        write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
+        write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
+        if (p.log_mode) {
+          log_commit(p, cu, s, cts, att_u, dig1(d.src, vs) + dig1(d.dst, vd), dig1(d.src, ns) + dig1(d.dst, nd));
+          if (p.log_mode == CSMV_LOG_FULL && p.max_vals >= 2) {
+            p.vals[cu * p.max_vals] = vs;
+            p.vals[cu * p.max_vals + 1] = vd;
+          }
+        }
+        ++cc.c_upd;
+        cu = kNoTx;
+        att_u = 0;
+        n_srv_ab = 0;
+      } else {
+        const bool ovf = (omask >> lane) & 1u;
+        cc.abort(ovf ? CSMV_AB_OVERFLOW : CSMV_AB_CONFLICT, true);
+        if (!ovf && p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
+      }
+    }
+    const uint32_t n = __popc(cmask);
+    if (n) {
+      if (p.publish == CSMV_PUBLISH_CLIENT) {
+        // Advance GTS by n once every earlier commit is visible:
+        // spin until GTS == first CTS - 1 ("GTS 1" = GTS+1).
+        __syncwarp();
+        fence_gpu();
+        uint32_t it = 0;
+        while (warp_ld_relaxed(p.gts) != base - 1) {
+          if ((++it & 255u) == 0) {
+            uint32_t bad = 0;
+            if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 2);
+            if (__shfl_sync(FULL, bad, 0)) break;
+          }
+          __nanosleep(32);
+        }
+        if (lane == 0) st_release(p.gts, base + n - 1);  // release also orders the write-backs
+      } else if (cts) {
+        st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
+      }
+    }
+  }
+  client_flush(p, cc);
+}
+
+}  // namespace csmvd

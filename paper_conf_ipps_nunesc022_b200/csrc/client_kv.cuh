@@ -1,0 +1,301 @@
+// client_kv.cuh -- the client warp of the MemcachedGPU workload.
+// Same lane state machine and round phases as client_bank.cuh; GET is the
+// read-only transaction, PUT the update transaction (docs/GENERATOR.md 4).
+#pragma once
+
+namespace csmvd {
+
+// GET(k) at snapshot s: scan set(k), stop at the matching key (then read
+// its value) or at the first empty way; never touches LRU.
+template <int NS>
+__device__ __forceinline__ int kv_get(const KParams& p, uint32_t key, uint32_t s, uint64_t& dg, uint32_t& hit) {
+  const uint32_t K = p.K, S = p.kv_S, A = p.kv_A;
+  uint32_t gk[4];
+  kv_key16(key, gk);
+  const uint32_t gset = kv_set(key, p.kv_T);
+  dg = 0;
+  hit = 0;
+  for (uint32_t w = 0; w < A; ++w) {
+    const uint32_t slot = gset * A + w;
+    uint32_t k4[4];
+    int r = kv_read_mw<NS, 4>(p.kv_key + (size_t)slot * NS * 4, K, s, true, k4);
+    if (r != RD_OK) return r;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) dg += dig_word(slot, j, k4[j]);
+    if (k4[0] == gk[0] && k4[1] == gk[1] && k4[2] == gk[2] && k4[3] == gk[3]) {
+      uint32_t val[8];
+      r = kv_read_mw<NS, 8>(p.kv_val + (size_t)slot * NS * 8, K, s, true, val);
+      if (r != RD_OK) return r;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) dg += dig_word(S + slot, j, val[j]);
+      hit = w + 1;
+      return RD_OK;
+    }
+    if (!(k4[0] | k4[1] | k4[2] | k4[3])) return RD_OK;
+  }
+  return RD_OK;
+}
+
+template <int NS>
+__device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scratch) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t cw = wib * p.n_client_ctas + (blockIdx.x - 1);
+  if (cw >= p.n_cw) return;
+  const uint64_t T = (uint64_t)p.n_cw * 32;
+  uint64_t cu = kNoTx;
+  uint64_t cr = (uint64_t)cw * 32 + lane;
+  uint32_t att_u = 0, att_r = 0, hold = 0, n_srv_ab = 0;
+  ClientCounters cc;
+  uint32_t round = 0;
+  const uint32_t K = p.K, S = p.kv_S, A = p.kv_A, Tn = p.kv_T;
+  const uint32_t lt = lanemask_lt();
+  const uint32_t streak = p.ro_streak;
+  // per-warp smem scratch, lane-minor: RS[kKvMaxRs][32], WS[4][32], NRS[32]
+  uint32_t* RS = scratch + (size_t)wib * 32 * (kKvMaxRs + 5);
+  uint32_t* WS = RS + kKvMaxRs * 32;
+  uint32_t* NRS = WS + 4 * 32;
+  uint32_t* my_ids = p.req_ids + (size_t)cw * p.maxid * 32;
+
+  for (;;) {
+    if (!__any_sync(FULL, cu != kNoTx || cr < p.n_tx)) break;
+    ++round;
+    ++cc.n_rounds;
+    uint32_t s = 0, err = 0;
+    if (lane == 0) {
+      s = ld_acquire(p.gts);  // TXBegin
+      err = ld_relaxed(&p.ctl->error);
+    }
+    s = __shfl_sync(FULL, s, 0);
+    if (__shfl_sync(FULL, err, 0)) break;
+
+    // ---- A: the pending PUT reads at s (read-set tracked)
+    int status = ST_NONE;
+    KvTx d{};
+    uint32_t kk[4] = {0, 0, 0, 0};
+    uint32_t victim = 0, tset = 0, clk = 0, nrs = 0;
+    uint64_t rdig = 0;
+    if (cu == kNoTx && cr < p.n_tx && gen_is_update(p.gen, cr)) {
+      cu = cr;
+      cr += T;
+    }
+    if (cu != kNoTx) {
+      if (hold) {
+        --hold;
+        status = ST_ABORT;
+      } else {
+        d = gen_kv(p.gen, cu);
+        kv_key16(d.key, kk);
+        tset = kv_set(d.key, Tn);
+        ++att_u;
+        int r = RD_OK;
+        victim = 0xFFFFFFFFu;
+        for (uint32_t w = 0; w < A && victim == 0xFFFFFFFFu; ++w) {
+          const uint32_t slot = tset * A + w;
+          uint32_t key[4];
+          r = kv_read_mw<NS, 4>(p.kv_key + (size_t)slot * NS * 4, K, s, false, key);
+          if (r != RD_OK) break;
+          RS[nrs++ * 32 + lane] = slot;
+#pragma unroll
+          for (int j = 0; j < 4; ++j) rdig += dig_word(slot, j, key[j]);
+          if ((key[0] == kk[0] && key[1] == kk[1] && key[2] == kk[2] && key[3] == kk[3]) ||
+              !(key[0] | key[1] | key[2] | key[3]))
+            victim = slot;
+        }
+        if (r == RD_OK && victim == 0xFFFFFFFFu) {
+          uint32_t best = 0;
+          for (uint32_t w = 0; w < A; ++w) {
+            const uint32_t slot = tset * A + w;
+            uint32_t l;
+            r = kv_read_1<NS>(p.kv_lru + (size_t)slot * NS, K, s, l);
+            if (r != RD_OK) break;
+            RS[nrs++ * 32 + lane] = 2 * S + slot;
+            rdig += dig1(2 * S + slot, l);
+            if (w == 0 || l < best) {
+              best = l;
+              victim = slot;
+            }
+          }
+        }
+        if (r == RD_OK) {
+          r = kv_read_1<NS>(p.kv_clk + (size_t)tset * NS, K, s, clk);
+          if (r == RD_OK) {
+            RS[nrs++ * 32 + lane] = 3 * S + tset;
+            rdig += dig1(3 * S + tset, clk);
+          }
+        }
+        if (r == RD_NEWER) {
+          cc.abort(CSMV_AB_EARLY, true);
+          status = ST_ABORT;
+          if (p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
+        } else if (r == RD_MISS) {
+          cc.abort(CSMV_AB_VERSION, true);
+          status = ST_ABORT;
+        } else {
+          WS[0 * 32 + lane] = victim;
+          WS[1 * 32 + lane] = S + victim;
+          WS[2 * 32 + lane] = 2 * S + victim;
+          WS[3 * 32 + lane] = 3 * S + tset;
+          NRS[lane] = nrs;
+          status = ST_CAND;
+        }
+      }
+    }
+    __syncwarp();
+
+    // ---- B: pre-validation: lane j is dropped if WS_i n (RS_j u WS_j)
+    // or WS_j n RS_i is non-empty for an earlier kept lane i
+    const uint32_t cand = __ballot_sync(FULL, status == ST_CAND);
+    uint32_t kept = cand;
+    if (!(p.debug & CSMV_DBG_NO_PREVAL)) {
+      kept = 0;
+      uint32_t rem = cand;
+      while (rem) {
+        const int i = __ffs(rem) - 1;
+        kept |= 1u << i;
+        bool conf = false;
+        if (((rem >> lane) & 1u) && lane > (uint32_t)i) {
+          const uint32_t nrs_i = NRS[i];
+          for (int a = 0; a < 4; ++a) {
+            const uint32_t x = WS[a * 32 + i];
+            for (uint32_t b = 0; b < nrs; ++b) conf |= RS[b * 32 + lane] == x;
+            for (int b = 0; b < 4; ++b) conf |= WS[b * 32 + lane] == x;
+          }
+          for (uint32_t b = 0; b < nrs_i; ++b) {
+            const uint32_t y = RS[b * 32 + i];
+            for (int a = 0; a < 4; ++a) conf |= WS[a * 32 + lane] == y;
+          }
+        }
+        rem &= ~__ballot_sync(FULL, conf) & ~(1u << i);
+      }
+    }
+    const bool mine = (kept >> lane) & 1u;
+    if (status == ST_CAND && !mine) cc.abort(CSMV_AB_PREVAL, true);
+    if (kept && mine) {
+      // request ids: RS u WS (bit 31: in WS)
+      uint32_t n = 0;
+      for (uint32_t b = 0; b < nrs; ++b) {
+        const uint32_t x = RS[b * 32 + lane];
+        bool w = false;
+#pragma unroll
+        for (int a = 0; a < 4; ++a) w |= WS[a * 32 + lane] == x;
+        my_ids[(size_t)n++ * 32 + lane] = x | (w ? kWriteBit : 0u);
+      }
+#pragma unroll
+      for (int a = 0; a < 4; ++a) {
+        const uint32_t x = WS[a * 32 + lane];
+        bool in_rs = false;
+        for (uint32_t b = 0; b < nrs; ++b) in_rs |= RS[b * 32 + lane] == x;
+        if (!in_rs) my_ids[(size_t)n++ * 32 + lane] = x | kWriteBit;
+      }
+      p.req_cnt[(size_t)cw * 32 + lane] = n;
+    }
+    if (kept) {
+      if (lane == 0) {
+        p.req_hdr[cw].snapshot = s;
+        p.req_hdr[cw].mask = kept;
+      }
+      __syncwarp();
+      fence_gpu();
+      if (lane == 0) st_relaxed(&p.req_seq[cw], round);
+    }
+
+    // ---- C: GETs at s while the batch is at the server
+    if (streak || cu == kNoTx) {
+      uint32_t n_ro = 0;
+      while (cr < p.n_tx) {
+        const KvTx g = gen_kv(p.gen, cr);
+        if (g.is_update) break;
+        if (streak ? n_ro >= streak : n_ro >= 1) break;
+        ++att_r;
+        ++n_ro;
+        uint64_t dg;
+        uint32_t hit;
+        if (kv_get<NS>(p, g.key, s, dg, hit) != RD_OK) {
+          cc.abort(CSMV_AB_VERSION, false);  // retried next round
+          break;
+        }
+        if (p.log_mode) log_commit(p, cr, s, 0, att_r, dg, hit);
+        ++cc.c_ro;
+        cc.ro_ck ^= dg;
+        cr += T;
+        att_r = 0;
+      }
+    }
+    if (!kept) continue;
+
+    // ---- D: response, write-back, GTS
+    uint32_t base = 0, cmask = 0, omask = 0;
+    {
+      uint32_t it = 0;
+      bool ok = true;
+      while (warp_ld_relaxed(&p.resp[cw].seq) != round) {
+        if ((++it & 255u) == 0) {
+          uint32_t bad = 0;
+          if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);
+          if (__shfl_sync(FULL, bad, 0)) {
+            ok = false;
+            break;
+          }
+        }
+        __nanosleep(64);
+      }
+      fence_gpu();
+      if (ok) {
+        base = ld_relaxed(&p.resp[cw].cts_base);
+        cmask = ld_relaxed(&p.resp[cw].commit_mask);
+        omask = ld_relaxed(&p.resp[cw].overflow_mask);
+      }
+    }
+    uint32_t cts = 0;
+    if (mine) {
+      if ((cmask >> lane) & 1u) {
+        // Client-side write-back: the paper's 4 writes.
+        cts = base + __popc(cmask & lt);
+        const uint32_t cn = clk + 1;
+        kv_write_mw<NS, 4>(p.kv_key + (size_t)victim * NS * 4, K, cts, kk);
+        kv_write_mw<NS, 8>(p.kv_val + (size_t)victim * NS * 8, K, cts, d.val);
+        kv_write_1<NS>(p.kv_lru + (size_t)victim * NS, K, cts, cn);
+        kv_write_1<NS>(p.kv_clk + (size_t)tset * NS, K, cts, cn);
+        if (p.log_mode) {
+          uint64_t wd = dig1(2 * S + victim, cn) + dig1(3 * S + tset, cn);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) wd += dig_word(victim, j, kk[j]);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) wd += dig_word(S + victim, j, d.val[j]);
+          log_commit(p, cu, s, cts, att_u, rdig, wd);
+        }
+        ++cc.c_upd;
+        cu = kNoTx;
+        att_u = 0;
+        n_srv_ab = 0;
+      } else {
+        const bool ovf = (omask >> lane) & 1u;
+        cc.abort(ovf ? CSMV_AB_OVERFLOW : CSMV_AB_CONFLICT, true);
+        if (!ovf && p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
+      }
+    }
+    const uint32_t n = __popc(cmask);
+    if (n) {
+      if (p.publish == CSMV_PUBLISH_CLIENT) {
+        __syncwarp();
+        fence_gpu();
+        uint32_t it = 0;
+        while (warp_ld_relaxed(p.gts) != base - 1) {
+          if ((++it & 255u) == 0) {
+            uint32_t bad = 0;
+            if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 2);
+            if (__shfl_sync(FULL, bad, 0)) break;
+          }
+          __nanosleep(32);
+        }
+        if (lane == 0) st_release(p.gts, base + n - 1);
+      } else if (cts) {
+        st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
+      }
+    }
+  }
+  client_flush(p, cc);
+}
+
+}  // namespace csmvd

@@ -451,6 +451,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.publish = w->publish;
   p.ro_streak = w->ro_streak;
   p.combine = w->server_combine ? w->server_combine : 1u;
+  p.backoff_max = w->backoff_max;
   p.debug = w->debug_flags;
   p.watchdog_ns = (uint64_t)(w->watchdog_ms ? w->watchdog_ms : 20000u) * 1000000ull;
 

@@ -215,186 +215,11 @@ __device__ __forceinline__ void client_flush(const KParams& p, const ClientCount
   }
 }
 
-template <int NS>
-__device__ void client_warp(const KParams& p, uint64_t t_begin) {
-  const uint32_t FULL = 0xFFFFFFFFu;
-  const uint32_t lane = threadIdx.x & 31;
-  const uint32_t cw = (threadIdx.x >> 5) * p.n_client_ctas + (blockIdx.x - 1);
-  if (cw >= p.n_cw) return;
-  const uint64_t T = (uint64_t)p.n_cw * 32;
-  uint64_t cur = (uint64_t)cw * 32 + lane;  // static assignment: tx = lane + k*T
-  uint32_t att = 0;
-  ClientCounters cc;
-  uint32_t round = 0;
-  uint32_t* my_ids = p.req_ids + (size_t)cw * 2 * 32;
-  const uint32_t K = p.K;
-  const uint32_t lt = lanemask_lt();
-  // ro_streak = 0: each lane runs one transaction per round (the paper's
-  // one-transaction-per-thread model).  ro_streak = R > 0: a lane runs up to
-  // R read-only transactions at the round's snapshot until it holds an
-  // update, so batches carry more updates.
-  const uint32_t streak = p.ro_streak;
+}  // namespace csmvd
 
-  for (;;) {
-    if (!__any_sync(FULL, cur < p.n_tx)) break;
-    ++round;
-    ++cc.n_rounds;
-    uint32_t s = 0, err = 0;
-    if (lane == 0) {
-      s = ld_acquire(p.gts);  // TXBegin: snapshot
-      err = ld_relaxed(&p.ctl->error);
-    }
-    s = __shfl_sync(FULL, s, 0);
-    if (__shfl_sync(FULL, err, 0)) break;
+#include "client_bank.cuh"
 
-    int status = ST_NONE;
-    BankTx d{};
-    Ring<NS> rs{}, rd{};
-    uint32_t vs = 0, vd = 0;
-    uint32_t n_ro = 0;
-    while (cur < p.n_tx) {
-      d = gen_bank(p.gen, cur);
-      if (!d.is_update) {
-        // Read-only transaction: reads at s, no read-set, no commit.
-        if (streak ? n_ro >= streak : n_ro >= 1) break;
-        ++att;
-        ++n_ro;
-        int64_t rsum;
-        uint64_t rdig;
-        if (!rot_scan<NS>(p, d.start, d.len, s, cur, rsum, rdig)) {
-          cc.abort(CSMV_AB_VERSION, false);  // retried next round
-          status = ST_ABORT;
-          break;
-        }
-        if (p.log_mode) log_commit(p, cur, s, 0, att, rdig, (uint64_t)rsum);
-        ++cc.c_ro;
-        cc.ro_ck ^= (uint64_t)rsum;
-        cur += T;
-        att = 0;
-        continue;
-      }
-      if (!streak && n_ro) break;  // paper mode: one transaction per round
-      ++att;
-      rs = ld_ring<NS>(p.rings + (size_t)d.src * NS);
-      rd = ld_ring<NS>(p.rings + (size_t)d.dst * NS);
-      const Sel qs = select_version<NS>(rs, s), qd = select_version<NS>(rd, s);
-      if (qs.newest > s || qd.newest > s) {
-        cc.abort(CSMV_AB_EARLY, true);  // a commit after s wrote it: validation must fail
-        status = ST_ABORT;
-      } else if (qs.best < 0 || qd.best < 0) {
-        cc.abort(CSMV_AB_VERSION, true);
-        status = ST_ABORT;
-      } else {
-        vs = (uint32_t)slot_at<NS>(rs, qs.best);
-        vd = (uint32_t)slot_at<NS>(rd, qd.best);
-        status = ST_CAND;
-      }
-      break;
-    }
-
-    // Client-side pre-validation: greedy in lane order, a lane is
-    // dropped if it shares an item with an earlier kept lane (RS = WS).
-    const uint32_t cand = __ballot_sync(FULL, status == ST_CAND);
-    uint32_t kept = cand;
-    if (!(p.debug & CSMV_DBG_NO_PREVAL)) {
-      kept = 0;
-      uint32_t rem = cand;
-      while (rem) {
-        const int i = __ffs(rem) - 1;
-        const uint32_t a = __shfl_sync(FULL, d.src, i), b = __shfl_sync(FULL, d.dst, i);
-        kept |= 1u << i;
-        const bool conf = ((rem >> lane) & 1u) && lane > (uint32_t)i &&
-                          (d.src == a || d.src == b || d.dst == a || d.dst == b);
-        rem &= ~__ballot_sync(FULL, conf) & ~(1u << i);
-      }
-    }
-    const bool mine = (kept >> lane) & 1u;
-    if (status == ST_CAND && !mine) cc.abort(CSMV_AB_PREVAL, true);
-    if (!kept) continue;
-
-    // Batch submit: ids, header, then the doorbell.
-    if (mine) {
-      my_ids[lane] = d.src | kWriteBit;
-      my_ids[32 + lane] = d.dst | kWriteBit;
-    }
-    if (lane == 0) {
-      p.req_hdr[cw].snapshot = s;
-      p.req_hdr[cw].mask = kept;
-    }
-    __syncwarp();
-    fence_gpu();
-    uint32_t base = 0, cmask = 0, omask = 0;
-    if (lane == 0) st_relaxed(&p.req_seq[cw], round);
-    {
-      // convergent wait on the response
-      uint32_t it = 0;
-      bool ok = true;
-      while (warp_ld_relaxed(&p.resp[cw].seq) != round) {
-        if ((++it & 255u) == 0) {
-          uint32_t bad = 0;
-          if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);
-          if (__shfl_sync(FULL, bad, 0)) {
-            ok = false;
-            break;
-          }
-        }
-        __nanosleep(64);
-      }
-      fence_gpu();  // acquire: response payload after its seq
-      if (ok) {
-        base = ld_relaxed(&p.resp[cw].cts_base);
-        cmask = ld_relaxed(&p.resp[cw].commit_mask);
-        omask = ld_relaxed(&p.resp[cw].overflow_mask);
-      }
-    }
-    uint32_t cts = 0;
-    if (mine) {
-      if ((cmask >> lane) & 1u) {
-        // Client-side write-back with CTS = base + rank.
-        cts = base + __popc(cmask & lt);
-        const uint32_t ns = vs - (uint32_t)d.amt, nd = vd + (uint32_t)d.amt;
-        write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
-        write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
-        if (p.log_mode) {
-          log_commit(p, cur, s, cts, att, dig1(d.src, vs) + dig1(d.dst, vd),
-                     dig1(d.src, ns) + dig1(d.dst, nd));
-          if (p.log_mode == CSMV_LOG_FULL && p.max_vals >= 2) {
-            p.vals[cur * p.max_vals] = vs;
-            p.vals[cur * p.max_vals + 1] = vd;
-          }
-        }
-        ++cc.c_upd;
-        cur += T;
-        att = 0;
-      } else {
-        cc.abort(((omask >> lane) & 1u) ? CSMV_AB_OVERFLOW : CSMV_AB_CONFLICT, true);
-      }
-    }
-    const uint32_t n = __popc(cmask);
-    if (n) {
-      if (p.publish == CSMV_PUBLISH_CLIENT) {
-        // Advance GTS by n once every earlier commit is visible:
-        // spin until GTS == first CTS - 1 ("GTS 1" = GTS+1).
-        __syncwarp();
-        fence_gpu();
-        uint32_t it = 0;
-        while (warp_ld_relaxed(p.gts) != base - 1) {
-          if ((++it & 255u) == 0) {
-            uint32_t bad = 0;
-            if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 2);
-            if (__shfl_sync(FULL, bad, 0)) break;
-          }
-          __nanosleep(32);
-        }
-        if (lane == 0) st_release(p.gts, base + n - 1);  // release also orders the write-backs
-      } else if (cts) {
-        st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
-      }
-    }
-  }
-
-  client_flush(p, cc);
-}
+namespace csmvd {
 
 // --------------------------------------------------------------------------
 // Server CTA

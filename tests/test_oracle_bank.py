@@ -232,15 +232,18 @@ def test_table_v_memory(golden_dir):
 
 @pytest.mark.parametrize("streak,expect,rounds,batches,preval", [
     # (tx: (snapshot, cts, attempts)) hand-traced, see docstring
-    (4, {0: (0, 0, 1), 2: (0, 0, 1), 4: (0, 1, 1), 1: (1, 2, 2), 3: (2, 3, 1), 5: (3, 0, 1)}, 4, 3, 1),
+    (4, {0: (0, 0, 1), 2: (0, 0, 1), 1: (0, 1, 1), 4: (1, 2, 1), 3: (1, 3, 1), 5: (1, 0, 1)}, 2, 2, 0),
     (0, {0: (0, 0, 1), 1: (0, 1, 1), 2: (1, 0, 1), 3: (1, 2, 1), 4: (2, 3, 1), 5: (2, 0, 1)}, 3, 3, 0),
 ])
 def test_ro_streak_hand_trace(streak, expect, rounds, batches, preval):
     """Two lanes; lane0 runs tx 0,2,4 and lane1 tx 1,3,5 (static assignment).
     tx0, tx2, tx5 are read-only, tx1 = 1->2, tx3 = 2->3, tx4 = 0->1.
-    streak 4: round 1 (s=0) lane0 runs ROTs 0 and 2 and holds tx4, lane1 holds
-    tx1; tx4 (items 0,1) is kept, tx1 (items 1,2) loses pre-validation; round 2
-    commits tx1, round 3 tx3, round 4 the ROT tx5 at s=3.
+    A round reads the pending updates first, then runs read-only
+    transactions (with ro_streak > 0 a lane runs ahead of its pending update).
+    streak 4: round 1 (s=0) lane1's tx1 commits (CTS 1) while lane0 runs ROTs
+    0 and 2 and stops at tx4; round 2 (s=1) tx4 (items 0,1) and tx3 (items
+    2,3) are disjoint and commit as one batch (CTS 2, 3) while lane1 runs
+    the ROT tx5 ahead of its pending tx3, at s=1.
     streak 0 (one tx per lane per round): rounds (tx0,tx1), (tx2,tx3), (tx4,tx5)."""
     cfg = oracle.bank_cfg(4, 4, ro_reads=2, ro_streak=streak)
     descs = R.desc_array([R.rot(0, 2), R.transfer(1, 2, 5), R.rot(1, 2), R.transfer(2, 3, 5),

@@ -20,8 +20,13 @@ def main(argv):
         else:
             kw[k] = int(v)
     cfg = workloads.PRESETS[name](**kw)
-    with csmv.Store(cfg.n_items, cfg.n_versions) as st:
+    if cfg.workload.kind == csmv.KIND_KV:
+        st = csmv.KvStore(cfg.n_items, cfg.workload.kv_ways, cfg.n_versions)
+        st.load(cfg.workload.kv_keys)
+    else:
+        st = csmv.Store(cfg.n_items, cfg.n_versions)
         st.load(cfg.init_values())
+    with st:
         for r in range(reps):
             t = time.time()
             s = st.run(cfg.workload, cfg.n_tx, cfg.seed + r)
