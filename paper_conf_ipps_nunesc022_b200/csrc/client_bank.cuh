@@ -25,7 +25,7 @@ template <int NS>
 __device__ void client_warp(const KParams& p, uint64_t t_begin) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
-  const uint32_t cw = (threadIdx.x >> 5) * p.n_client_ctas + (blockIdx.x - 1);
+  const uint32_t cw = (threadIdx.x >> 5) * p.n_client_ctas + (blockIdx.x - p.n_server_ctas);
   if (cw >= p.n_cw) return;
   const uint64_t T = (uint64_t)p.n_cw * 32;
   uint64_t cu = kNoTx;                       // pending update

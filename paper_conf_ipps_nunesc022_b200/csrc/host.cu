@@ -357,7 +357,6 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (w->p_update_ppm > 1000000) return set_err(CSMV_EINVAL, "csmv_run: p_update_ppm > 10^6");
   if (w->log_mode > CSMV_LOG_FULL || w->publish > CSMV_PUBLISH_SERVER)
     return set_err(CSMV_EINVAL, "csmv_run: bad log_mode/publish");
-  if (w->server != CSMV_SERVER_CTA) return set_err(CSMV_EINVAL, "csmv_run: cluster server not built yet");
   if (w->atr_mode != CSMV_ATR_HASH) return set_err(CSMV_EINVAL, "csmv_run: ATR list mode not built yet");
   if (n_tx >= (1ull << 32)) return set_err(CSMV_EINVAL, "csmv_run: n_tx must be < 2^32");
 
@@ -372,26 +371,46 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   int rc = make_gen(h, w, seed, &p.gen);
   if (rc) return rc;
 
-  // grid: CTA 0 = server, CTAs 1..C = clients, warps spread round-robin
-  uint32_t n_cw = w->client_warps ? w->client_warps : h->max_cw;
-  if (n_cw > h->max_cw) n_cw = h->max_cw;
-  if (n_cw == 0) return set_err(CSMV_EINVAL, "csmv_run: no client warps");
-  uint32_t n_ctas = (uint32_t)h->sm_count - 1;
-  if (n_cw < n_ctas) n_ctas = n_cw;
+  // server: one CTA or a thread-block cluster of C CTAs (DSMEM)
+  uint32_t n_srv = 1, clog2 = 0;
+  if (w->server == CSMV_SERVER_CLUSTER) {
+    n_srv = w->cluster_size ? w->cluster_size : 16u;
+    if (n_srv < 2 || n_srv > 16 || (n_srv & (n_srv - 1)))
+      return set_err(CSMV_EINVAL, "csmv_run: cluster_size must be 2, 4, 8 or 16");
+    while ((1u << clog2) < n_srv) ++clog2;
+  } else if (w->server != CSMV_SERVER_CTA) {
+    return set_err(CSMV_EINVAL, "csmv_run: unknown server kind %u", w->server);
+  }
   // server CTA: warp 0 receiver, warps 1..n_workers workers, last warp publisher
   uint32_t n_workers = w->server_workers ? w->server_workers : 4u;
   if (n_workers > kWarps - 2) n_workers = kWarps - 2;
+  uint32_t n_cw = w->client_warps ? w->client_warps : h->max_cw;
+  if (n_cw > h->max_cw) n_cw = h->max_cw;
+  if (n_cw == 0) return set_err(CSMV_EINVAL, "csmv_run: no client warps");
 
-  // recent-commit table: 4 entries per bucket (default 16384 entries, 144 KB)
-  uint32_t entries = w->atr_capacity ? w->atr_capacity : 16384u;
-  uint32_t rt_log2 = 1;
-  while ((4u << rt_log2) < entries && rt_log2 < 12) ++rt_log2;
-  size_t smem = server_smem_bytes(rt_log2, n_cw);
+  // recent-commit table: 4 entries per bucket, striped over the server CTAs
+  // (default 16384 entries = 144 KB per server CTA)
+  uint32_t entries = w->atr_capacity ? w->atr_capacity : 16384u * n_srv;
+  uint32_t rt_log2 = clog2 + 1;
+  while ((4u << rt_log2) < entries && rt_log2 < 12 + clog2) ++rt_log2;
+  const uint32_t per_srv = (n_cw + n_srv - 1) / n_srv;
+  size_t smem = server_smem_bytes(rt_log2 - clog2, per_srv);
   if (h->kind == CSMV_KIND_KV && smem < kv_client_smem_bytes()) smem = kv_client_smem_bytes();
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
-  int bps = 0;
-  CK(fused_occupancy(h->nslot, (uint32_t)h->kind, smem, &bps));
-  if (bps < 1) return set_err(CSMV_ECUDA, "csmv_run: fused kernel cannot be resident (smem %zu)", smem);
+
+  // grid: server CTAs first, then client CTAs (client warps spread round-robin)
+  p.kind = (uint32_t)h->kind;
+  p.n_server_ctas = n_srv;
+  int cap = 0;
+  CK(fused_capacity(p, h->nslot, smem, &cap));
+  if (cap < (int)n_srv + (int)n_srv)
+    return set_err(CSMV_ECUDA, "csmv_run: fused kernel cannot be resident (smem %zu, %d CTAs)", smem, cap);
+  uint32_t max_client_ctas = (uint32_t)cap - n_srv;
+  if (max_client_ctas > (uint32_t)h->sm_count - n_srv) max_client_ctas = (uint32_t)h->sm_count - n_srv;
+  if (n_cw > max_client_ctas * kWarps) n_cw = max_client_ctas * kWarps;
+  uint32_t n_ctas = n_cw < max_client_ctas ? n_cw : max_client_ctas;
+  if (n_srv > 1) n_ctas = (n_ctas + n_srv - 1) / n_srv * n_srv;  // grid a multiple of the cluster
+  if (n_ctas > max_client_ctas) n_ctas = max_client_ctas / n_srv * n_srv;
 
   // logs
   uint32_t max_vals = 0;
@@ -445,6 +464,8 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.n_tx = n_tx;
   p.n_cw = n_cw;
   p.n_client_ctas = n_ctas;
+  p.n_server_ctas = n_srv;
+  p.clog2 = clog2;
   p.n_workers = n_workers;
   p.rt_log2 = rt_log2;
   p.lastw = h->d_lastw;
@@ -460,7 +481,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   CK(cudaMemsetAsync(h->d_req_seq, 0, n_cw * sizeof(uint32_t), h->stream));
   CK(cudaMemsetAsync(h->d_resp, 0, n_cw * sizeof(Resp), h->stream));
   CK(cudaEventRecord(h->ev0, h->stream));
-  CK(launch_fused(p, h->nslot, 1 + n_ctas, smem, h->stream));
+  CK(launch_fused(p, h->nslot, n_srv + n_ctas, smem, h->stream));
   CK(cudaEventRecord(h->ev1, h->stream));
   CK(cudaStreamSynchronize(h->stream));
 
@@ -498,7 +519,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   s.server_busy_cycles = ds.busy_cycles;
   for (int i = 0; i < 8; ++i) s.server_phase_cycles[i] = ds.phase[i];
   s.client_warps = n_cw;
-  s.server_ctas = 1;
+  s.server_ctas = n_srv;
   s.server_workers = n_workers;
   s.atr_entries = 4u << rt_log2;
   s.sm_count = (uint32_t)h->sm_count;

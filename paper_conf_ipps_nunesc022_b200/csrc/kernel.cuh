@@ -77,9 +77,11 @@ struct KParams {
   GenParams gen;
   uint64_t n_tx;
   uint32_t n_cw;           // active client warps
-  uint32_t n_client_ctas;  // CTAs 1..n_client_ctas host clients
+  uint32_t n_client_ctas;  // CTAs n_server_ctas.. host clients
+  uint32_t n_server_ctas;  // 1, or the cluster size of a cluster server
+  uint32_t clog2;          // log2(n_server_ctas)
   uint32_t n_workers;      // server worker warps
-  uint32_t rt_log2;        // recent-commit table buckets (4 ways, 32 B each, + evmax)
+  uint32_t rt_log2;        // recent-commit table buckets, all server CTAs (4 ways, 32 B each, + evmax)
   uint32_t* lastw;         // per-item CTS of the last committed write
   uint32_t publish;
   uint32_t ro_streak;      // read-only transactions a lane may run per round (0 = one tx per round)
@@ -114,8 +116,9 @@ __host__ __device__ inline uint32_t queue_log2(uint32_t n_cw) {
 
 // smem the server CTA needs (every CTA of the fused grid gets the same):
 // recent-commit table, dispatch queue, receiver's last-seen doorbells, control words
-inline size_t server_smem_bytes(uint32_t rt_log2, uint32_t n_cw) {
-  return ((size_t)(32 + 4) << rt_log2) + ((size_t)8 << queue_log2(n_cw)) +
+// (per server CTA: its stripe of 2^local_log2 buckets and its slice of n_cw)
+inline size_t server_smem_bytes(uint32_t local_log2, uint32_t n_cw) {
+  return ((size_t)(32 + 4) << local_log2) + ((size_t)8 << queue_log2(n_cw)) +
          (((size_t)n_cw + 31) / 32 * 32) * 4 + 64;
 }
 
@@ -125,7 +128,9 @@ cudaError_t launch_fused(const KParams& p, uint32_t nslot, uint32_t grid, size_t
 cudaError_t launch_init_rings(uint64_t* rings, uint32_t nslot, const int32_t* init, uint64_t n,
                               uint32_t* gts, cudaStream_t st);
 cudaError_t launch_gen_descs(GenParams g, uint64_t tx0, uint64_t n, uint32_t* out, cudaStream_t st);
-cudaError_t fused_occupancy(uint32_t nslot, uint32_t kind, size_t smem, int* blocks_per_sm);
+// co-resident CTAs of the fused kernel for this configuration (server CTAs
+// included; a multiple of the cluster size for a cluster server)
+cudaError_t fused_capacity(const KParams& p, uint32_t nslot, size_t smem, int* ctas);
 cudaError_t launch_init_kv(const KParams& p, uint32_t nslot, const uint32_t* keys, const uint32_t* vals,
                            const uint32_t* lru, const uint32_t* clocks, cudaStream_t st);
 cudaError_t launch_kv_newest(const KParams& p, uint32_t nslot, uint32_t* keys, uint32_t* vals, uint32_t* lru,

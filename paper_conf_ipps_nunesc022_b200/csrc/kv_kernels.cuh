@@ -19,111 +19,6 @@ namespace csmvd {
 
 namespace csmvd {
 
-// Generic server worker (variable-length read/write sets): one batch per
-// critical section.  Validation reads lastw inside the critical section, so
-// it covers every commit up to the current tail exactly.
-__device__ void server_worker_generic(const KParams& p, uint64_t* queue, uint32_t qn_log2, SrvShared* sh,
-                                      uint64_t t_begin) {
-  const uint32_t FULL = 0xFFFFFFFFu;
-  const uint32_t lane = threadIdx.x & 31;
-  const uint32_t lt = lanemask_lt();
-  const uint32_t qmask = (1u << qn_log2) - 1;
-  const uint32_t dmask = (1u << kDoneLog2) - 1;
-  unsigned long long busy = 0, locked = 0, batches = 0;
-  for (;;) {
-    uint32_t slot = 0;
-    if (lane == 0) slot = atomicAdd(&sh->q_head, 1u);
-    slot = __shfl_sync(FULL, slot, 0);
-    uint64_t ent;
-    bool quit = false;
-    for (;;) {
-      ent = *(volatile uint64_t*)&queue[slot & qmask];
-      if ((uint32_t)(ent >> 32) == (slot >> qn_log2) + 1) break;
-      if (*(volatile uint32_t*)&sh->exit) {
-        quit = true;
-        break;
-      }
-      __nanosleep(64);
-    }
-    if (quit) break;
-    const uint32_t cw = (uint32_t)ent;
-    const long long t0 = clock64();
-    const uint32_t sq = ld_relaxed(p.req_seq + cw);
-    fence_gpu();
-    const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
-    const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
-    const bool mine = (mask >> lane) & 1u;
-    const uint32_t cnt = mine ? ld_relaxed(p.req_cnt + (size_t)cw * 32 + lane) : 0u;
-    uint32_t ids[kKvMaxId];
-#pragma unroll
-    for (uint32_t k = 0; k < kKvMaxId; ++k)
-      ids[k] = (k < cnt) ? ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + k) * 32 + lane) : 0u;
-    uint32_t x = s;
-#pragma unroll
-    for (uint32_t k = 0; k < kKvMaxId; ++k) x ^= ids[k];
-    if (__ballot_sync(FULL, x == 0x12345679u) == FULL) __nanosleep(1);
-    // ---- critical section
-    uint32_t ticket = 0;
-    if (lane == 0) ticket = atomicAdd(&sh->next_ticket, 1u);
-    ticket = __shfl_sync(FULL, ticket, 0);
-    while (*(volatile uint32_t*)&sh->now_serving != ticket) __nanosleep(16);
-    __syncwarp();
-    fence_cta();
-    const long long t1 = clock64();
-    const uint32_t t0c = *(volatile uint32_t*)&sh->tail;
-    uint32_t lw[kKvMaxId];
-#pragma unroll
-    for (uint32_t k = 0; k < kKvMaxId; ++k) lw[k] = (k < cnt) ? ld_relaxed(p.lastw + (ids[k] & ~kWriteBit)) : 0u;
-    bool conflict = false;
-#pragma unroll
-    for (uint32_t k = 0; k < kKvMaxId; ++k) conflict |= lw[k] > s;
-    if (p.debug & CSMV_DBG_NO_VALIDATE) conflict = false;
-    const bool commit = mine && !conflict;
-    const uint32_t cm = __ballot_sync(FULL, commit);
-    const uint32_t n = __popc(cm);
-    const uint32_t cts = t0c + 1 + __popc(cm & lt);
-    if (p.publish == CSMV_PUBLISH_SERVER && n) {
-      if (lane == 0) {
-        uint32_t it = 0;
-        while (t0c + n > sh->gts_seen + dmask) {
-          sh->gts_seen = ld_relaxed(p.gts);
-          if ((++it & 255u) == 0 && watchdog(p, t_begin, 4)) break;
-        }
-      }
-      __syncwarp();
-    }
-    if (commit) {
-#pragma unroll
-      for (uint32_t k = 0; k < kKvMaxId; ++k)
-        if (k < cnt && (ids[k] & kWriteBit)) p.lastw[ids[k] & ~kWriteBit] = cts;
-    }
-    __syncwarp();
-    fence_cta();
-    if (lane == 0) {
-      sh->tail = t0c + n;
-      fence_cta();
-      *(volatile uint32_t*)&sh->now_serving = ticket + 1;
-    }
-    const long long t2 = clock64();
-    if (lane == 0) {
-      st_relaxed(&p.resp[cw].cts_base, t0c + 1);
-      st_relaxed(&p.resp[cw].commit_mask, cm);
-      st_relaxed(&p.resp[cw].overflow_mask, 0u);
-      st_release(&p.resp[cw].seq, sq);
-    }
-    __syncwarp();
-    busy += (unsigned long long)(clock64() - t0);
-    locked += (unsigned long long)(t2 - t1);
-    ++batches;
-  }
-  if (lane == 0) {
-    atomicAdd(&p.stats->batches, batches);
-    atomicAdd(&p.stats->groups, batches);
-    atomicAdd(&p.stats->busy_cycles, busy);
-    atomicAdd(&p.stats->lock_cycles, locked);
-  }
-}
-
 // ---- setup and dump kernels
 template <int NS>
 __global__ void init_kv_rings(KParams p, const uint32_t* keys, const uint32_t* vals, const uint32_t* lru,

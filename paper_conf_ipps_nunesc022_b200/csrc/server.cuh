@@ -1,0 +1,574 @@
+// server.cuh -- the commit server.
+//
+// Single-CTA server (CL = false, the paper's one server SM) or a
+// thread-block-cluster server (CL = true): cluster 0 of the fused grid, C
+// CTAs.  In the cluster server
+//  * the recent-commit table (the on-chip level of the ATR) is striped over
+//    the C CTAs' shared memory by bucket (bucket b lives in CTA b mod C) and
+//    reached through distributed shared memory -- C times the capacity;
+//  * the CTS counter, ticket lock and publisher live in CTA 0 (SURVEY H5:
+//    validation + CTS reservation stay linearizable in one place);
+//  * every CTA runs a receiver warp for its slice of the client doorbells and
+//    its own worker warps, so receiving, payload loading and responding scale
+//    with C.
+// Included by kernel.cu after the shared helpers.
+#pragma once
+#include <cooperative_groups.h>
+
+namespace csmvd {
+
+namespace cg = cooperative_groups;
+
+struct SrvShared {
+  uint32_t tail;         // last CTS assigned (the CTS counter)   [CTA 0]
+  uint32_t next_ticket;  // ticket lock around validate+reserve+insert        [CTA 0]
+  uint32_t now_serving;  //                                                   [CTA 0]
+  uint32_t gts_seen;     // publisher progress seen by workers (back-pressure) [CTA 0]
+  uint32_t q_head;       // next dispatch-queue slot a worker claims          [per CTA]
+  uint32_t exit;         // receiver: all clients finished                    [per CTA]
+};
+
+// ---------------------------------------------------------------------------
+// The ATR, item-indexed and split in two levels:
+//  * lastw[x] in HBM: CTS of the last commit that wrote x -- the exact
+//    record of every committed write-set, all history;
+//  * rt in shared memory: 4-way buckets of (cts << 32 | item) holding recent
+//    writes plus, per bucket, evmax = the largest CTS ever evicted from it,
+//    so that commits made after a worker prefetched lastw (CTS > e_pre) are
+//    seen with on-chip latency.
+// Invariant: if the latest write c of item y (bucket b) is not in b, then
+// evmax[b] >= c (entries leave a bucket only through atomicExch, and the
+// evictor records the evicted CTS with atomicMax).
+// Validation of x for snapshot s (P:75 read-set, P:115 write-set), s <= e_pre:
+//    conflict  iff  lastw[x] (as of e_pre) > s  or  some way holds (x, c), c > s
+//    unknown   iff  not conflict and evmax[b] > e_pre -> abort, reason OVERFLOW
+// ---------------------------------------------------------------------------
+constexpr int kRtWays = 4;
+
+__device__ __forceinline__ uint32_t rt_bucket(uint32_t key, uint32_t rt_log2) {
+  return (key * 0x9E3779B1u) >> (32 - rt_log2);
+}
+
+struct SrvCtx {
+  uint64_t* rt;       // this CTA's stripe of buckets (kRtWays u64 each)
+  uint32_t* evmax;    // this CTA's stripe of eviction watermarks
+  uint32_t clog2;     // log2(server CTAs)
+  SrvShared* sh;      // this CTA's control block
+  SrvShared* sh0;     // CTA 0's control block (DSMEM in a cluster)
+  uint64_t* queue;    // this CTA's dispatch queue
+  uint32_t qn_log2;
+  uint32_t* last_seen;
+  uint32_t cw_lo, cw_hi;  // client warps this CTA's receiver serves
+};
+
+template <bool CL>
+__device__ __forceinline__ uint64_t* rt_at(const SrvCtx& c, uint32_t b) {
+  if constexpr (!CL) {
+    return c.rt + (size_t)b * kRtWays;
+  } else {
+    const uint32_t owner = b & ((1u << c.clog2) - 1), local = b >> c.clog2;
+    return cg::this_cluster().map_shared_rank(c.rt, owner) + (size_t)local * kRtWays;
+  }
+}
+
+template <bool CL>
+__device__ __forceinline__ uint32_t* ev_at(const SrvCtx& c, uint32_t b) {
+  if constexpr (!CL) {
+    return c.evmax + b;
+  } else {
+    const uint32_t owner = b & ((1u << c.clog2) - 1), local = b >> c.clog2;
+    return cg::this_cluster().map_shared_rank(c.evmax, owner) + local;
+  }
+}
+
+template <bool CL>
+__device__ __forceinline__ void srv_fence() {
+  if constexpr (CL) asm volatile("fence.acq_rel.cluster;" ::: "memory");
+  else fence_cta();
+}
+
+struct RtProbe {
+  int way;        // way to overwrite: the way holding x, else the oldest
+  bool conflict;
+  bool unknown;
+};
+
+template <bool CL>
+__device__ __forceinline__ RtProbe rt_probe(const SrvCtx& c, uint32_t bucket, uint32_t key, uint32_t s,
+                                            uint32_t e_pre, uint32_t lastw) {
+  const ulonglong2* e = reinterpret_cast<const ulonglong2*>(rt_at<CL>(c, bucket));
+  const ulonglong2 a = e[0], b = e[1];
+  const uint32_t ev = *ev_at<CL>(c, bucket);
+  const uint64_t w[4] = {a.x, a.y, b.x, b.y};
+  RtProbe r;
+  r.conflict = lastw > s;
+  int hit = -1, old = 0;
+  uint32_t oldc = 0xFFFFFFFFu;
+#pragma unroll
+  for (int i = 0; i < kRtWays; ++i) {
+    const uint32_t k = (uint32_t)w[i], cc = (uint32_t)(w[i] >> 32);
+    if (k == key) {
+      hit = i;
+      r.conflict |= cc > s;
+    }
+    if (cc < oldc) {
+      oldc = cc;
+      old = i;
+    }
+  }
+  r.unknown = !r.conflict && ev > e_pre;
+  r.way = hit >= 0 ? hit : old;
+  return r;
+}
+
+// Record (key, cts) into `way` of its bucket; an evicted entry of another
+// key raises evmax.  Exchanges by several lanes on one slot are serialised
+// by the hardware and each evictor sees the value it replaced.
+template <bool CL>
+__device__ __forceinline__ void rt_record(const SrvCtx& c, uint32_t bucket, int way, uint32_t key, uint32_t cts) {
+  const unsigned long long old =
+      atomicExch(reinterpret_cast<unsigned long long*>(rt_at<CL>(c, bucket) + way), ((unsigned long long)cts << 32) | key);
+  if ((uint32_t)old != key && (uint32_t)(old >> 32) != 0u) atomicMax(ev_at<CL>(c, bucket), (uint32_t)(old >> 32));
+}
+
+// ---------------------------------------------------------------------------
+// Receiver warp: sweeps its slice of the client doorbells with
+// coalesced loads and dispatches new requests to this CTA's workers through
+// a shared-memory queue (entry = lap << 32 | client warp; a worker that
+// claimed slot i waits for lap i / QN + 1).  At most one request per client
+// warp is outstanding, so QN >= slice slots never wrap onto an unconsumed
+// entry.
+// ---------------------------------------------------------------------------
+__device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t n = c.cw_hi - c.cw_lo;
+  const uint32_t rows = (n + 31) / 32;
+  const uint32_t lt = lanemask_lt();
+  const uint32_t qmask = (1u << c.qn_log2) - 1;
+  uint32_t tail = 0;
+  uint32_t idle = 0;
+  for (;;) {
+    bool found = false;
+    for (uint32_t r0 = 0; r0 < rows; r0 += 8) {
+      uint32_t seq[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const uint32_t i = (r0 + k) * 32 + lane;
+        seq[k] = (r0 + k < rows && i < n) ? ld_relaxed(p.req_seq + c.cw_lo + i) : 0u;
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const uint32_t i = (r0 + k) * 32 + lane;
+        const bool pend = r0 + k < rows && i < n && seq[k] != c.last_seen[i];
+        const uint32_t pm = __ballot_sync(FULL, pend);
+        if (pm) {
+          found = true;
+          if (pend) {
+            const uint32_t pos = tail + __popc(pm & lt);
+            c.last_seen[i] = seq[k];
+            *(volatile uint64_t*)&c.queue[pos & qmask] =
+                ((uint64_t)((pos >> c.qn_log2) + 1) << 32) | (c.cw_lo + i);
+          }
+          tail += __popc(pm);
+        }
+      }
+    }
+    if (found) {
+      idle = 0;
+      continue;
+    }
+    if ((++idle & 15u) == 0) {
+      uint32_t dw = 0, er = 0;
+      if (lane == 0) {
+        dw = ld_relaxed(&p.ctl->done_warps);
+        er = ld_relaxed(&p.ctl->error);
+        if (!er && dw < p.n_cw && watchdog(p, t_begin, 3)) er = 1;
+      }
+      dw = __shfl_sync(FULL, dw, 0);
+      er = __shfl_sync(FULL, er, 0);
+      if (dw >= p.n_cw || er) {
+        if (lane == 0) *(volatile uint32_t*)&c.sh->exit = 1;
+        return;
+      }
+    }
+  }
+}
+
+// Claim the next dispatched request of this CTA's queue (blocking).
+// Returns false when the receiver has finished.
+__device__ __forceinline__ bool claim_request(const SrvCtx& c, uint32_t& cw) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t qmask = (1u << c.qn_log2) - 1;
+  uint32_t slot = 0;
+  if ((threadIdx.x & 31) == 0) slot = atomicAdd(&c.sh->q_head, 1u);
+  slot = __shfl_sync(FULL, slot, 0);
+  for (;;) {  // convergent wait: every lane polls the same word (broadcast LDS)
+    const uint64_t ent = *(volatile uint64_t*)&c.queue[slot & qmask];
+    if ((uint32_t)(ent >> 32) == (slot >> c.qn_log2) + 1) {
+      cw = (uint32_t)ent;
+      return true;
+    }
+    if (*(volatile uint32_t*)&c.sh->exit) return false;
+    __nanosleep(64);
+  }
+}
+
+// Ticket lock around the commit critical section, in CTA 0's shared memory.
+template <bool CL>
+__device__ __forceinline__ uint32_t cs_enter(const SrvCtx& c) {
+  uint32_t ticket = 0;
+  if ((threadIdx.x & 31) == 0) ticket = atomicAdd(&c.sh0->next_ticket, 1u);
+  ticket = __shfl_sync(0xFFFFFFFFu, ticket, 0);
+  while (*(volatile uint32_t*)&c.sh0->now_serving != ticket) __nanosleep(16);
+  __syncwarp();
+  srv_fence<CL>();
+  return ticket;
+}
+
+template <bool CL>
+__device__ __forceinline__ void cs_leave(const SrvCtx& c, uint32_t ticket, uint32_t new_tail) {
+  __syncwarp();
+  srv_fence<CL>();
+  if ((threadIdx.x & 31) == 0) {
+    *(volatile uint32_t*)&c.sh0->tail = new_tail;
+    srv_fence<CL>();
+    *(volatile uint32_t*)&c.sh0->now_serving = ticket + 1;
+  }
+}
+
+// done-ring back-pressure (CSMV_PUBLISH_SERVER): CTS t may reuse slot
+// t & mask only once GTS >= t - 2^20
+__device__ __forceinline__ void done_ring_room(const KParams& p, const SrvCtx& c, uint32_t t, uint64_t t_begin) {
+  const uint32_t dmask = (1u << kDoneLog2) - 1;
+  if ((threadIdx.x & 31) == 0) {
+    uint32_t it = 0;
+    while (t > *(volatile uint32_t*)&c.sh0->gts_seen + dmask) {
+      *(volatile uint32_t*)&c.sh0->gts_seen = ld_relaxed(p.gts);
+      if ((++it & 255u) == 0 && watchdog(p, t_begin, 4)) break;
+    }
+  }
+  __syncwarp();
+}
+
+// ---------------------------------------------------------------------------
+// Bank worker warp.  Claims up to kMaxCombine dispatched batches (the first
+// blocking, the rest only if already queued), loads them outside the lock,
+// and commits them inside ONE critical section, one after another in queue
+// order -- exactly as if each had its own critical section: batch j is
+// validated after batch j-1's write-set was recorded, and receives the next
+// consecutive CTS range.  A batch is validated by the whole warp,
+// one lane per transaction, __ballot_sync for the commit mask.
+// ---------------------------------------------------------------------------
+template <bool CL>
+__device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+  constexpr int M = kMaxCombine;
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t lt = lanemask_lt();
+  const uint32_t qmask = (1u << c.qn_log2) - 1;
+  const uint32_t m_max = p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine);
+  unsigned long long busy = 0, locked = 0, batches = 0, groups = 0;
+  unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  for (;;) {
+    const long long tq = clock64();
+    uint32_t cwv[M];
+    if (!claim_request(c, cwv[0])) break;
+    // ---- combine: grab further requests that are already queued
+    uint32_t m = 1;
+#pragma unroll
+    for (int j = 1; j < M; ++j) {
+      uint32_t got = 0xFFFFFFFFu;
+      if (m == (uint32_t)j && m < m_max && lane == 0) {
+        const uint32_t h = *(volatile uint32_t*)&c.sh->q_head;
+        const uint64_t e = *(volatile uint64_t*)&c.queue[h & qmask];
+        if ((uint32_t)(e >> 32) == (h >> c.qn_log2) + 1 && atomicCAS(&c.sh->q_head, h, h + 1) == h) got = (uint32_t)e;
+      }
+      got = __shfl_sync(FULL, got, 0);
+      cwv[j] = got;
+      if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
+    }
+    const long long t0 = clock64();
+    // ---- load the batches: doorbell (acquire pattern), header, ids
+    uint32_t sq[M], sn[M], msk[M], id0[M], id1[M];
+#pragma unroll
+    for (int j = 0; j < M; ++j) sq[j] = (j < (int)m) ? ld_relaxed(p.req_seq + cwv[j]) : 0u;
+    fence_gpu();
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      sn[j] = msk[j] = id0[j] = id1[j] = 0;
+      if (j < (int)m) {
+        sn[j] = ld_relaxed(&p.req_hdr[cwv[j]].snapshot);
+        msk[j] = ld_relaxed(&p.req_hdr[cwv[j]].mask);
+      }
+    }
+    bool mine[M];
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      mine[j] = (msk[j] >> lane) & 1u;
+      if (mine[j]) {
+        id0[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + lane) & ~kWriteBit;
+        id1[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + 32 + lane) & ~kWriteBit;
+      }
+    }
+    const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
+    srv_fence<CL>();
+    uint32_t lw0[M], lw1[M], bk0[M], bk1[M];
+    uint32_t xor_all = e_pre;
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      lw0[j] = lw1[j] = 0;
+      if (mine[j]) {
+        lw0[j] = ld_relaxed(p.lastw + id0[j]);
+        lw1[j] = ld_relaxed(p.lastw + id1[j]);
+      }
+      bk0[j] = rt_bucket(id0[j], p.rt_log2);
+      bk1[j] = rt_bucket(id1[j], p.rt_log2);
+      xor_all ^= bk0[j] ^ bk1[j] ^ lw0[j] ^ lw1[j] ^ sn[j];
+    }
+    // The payload must have arrived before the lock is taken: a warp vote on
+    // values derived from it makes the loads complete here.
+    if (__ballot_sync(FULL, xor_all == 0x12345679u) == FULL) __nanosleep(1);
+    const long long tl = clock64();
+    // ---- critical section: validate, reserve CTS, record
+    const uint32_t ticket = cs_enter<CL>(c);
+    const long long t1 = clock64();
+    const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
+    uint32_t t = t0c;
+    uint32_t cm[M], om[M], base[M];
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      cm[j] = om[j] = 0;
+      base[j] = t + 1;
+      if (j >= (int)m) continue;
+      RtProbe q0{0, false, false}, q1{0, false, false};
+      if (mine[j]) {
+        q0 = rt_probe<CL>(c, bk0[j], id0[j], sn[j], e_pre, lw0[j]);
+        q1 = rt_probe<CL>(c, bk1[j], id1[j], sn[j], e_pre, lw1[j]);
+        if (bk1[j] == bk0[j] && q1.way == q0.way) q1.way = (q1.way + 1) & (kRtWays - 1);
+      }
+      bool ovf = mine[j] && (q0.unknown || q1.unknown);
+      bool conflict = mine[j] && (q0.conflict || q1.conflict);
+      if (p.debug & CSMV_DBG_NO_VALIDATE) ovf = conflict = false;
+      const bool commit = mine[j] && !ovf && !conflict;
+      cm[j] = __ballot_sync(FULL, commit);
+      om[j] = __ballot_sync(FULL, ovf);
+      const uint32_t cts = t + 1 + __popc(cm[j] & lt);
+      t += __popc(cm[j]);
+      if (commit) {
+        p.lastw[id0[j]] = cts;
+        p.lastw[id1[j]] = cts;
+        rt_record<CL>(c, bk0[j], q0.way, id0[j], cts);
+        rt_record<CL>(c, bk1[j], q1.way, id1[j], cts);
+      }
+      __syncwarp();  // batch j's records precede batch j+1's probes
+    }
+    const long long ta = clock64();
+    if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) done_ring_room(p, c, t, t_begin);
+    cs_leave<CL>(c, ticket, t);
+    const long long t2 = clock64();
+    // ---- respond: one fence, then the payloads and sequence words
+    if (lane == 0) {
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        if (j >= (int)m) break;
+        st_relaxed(&p.resp[cwv[j]].cts_base, base[j]);
+        st_relaxed(&p.resp[cwv[j]].commit_mask, cm[j]);
+        st_relaxed(&p.resp[cwv[j]].overflow_mask, om[j]);
+      }
+      fence_gpu();
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        if (j >= (int)m) break;
+        st_relaxed(&p.resp[cwv[j]].seq, sq[j]);
+      }
+    }
+    __syncwarp();
+    const long long t3 = clock64();
+    busy += (unsigned long long)(t3 - t0);
+    locked += (unsigned long long)(t2 - t1);
+    ph[0] += (unsigned long long)(t0 - tq);
+    ph[1] += (unsigned long long)(tl - t0);
+    ph[2] += (unsigned long long)(t1 - tl);
+    ph[3] += (unsigned long long)(t2 - t1);
+    ph[4] += (unsigned long long)(t3 - t2);
+    ph[5] += (unsigned long long)(ta - t1);
+    batches += m;
+    ++groups;
+  }
+  if (lane == 0) {
+    for (int i = 0; i < 8; ++i) atomicAdd(&p.stats->phase[i], ph[i]);
+    atomicAdd(&p.stats->batches, batches);
+    atomicAdd(&p.stats->groups, groups);
+    atomicAdd(&p.stats->busy_cycles, busy);
+    atomicAdd(&p.stats->lock_cycles, locked);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Generic worker (variable-length read/write sets, the KV workload): one
+// batch per critical section.  Validation reads lastw inside the critical
+// section, so it covers every commit up to the current tail exactly
+// (P:75).
+// ---------------------------------------------------------------------------
+template <bool CL>
+__device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t lt = lanemask_lt();
+  unsigned long long busy = 0, locked = 0, batches = 0;
+  for (;;) {
+    uint32_t cw;
+    if (!claim_request(c, cw)) break;
+    const long long t0 = clock64();
+    const uint32_t sq = ld_relaxed(p.req_seq + cw);
+    fence_gpu();
+    const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
+    const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
+    const bool mine = (mask >> lane) & 1u;
+    const uint32_t cnt = mine ? ld_relaxed(p.req_cnt + (size_t)cw * 32 + lane) : 0u;
+    uint32_t ids[kKvMaxId];
+#pragma unroll
+    for (uint32_t k = 0; k < kKvMaxId; ++k)
+      ids[k] = (k < cnt) ? ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + k) * 32 + lane) : 0u;
+    uint32_t x = s;
+#pragma unroll
+    for (uint32_t k = 0; k < kKvMaxId; ++k) x ^= ids[k];
+    if (__ballot_sync(FULL, x == 0x12345679u) == FULL) __nanosleep(1);
+    // ---- critical section
+    const uint32_t ticket = cs_enter<CL>(c);
+    const long long t1 = clock64();
+    const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
+    uint32_t lw[kKvMaxId];
+#pragma unroll
+    for (uint32_t k = 0; k < kKvMaxId; ++k) lw[k] = (k < cnt) ? ld_relaxed(p.lastw + (ids[k] & ~kWriteBit)) : 0u;
+    bool conflict = false;
+#pragma unroll
+    for (uint32_t k = 0; k < kKvMaxId; ++k) conflict |= lw[k] > s;
+    if (p.debug & CSMV_DBG_NO_VALIDATE) conflict = false;
+    const bool commit = mine && !conflict;
+    const uint32_t cm = __ballot_sync(FULL, commit);
+    const uint32_t n = __popc(cm);
+    const uint32_t cts = t0c + 1 + __popc(cm & lt);
+    if (p.publish == CSMV_PUBLISH_SERVER && n) done_ring_room(p, c, t0c + n, t_begin);
+    if (commit) {
+#pragma unroll
+      for (uint32_t k = 0; k < kKvMaxId; ++k)
+        if (k < cnt && (ids[k] & kWriteBit)) p.lastw[ids[k] & ~kWriteBit] = cts;
+    }
+    cs_leave<CL>(c, ticket, t0c + n);
+    const long long t2 = clock64();
+    if (lane == 0) {
+      st_relaxed(&p.resp[cw].cts_base, t0c + 1);
+      st_relaxed(&p.resp[cw].commit_mask, cm);
+      st_relaxed(&p.resp[cw].overflow_mask, 0u);
+      st_release(&p.resp[cw].seq, sq);
+    }
+    __syncwarp();
+    busy += (unsigned long long)(clock64() - t0);
+    locked += (unsigned long long)(t2 - t1);
+    ++batches;
+  }
+  if (lane == 0) {
+    atomicAdd(&p.stats->batches, batches);
+    atomicAdd(&p.stats->groups, batches);
+    atomicAdd(&p.stats->busy_cycles, busy);
+    atomicAdd(&p.stats->lock_cycles, locked);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// CSMV_PUBLISH_SERVER: advance GTS over the prefix of CTS whose write-backs
+// are done.  Same invariant as P:116 (GTS = c only once every commit <= c
+// has written back), without a client-side serial chain.  CTA 0 only.
+// ---------------------------------------------------------------------------
+__device__ void server_publisher(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t dmask = (1u << kDoneLog2) - 1;
+  uint32_t g = *(volatile uint32_t*)&c.sh->tail;
+  uint32_t spins = 0;
+  for (;;) {
+    uint32_t v[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) v[k] = ld_relaxed(p.done_ring + ((g + 1 + k * 32 + lane) & dmask));
+    uint32_t adv = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const uint32_t bad = __ballot_sync(FULL, v[k] != g + 1 + k * 32 + lane);
+      if (adv == (uint32_t)k * 32) adv += bad ? (uint32_t)(__ffs(bad) - 1) : 32u;
+    }
+    if (adv) {
+      fence_gpu();
+      g += adv;
+      if (lane == 0) st_release(p.gts, g);
+      continue;
+    }
+    if ((++spins & 63u) == 0) {
+      uint32_t dw = 0, er = 0;
+      if (lane == 0) {
+        dw = ld_relaxed(&p.ctl->done_warps);
+        er = ld_relaxed(&p.ctl->error);
+        if (!er && watchdog(p, t_begin, 5)) er = 1;
+      }
+      dw = __shfl_sync(FULL, dw, 0);
+      er = __shfl_sync(FULL, er, 0);
+      if (er) break;
+      if (dw >= p.n_cw && g == *(volatile uint32_t*)&c.sh->tail) break;
+    }
+  }
+}
+
+// Shared-memory layout of one server CTA (every CTA of the fused grid gets
+// the same dynamic allocation): rt stripe, evmax stripe, dispatch queue,
+// last-seen doorbells of its slice, control block.
+template <int KIND, bool CL>
+__device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
+  const uint32_t C = p.n_server_ctas;
+  const uint32_t rank = CL ? cg::this_cluster().block_rank() : 0u;
+  const uint32_t local_log2 = p.rt_log2 - p.clog2;
+  const uint32_t per = (p.n_cw + C - 1) / C;
+  SrvCtx c;
+  c.clog2 = p.clog2;
+  c.cw_lo = min(rank * per, p.n_cw);
+  c.cw_hi = min(c.cw_lo + per, p.n_cw);
+  c.qn_log2 = queue_log2(per);
+  c.rt = reinterpret_cast<uint64_t*>(smem);
+  const uint32_t rt_words = (uint32_t)kRtWays << local_log2;
+  c.queue = c.rt + rt_words;
+  c.evmax = reinterpret_cast<uint32_t*>(c.queue + (1u << c.qn_log2));
+  c.last_seen = c.evmax + (1u << local_log2);
+  const uint32_t ls_words = (per + 31) / 32 * 32;
+  c.sh = reinterpret_cast<SrvShared*>(c.last_seen + ls_words);
+  if constexpr (CL) c.sh0 = cg::this_cluster().map_shared_rank(c.sh, 0);
+  else c.sh0 = c.sh;
+  for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) c.rt[i] = 0xFFFFFFFFull;  // cts 0, no item
+  for (uint32_t i = threadIdx.x; i < (1u << local_log2); i += blockDim.x) c.evmax[i] = 0;
+  for (uint32_t i = threadIdx.x; i < (1u << c.qn_log2); i += blockDim.x) c.queue[i] = 0;
+  for (uint32_t i = threadIdx.x; i < ls_words; i += blockDim.x) c.last_seen[i] = 0;
+  if (threadIdx.x == 0) {
+    const uint32_t g0 = *p.gts;
+    c.sh->tail = g0;
+    c.sh->next_ticket = 0;
+    c.sh->now_serving = 0;
+    c.sh->gts_seen = g0;
+    c.sh->q_head = 0;
+    c.sh->exit = 0;
+  }
+  if constexpr (CL) cg::this_cluster().sync();
+  else __syncthreads();
+  const uint32_t warp = threadIdx.x >> 5;
+  if (warp == 0) {
+    server_receiver(p, c, t_begin);
+  } else if (warp <= p.n_workers) {
+    if constexpr (KIND == CSMV_KIND_KV) server_worker_generic<CL>(p, c, t_begin);
+    else server_worker<CL>(p, c, t_begin);
+  } else if (warp == p.n_workers + 1 && rank == 0 && p.publish == CSMV_PUBLISH_SERVER) {
+    server_publisher(p, c, t_begin);
+  }
+  if constexpr (CL) cg::this_cluster().sync();
+  else __syncthreads();
+  if (rank == 0 && threadIdx.x == 0) p.ctl->tail_final = c.sh->tail;
+}
+
+}  // namespace csmvd

@@ -1,0 +1,62 @@
+"""GPU parity of the thread-block-cluster server (the recent-commit table
+striped over C CTAs' shared memory through DSMEM, CTS counter in CTA 0) and
+of the single-CTA server on the same workloads (C5's server axis)."""
+import numpy as np
+import pytest
+
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+csmv = pytest.importorskip("paper_conf_ipps_nunesc022_b200.csmv")
+from paper_conf_ipps_nunesc022_b200 import workloads as W  # noqa: E402
+from tests.test_gpu_parity import check, closed_form, newest  # noqa: E402
+from tests.test_gpu_kv import ocfg_of, as_state, run as run_kv  # noqa: E402
+
+
+@pytest.mark.parametrize("cs", [2, 4, 8, 16])
+def test_bank_cluster_parity(cs):
+    cfg = W.c2(n_items=1 << 16, n_tx=1 << 18, server=csmv.SERVER_CLUSTER, cluster_size=cs,
+               publish=csmv.PUBLISH_SERVER, ro_streak=8, server_workers=6, server_combine=4,
+               client_warps=256)
+    rep, stats, log, rings, descs = check(cfg)
+    assert stats["server_ctas"] == cs
+    assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions), closed_form(cfg, descs, cfg.init_values()))
+
+
+def test_bank_cluster_contention_and_tiny_table():
+    """Hot items and a tiny striped table: OVERFLOW aborts appear, parity holds."""
+    cfg = W.c2(n_items=1 << 10, n_tx=1 << 17, server=csmv.SERVER_CLUSTER, cluster_size=4,
+               atr_capacity=64, p_update_ppm=700_000, client_warps=128, server_combine=4, server_workers=6)
+    rep, stats, *_ = check(cfg)
+    assert stats["aborts"]["overflow"]["update"] > 0
+
+
+def test_c3_cluster_parity():
+    cfg = W.c3(n_tx=1 << 17, server=csmv.SERVER_CLUSTER, cluster_size=8, client_warps=128,
+               ro_streak=8, server_combine=4, server_workers=6)
+    check(cfg)
+
+
+def test_kv_cluster_parity():
+    cfg = W.c4(n_items=1 << 13, n_tx=1 << 16, p_update_ppm=100_000, server=csmv.SERVER_CLUSTER,
+               cluster_size=4, client_warps=128, server_workers=6)
+    pre, stats, log, fin = run_kv(cfg)
+    oc = ocfg_of(cfg)
+    init = oracle.kv_preload(oc)
+    d = oracle.kv_gen(oc, cfg.seed, cfg.n_tx)
+    rep = oracle.kv_check(oc, init, d, log, final=as_state(fin, cfg.n_items, cfg.workload.kv_ways),
+                          claims=dict(committed_update=stats["committed_update"], committed_ro=stats["committed_ro"],
+                                      gts_final=stats["gts_final"], total_aborts=stats["total_aborts"]))
+    assert rep["ok"], rep
+
+
+def test_cluster_one_client_warp_is_deterministic():
+    """P7 holds with the cluster server too (the server's shape is invisible)."""
+    cfg = W.c1(client_warps=1, n_tx=2000, server=csmv.SERVER_CLUSTER, cluster_size=2, ro_streak=4)
+    from tests.test_gpu_parity import run_gpu, oracle_cfg
+    stats, log, (vals, mv), rings = run_gpu(cfg)
+    ocfg = oracle_cfg(cfg)
+    descs = oracle.bank_gen(ocfg, cfg.seed, cfg.n_tx)
+    plog, pvals, prings, pst = oracle.bank_predict(ocfg, cfg.init_values(), descs, 32, max_vals=mv)
+    assert np.array_equal(log, plog) and np.array_equal(rings, prings)
