@@ -125,6 +125,12 @@ class Clocks:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
+DESCR = {"C1": "C1: bank, 1,024 accounts, K=4, 8 client warps, 10k transfers + 10% total-sum ROTs",
+         "C2": "C2: bank, 1M accounts, K=4, 50% update, uniform, 64-read ROT scans",
+         "C3": "C3: bank, 4,096 accounts, K=4, 90% 64-read ROT scans, zipf 0.99 updates",
+         "C4": "C4: MemcachedGPU KV, 4M slots/keys, 16 ways, K=4, 99% GET, zipf 0.99"}
+
+
 def oracle_sample_rate(cfg, budget_s: float, chunk: int, tx_start: int = 0):
     """CPU oracle (1-warp deterministic schedule, single thread) on bounded
     chunks of the workload; returns (tx/s, txs, seconds)."""
@@ -133,15 +139,23 @@ def oracle_sample_rate(cfg, budget_s: float, chunk: int, tx_start: int = 0):
     import oracle
 
     w = cfg.workload
-    ocfg = oracle.bank_cfg(cfg.n_items, cfg.n_versions, dist=w.dist, zipf_theta_milli=w.zipf_theta_milli,
-                           p_update_ppm=w.p_update_ppm, ro_period=w.ro_period, ro_reads=w.ro_reads,
-                           amount_max=w.amount_max, ro_streak=w.ro_streak)
-    init = np.full(cfg.n_items, 1000, dtype=np.int32)
+    if w.kind == 1:  # KV (MemcachedGPU)
+        ocfg = oracle.kv_cfg(cfg.n_items, w.kv_ways, n_keys=w.kv_keys, n_versions=cfg.n_versions, dist=w.dist,
+                             zipf_theta_milli=w.zipf_theta_milli, p_update_ppm=w.p_update_ppm,
+                             ro_streak=w.ro_streak)
+        init = oracle.kv_preload(ocfg)
+        gen, predict = oracle.kv_gen, oracle.kv_predict
+    else:
+        ocfg = oracle.bank_cfg(cfg.n_items, cfg.n_versions, dist=w.dist, zipf_theta_milli=w.zipf_theta_milli,
+                               p_update_ppm=w.p_update_ppm, ro_period=w.ro_period, ro_reads=w.ro_reads,
+                               amount_max=w.amount_max, ro_streak=w.ro_streak)
+        init = np.full(cfg.n_items, 1000, dtype=np.int32)
+        gen, predict = oracle.bank_gen, oracle.bank_predict
     done, spent, tx0 = 0, 0.0, tx_start
     while True:
-        descs = oracle.bank_gen(ocfg, cfg.seed, chunk, tx0=tx0)
+        descs = gen(ocfg, cfg.seed, chunk, tx0=tx0)
         t = time.perf_counter()
-        oracle.bank_predict(ocfg, init, descs, 32)
+        predict(ocfg, init, descs, 32)
         spent += time.perf_counter() - t
         done += chunk
         tx0 += chunk
@@ -152,12 +166,25 @@ def oracle_sample_rate(cfg, budget_s: float, chunk: int, tx_start: int = 0):
 
 def make_cfg(args, world: int, rank: int):
     from paper_conf_ipps_nunesc022_b200 import partition, workloads
-    cfg = workloads.c2()
+    cfg = workloads.PRESETS[args.config]()
     n_tx = args.n_tx or cfg.n_tx
     cfg = cfg.with_(n_tx=n_tx, log_mode=0, ro_streak=TUNED["ro_streak"], publish=TUNED["publish"],
                     server_workers=TUNED["server_workers"], server_combine=TUNED["server_combine"])
     part = partition.partition(cfg.n_items, n_tx, cfg.seed, rank, world)
-    return cfg, partition.local_config(cfg, part), part
+    lcfg = partition.local_config(cfg, part)
+    if cfg.workload.kind == 1:   # KV: the partition is a smaller cache with its own key space
+        lcfg = lcfg.with_(kv_keys=lcfg.n_items - lcfg.n_items % cfg.workload.kv_ways,
+                          n_items=lcfg.n_items - lcfg.n_items % cfg.workload.kv_ways)
+    return cfg, lcfg, part
+
+
+# KV algorithmic bytes (paper VBox layout): a GET hitting at
+# the average way (A+1)/2 reads that many keys (head+ts+16 B) and the value
+# (head+ts+32 B); a PUT at most 2A+1 reads + 4 write-backs + ids.
+def kv_bytes(stats: dict, ways: int) -> float:
+    get = (ways + 1) / 2 * 24 + 40
+    put = (ways + 1) / 2 * 24 + 12 + (24 + 40 + 12 + 12) + 4 * ((ways + 1) / 2 + 4) + 4
+    return stats["committed_ro"] * get + stats["committed_update"] * put
 
 
 def bench_reference(args):
@@ -175,11 +202,11 @@ def bench_reference(args):
         total_tx += n
         total_s += s
     value = total_tx / total_s
-    sample = f"{args.steps} chunks of {chunk} consecutive C2 transactions (1M accounts, 50% update)"
+    sample = f"{args.steps} chunks of {chunk} consecutive {cfg.name} transactions ({cfg.n_items} items)"
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total_s / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
-            "data": "synthetic", "config": {"workload": "C2", "n_items": cfg.n_items,
+            "data": "synthetic", "config": {"workload": DESCR.get(cfg.name, cfg.name), "n_items": cfg.n_items,
                                             "n_versions": cfg.n_versions, "sample": sample},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -205,15 +232,22 @@ def bench_ours(args):
     dev = torch.device("cuda", torch.cuda.current_device())
     cfg, lcfg, part = make_cfg(args, world, rank)
     props = torch.cuda.get_device_properties(dev)
-    n_cw = args.client_warps or TUNED["client_warps_per_sm"] * (props.multi_processor_count - 1)
+    n_cw = args.client_warps or lcfg.workload.client_warps or \
+        TUNED["client_warps_per_sm"] * (props.multi_processor_count - 1)
     lcfg = lcfg.with_(client_warps=n_cw)
     w = lcfg.workload
+    is_kv = w.kind == csmv.KIND_KV
 
     stream = torch.cuda.current_stream()
-    store = csmv.Store(lcfg.n_items, lcfg.n_versions)
+    if is_kv:
+        store = csmv.KvStore(lcfg.n_items, w.kv_ways, lcfg.n_versions)
+        init = np.zeros(lcfg.n_items * 13 + lcfg.n_items // w.kv_ways, dtype=np.uint32)  # preload upload size
+        store.load(w.kv_keys)
+    else:
+        store = csmv.Store(lcfg.n_items, lcfg.n_versions)
+        init = np.full(lcfg.n_items, 1000, dtype=np.int32)
+        store.load(init)
     store.set_stream(stream.cuda_stream)
-    init = np.full(lcfg.n_items, 1000, dtype=np.int32)
-    store.load(init)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     def barrier():
@@ -247,7 +281,8 @@ def bench_ours(args):
     value = red["committed"] / (total_ms_max * 1e-3)
 
     # roofline of the dominant (only) kernel, csmv_fused
-    algo = sum(algorithmic_bytes(s, w.ro_reads, lcfg.n_items) for _, _, s in steps) / len(steps)
+    algo = sum(kv_bytes(s, w.kv_ways) if is_kv else algorithmic_bytes(s, w.ro_reads, lcfg.n_items)
+               for _, _, s in steps) / len(steps)
     kmean = sum(kern_ns) / len(kern_ns)
     achieved = algo / (kmean * 1e-9) / 1e9
     peak, peak_kind = peaks()
@@ -264,7 +299,7 @@ def bench_ours(args):
     t0 = time.perf_counter()
     e2e_committed = 0
     for i in range(e2e_steps):
-        store.load(init_pinned.numpy())
+        store.load(w.kv_keys if is_kv else init_pinned.numpy())
         s = store.run(w, lcfg.n_tx, lcfg.seed + 500 + i)
         e2e_committed += s["committed"]
     torch.cuda.synchronize()
@@ -283,13 +318,13 @@ def bench_ours(args):
     if world == 1 and not args.no_cpu_baseline:
         r, n, s = oracle_sample_rate(cfg, args.cpu_budget, 1 << 18)
         cpu = {"value": r, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"{n} consecutive C2 transactions ({s:.1f} s, 1M accounts, 1-warp schedule)"}
+               "sample": f"{n} consecutive {cfg.name} transactions ({s:.1f} s, 1-warp schedule, {cfg.n_items} items)"}
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": total_ms_max / args.steps, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
         "abort_rate": red["abort_rate"],
-        "config": {"workload": "C2: bank, 1M accounts, K=4, 50% update, uniform, 64-read ROT scans",
+        "config": {"workload": DESCR.get(cfg.name, cfg.name),
                    "n_items": cfg.n_items, "n_versions": cfg.n_versions, "n_tx_per_step": cfg.n_tx,
                    "client_warps_per_gpu": n_cw, "server_workers": w.server_workers,
                    "server_combine": w.server_combine,
@@ -326,6 +361,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
     ap.add_argument("--n-tx", type=int, default=0)
+    ap.add_argument("--config", choices=("C1", "C2", "C3", "C4"), default="C2",
+                    help="workload (default C2, the config BASELINE.json's metric is quoted on)")
     ap.add_argument("--client-warps", type=int, default=0)
     ap.add_argument("--cpu-budget", type=float, default=10.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")

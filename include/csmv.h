@@ -60,7 +60,8 @@ extern "C" {
 #define CSMV_PUBLISH_CLIENT 0u /* client advances GTS when GTS == CTS-1 */
 #define CSMV_PUBLISH_SERVER 1u /* a server warp advances GTS over finished write-backs */
 #define CSMV_ATR_HASH 0u       /* item-indexed ATR (set-associative, smem) */
-#define CSMV_ATR_LIST 1u       /* ATR as a list of write-sets, warp-striped scan */
+#define CSMV_ATR_LIST 1u       /* the paper's ATR: list of write-sets, collaborative validation */
+#define CSMV_ATR_LIST_NOCV 2u  /* the list ATR, one lane per transaction (CSMV-NoCV) */
 
 #define CSMV_DBG_NO_PREVAL 1u  /* negative control: skip client pre-validation */
 #define CSMV_DBG_NO_VALIDATE 2u/* negative control: server commits without validating */

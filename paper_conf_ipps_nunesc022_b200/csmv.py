@@ -21,7 +21,7 @@ DIST_UNIFORM, DIST_ZIPF = 0, 1
 LOG_NONE, LOG_DIGEST, LOG_FULL = 0, 1, 2
 SERVER_CTA, SERVER_CLUSTER = 0, 1
 PUBLISH_CLIENT, PUBLISH_SERVER = 0, 1
-ATR_HASH, ATR_LIST = 0, 1
+ATR_HASH, ATR_LIST, ATR_LIST_NOCV = 0, 1, 2
 DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER = 1, 2, 4
 ABORT_REASONS = ("preval", "conflict", "early", "overflow", "version")
 

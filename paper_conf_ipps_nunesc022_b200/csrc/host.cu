@@ -357,7 +357,9 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (w->p_update_ppm > 1000000) return set_err(CSMV_EINVAL, "csmv_run: p_update_ppm > 10^6");
   if (w->log_mode > CSMV_LOG_FULL || w->publish > CSMV_PUBLISH_SERVER)
     return set_err(CSMV_EINVAL, "csmv_run: bad log_mode/publish");
-  if (w->atr_mode != CSMV_ATR_HASH) return set_err(CSMV_EINVAL, "csmv_run: ATR list mode not built yet");
+  if (w->atr_mode > CSMV_ATR_LIST_NOCV) return set_err(CSMV_EINVAL, "csmv_run: unknown atr_mode %u", w->atr_mode);
+  if (w->atr_mode != CSMV_ATR_HASH && (h->kind != CSMV_KIND_BANK || w->server != CSMV_SERVER_CTA))
+    return set_err(CSMV_EINVAL, "csmv_run: the list ATR is built for the bank workload on the single-CTA server");
   if (n_tx >= (1ull << 32)) return set_err(CSMV_EINVAL, "csmv_run: n_tx must be < 2^32");
 
   uint32_t gts0 = 0;
@@ -472,6 +474,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.publish = w->publish;
   p.ro_streak = w->ro_streak;
   p.combine = w->server_combine ? w->server_combine : 1u;
+  p.atr_mode = w->atr_mode;
   p.backoff_max = w->backoff_max;
   p.debug = w->debug_flags;
   p.watchdog_ns = (uint64_t)(w->watchdog_ms ? w->watchdog_ms : 20000u) * 1000000ull;

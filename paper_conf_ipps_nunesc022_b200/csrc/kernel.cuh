@@ -87,6 +87,7 @@ struct KParams {
   uint32_t ro_streak;      // read-only transactions a lane may run per round (0 = one tx per round)
   uint32_t combine;        // batches per critical section (1..kMaxCombine)
   uint32_t backoff_max;    // rounds an update rejected by the server may sit out (0 = none)
+  uint32_t atr_mode;       // CSMV_ATR_HASH (item-indexed) / _LIST (paper, CV) / _LIST_NOCV
   uint32_t debug;
   uint64_t watchdog_ns;
   // KV workload (kind == CSMV_KIND_KV)

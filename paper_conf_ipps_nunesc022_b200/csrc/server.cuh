@@ -252,6 +252,52 @@ __device__ __forceinline__ void done_ring_room(const KParams& p, const SrvCtx& c
 }
 
 // ---------------------------------------------------------------------------
+// The paper's ATR (CSMV_ATR_LIST / CSMV_ATR_LIST_NOCV, single-CTA server):
+// a CTS-indexed ring of R write-set records in shared memory;
+// entry c holds the write-set of the commit with CTS c.  A transaction with
+// snapshot s is validated against the entries (s, t] -- every commit after
+// its snapshot; if the ring no longer holds them all
+// (t - s >= R) it aborts with the labelled reason OVERFLOW.
+//  * LIST (collaborative validation): the transactions of
+//    the batch are validated one after another; for each, every lane takes
+//    the same read/write-set entries e_t (a broadcast) and stripes over the
+//    ATR records, and __any_sync combines the lanes' findings;
+//  * LIST_NOCV (CSMV-NoCV): each lane validates its own
+//    transaction by scanning every record of the window itself.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void atr_list_validate(const KParams& p, const SrvCtx& c, uint32_t s, uint32_t t,
+                                                  bool mine, uint32_t a, uint32_t b, bool& ovf, bool& conflict) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t R = (uint32_t)kRtWays << (p.rt_log2 - p.clog2);
+  const uint64_t* atr = c.rt;
+  ovf = mine && (t - s >= R);
+  conflict = false;
+  if (p.atr_mode == CSMV_ATR_LIST) {
+    uint32_t need = __ballot_sync(FULL, mine && !ovf), found = 0;
+    while (need) {
+      const int i = __ffs(need) - 1;
+      need &= need - 1;
+      const uint32_t ea = __shfl_sync(FULL, a, i), eb = __shfl_sync(FULL, b, i);
+      bool f = false;
+      for (uint32_t q = s + 1 + lane; q - 1 < t; q += 32) {  // q in (s, t], striped over lanes
+        const uint64_t e = atr[q & (R - 1)];
+        const uint32_t w0 = (uint32_t)e, w1 = (uint32_t)(e >> 32);
+        f |= w0 == ea || w0 == eb || w1 == ea || w1 == eb;
+      }
+      if (__any_sync(FULL, f)) found |= 1u << i;
+    }
+    conflict = (found >> lane) & 1u;
+  } else if (mine && !ovf) {
+    for (uint32_t q = s + 1; q - 1 < t; ++q) {
+      const uint64_t e = atr[q & (R - 1)];
+      const uint32_t w0 = (uint32_t)e, w1 = (uint32_t)(e >> 32);
+      conflict |= w0 == a || w0 == b || w1 == a || w1 == b;
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
 // Bank worker warp.  Claims up to kMaxCombine dispatched batches (the first
 // blocking, the rest only if already queued), loads them outside the lock,
 // and commits them inside ONE critical section, one after another in queue
@@ -342,13 +388,18 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       base[j] = t + 1;
       if (j >= (int)m) continue;
       RtProbe q0{0, false, false}, q1{0, false, false};
-      if (mine[j]) {
-        q0 = rt_probe<CL>(c, bk0[j], id0[j], sn[j], e_pre, lw0[j]);
-        q1 = rt_probe<CL>(c, bk1[j], id1[j], sn[j], e_pre, lw1[j]);
-        if (bk1[j] == bk0[j] && q1.way == q0.way) q1.way = (q1.way + 1) & (kRtWays - 1);
+      bool ovf = false, conflict = false;
+      if (p.atr_mode == CSMV_ATR_HASH) {
+        if (mine[j]) {
+          q0 = rt_probe<CL>(c, bk0[j], id0[j], sn[j], e_pre, lw0[j]);
+          q1 = rt_probe<CL>(c, bk1[j], id1[j], sn[j], e_pre, lw1[j]);
+          if (bk1[j] == bk0[j] && q1.way == q0.way) q1.way = (q1.way + 1) & (kRtWays - 1);
+        }
+        ovf = mine[j] && (q0.unknown || q1.unknown);
+        conflict = mine[j] && (q0.conflict || q1.conflict);
+      } else {
+        atr_list_validate(p, c, sn[j], t, mine[j], id0[j], id1[j], ovf, conflict);
       }
-      bool ovf = mine[j] && (q0.unknown || q1.unknown);
-      bool conflict = mine[j] && (q0.conflict || q1.conflict);
       if (p.debug & CSMV_DBG_NO_VALIDATE) ovf = conflict = false;
       const bool commit = mine[j] && !ovf && !conflict;
       cm[j] = __ballot_sync(FULL, commit);
@@ -356,10 +407,14 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       const uint32_t cts = t + 1 + __popc(cm[j] & lt);
       t += __popc(cm[j]);
       if (commit) {
-        p.lastw[id0[j]] = cts;
-        p.lastw[id1[j]] = cts;
-        rt_record<CL>(c, bk0[j], q0.way, id0[j], cts);
-        rt_record<CL>(c, bk1[j], q1.way, id1[j], cts);
+        if (p.atr_mode == CSMV_ATR_HASH) {
+          p.lastw[id0[j]] = cts;
+          p.lastw[id1[j]] = cts;
+          rt_record<CL>(c, bk0[j], q0.way, id0[j], cts);
+          rt_record<CL>(c, bk1[j], q1.way, id1[j], cts);
+        } else {  // the paper's ATR: the write-set of commit `cts` at entry cts
+          c.rt[cts & ((uint32_t)(kRtWays << (p.rt_log2 - p.clog2)) - 1)] = ((uint64_t)id1[j] << 32) | id0[j];
+        }
       }
       __syncwarp();  // batch j's records precede batch j+1's probes
     }
