@@ -63,9 +63,21 @@ extern "C" {
 #define CSMV_ATR_LIST 1u       /* the paper's ATR: list of write-sets, collaborative validation */
 #define CSMV_ATR_LIST_NOCV 2u  /* the list ATR, one lane per transaction (CSMV-NoCV) */
 
+/* commit protocol (csmv_workload.commit) */
+#define CSMV_COMMIT_CSMV 0u    /* the paper's client-server batched commit */
+#define CSMV_COMMIT_ONLYCS 1u  /* CSMV-onlyCS ablation: the client-server design alone --
+                                  list ATR scanned per transaction (no CV), no client pre-validation,
+                                  one ATR insert per transaction, server-side write-back.  Bank only,
+                                  single-CTA server; atr_mode is ignored */
+#define CSMV_COMMIT_JVSTM 2u   /* JVSTM-GPU baseline: no server; every thread validates
+                                  against a global-memory ATR, reserves its CTS with a global CAS,
+                                  writes back and advances GTS in order itself.  Bank only */
+
 #define CSMV_DBG_NO_PREVAL 1u  /* negative control: skip client pre-validation */
 #define CSMV_DBG_NO_VALIDATE 2u/* negative control: server commits without validating */
 #define CSMV_DBG_JITTER 4u     /* random __nanosleep in client and server */
+#define CSMV_DBG_PHASES 8u     /* per-phase client clocks (csmv_stats_t.client_phase_cycles) */
+#define CSMV_DBG_KV_COMPACT 16u/* KV: ship PUT read-sets as {set clock} u WS at any ways (always above 16) */
 
 typedef struct csmv_workload {
     uint32_t kind;             /* CSMV_KIND_* */
@@ -92,6 +104,7 @@ typedef struct csmv_workload {
     uint32_t log_mode;         /* CSMV_LOG_* */
     uint32_t debug_flags;      /* CSMV_DBG_* */
     uint32_t watchdog_ms;      /* 0 = default (20000) */
+    uint32_t commit;           /* CSMV_COMMIT_* (0 = the paper's CSMV) */
 } csmv_workload;
 
 /* ---- statistics ---- */
@@ -118,6 +131,10 @@ typedef struct csmv_stats {
     uint64_t server_lock_cycles; /* cycles the commit critical section was held */
     uint64_t server_busy_cycles; /* cycles workers spent processing batches */
     uint64_t server_phase_cycles[8]; /* worker: queue wait, payload load, lock wait, critical section, respond */
+    uint64_t cas_failures;     /* CSMV_COMMIT_JVSTM: failed CTS reservations (global CAS) */
+    uint64_t client_phase_cycles[8]; /* CSMV_DBG_PHASES, summed over client warps (mean lane): read,
+                                    pre-validation | JVSTM validation+CAS, submit, read-only txs,
+                                    wait for server, write-back, GTS publish, divergence (JVSTM) */
     uint32_t client_warps;
     uint32_t server_ctas;
     uint32_t server_workers;

@@ -22,7 +22,9 @@ LOG_NONE, LOG_DIGEST, LOG_FULL = 0, 1, 2
 SERVER_CTA, SERVER_CLUSTER = 0, 1
 PUBLISH_CLIENT, PUBLISH_SERVER = 0, 1
 ATR_HASH, ATR_LIST, ATR_LIST_NOCV = 0, 1, 2
-DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER = 1, 2, 4
+COMMIT_CSMV, COMMIT_ONLYCS, COMMIT_JVSTM = 0, 1, 2
+DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER, DBG_PHASES, DBG_KV_COMPACT = 1, 2, 4, 8, 16
+CLIENT_PHASES = ("read", "preval", "submit", "rot", "wait_server", "writeback", "publish", "divergence")
 ABORT_REASONS = ("preval", "conflict", "early", "overflow", "version")
 
 LOG_DTYPE = np.dtype([("tx", "<u4"), ("snapshot", "<u4"), ("cts", "<u4"),
@@ -39,7 +41,7 @@ class _Workload(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in (
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
         "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers", "server_combine",
-        "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms")]
+        "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms", "commit")]
 
 
 class _Stats(C.Structure):
@@ -50,7 +52,8 @@ class _Stats(C.Structure):
                 ("elapsed_ns", C.c_uint64), ("ro_checksum", C.c_uint64),
                 ("store_bytes", C.c_uint64), ("store_bytes_paper", C.c_uint64),
                 ("server_lock_cycles", C.c_uint64), ("server_busy_cycles", C.c_uint64),
-                ("server_phase_cycles", C.c_uint64 * 8),
+                ("server_phase_cycles", C.c_uint64 * 8), ("cas_failures", C.c_uint64),
+                ("client_phase_cycles", C.c_uint64 * 8),
                 ("client_warps", C.c_uint32), ("server_ctas", C.c_uint32),
                 ("server_workers", C.c_uint32), ("atr_entries", C.c_uint32),
                 ("sm_count", C.c_uint32), ("kernel_launches", C.c_uint32)]
@@ -81,6 +84,7 @@ class Workload:
     log_mode: int = LOG_NONE
     debug_flags: int = 0
     watchdog_ms: int = 0
+    commit: int = COMMIT_CSMV
 
     def to_c(self) -> _Workload:
         return _Workload(*[getattr(self, f.name) for f in fields(self)])
@@ -132,7 +136,9 @@ def _ptr(a: np.ndarray):
 
 
 def stats_dict(s: _Stats) -> dict:
-    d = {f: getattr(s, f) for f, _ in _Stats._fields_ if f not in ("aborts", "server_phase_cycles")}
+    d = {f: getattr(s, f) for f, _ in _Stats._fields_
+         if f not in ("aborts", "server_phase_cycles", "client_phase_cycles")}
+    d["client_phase_cycles"] = dict(zip(CLIENT_PHASES, list(s.client_phase_cycles)))
     d["server_phase_cycles"] = dict(zip(("queue", "load", "lock_wait", "critical", "respond", "cs_validate", "cs_insert0", "cs_insert1"),
                                         list(s.server_phase_cycles)))
     d["aborts"] = {ABORT_REASONS[i]: {"ro": s.aborts[i][0], "update": s.aborts[i][1]}

@@ -15,11 +15,68 @@
 //   D  the response, client write-back, GTS advance.
 // An update rejected by the server may sit out `backoff` rounds
 // (backoff_max > 0); its lane keeps running read-only transactions.
+//
+// Commit-protocol ablations:
+//   CSMV_COMMIT_ONLYCS  B skips pre-validation and ships the new values; the
+//                       server validates, inserts and writes back one
+//                       transaction at a time (server_worker_onlycs);
+//   CSMV_COMMIT_JVSTM   no server: B is replaced by jv_commit, each lane
+//                       validating against the global ATR and reserving its
+//                       CTS with a global CAS, then writing back and
+//                       advancing GTS in CTS order itself (lane-divergent).
 #pragma once
 
 namespace csmvd {
 
 constexpr uint64_t kNoTx = ~0ull;
+
+// JVSTM-GPU commit of one transaction with snapshot s and RS = WS = {a, b}
+// (JVSTM's lock-free commit ported per thread): validate against
+// every record of the global ATR after s, reserve CTS t+1 with
+// a CAS on the ATR tail t, re-validating the records that appeared when the
+// CAS fails, then publish the write-set record at entry t+1.  Returns the
+// CTS, or 0 with `reason` set (CONFLICT; OVERFLOW when the ring no longer
+// holds every record after s; -1 if the run is being torn down).  Entry c is
+// overwritten only by CTS c + R, which needs tail >= c + R; the tail is <= t
+// throughout a scan that ends in a successful CAS at t, so t - s < R proves
+// every record read was the one of its CTS.
+__device__ __forceinline__ uint32_t jv_commit(const KParams& p, uint32_t s, uint32_t a, uint32_t b, int& reason,
+                                              uint32_t& fails, uint64_t t_begin) {
+  const uint32_t R = 1u << p.jv_log2, M = R - 1;
+  uint32_t t = ld_acquire(&p.ctl->jv_tail);
+  uint32_t q = s;
+  for (;;) {
+    if (t - s >= R) {
+      reason = CSMV_AB_OVERFLOW;
+      return 0;
+    }
+    for (uint32_t c = q + 1; c - 1 < t; ++c) {  // records (q, t]
+      uint32_t it = 0;
+      while (ld_acquire(p.jv_tag + (c & M)) != c) {
+        if ((++it & 1023u) == 0 && (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 6))) {
+          reason = -1;
+          return 0;
+        }
+        __nanosleep(32);
+      }
+      const uint64_t e = ld_relaxed64(p.jv_ws + (c & M));
+      const uint32_t w0 = (uint32_t)e, w1 = (uint32_t)(e >> 32);
+      if (!(p.debug & CSMV_DBG_NO_VALIDATE) && (w0 == a || w0 == b || w1 == a || w1 == b)) {
+        reason = CSMV_AB_CONFLICT;
+        return 0;
+      }
+    }
+    const uint32_t old = atomicCAS(&p.ctl->jv_tail, t, t + 1);
+    if (old == t) break;
+    ++fails;
+    q = t;
+    t = old;
+  }
+  const uint32_t cts = t + 1;
+  st_relaxed64(p.jv_ws + (cts & M), ((uint64_t)b << 32) | a);
+  st_release(p.jv_tag + (cts & M), cts);
+  return cts;
+}
 
 template <int NS>
 __device__ void client_warp(const KParams& p, uint64_t t_begin) {
@@ -37,9 +94,11 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
   const uint32_t K = p.K;
   const uint32_t lt = lanemask_lt();
   const uint32_t streak = p.ro_streak;
+  PhaseClock pc((p.debug & CSMV_DBG_PHASES) != 0);
 
   for (;;) {
     if (!__any_sync(FULL, cu != kNoTx || cr < p.n_tx)) break;
+    pc.start();
     ++round;
     ++cc.n_rounds;
     uint32_t s = 0, err = 0;
@@ -84,10 +143,47 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
       }
     }
 
+    pc.mark(PH_READ);
+    if (p.commit == CSMV_COMMIT_JVSTM) {
+      // ---- B': decentralized commit, every lane on its own
+      if (status == ST_CAND) {
+        int reason = 0;
+        const uint32_t cts = jv_commit(p, s, d.src, d.dst, reason, cc.cas_fail, t_begin);
+        pc.mark(PH_PREVAL);
+        if (cts) {
+          const uint32_t ns = vs - (uint32_t)d.amt, nd = vd + (uint32_t)d.amt;
+          write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
+          write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
+          pc.mark(PH_WRITEBACK);
+          if (p.log_mode) {
+            log_commit(p, cu, s, cts, att_u, dig1(d.src, vs) + dig1(d.dst, vd), dig1(d.src, ns) + dig1(d.dst, nd));
+            if (p.log_mode == CSMV_LOG_FULL && p.max_vals >= 2) {
+              p.vals[cu * p.max_vals] = vs;
+              p.vals[cu * p.max_vals + 1] = vd;
+            }
+          }
+          // in-order GTS advance by this thread
+          uint32_t it = 0;
+          while (ld_relaxed(p.gts) != cts - 1) {
+            if ((++it & 1023u) == 0 && (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 7))) break;
+            __nanosleep(32);
+          }
+          st_release(p.gts, cts);
+          pc.mark(PH_PUBLISH);
+          ++cc.c_upd;
+          cu = kNoTx;
+          att_u = 0;
+        } else if (reason >= 0) {
+          cc.abort(reason, true);
+        }
+      }
+      __syncwarp();
+      pc.mark(PH_DIVERGENCE);
+    }
     // ---- B: pre-validation, greedy in lane order (RS = WS = {src, dst})
-    const uint32_t cand = __ballot_sync(FULL, status == ST_CAND);
+    const uint32_t cand = p.commit == CSMV_COMMIT_JVSTM ? 0u : __ballot_sync(FULL, status == ST_CAND);
     uint32_t kept = cand;
-    if (!(p.debug & CSMV_DBG_NO_PREVAL)) {
+    if (!(p.debug & CSMV_DBG_NO_PREVAL) && p.commit == CSMV_COMMIT_CSMV) {
       kept = 0;
       uint32_t rem = cand;
       while (rem) {
@@ -101,10 +197,15 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
     }
     const bool mine = (kept >> lane) & 1u;
     if (status == ST_CAND && !mine) cc.abort(CSMV_AB_PREVAL, true);
+    if (p.commit != CSMV_COMMIT_JVSTM) pc.mark(PH_PREVAL);
     if (kept) {
       if (mine) {
         my_ids[lane] = d.src | kWriteBit;
         my_ids[32 + lane] = d.dst | kWriteBit;
+        if (p.commit == CSMV_COMMIT_ONLYCS) {  // the server writes back
+          p.req_vals[(size_t)cw * 64 + lane] = vs - (uint32_t)d.amt;
+          p.req_vals[(size_t)cw * 64 + 32 + lane] = vd + (uint32_t)d.amt;
+        }
       }
       if (lane == 0) {
         p.req_hdr[cw].snapshot = s;
@@ -113,6 +214,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
       __syncwarp();
       fence_gpu();
       if (lane == 0) st_relaxed(&p.req_seq[cw], round);
+      pc.mark(PH_SUBMIT);
     }
 
     // ---- C: read-only transactions at s
@@ -137,6 +239,8 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         att_r = 0;
       }
     }
+    __syncwarp();
+    pc.mark(PH_ROT);
     if (!kept) continue;
 
     // ---- D: the server's answer, write-back, GTS
@@ -162,14 +266,17 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         omask = ld_relaxed(&p.resp[cw].overflow_mask);
       }
     }
+    pc.mark(PH_WAIT);
     uint32_t cts = 0;
     if (mine) {
       if ((cmask >> lane) & 1u) {
         // Client-side write-back with CTS = base + rank.
         cts = base + __popc(cmask & lt);
         const uint32_t ns = vs - (uint32_t)d.amt, nd = vd + (uint32_t)d.amt;
-        write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
-        write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
+        if (p.commit != CSMV_COMMIT_ONLYCS) {
+          write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
+          write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
+        }
         if (p.log_mode) {
           log_commit(p, cu, s, cts, att_u, dig1(d.src, vs) + dig1(d.dst, vd), dig1(d.src, ns) + dig1(d.dst, nd));
           if (p.log_mode == CSMV_LOG_FULL && p.max_vals >= 2) {
@@ -187,6 +294,8 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         if (!ovf && p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
       }
     }
+    __syncwarp();
+    pc.mark(PH_WRITEBACK);
     const uint32_t n = __popc(cmask);
     if (n) {
       if (p.publish == CSMV_PUBLISH_CLIENT) {
@@ -204,12 +313,14 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
           __nanosleep(32);
         }
         if (lane == 0) st_release(p.gts, base + n - 1);  // release also orders the write-backs
-      } else if (cts) {
+      } else if (cts && p.commit != CSMV_COMMIT_ONLYCS) {
         st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
       }
     }
+    pc.mark(PH_PUBLISH);
   }
   client_flush(p, cc);
+  pc.flush(p);
 }
 
 }  // namespace csmvd

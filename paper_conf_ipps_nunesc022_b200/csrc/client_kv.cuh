@@ -1,6 +1,17 @@
 // client_kv.cuh -- the client warp of the MemcachedGPU workload.
 // Same lane state machine and round phases as client_bank.cuh; GET is the
 // read-only transaction, PUT the update transaction (docs/GENERATOR.md 4).
+//
+// Read-set representation.  With A <= kKvFullWays the PUT's read-set is
+// tracked item by item (smem scratch) and shipped whole, as in the paper.
+// Above that (up to 256 ways) -- or with CSMV_DBG_KV_COMPACT -- it is
+// shipped as {set clock} u WS: every item a PUT reads lies in its set t,
+// every PUT on set t reads and writes clock[t], and nothing else writes an
+// item of set t, so "a commit after s wrote an item of RS u WS" holds iff
+// "a commit after s wrote clock[t]" -- validation and
+// pre-validation (two PUTs conflict iff same set) decide exactly as
+// with the full sets (DESIGN.md readings; the 1-warp tests compare both
+// against the item-level reference predictor).
 #pragma once
 
 namespace csmvd {
@@ -51,6 +62,8 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
   const uint32_t K = p.K, S = p.kv_S, A = p.kv_A, Tn = p.kv_T;
   const uint32_t lt = lanemask_lt();
   const uint32_t streak = p.ro_streak;
+  const bool compact = A > kKvFullWays || (p.debug & CSMV_DBG_KV_COMPACT);
+  PhaseClock pc((p.debug & CSMV_DBG_PHASES) != 0);
   // per-warp smem scratch, lane-minor: RS[kKvMaxRs][32], WS[4][32], NRS[32]
   uint32_t* RS = scratch + (size_t)wib * 32 * (kKvMaxRs + 5);
   uint32_t* WS = RS + kKvMaxRs * 32;
@@ -59,6 +72,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
 
   for (;;) {
     if (!__any_sync(FULL, cu != kNoTx || cr < p.n_tx)) break;
+    pc.start();
     ++round;
     ++cc.n_rounds;
     uint32_t s = 0, err = 0;
@@ -95,7 +109,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           uint32_t key[4];
           r = kv_read_mw<NS, 4>(p.kv_key + (size_t)slot * NS * 4, K, s, false, key);
           if (r != RD_OK) break;
-          RS[nrs++ * 32 + lane] = slot;
+          if (!compact) RS[nrs++ * 32 + lane] = slot;
 #pragma unroll
           for (int j = 0; j < 4; ++j) rdig += dig_word(slot, j, key[j]);
           if ((key[0] == kk[0] && key[1] == kk[1] && key[2] == kk[2] && key[3] == kk[3]) ||
@@ -109,7 +123,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
             uint32_t l;
             r = kv_read_1<NS>(p.kv_lru + (size_t)slot * NS, K, s, l);
             if (r != RD_OK) break;
-            RS[nrs++ * 32 + lane] = 2 * S + slot;
+            if (!compact) RS[nrs++ * 32 + lane] = 2 * S + slot;
             rdig += dig1(2 * S + slot, l);
             if (w == 0 || l < best) {
               best = l;
@@ -120,7 +134,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         if (r == RD_OK) {
           r = kv_read_1<NS>(p.kv_clk + (size_t)tset * NS, K, s, clk);
           if (r == RD_OK) {
-            RS[nrs++ * 32 + lane] = 3 * S + tset;
+            if (!compact) RS[nrs++ * 32 + lane] = 3 * S + tset;
             rdig += dig1(3 * S + tset, clk);
           }
         }
@@ -132,22 +146,34 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           cc.abort(CSMV_AB_VERSION, true);
           status = ST_ABORT;
         } else {
-          WS[0 * 32 + lane] = victim;
-          WS[1 * 32 + lane] = S + victim;
-          WS[2 * 32 + lane] = 2 * S + victim;
-          WS[3 * 32 + lane] = 3 * S + tset;
-          NRS[lane] = nrs;
+          if (!compact) {
+            WS[0 * 32 + lane] = victim;
+            WS[1 * 32 + lane] = S + victim;
+            WS[2 * 32 + lane] = 2 * S + victim;
+            WS[3 * 32 + lane] = 3 * S + tset;
+            NRS[lane] = nrs;
+          }
           status = ST_CAND;
         }
       }
     }
     __syncwarp();
+    pc.mark(PH_READ);
 
     // ---- B: pre-validation: lane j is dropped if WS_i n (RS_j u WS_j)
     // or WS_j n RS_i is non-empty for an earlier kept lane i
     const uint32_t cand = __ballot_sync(FULL, status == ST_CAND);
     uint32_t kept = cand;
-    if (!(p.debug & CSMV_DBG_NO_PREVAL)) {
+    if (!(p.debug & CSMV_DBG_NO_PREVAL) && compact) {
+      kept = 0;
+      uint32_t rem = cand;
+      while (rem) {  // same set <=> conflicting read/write sets
+        const int i = __ffs(rem) - 1;
+        kept |= 1u << i;
+        const uint32_t ti = __shfl_sync(FULL, tset, i);
+        rem &= ~__ballot_sync(FULL, ((rem >> lane) & 1u) && lane > (uint32_t)i && tset == ti) & ~(1u << i);
+      }
+    } else if (!(p.debug & CSMV_DBG_NO_PREVAL)) {
       kept = 0;
       uint32_t rem = cand;
       while (rem) {
@@ -171,7 +197,14 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     }
     const bool mine = (kept >> lane) & 1u;
     if (status == ST_CAND && !mine) cc.abort(CSMV_AB_PREVAL, true);
-    if (kept && mine) {
+    pc.mark(PH_PREVAL);
+    if (kept && mine && compact) {
+      my_ids[0 * 32 + lane] = (3 * S + tset) | kWriteBit;  // read and written: stands for the set
+      my_ids[1 * 32 + lane] = victim | kWriteBit;
+      my_ids[2 * 32 + lane] = (S + victim) | kWriteBit;
+      my_ids[3 * 32 + lane] = (2 * S + victim) | kWriteBit;
+      p.req_cnt[(size_t)cw * 32 + lane] = 4;
+    } else if (kept && mine) {
       // request ids: RS u WS (bit 31: in WS)
       uint32_t n = 0;
       for (uint32_t b = 0; b < nrs; ++b) {
@@ -198,6 +231,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       __syncwarp();
       fence_gpu();
       if (lane == 0) st_relaxed(&p.req_seq[cw], round);
+      pc.mark(PH_SUBMIT);
     }
 
     // ---- C: GETs at s while the batch is at the server
@@ -222,6 +256,8 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         att_r = 0;
       }
     }
+    __syncwarp();
+    pc.mark(PH_ROT);
     if (!kept) continue;
 
     // ---- D: response, write-back, GTS
@@ -247,6 +283,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         omask = ld_relaxed(&p.resp[cw].overflow_mask);
       }
     }
+    pc.mark(PH_WAIT);
     uint32_t cts = 0;
     if (mine) {
       if ((cmask >> lane) & 1u) {
@@ -275,6 +312,8 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         if (!ovf && p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
       }
     }
+    __syncwarp();
+    pc.mark(PH_WRITEBACK);
     const uint32_t n = __popc(cmask);
     if (n) {
       if (p.publish == CSMV_PUBLISH_CLIENT) {
@@ -294,8 +333,10 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
       }
     }
+    pc.mark(PH_PUBLISH);
   }
   client_flush(p, cc);
+  pc.flush(p);
 }
 
 }  // namespace csmvd

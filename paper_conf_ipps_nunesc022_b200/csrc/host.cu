@@ -87,6 +87,9 @@ struct csmv {
   uint32_t* d_req_ids = nullptr;
   uint32_t* d_req_cnt = nullptr;
   Resp* d_resp = nullptr;
+  uint32_t* d_req_vals = nullptr;  // CSMV_COMMIT_ONLYCS (bank)
+  uint64_t* d_jv_ws = nullptr;     // CSMV_COMMIT_JVSTM global ATR (allocated on first use)
+  uint32_t* d_jv_tag = nullptr;
   // logs
   csmv_log_rec* d_log = nullptr;
   uint64_t log_cap = 0;
@@ -105,7 +108,7 @@ struct csmv {
 static void free_all(csmv* h) {
   void* ps[] = {h->d_rings, h->d_key, h->d_val, h->d_lru, h->d_clk, h->d_lastw, h->d_gts, h->d_ctl,
                 h->d_stats, h->d_done, h->d_req_seq, h->d_req_hdr, h->d_req_ids, h->d_req_cnt,
-                h->d_resp, h->d_log, h->d_vals, h->d_zipf};
+                h->d_resp, h->d_log, h->d_vals, h->d_zipf, h->d_req_vals, h->d_jv_ws, h->d_jv_tag};
   for (void* q : ps) cudaFree(q);
   if (h->ev0) cudaEventDestroy(h->ev0);
   if (h->ev1) cudaEventDestroy(h->ev1);
@@ -180,6 +183,8 @@ csmv_t* csmv_create(uint64_t n_items, uint32_t n_versions) {
   h->maxid = 2;
   if (cudaMalloc(&h->d_rings, n_items * h->nslot * sizeof(uint64_t)) != cudaSuccess) return create_fail(h, "rings");
   if (!alloc_common(h)) return create_fail(h, "control buffers");
+  if (cudaMalloc(&h->d_req_vals, (size_t)h->max_cw * 64 * sizeof(uint32_t)) != cudaSuccess)
+    return create_fail(h, "request values");
   return h;
 }
 
@@ -361,6 +366,15 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (w->atr_mode != CSMV_ATR_HASH && (h->kind != CSMV_KIND_BANK || w->server != CSMV_SERVER_CTA))
     return set_err(CSMV_EINVAL, "csmv_run: the list ATR is built for the bank workload on the single-CTA server");
   if (n_tx >= (1ull << 32)) return set_err(CSMV_EINVAL, "csmv_run: n_tx must be < 2^32");
+  if (w->commit > CSMV_COMMIT_JVSTM) return set_err(CSMV_EINVAL, "csmv_run: unknown commit %u", w->commit);
+  const bool jvstm = w->commit == CSMV_COMMIT_JVSTM;
+  if (w->commit != CSMV_COMMIT_CSMV && (h->kind != CSMV_KIND_BANK || w->server != CSMV_SERVER_CTA))
+    return set_err(CSMV_EINVAL, "csmv_run: the onlyCS / JVSTM-GPU ablations are built for the bank workload "
+                                "with the single-CTA server setting");
+  if (jvstm && !h->d_jv_ws) {
+    CK(cudaMalloc(&h->d_jv_ws, sizeof(uint64_t) << kJvLog2));
+    CK(cudaMalloc(&h->d_jv_tag, sizeof(uint32_t) << kJvLog2));
+  }
 
   uint32_t gts0 = 0;
   CK(cudaMemcpyAsync(&gts0, h->d_gts, 4, cudaMemcpyDeviceToHost, h->stream));
@@ -373,8 +387,9 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   int rc = make_gen(h, w, seed, &p.gen);
   if (rc) return rc;
 
-  // server: one CTA or a thread-block cluster of C CTAs (DSMEM)
-  uint32_t n_srv = 1, clog2 = 0;
+  // server: one CTA, a thread-block cluster of C CTAs (DSMEM), or
+  // none (JVSTM-GPU: every CTA is a client)
+  uint32_t n_srv = jvstm ? 0u : 1u, clog2 = 0;
   if (w->server == CSMV_SERVER_CLUSTER) {
     n_srv = w->cluster_size ? w->cluster_size : 16u;
     if (n_srv < 2 || n_srv > 16 || (n_srv & (n_srv - 1)))
@@ -395,7 +410,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   uint32_t entries = w->atr_capacity ? w->atr_capacity : 16384u * n_srv;
   uint32_t rt_log2 = clog2 + 1;
   while ((4u << rt_log2) < entries && rt_log2 < 12 + clog2) ++rt_log2;
-  const uint32_t per_srv = (n_cw + n_srv - 1) / n_srv;
+  const uint32_t per_srv = n_srv ? (n_cw + n_srv - 1) / n_srv : 0u;
   size_t smem = server_smem_bytes(rt_log2 - clog2, per_srv);
   if (h->kind == CSMV_KIND_KV && smem < kv_client_smem_bytes()) smem = kv_client_smem_bytes();
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
@@ -412,7 +427,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (n_cw > max_client_ctas * kWarps) n_cw = max_client_ctas * kWarps;
   uint32_t n_ctas = n_cw < max_client_ctas ? n_cw : max_client_ctas;
   if (n_srv > 1) n_ctas = (n_ctas + n_srv - 1) / n_srv * n_srv;  // grid a multiple of the cluster
-  if (n_ctas > max_client_ctas) n_ctas = max_client_ctas / n_srv * n_srv;
+  if (n_srv > 1 && n_ctas > max_client_ctas) n_ctas = max_client_ctas / n_srv * n_srv;
 
   // logs
   uint32_t max_vals = 0;
@@ -477,9 +492,18 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.atr_mode = w->atr_mode;
   p.backoff_max = w->backoff_max;
   p.debug = w->debug_flags;
+  p.commit = w->commit;
+  p.req_vals = h->d_req_vals;
+  p.jv_ws = h->d_jv_ws;
+  p.jv_tag = h->d_jv_tag;
+  p.jv_log2 = kJvLog2;
   p.watchdog_ns = (uint64_t)(w->watchdog_ms ? w->watchdog_ms : 20000u) * 1000000ull;
 
   CK(cudaMemsetAsync(h->d_ctl, 0, sizeof(Ctl), h->stream));
+  if (jvstm) {  // the global ATR starts empty at the current GTS
+    CK(cudaMemcpyAsync(&h->d_ctl->jv_tail, &gts0, 4, cudaMemcpyHostToDevice, h->stream));
+    CK(cudaMemsetAsync(h->d_jv_tag, 0, sizeof(uint32_t) << kJvLog2, h->stream));
+  }
   CK(cudaMemsetAsync(h->d_stats, 0, sizeof(DevStats), h->stream));
   CK(cudaMemsetAsync(h->d_req_seq, 0, n_cw * sizeof(uint32_t), h->stream));
   CK(cudaMemsetAsync(h->d_resp, 0, n_cw * sizeof(Resp), h->stream));
@@ -521,6 +545,9 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   s.server_lock_cycles = ds.lock_cycles;
   s.server_busy_cycles = ds.busy_cycles;
   for (int i = 0; i < 8; ++i) s.server_phase_cycles[i] = ds.phase[i];
+  s.cas_failures = ds.cas_fail;
+  for (int i = 0; i < 8; ++i) s.client_phase_cycles[i] = ds.client_phase[i];
+  if (jvstm) ctl.tail_final = ctl.jv_tail;
   s.client_warps = n_cw;
   s.server_ctas = n_srv;
   s.server_workers = n_workers;

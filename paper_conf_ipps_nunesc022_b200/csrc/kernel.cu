@@ -161,7 +161,7 @@ __device__ __forceinline__ bool rot_scan(const KParams& p, uint32_t start, uint3
 // Client warp
 // --------------------------------------------------------------------------
 struct ClientCounters {
-  uint32_t c_upd = 0, c_ro = 0, n_rounds = 0;
+  uint32_t c_upd = 0, c_ro = 0, n_rounds = 0, cas_fail = 0;
   uint32_t ab[CSMV_N_ABORT][2];
   uint64_t ro_ck = 0;
   __device__ ClientCounters() {
@@ -172,6 +172,53 @@ struct ClientCounters {
 #pragma unroll
     for (int i = 0; i < (int)CSMV_N_ABORT; ++i)
       if (reason == i) ++ab[i][upd ? 1 : 0];
+  }
+};
+
+// Per-phase client clocks (CSMV_DBG_PHASES; the shape of Tables I and III,
+// P:136-147).  Every lane accumulates; the flush reports the
+// mean over lanes, so warp-convergent phases read as the warp's time and
+// lane-divergent ones (JVSTM-GPU) as the mean lane's.
+enum : int {
+  PH_READ = 0,     // A: snapshot + update reads
+  PH_PREVAL,       // B: pre-validation          | JVSTM: validation + CTS CAS
+  PH_SUBMIT,       // B: request + doorbell      | JVSTM: ATR record insert
+  PH_ROT,          // C: read-only transactions
+  PH_WAIT,         // D: waiting for the server
+  PH_WRITEBACK,    // D: write-back
+  PH_PUBLISH,      // D: GTS advance / done flag
+  PH_DIVERGENCE,   // JVSTM: a lane's wait from its own commit end to reconvergence
+};
+
+struct PhaseClock {
+  unsigned long long ph[8];
+  long long t;
+  bool on;
+  __device__ explicit PhaseClock(bool enabled) : t(0), on(enabled) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) ph[i] = 0;
+  }
+  __device__ __forceinline__ void start() {
+    if (on) t = clock64();
+  }
+  __device__ __forceinline__ void mark(int k) {
+    if (on) {
+      const long long n = clock64();
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        if (i == k) ph[i] += (unsigned long long)(n - t);
+      t = n;
+    }
+  }
+  __device__ __forceinline__ void flush(const KParams& p) const {
+    if (!on) return;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      unsigned long long v = ph[i];
+#pragma unroll
+      for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, o);
+      if ((threadIdx.x & 31) == 0 && v) atomicAdd(&p.stats->client_phase[i], v / 32);
+    }
   }
 };
 
@@ -192,6 +239,7 @@ __device__ __forceinline__ void client_flush(const KParams& p, const ClientCount
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t s_upd = __reduce_add_sync(FULL, cc.c_upd), s_ro = __reduce_add_sync(FULL, cc.c_ro);
+  const uint32_t s_cf = __reduce_add_sync(FULL, cc.cas_fail);
   uint32_t s_ab[CSMV_N_ABORT][2];
 #pragma unroll
   for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
@@ -209,6 +257,7 @@ __device__ __forceinline__ void client_flush(const KParams& p, const ClientCount
       if (s_ab[i][1]) atomicAdd(&p.stats->aborts[i][1], (unsigned long long)s_ab[i][1]);
     }
     atomicAdd(&p.stats->rounds, (unsigned long long)cc.n_rounds);
+    if (s_cf) atomicAdd(&p.stats->cas_fail, (unsigned long long)s_cf);
     atomicXor(&p.stats->ro_checksum, (unsigned long long)ro_ck);
     __threadfence();
     atomicAdd(&p.ctl->done_warps, 1u);
@@ -233,7 +282,7 @@ template <int NS, int KIND, bool CL>
 __global__ void __launch_bounds__(kBlock, 1) csmv_fused(const KParams p) {
   extern __shared__ __align__(16) uint8_t smem[];
   const uint64_t t_begin = globaltimer();
-  if (blockIdx.x < p.n_server_ctas) server_cta<KIND, CL>(p, smem, t_begin);
+  if (blockIdx.x < p.n_server_ctas) server_cta<NS, KIND, CL>(p, smem, t_begin);
   else if constexpr (KIND == CSMV_KIND_KV) client_warp_kv<NS>(p, t_begin, reinterpret_cast<uint32_t*>(smem));
   else client_warp<NS>(p, t_begin);
 }

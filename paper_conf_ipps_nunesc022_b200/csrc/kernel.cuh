@@ -15,6 +15,8 @@
 //   lastw     u32[n_items]          CTS of the last commit that wrote the item
 //                                   (server-private level of the ATR)
 //   log       csmv_log_rec[n_tx]    parity runs only
+//   req_vals  u32[n_cw][2][32]      CSMV_COMMIT_ONLYCS: values for the server write-back
+//   jv_ws/jv_tag u64/u32[2^22]      CSMV_COMMIT_JVSTM: the global-memory ATR
 #pragma once
 #include <cstdint>
 
@@ -35,6 +37,7 @@ struct Ctl {
   uint32_t done_warps;  // client warps that finished
   uint32_t tail_final;  // server: last CTS assigned
   uint32_t where;       // which spin loop fired the watchdog
+  uint32_t jv_tail;     // CSMV_COMMIT_JVSTM: last CTS reserved (global CAS target)
 };
 
 struct ReqHdr {
@@ -56,6 +59,8 @@ struct DevStats {
   unsigned long long ro_checksum;
   unsigned long long lock_cycles, busy_cycles;
   unsigned long long phase[8];  // server worker: queue wait, load, lock wait, critical, respond
+  unsigned long long cas_fail;  // CSMV_COMMIT_JVSTM: failed CTS reservations
+  unsigned long long client_phase[8];  // CSMV_DBG_PHASES: client cycles by phase (mean lane)
 };
 
 struct KParams {
@@ -99,11 +104,18 @@ struct KParams {
   uint64_t* kv_clk;           // u64[T][NS]
   uint32_t* req_cnt;          // ids per lane [n_cw][32] (generic requests)
   uint32_t maxid;             // id rows per request slot
+  // commit-protocol ablations (CSMV_COMMIT_*)
+  uint32_t commit;
+  uint32_t* req_vals;         // ONLYCS: new values [n_cw][2][32] for the server-side write-back
+  uint64_t* jv_ws;            // JVSTM: global ATR, write-set of CTS c at c & (2^jv_log2 - 1)
+  uint32_t* jv_tag;           //        entry tag = c once the record of c is written
+  uint32_t jv_log2;
 };
 
-constexpr uint32_t kKvMaxWays = 16;               // KV ways supported by the device path
-constexpr uint32_t kKvMaxRs = 2 * kKvMaxWays + 1;  // keys + LRU stamps + clock
-constexpr uint32_t kKvMaxId = 2 * kKvMaxWays + 2;  // RS u WS
+constexpr uint32_t kKvMaxWays = 256;              // KV ways supported by the device path
+constexpr uint32_t kKvFullWays = 16;              // up to here PUT read-sets are shipped item by item
+constexpr uint32_t kKvMaxRs = 2 * kKvFullWays + 1;  // keys + LRU stamps + clock
+constexpr uint32_t kKvMaxId = 2 * kKvFullWays + 2;  // RS u WS
 
 // client smem scratch per warp (KV read/write sets of its update lanes)
 inline size_t kv_client_smem_bytes() { return (size_t)kWarps * 32 * (kKvMaxRs + 4 + 1) * 4; }
@@ -124,6 +136,8 @@ inline size_t server_smem_bytes(uint32_t local_log2, uint32_t n_cw) {
 }
 
 // host-callable launchers (kernel.cu)
+constexpr uint32_t kJvLog2 = 22;       // JVSTM global ATR entries
+
 cudaError_t launch_fused(const KParams& p, uint32_t nslot, uint32_t grid, size_t smem,
                          cudaStream_t st);
 cudaError_t launch_init_rings(uint64_t* rings, uint32_t nslot, const int32_t* init, uint64_t n,

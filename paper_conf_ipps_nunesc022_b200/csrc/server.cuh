@@ -472,8 +472,10 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t lt = lanemask_lt();
   unsigned long long busy = 0, locked = 0, batches = 0;
+  unsigned long long ph[5] = {0, 0, 0, 0, 0};
   for (;;) {
     uint32_t cw;
+    const long long tq = clock64();
     if (!claim_request(c, cw)) break;
     const long long t0 = clock64();
     const uint32_t sq = ld_relaxed(p.req_seq + cw);
@@ -490,6 +492,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
 #pragma unroll
     for (uint32_t k = 0; k < kKvMaxId; ++k) x ^= ids[k];
     if (__ballot_sync(FULL, x == 0x12345679u) == FULL) __nanosleep(1);
+    const long long tl = clock64();
     // ---- critical section
     const uint32_t ticket = cs_enter<CL>(c);
     const long long t1 = clock64();
@@ -517,6 +520,111 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
       st_relaxed(&p.resp[cw].cts_base, t0c + 1);
       st_relaxed(&p.resp[cw].commit_mask, cm);
       st_relaxed(&p.resp[cw].overflow_mask, 0u);
+      st_release(&p.resp[cw].seq, sq);
+    }
+    __syncwarp();
+    const long long t3 = clock64();
+    busy += (unsigned long long)(t3 - t0);
+    locked += (unsigned long long)(t2 - t1);
+    ph[0] += (unsigned long long)(t0 - tq);
+    ph[1] += (unsigned long long)(tl - t0);
+    ph[2] += (unsigned long long)(t1 - tl);
+    ph[3] += (unsigned long long)(t2 - t1);
+    ph[4] += (unsigned long long)(t3 - t2);
+    ++batches;
+  }
+  if (lane == 0) {
+    for (int i = 0; i < 5; ++i) atomicAdd(&p.stats->phase[i], ph[i]);
+    atomicAdd(&p.stats->batches, batches);
+    atomicAdd(&p.stats->groups, batches);
+    atomicAdd(&p.stats->busy_cycles, busy);
+    atomicAdd(&p.stats->lock_cycles, locked);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// CSMV-onlyCS worker: the client-server design with the paper's
+// complementary mechanisms removed -- no collaborative validation (the lane
+// of the transaction scans the list ATR alone), no batched ATR insert
+// (each transaction is validated and, if it commits, inserted before the
+// next one is looked at; this also catches the intra-batch conflicts the
+// missing client pre-validation would have caught), and server-side
+// write-back of the new versions (instead of the client's).  Bank,
+// single-CTA server; the ATR is the CTS-indexed ring of CSMV_ATR_LIST.
+// ---------------------------------------------------------------------------
+template <int NS>
+__device__ void server_worker_onlycs(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t lt = lanemask_lt();
+  const uint32_t R = (uint32_t)kRtWays << p.rt_log2;
+  const uint32_t dmask = (1u << kDoneLog2) - 1;
+  unsigned long long busy = 0, locked = 0, batches = 0;
+  for (;;) {
+    uint32_t cw;
+    if (!claim_request(c, cw)) break;
+    const long long t0 = clock64();
+    const uint32_t sq = ld_relaxed(p.req_seq + cw);
+    fence_gpu();
+    const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
+    const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
+    const bool mine = (mask >> lane) & 1u;
+    uint32_t a = 0, b = 0, na = 0, nb = 0;
+    if (mine) {
+      a = ld_relaxed(p.req_ids + (size_t)cw * 64 + lane) & ~kWriteBit;
+      b = ld_relaxed(p.req_ids + (size_t)cw * 64 + 32 + lane) & ~kWriteBit;
+      na = ld_relaxed(p.req_vals + (size_t)cw * 64 + lane);
+      nb = ld_relaxed(p.req_vals + (size_t)cw * 64 + 32 + lane);
+    }
+    if (__ballot_sync(FULL, (a ^ b ^ na ^ nb ^ s) == 0x12345679u) == FULL) __nanosleep(1);
+    const uint32_t ticket = cs_enter<false>(c);
+    const long long t1 = clock64();
+    const uint32_t base = *(volatile uint32_t*)&c.sh0->tail + 1;
+    uint32_t t = base - 1, cm = 0, om = 0, rem = mask;
+    while (rem) {  // one transaction at a time, in lane order
+      const int i = __ffs(rem) - 1;
+      rem &= rem - 1;
+      uint32_t ok = 0, ovf = 0;
+      if (lane == (uint32_t)i) {
+        ovf = (t - s >= R) ? 1u : 0u;
+        ok = ovf ? 0u : 1u;
+        if (!(p.debug & CSMV_DBG_NO_VALIDATE)) {
+          for (uint32_t q = s + 1; ok && q - 1 < t; ++q) {  // every commit after s
+            const uint64_t e = c.rt[q & (R - 1)];
+            const uint32_t w0 = (uint32_t)e, w1 = (uint32_t)(e >> 32);
+            if (w0 == a || w0 == b || w1 == a || w1 == b) ok = 0;
+          }
+        }
+        if (ok) c.rt[(t + 1) & (R - 1)] = ((uint64_t)b << 32) | a;  // insert this write-set alone
+      }
+      ok = __shfl_sync(FULL, ok, i);
+      ovf = __shfl_sync(FULL, ovf, i);
+      if (ok) {
+        cm |= 1u << i;
+        ++t;
+      } else if (ovf) {
+        om |= 1u << i;
+      }
+      __syncwarp();
+    }
+    if (p.publish == CSMV_PUBLISH_SERVER && t + 1 != base) done_ring_room(p, c, t, t_begin);
+    cs_leave<false>(c, ticket, t);
+    const long long t2 = clock64();
+    // server-side write-back; every earlier writer of a and b has published
+    // (the snapshot s covers it), so the ring read here is current
+    if ((cm >> lane) & 1u) {
+      const uint32_t cts = base + __popc(cm & lt);
+      const Ring<NS> ra = ld_ring<NS>(p.rings + (size_t)a * NS), rb = ld_ring<NS>(p.rings + (size_t)b * NS);
+      write_back<NS>(p.rings + (size_t)a * NS, ra, p.K, cts, na);
+      write_back<NS>(p.rings + (size_t)b * NS, rb, p.K, cts, nb);
+      if (p.publish == CSMV_PUBLISH_SERVER) st_release(p.done_ring + (cts & dmask), cts);
+    }
+    __syncwarp();
+    fence_gpu();  // the write-backs precede the response (the client publishes GTS after it)
+    if (lane == 0) {
+      st_relaxed(&p.resp[cw].cts_base, base);
+      st_relaxed(&p.resp[cw].commit_mask, cm);
+      st_relaxed(&p.resp[cw].overflow_mask, om);
       st_release(&p.resp[cw].seq, sq);
     }
     __syncwarp();
@@ -577,7 +685,7 @@ __device__ void server_publisher(const KParams& p, const SrvCtx& c, uint64_t t_b
 // Shared-memory layout of one server CTA (every CTA of the fused grid gets
 // the same dynamic allocation): rt stripe, evmax stripe, dispatch queue,
 // last-seen doorbells of its slice, control block.
-template <int KIND, bool CL>
+template <int NS, int KIND, bool CL>
 __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   const uint32_t C = p.n_server_ctas;
   const uint32_t rank = CL ? cg::this_cluster().block_rank() : 0u;
@@ -617,6 +725,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     server_receiver(p, c, t_begin);
   } else if (warp <= p.n_workers) {
     if constexpr (KIND == CSMV_KIND_KV) server_worker_generic<CL>(p, c, t_begin);
+    else if (!CL && p.commit == CSMV_COMMIT_ONLYCS) server_worker_onlycs<NS>(p, c, t_begin);
     else server_worker<CL>(p, c, t_begin);
   } else if (warp == p.n_workers + 1 && rank == 0 && p.publish == CSMV_PUBLISH_SERVER) {
     server_publisher(p, c, t_begin);

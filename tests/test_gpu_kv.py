@@ -95,3 +95,61 @@ def test_kv_no_validate_is_caught():
     oc = ocfg_of(cfg)
     rep = oracle.kv_check(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), log)
     assert not rep["ok"]
+
+
+# ---- compact PUT read-sets ({set clock} u WS) and wide sets (4..256 ways) ----
+def _check_kv(cfg):
+    pre, stats, log, fin = run(cfg)
+    oc = ocfg_of(cfg)
+    init = oracle.kv_preload(oc)
+    d = oracle.kv_gen(oc, cfg.seed, cfg.n_tx)
+    rep = oracle.kv_check(oc, init, d, log, final=as_state(fin, cfg.n_items, cfg.workload.kv_ways),
+                          claims=dict(committed_update=stats["committed_update"],
+                                      committed_ro=stats["committed_ro"], gts_final=stats["gts_final"],
+                                      total_aborts=stats["total_aborts"]))
+    assert rep["ok"], (rep, stats)
+    return stats
+
+
+@pytest.mark.parametrize("ways", [8, 16])
+def test_kv_compact_one_warp_matches_item_level_predictor(ways):
+    """The oracle's predictor pre-validates item by item; the compact
+    representation must keep and abort exactly the same lanes."""
+    cfg = W.c4(n_items=1 << 11, kv_ways=ways, n_tx=4000, p_update_ppm=300_000, client_warps=1, ro_streak=4,
+               debug_flags=csmv.DBG_KV_COMPACT)
+    pre, stats, log, fin = run(cfg)
+    oc = ocfg_of(cfg)
+    plog, pfin, ps = oracle.kv_predict(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), 32)
+    assert np.array_equal(log, plog)
+    for a, b in zip(fin, (pfin.keys, pfin.vals, pfin.lru, pfin.clocks)):
+        assert np.array_equal(a, b)
+    assert stats["total_aborts"] == ps["aborts_preval"]
+
+
+@pytest.mark.parametrize("ways", [32, 256])
+def test_kv_wide_sets_one_warp(ways):
+    cfg = W.c4(n_items=ways * 64, kv_ways=ways, kv_keys=ways * 64, n_tx=3000, p_update_ppm=300_000,
+               client_warps=1, ro_streak=4)
+    pre, stats, log, fin = run(cfg)
+    oc = ocfg_of(cfg)
+    plog, pfin, ps = oracle.kv_predict(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), 32)
+    assert np.array_equal(log, plog)
+    for a, b in zip(fin, (pfin.keys, pfin.vals, pfin.lru, pfin.clocks)):
+        assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("ways,p_update", [(16, 50_000), (64, 2_000), (256, 2_000), (256, 100_000)])
+def test_kv_wide_sets_parity(ways, p_update):
+    flags = csmv.DBG_KV_COMPACT if ways <= 16 else 0
+    cfg = W.c4(n_items=1 << 16, kv_ways=ways, kv_keys=1 << 16, n_tx=1 << 16, p_update_ppm=p_update,
+               client_warps=256, server_workers=6, ro_streak=4, debug_flags=flags)
+    _check_kv(cfg)
+
+
+def test_kv_wide_negative_control():
+    cfg = W.c4(n_items=1 << 10, kv_ways=64, kv_keys=1 << 10, n_tx=1 << 14, p_update_ppm=600_000, client_warps=64,
+               debug_flags=csmv.DBG_NO_VALIDATE, dist=0)
+    pre, stats, log, fin = run(cfg)
+    oc = ocfg_of(cfg)
+    rep = oracle.kv_check(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), log)
+    assert not rep["ok"]
