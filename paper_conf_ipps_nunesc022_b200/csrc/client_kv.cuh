@@ -26,23 +26,39 @@ __device__ __forceinline__ int kv_get(const KParams& p, uint32_t key, uint32_t s
   const uint32_t gset = kv_set(key, p.kv_T);
   dg = 0;
   hit = 0;
-  for (uint32_t w = 0; w < A; ++w) {
-    const uint32_t slot = gset * A + w;
-    uint32_t k4[4];
-    int r = kv_read_mw<NS, 4>(p.kv_key + (size_t)slot * NS * 4, K, s, true, k4);
-    if (r != RD_OK) return r;
+  // U ways in flight per lane (the scan stops at a match or an empty way;
+  // the over-read of at most U-1 ways is the price of U x fewer round trips)
+  constexpr int U = NS <= 4 ? 4 : (NS == 8 ? 2 : 1);
+  for (uint32_t w0 = 0; w0 < A; w0 += U) {
+    Ring<4> r[U][NS];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) dg += dig_word(slot, j, k4[j]);
-    if (k4[0] == gk[0] && k4[1] == gk[1] && k4[2] == gk[2] && k4[3] == gk[3]) {
-      uint32_t val[8];
-      r = kv_read_mw<NS, 8>(p.kv_val + (size_t)slot * NS * 8, K, s, true, val);
-      if (r != RD_OK) return r;
+    for (int u = 0; u < U; ++u) {
+      if (w0 + u < A) {
+        const uint64_t* ring = p.kv_key + (size_t)(gset * A + w0 + u) * NS * 4;
 #pragma unroll
-      for (int j = 0; j < 8; ++j) dg += dig_word(S + slot, j, val[j]);
-      hit = w + 1;
-      return RD_OK;
+        for (int j = 0; j < NS; ++j) r[u][j] = ld_ring<4>(ring + j * 4);
+      }
     }
-    if (!(k4[0] | k4[1] | k4[2] | k4[3])) return RD_OK;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (w0 + u >= A) break;
+      const uint32_t slot = gset * A + w0 + u;
+      uint32_t k4[4];
+      int rr = kv_key_pick<NS>(p.kv_key + (size_t)slot * NS * 4, r[u], K, s, k4);
+      if (rr != RD_OK) return rr;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) dg += dig_word(slot, j, k4[j]);
+      if (k4[0] == gk[0] && k4[1] == gk[1] && k4[2] == gk[2] && k4[3] == gk[3]) {
+        uint32_t val[8];
+        rr = kv_read_mw<NS, 8>(p.kv_val + (size_t)slot * NS * 8, K, s, true, val);
+        if (rr != RD_OK) return rr;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) dg += dig_word(S + slot, j, val[j]);
+        hit = w0 + u + 1;
+        return RD_OK;
+      }
+      if (!(k4[0] | k4[1] | k4[2] | k4[3])) return RD_OK;
+    }
   }
   return RD_OK;
 }

@@ -242,6 +242,8 @@ int csmv_load(csmv_t* h, const int32_t* init, uint64_t n) {
   CK(cudaMemcpyAsync(d_init, init, n * sizeof(int32_t), cudaMemcpyHostToDevice, h->stream));
   CK(launch_init_rings(h->d_rings, h->nslot, d_init, n, h->d_gts, h->stream));
   CK(cudaMemsetAsync(h->d_lastw, 0, n * sizeof(uint32_t), h->stream));
+  // CTS restart at 1: stale done flags of an earlier run would publish GTS early
+  CK(cudaMemsetAsync(h->d_done, 0, sizeof(uint32_t) << kDoneLog2, h->stream));
   CK(cudaFreeAsync(d_init, h->stream));
   CK(cudaStreamSynchronize(h->stream));
   h->loaded = true;
@@ -307,6 +309,7 @@ int csmv_load_kv(csmv_t* h, uint64_t n_keys) {
     e = launch_init_kv(kv_params(h), h->nslot, d, d + (size_t)S * 4, d + (size_t)S * 12, d + (size_t)S * 13,
                        h->stream);
   if (e == cudaSuccess) e = cudaMemsetAsync(h->d_lastw, 0, h->n_items * 4, h->stream);
+  if (e == cudaSuccess) e = cudaMemsetAsync(h->d_done, 0, sizeof(uint32_t) << kDoneLog2, h->stream);
   if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
   cudaFree(d);
   if (e != cudaSuccess) return set_err(CSMV_ECUDA, "csmv_load_kv: %s", cudaGetErrorString(e));

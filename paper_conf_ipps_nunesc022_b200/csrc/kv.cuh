@@ -92,6 +92,61 @@ __device__ __forceinline__ int kv_read_mw(const uint64_t* ring, uint32_t K, uint
   return RD_OK;
 }
 
+// GET-side read of a key item (W = 4) at snapshot s from its whole ring,
+// loaded in one pass (NS x 32 B, independent 256-bit loads) -- one memory
+// round trip per way instead of kv_read_mw's two.  A slot counts only if
+// all its words carry the same ts; a torn slot (a write-back in flight: its
+// new words carry a CTS > s) that may hide the version visible at s makes
+// the read a miss.  When a version newer than s is present the chosen slot
+// is re-read (address-dependent on the first loads, so ordered after them):
+// still intact means no version in (cts, s] was recycled meanwhile (oldest-
+// first recycling) -- the argument of rot_scan.
+template <int NS>
+__device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (&r)[NS], uint32_t K, uint32_t s,
+                                           uint32_t (&out)[4]) {
+  int cand = -1;
+  uint32_t cts = 0, newest = 0, torn_max = 0;
+  bool torn = false;
+#pragma unroll
+  for (int j = 0; j < NS; ++j) {
+    if ((uint32_t)j >= K) continue;
+    const uint32_t t0 = (uint32_t)(r[j].s[0] >> 32);
+    bool intact = true;
+#pragma unroll
+    for (int w = 0; w < 4; ++w) {
+      const uint32_t tw = (uint32_t)(r[j].s[w] >> 32);
+      intact &= tw == t0;
+      if (tw != kEmptyTs) newest = max(newest, tw);
+      if (tw <= s) torn_max = max(torn_max, tw);
+    }
+    if (!intact) {
+      torn = true;
+      continue;
+    }
+    if (t0 != kEmptyTs && t0 <= s && (cand < 0 || t0 > cts)) {
+      cand = j;
+      cts = t0;
+    }
+  }
+  if (cand < 0 || (torn && torn_max > cts)) return RD_MISS;
+  if (newest > s) {
+    const Ring<4> q = ld_ring<4>(ring + cand * 4);
+#pragma unroll
+    for (int w = 0; w < 4; ++w) {
+      if ((uint32_t)(q.s[w] >> 32) != cts) return RD_MISS;
+      out[w] = (uint32_t)q.s[w];
+    }
+    return RD_OK;
+  }
+#pragma unroll
+  for (int j = 0; j < NS; ++j)
+    if (j == cand) {
+#pragma unroll
+      for (int w = 0; w < 4; ++w) out[w] = (uint32_t)r[j].s[w];
+    }
+  return RD_OK;
+}
+
 // Install version (cts, data) over the first unused slot, else the oldest
 // (P:291).  The writer owns the item (WW check).
 template <int NS, int W>

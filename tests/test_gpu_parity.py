@@ -183,3 +183,24 @@ def test_runs_continue_from_store():
         s2 = st.run(cfg.workload, cfg.n_tx, 2)
         assert s2["gts_start"] == s1["gts_final"]
         assert s2["gts_final"] == s1["gts_final"] + s2["committed_update"]
+
+
+@pytest.mark.parametrize("publish", [csmv.PUBLISH_CLIENT, csmv.PUBLISH_SERVER])
+def test_reload_then_rerun(publish):
+    """csmv_load restarts CTS at 1: nothing left from the previous run (done
+    flags of the server publisher, lastw) may leak into the next one."""
+    cfg = W.c2(n_items=1 << 12, n_tx=1 << 15, publish=publish, client_warps=32, ro_streak=4, watchdog_ms=20_000)
+    init = cfg.init_values()
+    ocfg = oracle_cfg(cfg)
+    with csmv.Store(cfg.n_items, cfg.n_versions) as st:
+        for seed in (1, 2):
+            st.load(init)
+            stats = st.run(cfg.workload, cfg.n_tx, seed)
+            log = st.log(cfg.n_tx)
+            rings = st.dump()
+            descs = oracle.bank_gen(ocfg, seed, cfg.n_tx)
+            rep = oracle.bank_check(ocfg, init, descs, log, rings=rings,
+                                    claims=dict(committed_update=stats["committed_update"],
+                                                committed_ro=stats["committed_ro"], gts_final=stats["gts_final"],
+                                                total_aborts=stats["total_aborts"]))
+            assert rep["ok"], (seed, rep)

@@ -11,6 +11,8 @@
 #include "../../paper_conf_ipps_nunesc022_b200/csrc/ptx.cuh"
 namespace csmvd {
 __device__ __forceinline__ bool watchdog(const KParams&, uint64_t, uint32_t) { return false; }
+template <int NS>
+__device__ void write_back(uint64_t*, const Ring<NS>&, uint32_t, uint32_t, uint32_t) {}
 }
 #include "../../paper_conf_ipps_nunesc022_b200/csrc/server.cuh"
 using namespace csmvd;
@@ -40,7 +42,8 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
     const uint32_t b0 = rt_bucket(id0, 12), b1 = rt_bucket(id1, 12);
     const bool mine = lane < 29;
     uint32_t ticket = 0;
-    if (mode == 4) {
+    const bool locked = mode >= 4;
+    if (locked) {
       ticket = cs_enter<false>(c);
       t = *(volatile uint32_t*)&sh.tail;
     }
@@ -56,7 +59,7 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
     const uint32_t cm = __ballot_sync(0xFFFFFFFFu, commit);
     const uint32_t cts = t + 1 + __popc(cm & lt);
     t += __popc(cm);
-    if (commit && mode >= 3) {
+    if (commit && mode >= 3 && mode != 5) {
       lastw[id0 & 0xFFFFF] = cts;
       lastw[id1 & 0xFFFFF] = cts;
     }
@@ -66,12 +69,12 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
     }
     __syncwarp();
     acc += clock64() - a;
-    if (mode == 4) cs_leave<false>(c, ticket, t);
+    if (locked) cs_leave<false>(c, ticket, t);
     sink += cm;
   }
   const long long a1 = clock64();
   if (lane == 0 && warp == 0) {
-    out[0] = mode == 4 ? (a1 - a0) / ((long long)iters * nw) : acc / iters;
+    out[0] = mode >= 4 ? (a1 - a0) / ((long long)iters * nw) : acc / iters;
     out[1] = acc / iters;
     out[2] = sink;
   }
@@ -94,6 +97,9 @@ int main() {
     bench<<<1, 256, smem>>>(lw, o, 4, 20000, nw);
     cudaDeviceSynchronize();
     printf("locked chain, %d warps: %llu cycles/batch (body %llu)\n", nw, o[0], o[1]);
+    bench<<<1, 256, smem>>>(lw, o, 5, 20000, nw);
+    cudaDeviceSynchronize();
+    printf("locked chain, no lastw stores, %d warps: %llu cycles/batch (body %llu)\n", nw, o[0], o[1]);
   }
   printf("err=%s\n", cudaGetErrorString(cudaGetLastError()));
 }
