@@ -1,31 +1,30 @@
 // kernel.cu -- the fused persistent CSMV kernel for sm_100a.
 //
 // One cooperative grid holds both roles of the paper's client-server split
-// (P:99-105): CTA 0 is the server SM, CTAs 1..C are client SMs.  Fusing the
-// roles into one launch guarantees co-residency of a server that spins on
-// its clients (the paper launches two kernels; separate kernels deadlock when
-// a profiler serialises them).
+// (P:99-105): CTAs 0..C-1 are the server (C = 1, the paper's one SM, or a
+// thread-block cluster), the rest are client SMs.  Fusing the roles into one
+// launch guarantees co-residency of a server that spins on its clients (the
+// paper launches two kernels; separate kernels deadlock when a profiler
+// serialises them).  CSMV_COMMIT_JVSTM launches clients only.
 //
-// Client warp, one round (section III):
+// Client warp, one round (client_bank.cuh / client_kv.cuh):
 //   TXBegin     s <- GTS (one acquire load per warp round)
 //   TXRead      newest version with ts <= s from the VBox ring
-//               read-only lanes finish here, no commit
 //   pre-validation of the warp's update lanes (shuffle/ballot)
-//   submit the batch (request slot + doorbell), wait for the response P:101
-//   write-back of the new versions by the client
+//   submit the batch (request slot + doorbell)
+//   read-only transactions at s while the batch is at the server
+//   the response, client write-back of the new versions
 //   ordered GTS advance by n (CSMV_PUBLISH_CLIENT) or a done
 //   flag per CTS for the server publisher (CSMV_PUBLISH_SERVER)
-//   aborted lanes retry with a fresh snapshot next round
+//   aborted transactions retry with a fresh snapshot next round
 //
-// Server CTA: worker warps each own a contiguous slice of client doorbells
-// (receiving and working are merged per warp); a batch is
-// validated by the whole warp (one lane per transaction, __ballot_sync /
-// __match_any_sync) against the ATR, which lives in shared memory as an
-// item-indexed set-associative table of (item, last CTS) covering every
-// commit after the watermark W_low;
-// consecutive CTS are reserved and the write-sets inserted inside one
-// shared-memory critical section.  No global atomics on the
-// commit path.
+// Server (server.cuh): a receiver warp per server CTA dispatches doorbells to
+// worker warps; a worker validates whole batches (one lane per transaction,
+// __ballot_sync) against the two-level item-indexed ATR (HBM lastw + smem
+// recent-commit table; or the paper's list ATR), reserves consecutive CTS
+// and records the write-sets inside a shared-memory ticket-locked critical
+// section.  No global atomics on
+// the commit path.
 #include <cuda_runtime.h>
 
 #include "kernel.cuh"

@@ -57,7 +57,7 @@ def run_point(cfg, check: bool):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--n-tx", type=int, default=1 << 22)
+    ap.add_argument("--n-tx", type=int, default=1 << 21)
     ap.add_argument("--check", action="store_true")
     ap.add_argument("--out", default="")
     ap.add_argument("--servers", default="0,1")
@@ -67,7 +67,7 @@ def main():
     f = open(args.out, "w") if args.out else None
     for cfg in workloads.c5_points(args.n_tx, servers=servers):
         cw = max(16, min(TUNED["client_warps"], cfg.n_items // 64))  # in-flight updates << items (Q29)
-        cfg = cfg.with_(cluster_size=args.cluster_size, watchdog_ms=300_000, **dict(TUNED, client_warps=cw))
+        cfg = cfg.with_(cluster_size=args.cluster_size, watchdog_ms=60_000, **dict(TUNED, client_warps=cw))
         try:
             r = run_point(cfg, args.check)
         except Exception as e:  # report and continue the sweep
