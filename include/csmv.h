@@ -105,6 +105,9 @@ typedef struct csmv_workload {
     uint32_t debug_flags;      /* CSMV_DBG_* */
     uint32_t watchdog_ms;      /* 0 = default (20000) */
     uint32_t commit;           /* CSMV_COMMIT_* (0 = the paper's CSMV) */
+    uint32_t ro_adaptive;      /* 1: a lane stops its read-only run (at most ro_streak) as soon as the
+                                  server has answered the warp's batch -- rounds track the server
+                                  round trip (timing-dependent schedule; 0 = fixed, deterministic) */
 } csmv_workload;
 
 /* ---- statistics ---- */

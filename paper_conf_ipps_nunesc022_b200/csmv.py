@@ -41,7 +41,8 @@ class _Workload(C.Structure):
     _fields_ = [(n, C.c_uint32) for n in (
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
         "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers", "server_combine",
-        "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms", "commit")]
+        "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms", "commit",
+        "ro_adaptive")]
 
 
 class _Stats(C.Structure):
@@ -85,6 +86,7 @@ class Workload:
     debug_flags: int = 0
     watchdog_ms: int = 0
     commit: int = COMMIT_CSMV
+    ro_adaptive: int = 0
 
     def to_c(self) -> _Workload:
         return _Workload(*[getattr(self, f.name) for f in fields(self)])

@@ -237,6 +237,8 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         cc.ro_ck ^= (uint64_t)rsum;
         cr += T;
         att_r = 0;
+        // ro_adaptive: the batch has been answered -> finish the round
+        if (p.ro_adaptive && kept && ld_relaxed(&p.resp[cw].seq) == round) break;
       }
     }
     __syncwarp();

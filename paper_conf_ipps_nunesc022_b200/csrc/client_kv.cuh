@@ -270,6 +270,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         cc.ro_ck ^= dg;
         cr += T;
         att_r = 0;
+        if (p.ro_adaptive && kept && ld_relaxed(&p.resp[cw].seq) == round) break;
       }
     }
     __syncwarp();

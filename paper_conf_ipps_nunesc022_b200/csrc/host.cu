@@ -496,6 +496,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.backoff_max = w->backoff_max;
   p.debug = w->debug_flags;
   p.commit = w->commit;
+  p.ro_adaptive = w->ro_adaptive;
   p.req_vals = h->d_req_vals;
   p.jv_ws = h->d_jv_ws;
   p.jv_tag = h->d_jv_tag;

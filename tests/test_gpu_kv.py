@@ -153,3 +153,9 @@ def test_kv_wide_negative_control():
     oc = ocfg_of(cfg)
     rep = oracle.kv_check(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), log)
     assert not rep["ok"]
+
+
+def test_kv_ro_adaptive_parity():
+    cfg = W.c4(n_items=1 << 14, n_tx=1 << 17, p_update_ppm=20_000, client_warps=256, server_workers=6,
+               ro_streak=32, ro_adaptive=1)
+    _check_kv(cfg)

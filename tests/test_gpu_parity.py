@@ -204,3 +204,14 @@ def test_reload_then_rerun(publish):
                                                 committed_ro=stats["committed_ro"], gts_final=stats["gts_final"],
                                                 total_aborts=stats["total_aborts"]))
             assert rep["ok"], (seed, rep)
+
+
+@pytest.mark.parametrize("preset,streak", [("c2", 16), ("c3", 32)])
+def test_ro_adaptive_parity(preset, streak):
+    """ro_adaptive: read-only runs end when the batch is answered (a
+    timing-dependent schedule) -- still every history replays exactly."""
+    mk = getattr(W, preset)
+    cfg = mk(n_items=1 << 12, n_tx=1 << 17, client_warps=128, ro_streak=streak, ro_adaptive=1,
+             server_workers=6, server_combine=4, publish=csmv.PUBLISH_SERVER)
+    rep, stats, log, rings, descs = check(cfg)
+    assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions), closed_form(cfg, descs, cfg.init_values()))
