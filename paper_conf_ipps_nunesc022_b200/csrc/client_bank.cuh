@@ -176,6 +176,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         } else if (reason >= 0) {
           cc.abort(reason, true);
         }
+        status = ST_NONE;  // decided here: not a pre-validation loser below
       }
       __syncwarp();
       pc.mark(PH_DIVERGENCE);
