@@ -77,7 +77,8 @@ extern "C" {
 #define CSMV_DBG_NO_VALIDATE 2u/* negative control: server commits without validating */
 #define CSMV_DBG_JITTER 4u     /* random __nanosleep in client and server */
 #define CSMV_DBG_PHASES 8u     /* per-phase client clocks (csmv_stats_t.client_phase_cycles) */
-#define CSMV_DBG_KV_COMPACT 16u/* KV: ship PUT read-sets as {set clock} u WS at any ways (always above 16) */
+#define CSMV_DBG_KV_ITEMSETS 16u /* KV, A <= 16: ship PUT read/write sets item by item (the paper's literal
+                                    form); default {set clock} u WS, which decides identically */
 
 typedef struct csmv_workload {
     uint32_t kind;             /* CSMV_KIND_* */

@@ -2,10 +2,11 @@
 // Same lane state machine and round phases as client_bank.cuh; GET is the
 // read-only transaction, PUT the update transaction (docs/GENERATOR.md 4).
 //
-// Read-set representation.  With A <= kKvFullWays the PUT's read-set is
-// tracked item by item (smem scratch) and shipped whole, as in the paper.
-// Above that (up to 256 ways) -- or with CSMV_DBG_KV_COMPACT -- it is
-// shipped as {set clock} u WS: every item a PUT reads lies in its set t,
+// Read-set representation.  By default (and always above kKvFullWays ways,
+// up to 256) a PUT's read/write set is shipped as {set clock} u WS;
+// with CSMV_DBG_KV_ITEMSETS (A <= 16) it is tracked item by item (smem
+// scratch) and shipped whole, the paper's literal form.  The two decide
+// identically: every item a PUT reads lies in its set t,
 // every PUT on set t reads and writes clock[t], and nothing else writes an
 // item of set t, so "a commit after s wrote an item of RS u WS" holds iff
 // "a commit after s wrote clock[t]" -- validation and
@@ -78,7 +79,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
   const uint32_t K = p.K, S = p.kv_S, A = p.kv_A, Tn = p.kv_T;
   const uint32_t lt = lanemask_lt();
   const uint32_t streak = p.ro_streak;
-  const bool compact = A > kKvFullWays || (p.debug & CSMV_DBG_KV_COMPACT);
+  const bool compact = A > kKvFullWays || !(p.debug & CSMV_DBG_KV_ITEMSETS);
   PhaseClock pc((p.debug & CSMV_DBG_PHASES) != 0);
   // per-warp smem scratch, lane-minor: RS[kKvMaxRs][32], WS[4][32], NRS[32]
   uint32_t* RS = scratch + (size_t)wib * 32 * (kKvMaxRs + 5);

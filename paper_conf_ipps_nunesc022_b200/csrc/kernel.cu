@@ -117,7 +117,7 @@ __device__ __forceinline__ bool watchdog(const KParams& p, uint64_t t0, uint32_t
 template <int NS>
 __device__ __forceinline__ bool rot_scan(const KParams& p, uint32_t start, uint32_t len, uint32_t s,
                                          uint64_t tx, int64_t& sum, uint64_t& dg) {
-  constexpr int U = 4;
+  constexpr int U = NS <= 4 ? 8 : (NS == 8 ? 4 : 2);  // rings in flight per lane (memory-level parallelism)
   sum = 0;
   dg = 0;
   const uint32_t N = p.n_items;

@@ -24,7 +24,6 @@ struct SrvShared {
   uint32_t next_ticket;  // ticket lock around validate+reserve+insert        [CTA 0]
   uint32_t now_serving;  //                                                   [CTA 0]
   uint32_t gts_seen;     // publisher progress seen by workers (back-pressure) [CTA 0]
-  uint32_t evmax;        // largest CTS ever evicted from the recent table     [CTA 0]
   uint32_t q_head;       // next dispatch-queue slot a worker claims          [per CTA]
   uint32_t exit;         // receiver: all clients finished                    [per CTA]
 };
@@ -34,19 +33,15 @@ struct SrvShared {
 //  * lastw[x] in HBM: CTS of the last commit that wrote x -- the exact
 //    record of every committed write-set, all history;
 //  * rt in shared memory: 4-way buckets of (cts << 32 | item) holding recent
-//    writes (oldest-first replacement), plus ONE watermark evmax = the
-//    largest CTS ever evicted from any bucket, so that commits made after a
-//    worker prefetched lastw (CTS > e_pre) are seen with on-chip latency
-//    (P:105).  Oldest-first replacement keeps evicted CTS far behind the
-//    tail, so a single watermark is as effective as one per bucket and
-//    costs no load per probe and no atomic per record.
-// Invariant: if the latest write c of item y is not in its bucket, then
-// evmax >= c (entries leave a bucket only through atomicExch inside the
-// critical section, and the holder folds every evicted CTS into evmax
-// before it releases the lock).
+//    writes plus, per bucket, evmax = the largest CTS ever evicted from it,
+//    so that commits made after a worker prefetched lastw (CTS > e_pre) are
+//    seen with on-chip latency.
+// Invariant: if the latest write c of item y (bucket b) is not in b, then
+// evmax[b] >= c (entries leave a bucket only through atomicExch, and the
+// evictor records the evicted CTS with atomicMax).
 // Validation of x for snapshot s (P:75 read-set, P:115 write-set), s <= e_pre:
 //    conflict  iff  lastw[x] (as of e_pre) > s  or  some way holds (x, c), c > s
-//    unknown   iff  not conflict and evmax > e_pre -> abort, reason OVERFLOW
+//    unknown   iff  not conflict and evmax[b] > e_pre -> abort, reason OVERFLOW
 // ---------------------------------------------------------------------------
 constexpr int kRtWays = 4;
 
@@ -56,6 +51,7 @@ __device__ __forceinline__ uint32_t rt_bucket(uint32_t key, uint32_t rt_log2) {
 
 struct SrvCtx {
   uint64_t* rt;       // this CTA's stripe of buckets (kRtWays u64 each)
+  uint32_t* evmax;    // this CTA's stripe of eviction watermarks
   uint32_t clog2;     // log2(server CTAs)
   SrvShared* sh;      // this CTA's control block
   SrvShared* sh0;     // CTA 0's control block (DSMEM in a cluster)
@@ -76,6 +72,16 @@ __device__ __forceinline__ uint64_t* rt_at(const SrvCtx& c, uint32_t b) {
 }
 
 template <bool CL>
+__device__ __forceinline__ uint32_t* ev_at(const SrvCtx& c, uint32_t b) {
+  if constexpr (!CL) {
+    return c.evmax + b;
+  } else {
+    const uint32_t owner = b & ((1u << c.clog2) - 1), local = b >> c.clog2;
+    return cg::this_cluster().map_shared_rank(c.evmax, owner) + local;
+  }
+}
+
+template <bool CL>
 __device__ __forceinline__ void srv_fence() {
   if constexpr (CL) asm volatile("fence.acq_rel.cluster;" ::: "memory");
   else fence_cta();
@@ -87,13 +93,27 @@ struct RtProbe {
   bool unknown;
 };
 
-// ev: the eviction watermark as of this point of the critical section
+// A bucket as loaded: its 4 ways and its eviction watermark.  Loading and
+// evaluating are split so that callers can put several loads in flight.
+struct RtBucket {
+  ulonglong2 a, b;
+  uint32_t ev;
+};
+
 template <bool CL>
-__device__ __forceinline__ RtProbe rt_probe(const SrvCtx& c, uint32_t bucket, uint32_t key, uint32_t s,
-                                            uint32_t e_pre, uint32_t lastw, uint32_t ev) {
+__device__ __forceinline__ RtBucket rt_load(const SrvCtx& c, uint32_t bucket) {
   const ulonglong2* e = reinterpret_cast<const ulonglong2*>(rt_at<CL>(c, bucket));
-  const ulonglong2 a = e[0], b = e[1];
-  const uint64_t w[4] = {a.x, a.y, b.x, b.y};
+  RtBucket q;
+  q.a = e[0];
+  q.b = e[1];
+  q.ev = *ev_at<CL>(c, bucket);
+  return q;
+}
+
+__device__ __forceinline__ RtProbe rt_eval(const RtBucket& q, uint32_t key, uint32_t s, uint32_t e_pre,
+                                           uint32_t lastw) {
+  const uint64_t w[4] = {q.a.x, q.a.y, q.b.x, q.b.y};
+  const uint32_t ev = q.ev;
   RtProbe r;
   r.conflict = lastw > s;
   int hit = -1, old = 0;
@@ -115,16 +135,20 @@ __device__ __forceinline__ RtProbe rt_probe(const SrvCtx& c, uint32_t bucket, ui
   return r;
 }
 
-// Record (key, cts) into `way` of its bucket; returns the CTS of an evicted
-// entry of another key (0 if none), which the caller folds into evmax.
-// Exchanges by several lanes on one slot are serialised by the hardware and
-// each evictor sees the value it replaced.
 template <bool CL>
-__device__ __forceinline__ uint32_t rt_record(const SrvCtx& c, uint32_t bucket, int way, uint32_t key,
-                                              uint32_t cts) {
+__device__ __forceinline__ RtProbe rt_probe(const SrvCtx& c, uint32_t bucket, uint32_t key, uint32_t s,
+                                            uint32_t e_pre, uint32_t lastw) {
+  return rt_eval(rt_load<CL>(c, bucket), key, s, e_pre, lastw);
+}
+
+// Record (key, cts) into `way` of its bucket; an evicted entry of another
+// key raises evmax.  Exchanges by several lanes on one slot are serialised
+// by the hardware and each evictor sees the value it replaced.
+template <bool CL>
+__device__ __forceinline__ void rt_record(const SrvCtx& c, uint32_t bucket, int way, uint32_t key, uint32_t cts) {
   const unsigned long long old =
       atomicExch(reinterpret_cast<unsigned long long*>(rt_at<CL>(c, bucket) + way), ((unsigned long long)cts << 32) | key);
-  return ((uint32_t)old != key) ? (uint32_t)(old >> 32) : 0u;
+  if ((uint32_t)old != key && (uint32_t)(old >> 32) != 0u) atomicMax(ev_at<CL>(c, bucket), (uint32_t)(old >> 32));
 }
 
 // ---------------------------------------------------------------------------
@@ -376,7 +400,6 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     const uint32_t ticket = cs_enter<CL>(c);
     const long long t1 = clock64();
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
-    uint32_t ev = *(volatile uint32_t*)&c.sh0->evmax;
     uint32_t t = t0c;
     uint32_t cm[M], om[M], base[M];
 #pragma unroll
@@ -388,8 +411,8 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       bool ovf = false, conflict = false;
       if (p.atr_mode == CSMV_ATR_HASH) {
         if (mine[j]) {
-          q0 = rt_probe<CL>(c, bk0[j], id0[j], sn[j], e_pre, lw0[j], ev);
-          q1 = rt_probe<CL>(c, bk1[j], id1[j], sn[j], e_pre, lw1[j], ev);
+          q0 = rt_probe<CL>(c, bk0[j], id0[j], sn[j], e_pre, lw0[j]);
+          q1 = rt_probe<CL>(c, bk1[j], id1[j], sn[j], e_pre, lw1[j]);
           if (bk1[j] == bk0[j] && q1.way == q0.way) q1.way = (q1.way + 1) & (kRtWays - 1);
         }
         ovf = mine[j] && (q0.unknown || q1.unknown);
@@ -403,20 +426,18 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       om[j] = __ballot_sync(FULL, ovf);
       const uint32_t cts = t + 1 + __popc(cm[j] & lt);
       t += __popc(cm[j]);
-      uint32_t evicted = 0;
       if (commit) {
         if (p.atr_mode == CSMV_ATR_HASH) {
           p.lastw[id0[j]] = cts;
           p.lastw[id1[j]] = cts;
-          evicted = max(rt_record<CL>(c, bk0[j], q0.way, id0[j], cts), rt_record<CL>(c, bk1[j], q1.way, id1[j], cts));
+          rt_record<CL>(c, bk0[j], q0.way, id0[j], cts);
+          rt_record<CL>(c, bk1[j], q1.way, id1[j], cts);
         } else {  // the paper's ATR: the write-set of commit `cts` at entry cts
           c.rt[cts & ((uint32_t)(kRtWays << (p.rt_log2 - p.clog2)) - 1)] = ((uint64_t)id1[j] << 32) | id0[j];
         }
       }
-      if (p.atr_mode == CSMV_ATR_HASH) ev = max(ev, __reduce_max_sync(FULL, evicted));
       __syncwarp();  // batch j's records precede batch j+1's probes
     }
-    if (p.atr_mode == CSMV_ATR_HASH && (threadIdx.x & 31) == 0) *(volatile uint32_t*)&c.sh0->evmax = ev;
     const long long ta = clock64();
     if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) done_ring_room(p, c, t, t_begin);
     cs_leave<CL>(c, ticket, t);
@@ -471,7 +492,11 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t lt = lanemask_lt();
   unsigned long long busy = 0, locked = 0, batches = 0;
-  unsigned long long ph[5] = {0, 0, 0, 0, 0};
+  unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  // {set clock} u WS requests (client_kv.cuh): ids[0] is the clock of the
+  // PUT's set, read and written by every PUT of that set while nothing else
+  // writes the set -- it alone decides validation (DESIGN.md readings)
+  const bool compact = p.kv_A > kKvFullWays || !(p.debug & CSMV_DBG_KV_ITEMSETS);
   for (;;) {
     uint32_t cw;
     const long long tq = clock64();
@@ -483,6 +508,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
     const bool mine = (mask >> lane) & 1u;
     const uint32_t cnt = mine ? ld_relaxed(p.req_cnt + (size_t)cw * 32 + lane) : 0u;
+    const uint32_t nval = compact ? min(cnt, 1u) : cnt;  // ids to validate
     uint32_t ids[kKvMaxId];
 #pragma unroll
     for (uint32_t k = 0; k < kKvMaxId; ++k)
@@ -493,7 +519,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     uint32_t x = s ^ e_pre;
 #pragma unroll
     for (uint32_t k = 0; k < kKvMaxId; ++k) {
-      lw[k] = (k < cnt) ? ld_relaxed(p.lastw + (ids[k] & ~kWriteBit)) : 0u;
+      lw[k] = (k < nval) ? ld_relaxed(p.lastw + (ids[k] & ~kWriteBit)) : 0u;
       x ^= ids[k] ^ lw[k];
     }
     if (__ballot_sync(FULL, x == 0x12345679u) == FULL) __nanosleep(1);  // payload complete before the lock
@@ -502,15 +528,22 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     const uint32_t ticket = cs_enter<CL>(c);
     const long long t1 = clock64();
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
-    uint32_t ev = *(volatile uint32_t*)&c.sh0->evmax;
     bool conflict = false, unknown = false;
+    // four buckets in flight per step; warp-uniform exit after the longest set
 #pragma unroll
-    for (uint32_t k = 0; k < kKvMaxId; ++k) {
-      if (k < cnt) {
-        const uint32_t id = ids[k] & ~kWriteBit;
-        const RtProbe q = rt_probe<CL>(c, rt_bucket(id, p.rt_log2), id, s, e_pre, lw[k], ev);
-        conflict |= q.conflict;
-        unknown |= q.unknown;
+    for (uint32_t k0 = 0; k0 < kKvMaxId; k0 += 4) {
+      if (!__any_sync(FULL, k0 < nval)) break;
+      RtBucket q[4];
+#pragma unroll
+      for (uint32_t u = 0; u < 4; ++u)
+        if (k0 + u < kKvMaxId && k0 + u < nval) q[u] = rt_load<CL>(c, rt_bucket(ids[k0 + u] & ~kWriteBit, p.rt_log2));
+#pragma unroll
+      for (uint32_t u = 0; u < 4; ++u) {
+        if (k0 + u < kKvMaxId && k0 + u < nval) {
+          const RtProbe r = rt_eval(q[u], ids[k0 + u] & ~kWriteBit, s, e_pre, lw[k0 + u]);
+          conflict |= r.conflict;
+          unknown |= r.unknown;
+        }
       }
     }
     if (p.debug & CSMV_DBG_NO_VALIDATE) conflict = unknown = false;
@@ -520,21 +553,22 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     const uint32_t om = __ballot_sync(FULL, ovf);
     const uint32_t n = __popc(cm);
     const uint32_t cts = t0c + 1 + __popc(cm & lt);
+    const long long tv = clock64();
     if (p.publish == CSMV_PUBLISH_SERVER && n) done_ring_room(p, c, t0c + n, t_begin);
-    uint32_t evicted = 0;
     if (commit) {
 #pragma unroll
       for (uint32_t k = 0; k < kKvMaxId; ++k) {
         if (k < cnt && (ids[k] & kWriteBit)) {
           const uint32_t id = ids[k] & ~kWriteBit, b = rt_bucket(id, p.rt_log2);
-          p.lastw[id] = cts;
-          const RtProbe q = rt_probe<CL>(c, b, id, 0u, 0u, 0u, 0u);  // the way to (re)use
-          evicted = max(evicted, rt_record<CL>(c, b, q.way, id, cts));
+          p.lastw[id] = cts;  // every written item, so lastw stays exact for any later run
+          if (k < nval || !compact) {
+            const RtProbe q = rt_probe<CL>(c, b, id, 0u, 0u, 0u);  // the way to (re)use
+            rt_record<CL>(c, b, q.way, id, cts);
+          }
         }
       }
     }
-    ev = max(ev, __reduce_max_sync(FULL, evicted));
-    if (lane == 0) *(volatile uint32_t*)&c.sh0->evmax = ev;
+    const long long tr = clock64();
     cs_leave<CL>(c, ticket, t0c + n);
     const long long t2 = clock64();
     if (lane == 0) {
@@ -552,10 +586,13 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     ph[2] += (unsigned long long)(t1 - tl);
     ph[3] += (unsigned long long)(t2 - t1);
     ph[4] += (unsigned long long)(t3 - t2);
+    ph[5] += (unsigned long long)(tv - t1);
+    ph[6] += (unsigned long long)(tr - tv);
+    ph[7] += (unsigned long long)(t2 - tr);
     ++batches;
   }
   if (lane == 0) {
-    for (int i = 0; i < 5; ++i) atomicAdd(&p.stats->phase[i], ph[i]);
+    for (int i = 0; i < 8; ++i) atomicAdd(&p.stats->phase[i], ph[i]);
     atomicAdd(&p.stats->batches, batches);
     atomicAdd(&p.stats->groups, batches);
     atomicAdd(&p.stats->busy_cycles, busy);
@@ -704,7 +741,7 @@ __device__ void server_publisher(const KParams& p, const SrvCtx& c, uint64_t t_b
 }
 
 // Shared-memory layout of one server CTA (every CTA of the fused grid gets
-// the same dynamic allocation): rt stripe, dispatch queue,
+// the same dynamic allocation): rt stripe, evmax stripe, dispatch queue,
 // last-seen doorbells of its slice, control block.
 template <int NS, int KIND, bool CL>
 __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
@@ -720,12 +757,14 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   c.rt = reinterpret_cast<uint64_t*>(smem);
   const uint32_t rt_words = (uint32_t)kRtWays << local_log2;
   c.queue = c.rt + rt_words;
-  c.last_seen = reinterpret_cast<uint32_t*>(c.queue + (1u << c.qn_log2));
+  c.evmax = reinterpret_cast<uint32_t*>(c.queue + (1u << c.qn_log2));
+  c.last_seen = c.evmax + (1u << local_log2);
   const uint32_t ls_words = (per + 31) / 32 * 32;
   c.sh = reinterpret_cast<SrvShared*>(c.last_seen + ls_words);
   if constexpr (CL) c.sh0 = cg::this_cluster().map_shared_rank(c.sh, 0);
   else c.sh0 = c.sh;
   for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) c.rt[i] = 0xFFFFFFFFull;  // cts 0, no item
+  for (uint32_t i = threadIdx.x; i < (1u << local_log2); i += blockDim.x) c.evmax[i] = 0;
   for (uint32_t i = threadIdx.x; i < (1u << c.qn_log2); i += blockDim.x) c.queue[i] = 0;
   for (uint32_t i = threadIdx.x; i < ls_words; i += blockDim.x) c.last_seen[i] = 0;
   if (threadIdx.x == 0) {
@@ -734,7 +773,6 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     c.sh->next_ticket = 0;
     c.sh->now_serving = 0;
     c.sh->gts_seen = g0;
-    c.sh->evmax = 0;
     c.sh->q_head = 0;
     c.sh->exit = 0;
   }

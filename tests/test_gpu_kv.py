@@ -45,11 +45,12 @@ def test_preload_parity(S, A):
         assert np.array_equal(a, b)
 
 
-@pytest.mark.parametrize("p_update,streak,k", [(10_000, 0, 4), (10_000, 8, 4), (200_000, 4, 4),
-                                               (500_000, 0, 2), (50_000, 8, 8)])
-def test_kv_parity(p_update, streak, k):
+@pytest.mark.parametrize("p_update,streak,k,flags", [(10_000, 0, 4, 0), (10_000, 8, 4, 0), (200_000, 4, 4, 0),
+                                                     (500_000, 0, 2, 0), (50_000, 8, 8, 0), (10_000, 8, 4, 16),
+                                                     (200_000, 4, 4, 16)])
+def test_kv_parity(p_update, streak, k, flags):
     cfg = W.c4(n_items=1 << 14, n_tx=1 << 17, p_update_ppm=p_update, ro_streak=streak, n_versions=k,
-               client_warps=256, server_workers=6)
+               client_warps=256, server_workers=6, debug_flags=flags)
     pre, stats, log, fin = run(cfg)
     oc = ocfg_of(cfg)
     init = oracle.kv_preload(oc)
@@ -62,10 +63,14 @@ def test_kv_parity(p_update, streak, k):
     assert stats["committed_update"] == int(d["is_update"].sum())
 
 
+@pytest.mark.parametrize("flags", [0, csmv.DBG_KV_ITEMSETS])
 @pytest.mark.parametrize("streak", [0, 4])
-def test_kv_one_warp_deterministic(streak):
+def test_kv_one_warp_deterministic(streak, flags):
+    """Both request forms ({set clock} u WS by default, item by item with
+    DBG_KV_ITEMSETS) keep and abort exactly the lanes the oracle's item-level
+    predictor does."""
     cfg = W.c4(n_items=1 << 11, kv_ways=8, n_tx=4000, p_update_ppm=300_000, client_warps=1,
-               ro_streak=streak)
+               ro_streak=streak, debug_flags=flags)
     pre, stats, log, fin = run(cfg)
     oc = ocfg_of(cfg)
     init = oracle.kv_preload(oc)
@@ -111,12 +116,10 @@ def _check_kv(cfg):
     return stats
 
 
-@pytest.mark.parametrize("ways", [8, 16])
-def test_kv_compact_one_warp_matches_item_level_predictor(ways):
-    """The oracle's predictor pre-validates item by item; the compact
-    representation must keep and abort exactly the same lanes."""
+@pytest.mark.parametrize("ways", [4, 16])
+def test_kv_itemsets_one_warp_matches_item_level_predictor(ways):
     cfg = W.c4(n_items=1 << 11, kv_ways=ways, n_tx=4000, p_update_ppm=300_000, client_warps=1, ro_streak=4,
-               debug_flags=csmv.DBG_KV_COMPACT)
+               debug_flags=csmv.DBG_KV_ITEMSETS)
     pre, stats, log, fin = run(cfg)
     oc = ocfg_of(cfg)
     plog, pfin, ps = oracle.kv_predict(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), 32)
@@ -138,9 +141,9 @@ def test_kv_wide_sets_one_warp(ways):
         assert np.array_equal(a, b)
 
 
-@pytest.mark.parametrize("ways,p_update", [(16, 50_000), (64, 2_000), (256, 2_000), (256, 100_000)])
-def test_kv_wide_sets_parity(ways, p_update):
-    flags = csmv.DBG_KV_COMPACT if ways <= 16 else 0
+@pytest.mark.parametrize("ways,p_update,flags", [(16, 50_000, 0), (16, 50_000, 16), (64, 2_000, 0),
+                                                 (256, 2_000, 0), (256, 100_000, 0)])
+def test_kv_wide_sets_parity(ways, p_update, flags):
     cfg = W.c4(n_items=1 << 16, kv_ways=ways, kv_keys=1 << 16, n_tx=1 << 16, p_update_ppm=p_update,
                client_warps=256, server_workers=6, ro_streak=4, debug_flags=flags)
     _check_kv(cfg)
