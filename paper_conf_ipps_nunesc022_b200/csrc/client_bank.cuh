@@ -211,6 +211,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
       if (lane == 0) {
         p.req_hdr[cw].snapshot = s;
         p.req_hdr[cw].mask = kept;
+        p.req_hdr[cw].round = round;
       }
       __syncwarp();
       fence_gpu();
@@ -239,7 +240,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         cr += T;
         att_r = 0;
         // ro_adaptive: the batch has been answered -> finish the round
-        if (p.ro_adaptive && kept && ld_relaxed(&p.resp[cw].seq) == round) break;
+        if (p.ro_adaptive && kept && (uint32_t)(ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
       }
     }
     __syncwarp();
@@ -248,28 +249,8 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
 
     // ---- D: the server's answer, write-back, GTS
     uint32_t base = 0, cmask = 0, omask = 0;
-    {
-      uint32_t it = 0;
-      bool ok = true;
-      while (warp_ld_relaxed(&p.resp[cw].seq) != round) {
-        if ((++it & 255u) == 0) {
-          uint32_t bad = 0;
-          if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);
-          if (__shfl_sync(FULL, bad, 0)) {
-            ok = false;
-            break;
-          }
-        }
-        __nanosleep(64);
-      }
-      fence_gpu();  // acquire: response payload after its seq
-      if (ok) {
-        base = ld_relaxed(&p.resp[cw].cts_base);
-        cmask = ld_relaxed(&p.resp[cw].commit_mask);
-        omask = ld_relaxed(&p.resp[cw].overflow_mask);
-      }
-    }
-    pc.mark(PH_WAIT);
+    wait_response(p, cw, round, t_begin, base, cmask, omask);
+    if (p.commit == CSMV_COMMIT_ONLYCS) fence_gpu();  // acquire: the server's write-backs
     uint32_t cts = 0;
     if (mine) {
       if ((cmask >> lane) & 1u) {

@@ -45,7 +45,7 @@ __device__ __forceinline__ int kv_get(const KParams& p, uint32_t key, uint32_t s
       if (w0 + u >= A) break;
       const uint32_t slot = gset * A + w0 + u;
       uint32_t k4[4];
-      int rr = kv_key_pick<NS>(p.kv_key + (size_t)slot * NS * 4, r[u], K, s, k4);
+      int rr = kv_key_pick<NS>(p.kv_key + (size_t)slot * NS * 4, r[u], K, s, true, k4);
       if (rr != RD_OK) return rr;
 #pragma unroll
       for (int j = 0; j < 4; ++j) dg += dig_word(slot, j, k4[j]);
@@ -121,30 +121,63 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         ++att_u;
         int r = RD_OK;
         victim = 0xFFFFFFFFu;
-        for (uint32_t w = 0; w < A && victim == 0xFFFFFFFFu; ++w) {
-          const uint32_t slot = tset * A + w;
-          uint32_t key[4];
-          r = kv_read_mw<NS, 4>(p.kv_key + (size_t)slot * NS * 4, K, s, false, key);
-          if (r != RD_OK) break;
-          if (!compact) RS[nrs++ * 32 + lane] = slot;
+        // key scan, U ways in flight (as in kv_get), stop at match or empty
+        constexpr int U = 1;
+        for (uint32_t w0 = 0; w0 < A && victim == 0xFFFFFFFFu && r == RD_OK; w0 += U) {
+          Ring<4> rk[U][NS];
 #pragma unroll
-          for (int j = 0; j < 4; ++j) rdig += dig_word(slot, j, key[j]);
-          if ((key[0] == kk[0] && key[1] == kk[1] && key[2] == kk[2] && key[3] == kk[3]) ||
-              !(key[0] | key[1] | key[2] | key[3]))
-            victim = slot;
+          for (int u = 0; u < U; ++u) {
+            if (w0 + u < A) {
+              const uint64_t* ring = p.kv_key + (size_t)(tset * A + w0 + u) * NS * 4;
+#pragma unroll
+              for (int j = 0; j < NS; ++j) rk[u][j] = ld_ring<4>(ring + j * 4);
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            if (w0 + u >= A || victim != 0xFFFFFFFFu || r != RD_OK) break;
+            const uint32_t slot = tset * A + w0 + u;
+            uint32_t key[4];
+            r = kv_key_pick<NS>(p.kv_key + (size_t)slot * NS * 4, rk[u], K, s, false, key);
+            if (r != RD_OK) break;
+            if (!compact) RS[nrs++ * 32 + lane] = slot;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) rdig += dig_word(slot, j, key[j]);
+            if ((key[0] == kk[0] && key[1] == kk[1] && key[2] == kk[2] && key[3] == kk[3]) ||
+                !(key[0] | key[1] | key[2] | key[3]))
+              victim = slot;
+          }
         }
         if (r == RD_OK && victim == 0xFFFFFFFFu) {
+          // LRU scan of the full set; a one-word ring needs one pass (a newer
+          // version anywhere aborts the PUT anyway)
+          constexpr int UL = 4;
           uint32_t best = 0;
-          for (uint32_t w = 0; w < A; ++w) {
-            const uint32_t slot = tset * A + w;
-            uint32_t l;
-            r = kv_read_1<NS>(p.kv_lru + (size_t)slot * NS, K, s, l);
-            if (r != RD_OK) break;
-            if (!compact) RS[nrs++ * 32 + lane] = 2 * S + slot;
-            rdig += dig1(2 * S + slot, l);
-            if (w == 0 || l < best) {
-              best = l;
-              victim = slot;
+          for (uint32_t w0 = 0; w0 < A && r == RD_OK; w0 += UL) {
+            Ring<NS> rl[UL];
+#pragma unroll
+            for (int u = 0; u < UL; ++u)
+              if (w0 + u < A) rl[u] = ld_ring<NS>(p.kv_lru + (size_t)(tset * A + w0 + u) * NS);
+#pragma unroll
+            for (int u = 0; u < UL; ++u) {
+              if (w0 + u >= A) break;
+              const uint32_t slot = tset * A + w0 + u;
+              const Sel q = select_version<NS>(rl[u], s);
+              if (q.newest > s) {
+                r = RD_NEWER;
+                break;
+              }
+              if (q.best < 0 || (uint32_t)q.best >= K) {
+                r = RD_MISS;
+                break;
+              }
+              const uint32_t l = (uint32_t)slot_at<NS>(rl[u], q.best);
+              if (!compact) RS[nrs++ * 32 + lane] = 2 * S + slot;
+              rdig += dig1(2 * S + slot, l);
+              if (w0 + u == 0 || l < best) {
+                best = l;
+                victim = slot;
+              }
             }
           }
         }
@@ -244,6 +277,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       if (lane == 0) {
         p.req_hdr[cw].snapshot = s;
         p.req_hdr[cw].mask = kept;
+        p.req_hdr[cw].round = round;
       }
       __syncwarp();
       fence_gpu();
@@ -271,7 +305,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         cc.ro_ck ^= dg;
         cr += T;
         att_r = 0;
-        if (p.ro_adaptive && kept && ld_relaxed(&p.resp[cw].seq) == round) break;
+        if (p.ro_adaptive && kept && (uint32_t)(ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
       }
     }
     __syncwarp();
@@ -280,28 +314,8 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
 
     // ---- D: response, write-back, GTS
     uint32_t base = 0, cmask = 0, omask = 0;
-    {
-      uint32_t it = 0;
-      bool ok = true;
-      while (warp_ld_relaxed(&p.resp[cw].seq) != round) {
-        if ((++it & 255u) == 0) {
-          uint32_t bad = 0;
-          if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);
-          if (__shfl_sync(FULL, bad, 0)) {
-            ok = false;
-            break;
-          }
-        }
-        __nanosleep(64);
-      }
-      fence_gpu();
-      if (ok) {
-        base = ld_relaxed(&p.resp[cw].cts_base);
-        cmask = ld_relaxed(&p.resp[cw].commit_mask);
-        omask = ld_relaxed(&p.resp[cw].overflow_mask);
-      }
-    }
-    pc.mark(PH_WAIT);
+    wait_response(p, cw, round, t_begin, base, cmask, omask);
+    if (p.commit == CSMV_COMMIT_ONLYCS) fence_gpu();  // acquire: the server's write-backs
     uint32_t cts = 0;
     if (mine) {
       if ((cmask >> lane) & 1u) {

@@ -103,6 +103,41 @@ __device__ __forceinline__ uint32_t warp_ld_relaxed(const uint32_t* p) {
   return __shfl_sync(0xFFFFFFFFu, v, 0);
 }
 
+__device__ __forceinline__ uint64_t warp_ld_relaxed64(const uint64_t* p) {
+  uint64_t v = 0;
+  if ((threadIdx.x & 31) == 0) v = ld_relaxed64(p);
+  return __shfl_sync(0xFFFFFFFFu, v, 0);
+}
+
+__device__ __forceinline__ bool watchdog(const KParams& p, uint64_t t0, uint32_t where);
+
+// Wait for the server's answer to request `round` of client warp cw (all
+// three words tagged with round).  false if the run is being torn down.
+__device__ __forceinline__ bool wait_response(const KParams& p, uint32_t cw, uint32_t round, uint64_t t_begin,
+                                              uint32_t& base, uint32_t& cmask, uint32_t& omask) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  uint32_t it = 0;
+  uint64_t b, c, o;
+  for (;;) {
+    b = warp_ld_relaxed64(&p.resp[cw].base);
+    if ((uint32_t)(b >> 32) == round) {
+      c = warp_ld_relaxed64(&p.resp[cw].commit);
+      o = warp_ld_relaxed64(&p.resp[cw].ovf);
+      if ((uint32_t)(c >> 32) == round && (uint32_t)(o >> 32) == round) break;
+    }
+    if ((++it & 255u) == 0) {
+      uint32_t bad = 0;
+      if ((threadIdx.x & 31) == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);
+      if (__shfl_sync(FULL, bad, 0)) return false;
+    }
+    __nanosleep(64);
+  }
+  base = (uint32_t)b;
+  cmask = (uint32_t)c;
+  omask = (uint32_t)o;
+  return true;
+}
+
 __device__ __forceinline__ bool watchdog(const KParams& p, uint64_t t0, uint32_t where) {
   if (globaltimer() - t0 > p.watchdog_ns) {
     if (atomicCAS(&p.ctl->error, 0u, 1u) == 0u) p.ctl->where = where;

@@ -40,16 +40,22 @@ struct Ctl {
   uint32_t jv_tail;     // CSMV_COMMIT_JVSTM: last CTS reserved (global CAS target)
 };
 
-struct ReqHdr {
+struct ReqHdr {        // written before the doorbell
   uint32_t snapshot;
   uint32_t mask;
+  uint32_t round;      // = the doorbell value; tags the response
+  uint32_t pad;
 };
 
+// The response: every word carries the request's round in its upper half,
+// so the client accepts it word by word -- no release/acquire pair and no
+// fence on the server's respond path (the client needs nothing else the
+// server wrote; CSMV_COMMIT_ONLYCS fences its write-backs first).
 struct Resp {
-  uint32_t cts_base;
-  uint32_t commit_mask;
-  uint32_t overflow_mask;
-  uint32_t seq;
+  uint64_t base;       // round << 32 | first CTS of the batch
+  uint64_t commit;     // round << 32 | commit mask
+  uint64_t ovf;        // round << 32 | overflow mask
+  uint64_t pad;
 };
 
 struct DevStats {

@@ -101,9 +101,11 @@ __device__ __forceinline__ int kv_read_mw(const uint64_t* ring, uint32_t K, uint
 // is re-read (address-dependent on the first loads, so ordered after them):
 // still intact means no version in (cts, s] was recycled meanwhile (oldest-
 // first recycling) -- the argument of rot_scan.
+// rot = false (a PUT's read): any version newer than s -> RD_NEWER, as in
+// kv_read_mw (a torn slot carries a newer ts, so it is covered too).
 template <int NS>
 __device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (&r)[NS], uint32_t K, uint32_t s,
-                                           uint32_t (&out)[4]) {
+                                           bool rot, uint32_t (&out)[4]) {
   int cand = -1;
   uint32_t cts = 0, newest = 0, torn_max = 0;
   bool torn = false;
@@ -128,6 +130,7 @@ __device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (
       cts = t0;
     }
   }
+  if (!rot && newest > s) return RD_NEWER;
   if (cand < 0 || (torn && torn_max > cts)) return RD_MISS;
   if (newest > s) {
     const Ring<4> q = ld_ring<4>(ring + cand * 4);

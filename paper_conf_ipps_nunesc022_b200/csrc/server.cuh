@@ -169,7 +169,7 @@ __device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64_t t_be
   uint32_t tail = 0;
   uint32_t idle = 0;
   for (;;) {
-    bool found = false;
+    bool found = false, fenced = false;
     for (uint32_t r0 = 0; r0 < rows; r0 += 8) {
       uint32_t seq[8];
 #pragma unroll
@@ -184,6 +184,10 @@ __device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64_t t_be
         const uint32_t pm = __ballot_sync(FULL, pend);
         if (pm) {
           found = true;
+          if (!fenced) {  // acquire: the payloads of the doorbells just seen precede
+            fence_gpu();  // every worker's reads of them (queue -> fence.cta -> loads)
+            fenced = true;
+          }
           if (pend) {
             const uint32_t pos = tail + __popc(pm & lt);
             c.last_seen[i] = seq[k];
@@ -355,27 +359,26 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
     }
     const long long t0 = clock64();
-    // ---- load the batches: doorbell (acquire pattern), header, ids
+    // ---- load the batches: header and ids together (the receiver's fence
+    // ordered them after the doorbells; ours orders them after the queue)
+    fence_cta();
     uint32_t sq[M], sn[M], msk[M], id0[M], id1[M];
 #pragma unroll
-    for (int j = 0; j < M; ++j) sq[j] = (j < (int)m) ? ld_relaxed(p.req_seq + cwv[j]) : 0u;
-    fence_gpu();
-#pragma unroll
     for (int j = 0; j < M; ++j) {
-      sn[j] = msk[j] = id0[j] = id1[j] = 0;
+      sq[j] = sn[j] = msk[j] = id0[j] = id1[j] = 0;
       if (j < (int)m) {
         sn[j] = ld_relaxed(&p.req_hdr[cwv[j]].snapshot);
         msk[j] = ld_relaxed(&p.req_hdr[cwv[j]].mask);
+        sq[j] = ld_relaxed(&p.req_hdr[cwv[j]].round);
+        id0[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + lane) & ~kWriteBit;
+        id1[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + 32 + lane) & ~kWriteBit;
       }
     }
     bool mine[M];
 #pragma unroll
     for (int j = 0; j < M; ++j) {
       mine[j] = (msk[j] >> lane) & 1u;
-      if (mine[j]) {
-        id0[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + lane) & ~kWriteBit;
-        id1[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + 32 + lane) & ~kWriteBit;
-      }
+      if (!mine[j]) id0[j] = id1[j] = 0;
     }
     const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
     srv_fence<CL>();
@@ -442,20 +445,16 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) done_ring_room(p, c, t, t_begin);
     cs_leave<CL>(c, ticket, t);
     const long long t2 = clock64();
-    // ---- respond: one fence, then the payloads and sequence words
-    if (lane == 0) {
+    // ---- respond: round-tagged words, no fence (kernel.cuh Resp)
+    if (lane < (uint32_t)m) {
 #pragma unroll
       for (int j = 0; j < M; ++j) {
-        if (j >= (int)m) break;
-        st_relaxed(&p.resp[cwv[j]].cts_base, base[j]);
-        st_relaxed(&p.resp[cwv[j]].commit_mask, cm[j]);
-        st_relaxed(&p.resp[cwv[j]].overflow_mask, om[j]);
-      }
-      fence_gpu();
-#pragma unroll
-      for (int j = 0; j < M; ++j) {
-        if (j >= (int)m) break;
-        st_relaxed(&p.resp[cwv[j]].seq, sq[j]);
+        if ((uint32_t)j == lane) {
+          const uint64_t tag = (uint64_t)sq[j] << 32;
+          st_relaxed64(&p.resp[cwv[j]].base, tag | base[j]);
+          st_relaxed64(&p.resp[cwv[j]].commit, tag | cm[j]);
+          st_relaxed64(&p.resp[cwv[j]].ovf, tag | om[j]);
+        }
       }
     }
     __syncwarp();
@@ -502,17 +501,18 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     const long long tq = clock64();
     if (!claim_request(c, cw)) break;
     const long long t0 = clock64();
-    const uint32_t sq = ld_relaxed(p.req_seq + cw);
-    fence_gpu();
+    fence_cta();  // after the receiver's acquire (see server_receiver)
+    const uint32_t sq = ld_relaxed(&p.req_hdr[cw].round);
     const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
     const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
-    const bool mine = (mask >> lane) & 1u;
-    const uint32_t cnt = mine ? ld_relaxed(p.req_cnt + (size_t)cw * 32 + lane) : 0u;
-    const uint32_t nval = compact ? min(cnt, 1u) : cnt;  // ids to validate
-    uint32_t ids[kKvMaxId];
+    const uint32_t cnt_raw = ld_relaxed(p.req_cnt + (size_t)cw * 32 + lane);
+    uint32_t ids[kKvMaxId];  // loaded with the header; rows past a lane's count are ignored
 #pragma unroll
     for (uint32_t k = 0; k < kKvMaxId; ++k)
-      ids[k] = (k < cnt) ? ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + k) * 32 + lane) : 0u;
+      ids[k] = (!compact || k < 4) ? ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + k) * 32 + lane) : 0u;
+    const bool mine = (mask >> lane) & 1u;
+    const uint32_t cnt = mine ? cnt_raw : 0u;
+    const uint32_t nval = compact ? min(cnt, 1u) : cnt;  // ids to validate
     const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
     srv_fence<CL>();
     uint32_t lw[kKvMaxId];
@@ -571,11 +571,11 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     const long long tr = clock64();
     cs_leave<CL>(c, ticket, t0c + n);
     const long long t2 = clock64();
-    if (lane == 0) {
-      st_relaxed(&p.resp[cw].cts_base, t0c + 1);
-      st_relaxed(&p.resp[cw].commit_mask, cm);
-      st_relaxed(&p.resp[cw].overflow_mask, om);
-      st_release(&p.resp[cw].seq, sq);
+    if (lane == 0) {  // round-tagged words, no fence (kernel.cuh Resp)
+      const uint64_t tag = (uint64_t)sq << 32;
+      st_relaxed64(&p.resp[cw].base, tag | (t0c + 1));
+      st_relaxed64(&p.resp[cw].commit, tag | cm);
+      st_relaxed64(&p.resp[cw].ovf, tag | om);
     }
     __syncwarp();
     const long long t3 = clock64();
@@ -622,8 +622,8 @@ __device__ void server_worker_onlycs(const KParams& p, const SrvCtx& c, uint64_t
     uint32_t cw;
     if (!claim_request(c, cw)) break;
     const long long t0 = clock64();
-    const uint32_t sq = ld_relaxed(p.req_seq + cw);
-    fence_gpu();
+    fence_cta();  // after the receiver's acquire (see server_receiver)
+    const uint32_t sq = ld_relaxed(&p.req_hdr[cw].round);
     const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
     const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
     const bool mine = (mask >> lane) & 1u;
@@ -679,11 +679,11 @@ __device__ void server_worker_onlycs(const KParams& p, const SrvCtx& c, uint64_t
     }
     __syncwarp();
     fence_gpu();  // the write-backs precede the response (the client publishes GTS after it)
-    if (lane == 0) {
-      st_relaxed(&p.resp[cw].cts_base, base);
-      st_relaxed(&p.resp[cw].commit_mask, cm);
-      st_relaxed(&p.resp[cw].overflow_mask, om);
-      st_release(&p.resp[cw].seq, sq);
+    if (lane == 0) {  // round-tagged words after the fence above
+      const uint64_t tag = (uint64_t)sq << 32;
+      st_relaxed64(&p.resp[cw].base, tag | base);
+      st_relaxed64(&p.resp[cw].commit, tag | cm);
+      st_relaxed64(&p.resp[cw].ovf, tag | om);
     }
     __syncwarp();
     busy += (unsigned long long)(clock64() - t0);
