@@ -251,6 +251,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
     uint32_t base = 0, cmask = 0, omask = 0;
     wait_response(p, cw, round, t_begin, base, cmask, omask);
     if (p.commit == CSMV_COMMIT_ONLYCS) fence_gpu();  // acquire: the server's write-backs
+    pc.mark(PH_WAIT);
     uint32_t cts = 0;
     if (mine) {
       if ((cmask >> lane) & 1u) {

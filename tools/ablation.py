@@ -28,7 +28,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
 
 VARIANTS = {
-    "csmv-b200": dict(atr_mode=csmv.ATR_HASH, server_combine=4, server_workers=6, ro_streak=8,
+    "csmv-b200": dict(atr_mode=csmv.ATR_HASH, server_combine=4, server_workers=6, ro_streak=8, ro_adaptive=1,
                       publish=csmv.PUBLISH_SERVER),
     "csmv": dict(atr_mode=csmv.ATR_LIST, server_combine=1, ro_streak=0, publish=csmv.PUBLISH_CLIENT),
     "nocv": dict(atr_mode=csmv.ATR_LIST_NOCV, server_combine=1, ro_streak=0, publish=csmv.PUBLISH_CLIENT),
