@@ -162,3 +162,9 @@ def test_kv_ro_adaptive_parity():
     cfg = W.c4(n_items=1 << 14, n_tx=1 << 17, p_update_ppm=20_000, client_warps=256, server_workers=6,
                ro_streak=32, ro_adaptive=1)
     _check_kv(cfg)
+
+
+def test_kv_small_atr():
+    cfg = W.c4(n_items=1 << 14, n_tx=1 << 17, p_update_ppm=100_000, client_warps=256, server_workers=6,
+               atr_capacity=256, dist=0)
+    _check_kv(cfg)

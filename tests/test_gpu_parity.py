@@ -215,3 +215,14 @@ def test_ro_adaptive_parity(preset, streak):
              server_workers=6, server_combine=4, publish=csmv.PUBLISH_SERVER)
     rep, stats, log, rings, descs = check(cfg)
     assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions), closed_form(cfg, descs, cfg.init_values()))
+
+
+@pytest.mark.parametrize("cap", [256, 1024])
+def test_small_atr_bucket_races(cap):
+    """Few buckets: lanes of one batch often race for the same way of a
+    bucket, so displaced entries are re-inserted (server.cuh rt_record) or
+    fold into the irregular-eviction watermark -- never lost."""
+    cfg = W.c2(n_items=1 << 14, n_tx=1 << 17, atr_capacity=cap, server_combine=4, server_workers=6,
+               client_warps=256, ro_streak=4, publish=csmv.PUBLISH_SERVER)
+    rep, stats, log, rings, descs = check(cfg)
+    assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions), closed_form(cfg, descs, cfg.init_values()))
