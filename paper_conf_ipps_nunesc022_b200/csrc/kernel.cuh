@@ -92,7 +92,7 @@ struct KParams {
   uint32_t n_server_ctas;  // 1, or the cluster size of a cluster server
   uint32_t clog2;          // log2(n_server_ctas)
   uint32_t n_workers;      // server worker warps
-  uint32_t rt_log2;        // recent-commit table buckets, all server CTAs (4 ways, 32 B each)
+  uint32_t rt_log2;        // recent-commit table buckets, all server CTAs (4 ways, 32 B each, + evmax)
   uint32_t* lastw;         // per-item CTS of the last committed write
   uint32_t publish;
   uint32_t ro_streak;      // read-only transactions a lane may run per round (0 = one tx per round)
@@ -138,7 +138,7 @@ __host__ __device__ inline uint32_t queue_log2(uint32_t n_cw) {
 // recent-commit table, dispatch queue, receiver's last-seen doorbells, control words
 // (per server CTA: its stripe of 2^local_log2 buckets and its slice of n_cw)
 inline size_t server_smem_bytes(uint32_t local_log2, uint32_t n_cw) {
-  return ((size_t)32 << local_log2) + ((size_t)8 << queue_log2(n_cw)) +
+  return ((size_t)(32 + 4) << local_log2) + ((size_t)8 << queue_log2(n_cw)) +
          (((size_t)n_cw + 31) / 32 * 32) * 4 + 64;
 }
 

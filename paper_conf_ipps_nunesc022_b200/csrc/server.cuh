@@ -24,7 +24,6 @@ struct SrvShared {
   uint32_t next_ticket;  // ticket lock around validate+reserve+insert        [CTA 0]
   uint32_t now_serving;  //                                                   [CTA 0]
   uint32_t gts_seen;     // publisher progress seen by workers (back-pressure) [CTA 0]
-  uint32_t evx;          // largest CTS evicted irregularly from the table     [CTA 0]
   uint32_t q_head;       // next dispatch-queue slot a worker claims          [per CTA]
   uint32_t exit;         // receiver: all clients finished                    [per CTA]
 };
@@ -34,24 +33,15 @@ struct SrvShared {
 //  * lastw[x] in HBM: CTS of the last commit that wrote x -- the exact
 //    record of every committed write-set, all history;
 //  * rt in shared memory: 4-way buckets of (cts << 32 | item) holding recent
-//    writes, so that commits made after a worker prefetched lastw (CTS >
-//    e_pre) are seen with on-chip latency.
-// Replacement: a write of x overwrites x's own way, else the way with the
-// smallest CTS.  Entries are only ever replaced by newer ones, so a bucket's
-// minimum CTS never decreases, and a regular eviction removes the minimum:
-// every entry left behind (and every later one) has a CTS >= the evicted
-// one.  Invariant: if the latest write c of item y is not in its bucket b,
-// then min_cts(b) >= c, or evx >= c, where evx (one word, CTA 0) collects
-// the CTS of the irregular evictions -- an entry replaced although it was
-// not the minimum (two lanes of one batch racing for a way, or both items
-// of one transaction in one bucket); rt_record detects those by comparing
-// what atomicExch returned with what the probe saw.
+//    writes plus, per bucket, evmax = the largest CTS ever evicted from it,
+//    so that commits made after a worker prefetched lastw (CTS > e_pre) are
+//    seen with on-chip latency.
+// Invariant: if the latest write c of item y (bucket b) is not in b, then
+// evmax[b] >= c (entries leave a bucket only through atomicExch, and the
+// evictor records the evicted CTS with atomicMax).
 // Validation of x for snapshot s (P:75 read-set, P:115 write-set), s <= e_pre:
 //    conflict  iff  lastw[x] (as of e_pre) > s  or  some way holds (x, c), c > s
-//    unknown   iff  not conflict and (min_cts(b) > e_pre or evx > e_pre)
-//              -> abort, reason OVERFLOW
-// A bucket is a 32-byte load and a record one atomicExch: no per-bucket
-// watermark to load or to raise with a second atomic.
+//    unknown   iff  not conflict and evmax[b] > e_pre -> abort, reason OVERFLOW
 // ---------------------------------------------------------------------------
 constexpr int kRtWays = 4;
 
@@ -61,6 +51,7 @@ __device__ __forceinline__ uint32_t rt_bucket(uint32_t key, uint32_t rt_log2) {
 
 struct SrvCtx {
   uint64_t* rt;       // this CTA's stripe of buckets (kRtWays u64 each)
+  uint32_t* evmax;    // this CTA's stripe of eviction watermarks
   uint32_t clog2;     // log2(server CTAs)
   SrvShared* sh;      // this CTA's control block
   SrvShared* sh0;     // CTA 0's control block (DSMEM in a cluster)
@@ -81,6 +72,16 @@ __device__ __forceinline__ uint64_t* rt_at(const SrvCtx& c, uint32_t b) {
 }
 
 template <bool CL>
+__device__ __forceinline__ uint32_t* ev_at(const SrvCtx& c, uint32_t b) {
+  if constexpr (!CL) {
+    return c.evmax + b;
+  } else {
+    const uint32_t owner = b & ((1u << c.clog2) - 1), local = b >> c.clog2;
+    return cg::this_cluster().map_shared_rank(c.evmax, owner) + local;
+  }
+}
+
+template <bool CL>
 __device__ __forceinline__ void srv_fence() {
   if constexpr (CL) asm volatile("fence.acq_rel.cluster;" ::: "memory");
   else fence_cta();
@@ -90,14 +91,13 @@ struct RtProbe {
   int way;        // way to overwrite: the way holding x, else the oldest
   bool conflict;
   bool unknown;
-  uint64_t old;   // the entry seen at `way`
-  uint32_t minc;  // the bucket's smallest CTS as seen
 };
 
-// A bucket as loaded (two 16-byte loads).  Loading and evaluating are split
-// so that callers can put several loads in flight.
+// A bucket as loaded: its 4 ways and its eviction watermark.  Loading and
+// evaluating are split so that callers can put several loads in flight.
 struct RtBucket {
   ulonglong2 a, b;
+  uint32_t ev;
 };
 
 template <bool CL>
@@ -106,13 +106,14 @@ __device__ __forceinline__ RtBucket rt_load(const SrvCtx& c, uint32_t bucket) {
   RtBucket q;
   q.a = e[0];
   q.b = e[1];
+  q.ev = *ev_at<CL>(c, bucket);
   return q;
 }
 
-// evx: the irregular-eviction watermark as of this point of the critical section
 __device__ __forceinline__ RtProbe rt_eval(const RtBucket& q, uint32_t key, uint32_t s, uint32_t e_pre,
-                                           uint32_t lastw, uint32_t evx) {
+                                           uint32_t lastw) {
   const uint64_t w[4] = {q.a.x, q.a.y, q.b.x, q.b.y};
+  const uint32_t ev = q.ev;
   RtProbe r;
   r.conflict = lastw > s;
   int hit = -1, old = 0;
@@ -129,46 +130,25 @@ __device__ __forceinline__ RtProbe rt_eval(const RtBucket& q, uint32_t key, uint
       old = i;
     }
   }
-  r.unknown = !r.conflict && (oldc > e_pre || evx > e_pre);
+  r.unknown = !r.conflict && ev > e_pre;
   r.way = hit >= 0 ? hit : old;
-  r.old = w[0];
-#pragma unroll
-  for (int i = 1; i < kRtWays; ++i) r.old = (r.way == i) ? w[i] : r.old;
-  r.minc = oldc;
   return r;
 }
 
 template <bool CL>
 __device__ __forceinline__ RtProbe rt_probe(const SrvCtx& c, uint32_t bucket, uint32_t key, uint32_t s,
-                                            uint32_t e_pre, uint32_t lastw, uint32_t evx) {
-  return rt_eval(rt_load<CL>(c, bucket), key, s, e_pre, lastw, evx);
+                                            uint32_t e_pre, uint32_t lastw) {
+  return rt_eval(rt_load<CL>(c, bucket), key, s, e_pre, lastw);
 }
 
-// Record (key, cts) over q.way of its bucket.  A regular eviction (the
-// entry the probe saw, holding the bucket minimum) needs nothing more.  An
-// entry displaced otherwise -- another lane of this batch took the same way
-// first, or q.way was moved off the minimum -- is put back over the
-// bucket's current minimum (or its own key's older entry), a few times at
-// most; an entry still displaced after that is returned (its CTS) for the
-// caller to fold into evx before the next validation.
+// Record (key, cts) into `way` of its bucket; an evicted entry of another
+// key raises evmax.  Exchanges by several lanes on one slot are serialised
+// by the hardware and each evictor sees the value it replaced.
 template <bool CL>
-__device__ __forceinline__ uint32_t rt_record(const SrvCtx& c, uint32_t bucket, const RtProbe& q, uint32_t key,
-                                              uint32_t cts) {
-  unsigned long long* slot = reinterpret_cast<unsigned long long*>(rt_at<CL>(c, bucket));
-  unsigned long long old = atomicExch(slot + q.way, ((unsigned long long)cts << 32) | key);
-  if ((uint32_t)old == key) return 0u;  // x's own older entry
-  uint64_t expect = q.old;
-  uint32_t minc = q.minc;
-  for (int it = 0; it < 4; ++it) {
-    if (old == expect && (uint32_t)(old >> 32) == minc) return 0u;
-    const RtProbe r = rt_eval(rt_load<CL>(c, bucket), (uint32_t)old, 0u, 0u, 0u, 0u);
-    const unsigned long long nxt = atomicExch(slot + r.way, old);
-    if ((uint32_t)nxt == (uint32_t)old) return 0u;  // replaced the displaced key's own older entry
-    expect = r.old;
-    minc = r.minc;
-    old = nxt;
-  }
-  return (old == expect && (uint32_t)(old >> 32) == minc) ? 0u : (uint32_t)(old >> 32);
+__device__ __forceinline__ void rt_record(const SrvCtx& c, uint32_t bucket, int way, uint32_t key, uint32_t cts) {
+  const unsigned long long old =
+      atomicExch(reinterpret_cast<unsigned long long*>(rt_at<CL>(c, bucket) + way), ((unsigned long long)cts << 32) | key);
+  if ((uint32_t)old != key && (uint32_t)(old >> 32) != 0u) atomicMax(ev_at<CL>(c, bucket), (uint32_t)(old >> 32));
 }
 
 // ---------------------------------------------------------------------------
@@ -423,7 +403,6 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     const uint32_t ticket = cs_enter<CL>(c);
     const long long t1 = clock64();
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
-    uint32_t evx = *(volatile uint32_t*)&c.sh0->evx;
     uint32_t t = t0c;
     uint32_t cm[M], om[M], base[M];
 #pragma unroll
@@ -431,16 +410,13 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       cm[j] = om[j] = 0;
       base[j] = t + 1;
       if (j >= (int)m) continue;
-      RtProbe q0{0, false, false, 0ull, 0u}, q1{0, false, false, 0ull, 0u};
+      RtProbe q0{0, false, false}, q1{0, false, false};
       bool ovf = false, conflict = false;
       if (p.atr_mode == CSMV_ATR_HASH) {
         if (mine[j]) {
-          q0 = rt_probe<CL>(c, bk0[j], id0[j], sn[j], e_pre, lw0[j], evx);
-          q1 = rt_probe<CL>(c, bk1[j], id1[j], sn[j], e_pre, lw1[j], evx);
-          if (bk1[j] == bk0[j] && q1.way == q0.way) {  // both items in one bucket: q1 takes the next way
-            q1.way = (q1.way + 1) & (kRtWays - 1);
-            q1.old = ~0ull;  // an irregular eviction
-          }
+          q0 = rt_probe<CL>(c, bk0[j], id0[j], sn[j], e_pre, lw0[j]);
+          q1 = rt_probe<CL>(c, bk1[j], id1[j], sn[j], e_pre, lw1[j]);
+          if (bk1[j] == bk0[j] && q1.way == q0.way) q1.way = (q1.way + 1) & (kRtWays - 1);
         }
         ovf = mine[j] && (q0.unknown || q1.unknown);
         conflict = mine[j] && (q0.conflict || q1.conflict);
@@ -453,20 +429,18 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       om[j] = __ballot_sync(FULL, ovf);
       const uint32_t cts = t + 1 + __popc(cm[j] & lt);
       t += __popc(cm[j]);
-      uint32_t irr = 0;
       if (commit) {
         if (p.atr_mode == CSMV_ATR_HASH) {
           p.lastw[id0[j]] = cts;
           p.lastw[id1[j]] = cts;
-          irr = max(rt_record<CL>(c, bk0[j], q0, id0[j], cts), rt_record<CL>(c, bk1[j], q1, id1[j], cts));
+          rt_record<CL>(c, bk0[j], q0.way, id0[j], cts);
+          rt_record<CL>(c, bk1[j], q1.way, id1[j], cts);
         } else {  // the paper's ATR: the write-set of commit `cts` at entry cts
           c.rt[cts & ((uint32_t)(kRtWays << (p.rt_log2 - p.clog2)) - 1)] = ((uint64_t)id1[j] << 32) | id0[j];
         }
       }
-      if (p.atr_mode == CSMV_ATR_HASH) evx = max(evx, __reduce_max_sync(FULL, irr));
       __syncwarp();  // batch j's records precede batch j+1's probes
     }
-    if ((threadIdx.x & 31) == 0) *(volatile uint32_t*)&c.sh0->evx = evx;
     const long long ta = clock64();
     if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) done_ring_room(p, c, t, t_begin);
     cs_leave<CL>(c, ticket, t);
@@ -554,7 +528,6 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     const uint32_t ticket = cs_enter<CL>(c);
     const long long t1 = clock64();
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
-    uint32_t evx = *(volatile uint32_t*)&c.sh0->evx;
     bool conflict = false, unknown = false;
     // four buckets in flight per step; warp-uniform exit after the longest set
 #pragma unroll
@@ -567,7 +540,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
 #pragma unroll
       for (uint32_t u = 0; u < 4; ++u) {
         if (k0 + u < kKvMaxId && k0 + u < nval) {
-          const RtProbe r = rt_eval(q[u], ids[k0 + u] & ~kWriteBit, s, e_pre, lw[k0 + u], evx);
+          const RtProbe r = rt_eval(q[u], ids[k0 + u] & ~kWriteBit, s, e_pre, lw[k0 + u]);
           conflict |= r.conflict;
           unknown |= r.unknown;
         }
@@ -582,7 +555,6 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     const uint32_t cts = t0c + 1 + __popc(cm & lt);
     const long long tv = clock64();
     if (p.publish == CSMV_PUBLISH_SERVER && n) done_ring_room(p, c, t0c + n, t_begin);
-    uint32_t irr = 0;
     if (commit) {
 #pragma unroll
       for (uint32_t k = 0; k < kKvMaxId; ++k) {
@@ -590,15 +562,13 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
           const uint32_t id = ids[k] & ~kWriteBit, b = rt_bucket(id, p.rt_log2);
           p.lastw[id] = cts;  // every written item, so lastw stays exact for any later run
           if (k < nval || !compact) {
-            const RtProbe q = rt_probe<CL>(c, b, id, 0u, 0u, 0u, 0u);  // the way to (re)use, now
-            irr = max(irr, rt_record<CL>(c, b, q, id, cts));
+            const RtProbe q = rt_probe<CL>(c, b, id, 0u, 0u, 0u);  // the way to (re)use
+            rt_record<CL>(c, b, q.way, id, cts);
           }
         }
       }
     }
     const long long tr = clock64();
-    evx = max(evx, __reduce_max_sync(FULL, irr));
-    if (lane == 0) *(volatile uint32_t*)&c.sh0->evx = evx;
     cs_leave<CL>(c, ticket, t0c + n);
     const long long t2 = clock64();
     if (lane == 0) {  // round-tagged words, no fence (kernel.cuh Resp)
@@ -771,7 +741,7 @@ __device__ void server_publisher(const KParams& p, const SrvCtx& c, uint64_t t_b
 }
 
 // Shared-memory layout of one server CTA (every CTA of the fused grid gets
-// the same dynamic allocation): rt stripe, dispatch queue,
+// the same dynamic allocation): rt stripe, evmax stripe, dispatch queue,
 // last-seen doorbells of its slice, control block.
 template <int NS, int KIND, bool CL>
 __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
@@ -787,12 +757,14 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   c.rt = reinterpret_cast<uint64_t*>(smem);
   const uint32_t rt_words = (uint32_t)kRtWays << local_log2;
   c.queue = c.rt + rt_words;
-  c.last_seen = reinterpret_cast<uint32_t*>(c.queue + (1u << c.qn_log2));
+  c.evmax = reinterpret_cast<uint32_t*>(c.queue + (1u << c.qn_log2));
+  c.last_seen = c.evmax + (1u << local_log2);
   const uint32_t ls_words = (per + 31) / 32 * 32;
   c.sh = reinterpret_cast<SrvShared*>(c.last_seen + ls_words);
   if constexpr (CL) c.sh0 = cg::this_cluster().map_shared_rank(c.sh, 0);
   else c.sh0 = c.sh;
   for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) c.rt[i] = 0xFFFFFFFFull;  // cts 0, no item
+  for (uint32_t i = threadIdx.x; i < (1u << local_log2); i += blockDim.x) c.evmax[i] = 0;
   for (uint32_t i = threadIdx.x; i < (1u << c.qn_log2); i += blockDim.x) c.queue[i] = 0;
   for (uint32_t i = threadIdx.x; i < ls_words; i += blockDim.x) c.last_seen[i] = 0;
   if (threadIdx.x == 0) {
@@ -801,7 +773,6 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     c.sh->next_ticket = 0;
     c.sh->now_serving = 0;
     c.sh->gts_seen = g0;
-    c.sh->evx = 0;
     c.sh->q_head = 0;
     c.sh->exit = 0;
   }

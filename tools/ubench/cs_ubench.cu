@@ -23,8 +23,10 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
   SrvCtx c;
   c.clog2 = 0;
   c.rt = reinterpret_cast<uint64_t*>(smem);
+  c.evmax = reinterpret_cast<uint32_t*>(c.rt + 4 * 4096);
   c.sh = c.sh0 = &sh;
   for (int i = threadIdx.x; i < 4 * 4096; i += blockDim.x) c.rt[i] = 0xFFFFFFFFull;
+  for (int i = threadIdx.x; i < 4096; i += blockDim.x) c.evmax[i] = 0;
   if (threadIdx.x == 0) sh.tail = sh.next_ticket = sh.now_serving = 0;
   __syncthreads();
   const uint32_t warp = threadIdx.x / 32;
@@ -47,10 +49,10 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
     }
     const long long a = clock64();
     const uint32_t s = t > 50 ? t - 50 : 0, e_pre = t;
-    RtProbe q0{0, false, false, 0ull, 0u}, q1{0, false, false, 0ull, 0u};
+    RtProbe q0{0, false, false}, q1{0, false, false};
     if (mode >= 1 && mine) {
-      q0 = rt_probe<false>(c, b0, id0, s, e_pre, 0, 0);
-      q1 = rt_probe<false>(c, b1, id1, s, e_pre, 0, 0);
+      q0 = rt_probe<false>(c, b0, id0, s, e_pre, 0);
+      q1 = rt_probe<false>(c, b1, id1, s, e_pre, 0);
       if (b1 == b0 && q1.way == q0.way) q1.way = (q1.way + 1) & 3;
     }
     const bool commit = mine && !q0.conflict && !q1.conflict && !q0.unknown && !q1.unknown;
@@ -62,7 +64,8 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
       lastw[id1 & 0xFFFFF] = cts;
     }
     if (commit && mode >= 2) {
-      sink += rt_record<false>(c, b0, q0, id0, cts) + rt_record<false>(c, b1, q1, id1, cts);
+      rt_record<false>(c, b0, q0.way, id0, cts);
+      rt_record<false>(c, b1, q1.way, id1, cts);
     }
     __syncwarp();
     acc += clock64() - a;
