@@ -298,8 +298,11 @@ def bench_ours(args):
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     e2e_committed = 0
+    t_load = 0.0
     for i in range(e2e_steps):
+        tl = time.perf_counter()
         store.load(w.kv_keys if is_kv else init_pinned.numpy())
+        t_load += time.perf_counter() - tl
         s = store.run(w, lcfg.n_tx, lcfg.seed + 500 + i)
         e2e_committed += s["committed"]
     torch.cuda.synchronize()
@@ -340,7 +343,8 @@ def bench_ours(args):
                          "critical_section_cycles_per_batch": cs_cycles,
                          "updates_per_batch": red["committed_update"] / max(1, red["batches"])},
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(init.nbytes),
-                "d2h_bytes_per_step": 400},
+                "d2h_bytes_per_step": 400, "steps": e2e_steps,
+                "load_ms_per_step": 1e3 * t_load / e2e_steps, "wall_ms_per_step": 1e3 * e2e_s / e2e_steps},
         "gpu_launches": args.steps * int(last["kernel_launches"]),
         "clocks": clk.summary(),
         "kernel_ms_per_step": statistics.mean(kern_ns) / 1e6,
