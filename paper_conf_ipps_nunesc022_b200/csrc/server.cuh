@@ -42,14 +42,8 @@ struct SrvShared {
 // Validation of x for snapshot s (P:75 read-set, P:115 write-set), s <= e_pre:
 //    conflict  iff  lastw[x] (as of e_pre) > s  or  some way holds (x, c), c > s
 //    unknown   iff  not conflict and evmax[b] > e_pre -> abort, reason OVERFLOW
-// Bounded prefetch age: a batch whose e_pre lags the tail at its critical
-// section (t0) by more than kEvLag aborts with OVERFLOW; so every current
-// and later validator has e_pre >= t0 - kEvLag, lastw already covers an
-// evicted CTS <= t0 - kEvLag for all of them, and only younger evictions
-// need the atomicMax (most evictions are far older: C2 ~8K CTS).
 // ---------------------------------------------------------------------------
 constexpr int kRtWays = 4;
-constexpr uint32_t kEvLag = 2048;  // prefetch age bound (CTS), see above
 
 __device__ __forceinline__ uint32_t rt_bucket(uint32_t key, uint32_t rt_log2) {
   return (key * 0x9E3779B1u) >> (32 - rt_log2);
@@ -108,21 +102,11 @@ struct RtBucket {
 
 template <bool CL>
 __device__ __forceinline__ RtBucket rt_load(const SrvCtx& c, uint32_t bucket) {
+  const ulonglong2* e = reinterpret_cast<const ulonglong2*>(rt_at<CL>(c, bucket));
   RtBucket q;
-  if constexpr (CL) {
-    const ulonglong2* e = reinterpret_cast<const ulonglong2*>(rt_at<CL>(c, bucket));
-    q.a = e[0];
-    q.b = e[1];
-    q.ev = *ev_at<CL>(c, bucket);
-  } else {
-    // volatile asm keeps the three loads of one or more buckets issued back
-    // to back (ptxas otherwise serialises the latency of consecutive probes)
-    const uint32_t e = (uint32_t)__cvta_generic_to_shared(rt_at<CL>(c, bucket));
-    const uint32_t v = (uint32_t)__cvta_generic_to_shared(ev_at<CL>(c, bucket));
-    asm volatile("ld.volatile.shared.v2.u64 {%0,%1}, [%2];" : "=l"(q.a.x), "=l"(q.a.y) : "r"(e) : "memory");
-    asm volatile("ld.volatile.shared.v2.u64 {%0,%1}, [%2+16];" : "=l"(q.b.x), "=l"(q.b.y) : "r"(e) : "memory");
-    asm volatile("ld.volatile.shared.u32 %0, [%1];" : "=r"(q.ev) : "r"(v) : "memory");
-  }
+  q.a = e[0];
+  q.b = e[1];
+  q.ev = *ev_at<CL>(c, bucket);
   return q;
 }
 
@@ -158,20 +142,14 @@ __device__ __forceinline__ RtProbe rt_probe(const SrvCtx& c, uint32_t bucket, ui
 }
 
 // Record (key, cts) into `way` of its bucket; an evicted entry of another
-// key younger than `covered` (= t0 - kEvLag, what lastw covers for every
-// current and later validator) raises evmax.  Exchanges by several lanes on
-// one slot are serialised by the hardware and each evictor sees the value
-// it replaced.
+// key raises evmax.  Exchanges by several lanes on one slot are serialised
+// by the hardware and each evictor sees the value it replaced.
 template <bool CL>
-__device__ __forceinline__ void rt_record(const SrvCtx& c, uint32_t bucket, int way, uint32_t key, uint32_t cts,
-                                          uint32_t covered) {
+__device__ __forceinline__ void rt_record(const SrvCtx& c, uint32_t bucket, int way, uint32_t key, uint32_t cts) {
   const unsigned long long old =
       atomicExch(reinterpret_cast<unsigned long long*>(rt_at<CL>(c, bucket) + way), ((unsigned long long)cts << 32) | key);
-  if ((uint32_t)old != key && (uint32_t)(old >> 32) > covered) atomicMax(ev_at<CL>(c, bucket), (uint32_t)(old >> 32));
+  if ((uint32_t)old != key && (uint32_t)(old >> 32) != 0u) atomicMax(ev_at<CL>(c, bucket), (uint32_t)(old >> 32));
 }
-
-// What lastw covers for every validator from a critical section that began at tail t0.
-__device__ __forceinline__ uint32_t ev_covered(uint32_t t0) { return t0 > kEvLag ? t0 - kEvLag : 0u; }
 
 // ---------------------------------------------------------------------------
 // Receiver warp: sweeps its slice of the client doorbells with
@@ -425,8 +403,6 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     const uint32_t ticket = cs_enter<CL>(c);
     const long long t1 = clock64();
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
-    const bool stale = t0c - e_pre > kEvLag;  // prefetch too old: abort (OVERFLOW)
-    const uint32_t covered = ev_covered(t0c);
     uint32_t t = t0c;
     uint32_t cm[M], om[M], base[M];
 #pragma unroll
@@ -438,13 +414,13 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       bool ovf = false, conflict = false;
       if (p.atr_mode == CSMV_ATR_HASH) {
         if (mine[j]) {
-          const RtBucket b0 = rt_load<CL>(c, bk0[j]), b1 = rt_load<CL>(c, bk1[j]);  // both in flight
+          const RtBucket b0 = rt_load<CL>(c, bk0[j]), b1 = rt_load<CL>(c, bk1[j]);
           q0 = rt_eval(b0, id0[j], sn[j], e_pre, lw0[j]);
           q1 = rt_eval(b1, id1[j], sn[j], e_pre, lw1[j]);
           if (bk1[j] == bk0[j] && q1.way == q0.way) q1.way = (q1.way + 1) & (kRtWays - 1);
         }
+        ovf = mine[j] && (q0.unknown || q1.unknown);
         conflict = mine[j] && (q0.conflict || q1.conflict);
-        ovf = mine[j] && !conflict && (q0.unknown || q1.unknown || stale);
       } else {
         atr_list_validate(p, c, sn[j], t, mine[j], id0[j], id1[j], ovf, conflict);
       }
@@ -458,8 +434,8 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
         if (p.atr_mode == CSMV_ATR_HASH) {
           p.lastw[id0[j]] = cts;
           p.lastw[id1[j]] = cts;
-          rt_record<CL>(c, bk0[j], q0.way, id0[j], cts, covered);
-          rt_record<CL>(c, bk1[j], q1.way, id1[j], cts, covered);
+          rt_record<CL>(c, bk0[j], q0.way, id0[j], cts);
+          rt_record<CL>(c, bk1[j], q1.way, id1[j], cts);
         } else {  // the paper's ATR: the write-set of commit `cts` at entry cts
           c.rt[cts & ((uint32_t)(kRtWays << (p.rt_log2 - p.clog2)) - 1)] = ((uint64_t)id1[j] << 32) | id0[j];
         }
@@ -553,8 +529,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     const uint32_t ticket = cs_enter<CL>(c);
     const long long t1 = clock64();
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
-    const uint32_t covered = ev_covered(t0c);
-    bool conflict = false, unknown = t0c - e_pre > kEvLag;  // prefetch too old: OVERFLOW
+    bool conflict = false, unknown = false;
     // four buckets in flight per step; warp-uniform exit after the longest set
 #pragma unroll
     for (uint32_t k0 = 0; k0 < kKvMaxId; k0 += 4) {
@@ -589,7 +564,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
           p.lastw[id] = cts;  // every written item, so lastw stays exact for any later run
           if (k < nval || !compact) {
             const RtProbe q = rt_probe<CL>(c, b, id, 0u, 0u, 0u);  // the way to (re)use
-            rt_record<CL>(c, b, q.way, id, cts, covered);
+            rt_record<CL>(c, b, q.way, id, cts);
           }
         }
       }

@@ -64,8 +64,8 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
       lastw[id1 & 0xFFFFF] = cts;
     }
     if (commit && mode >= 2) {
-      rt_record<false>(c, b0, q0.way, id0, cts, t > 8192 ? t - 8192 : 0);
-      rt_record<false>(c, b1, q1.way, id1, cts, t > 8192 ? t - 8192 : 0);
+      rt_record<false>(c, b0, q0.way, id0, cts);
+      rt_record<false>(c, b1, q1.way, id1, cts);
     }
     __syncwarp();
     acc += clock64() - a;
