@@ -51,6 +51,7 @@ __device__ __forceinline__ uint32_t rt_bucket(uint32_t key, uint32_t rt_log2) {
 
 struct SrvCtx {
   uint64_t* rt;       // this CTA's stripe of buckets (kRtWays u64 each)
+  uint32_t rt32;      // rt as a shared-window address
   uint32_t* evmax;    // this CTA's stripe of eviction watermarks
   uint32_t clog2;     // log2(server CTAs)
   SrvShared* sh;      // this CTA's control block
@@ -149,6 +150,57 @@ __device__ __forceinline__ void rt_record(const SrvCtx& c, uint32_t bucket, int 
   const unsigned long long old =
       atomicExch(reinterpret_cast<unsigned long long*>(rt_at<CL>(c, bucket) + way), ((unsigned long long)cts << 32) | key);
   if ((uint32_t)old != key && (uint32_t)(old >> 32) != 0u) atomicMax(ev_at<CL>(c, bucket), (uint32_t)(old >> 32));
+}
+
+// ---------------------------------------------------------------------------
+// Recent-write filter (the on-chip level of the ATR for the bank worker).
+// The same smem as the table above, read as 2^(rt_log2+3) u32 slots striped
+// over the server CTAs: slot i holds the largest CTS of any committed write
+// whose item hashes to i under one of kFiltK hash functions (a batch stores
+// its LAST CTS for all of its writes, so lanes that share a slot store the
+// same value and plain stores suffice -- the critical-section holder is the
+// only writer).  Values only grow.  For a transaction with snapshot s,
+// validated with lastw prefetched at tail e_pre >= s:
+//    conflict  iff  lastw[x] > s                        (exact, every CTS <= e_pre)
+//    unknown   iff  no conflict and min_k F[h_k(x)] > e_pre
+// A write of x after e_pre raises all k slots of x above e_pre, so "no
+// unknown" proves there was none; "unknown" aborts with the labelled reason
+// OVERFLOW -- a true conflict inside the window, or a false
+// positive with probability ~(k W / slots)^k for W writes in the window.
+// Per item: k loads and k stores, no atomics, no eviction.
+// ---------------------------------------------------------------------------
+constexpr int kFiltK = 3;
+
+// slot k of item x: multiplicative hashes with three odd constants
+__device__ __forceinline__ uint32_t filt_slot(uint32_t x, int k, uint32_t slots_log2) {
+  const uint32_t C[3] = {0x9E3779B1u, 0x85EBCA77u, 0xC2B2AE3Du};
+  return (x * C[k]) >> (32 - slots_log2);
+}
+
+// 32-bit shared-window address of filter slot i (a shared::cluster address
+// of the owning CTA for the cluster server)
+template <bool CL>
+__device__ __forceinline__ uint32_t filt_addr(const SrvCtx& c, uint32_t i) {
+  if constexpr (!CL) {
+    return c.rt32 + 4u * i;
+  } else {
+    const uint32_t owner = i & ((1u << c.clog2) - 1), local = c.rt32 + 4u * (i >> c.clog2);
+    uint32_t a;
+    asm("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(a) : "r"(local), "r"(owner));
+    return a;
+  }
+}
+template <bool CL>
+__device__ __forceinline__ uint32_t filt_ld(uint32_t a) {
+  uint32_t v;
+  if constexpr (CL) asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  else asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+template <bool CL>
+__device__ __forceinline__ void filt_st(uint32_t a, uint32_t v) {
+  if constexpr (CL) asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+  else asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
 
 // ---------------------------------------------------------------------------
@@ -382,19 +434,30 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     }
     const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
     srv_fence<CL>();
-    uint32_t lw0[M], lw1[M], bk0[M], bk1[M];
+    const bool hash = p.atr_mode == CSMV_ATR_HASH;
+    const bool novalid = (p.debug & CSMV_DBG_NO_VALIDATE) != 0;
+    // HASH: the exact part of the validation (lastw, every CTS <= e_pre) and
+    // the filter slot addresses are settled before the lock
+    bool chk[M];
+    uint32_t fa[M][kFiltK], fb[M][kFiltK];
     uint32_t xor_all = e_pre;
+    const uint32_t fl2 = p.rt_log2 + 3;
 #pragma unroll
     for (int j = 0; j < M; ++j) {
-      lw0[j] = lw1[j] = 0;
-      if (mine[j]) {
-        lw0[j] = ld_relaxed(p.lastw + id0[j]);
-        lw1[j] = ld_relaxed(p.lastw + id1[j]);
+      uint32_t lw0 = 0, lw1 = 0;
+      if (mine[j] && hash) {
+        lw0 = ld_relaxed(p.lastw + id0[j]);
+        lw1 = ld_relaxed(p.lastw + id1[j]);
       }
-      bk0[j] = rt_bucket(id0[j], p.rt_log2);
-      bk1[j] = rt_bucket(id1[j], p.rt_log2);
-      xor_all ^= bk0[j] ^ bk1[j] ^ lw0[j] ^ lw1[j] ^ sn[j];
+      chk[j] = mine[j] && (novalid || (lw0 <= sn[j] && lw1 <= sn[j]));
+#pragma unroll
+      for (int k = 0; k < kFiltK; ++k) {
+        fa[j][k] = filt_addr<CL>(c, filt_slot(id0[j], k, fl2));
+        fb[j][k] = filt_addr<CL>(c, filt_slot(id1[j], k, fl2));
+      }
+      xor_all ^= lw0 ^ lw1 ^ sn[j];
     }
+    const uint32_t e_chk = novalid ? 0xFFFFFFFFu : e_pre;
     // The payload must have arrived before the lock is taken: a warp vote on
     // values derived from it makes the loads complete here.
     if (__ballot_sync(FULL, xor_all == 0x12345679u) == FULL) __nanosleep(1);
@@ -405,42 +468,59 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
     uint32_t t = t0c;
     uint32_t cm[M], om[M], base[M];
+    if (hash) {
+      // batch j: a write after e_pre to one of its items raised all of that
+      // item's slots above e_pre (earlier batches of this section included)
 #pragma unroll
-    for (int j = 0; j < M; ++j) {
-      cm[j] = om[j] = 0;
-      base[j] = t + 1;
-      if (j >= (int)m) continue;
-      RtProbe q0{0, false, false}, q1{0, false, false};
-      bool ovf = false, conflict = false;
-      if (p.atr_mode == CSMV_ATR_HASH) {
-        if (mine[j]) {
-          const RtBucket b0 = rt_load<CL>(c, bk0[j]), b1 = rt_load<CL>(c, bk1[j]);
-          q0 = rt_eval(b0, id0[j], sn[j], e_pre, lw0[j]);
-          q1 = rt_eval(b1, id1[j], sn[j], e_pre, lw1[j]);
-          if (bk1[j] == bk0[j] && q1.way == q0.way) q1.way = (q1.way + 1) & (kRtWays - 1);
+      for (int j = 0; j < M; ++j) {
+        cm[j] = om[j] = 0;
+        base[j] = t + 1;
+        if (j < (int)m) {
+          uint32_t va[kFiltK] = {0u, 0u, 0u}, vb[kFiltK] = {0u, 0u, 0u};
+          if (chk[j]) {
+#pragma unroll
+            for (int k = 0; k < kFiltK; ++k) {
+              va[k] = filt_ld<CL>(fa[j][k]);
+              vb[k] = filt_ld<CL>(fb[j][k]);
+            }
+          }
+          const uint32_t lo = max(min(va[0], min(va[1], va[2])), min(vb[0], min(vb[1], vb[2])));
+          const bool ovf = chk[j] && lo > e_chk;
+          const bool commit = chk[j] && !ovf;
+          cm[j] = __ballot_sync(FULL, commit);
+          om[j] = __ballot_sync(FULL, ovf);
+          const uint32_t cts = t + 1 + __popc(cm[j] & lt);
+          t += __popc(cm[j]);
+          if (commit) {
+#pragma unroll
+            for (int k = 0; k < kFiltK; ++k) {  // the batch's last CTS: equal values, race-free
+              filt_st<CL>(fa[j][k], t);
+              filt_st<CL>(fb[j][k], t);
+            }
+            p.lastw[id0[j]] = cts;
+            p.lastw[id1[j]] = cts;
+          }
+          __syncwarp();  // batch j's records precede batch j+1's probes
         }
-        ovf = mine[j] && (q0.unknown || q1.unknown);
-        conflict = mine[j] && (q0.conflict || q1.conflict);
-      } else {
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        cm[j] = om[j] = 0;
+        base[j] = t + 1;
+        if (j >= (int)m) continue;
+        bool ovf = false, conflict = false;
         atr_list_validate(p, c, sn[j], t, mine[j], id0[j], id1[j], ovf, conflict);
+        if (novalid) ovf = conflict = false;
+        const bool commit = mine[j] && !ovf && !conflict;
+        cm[j] = __ballot_sync(FULL, commit);
+        om[j] = __ballot_sync(FULL, ovf);
+        const uint32_t cts = t + 1 + __popc(cm[j] & lt);
+        t += __popc(cm[j]);
+        // the paper's ATR: the write-set of commit `cts` at entry cts
+        if (commit) c.rt[cts & ((uint32_t)(kRtWays << (p.rt_log2 - p.clog2)) - 1)] = ((uint64_t)id1[j] << 32) | id0[j];
+        __syncwarp();  // batch j's records precede batch j+1's validation
       }
-      if (p.debug & CSMV_DBG_NO_VALIDATE) ovf = conflict = false;
-      const bool commit = mine[j] && !ovf && !conflict;
-      cm[j] = __ballot_sync(FULL, commit);
-      om[j] = __ballot_sync(FULL, ovf);
-      const uint32_t cts = t + 1 + __popc(cm[j] & lt);
-      t += __popc(cm[j]);
-      if (commit) {
-        if (p.atr_mode == CSMV_ATR_HASH) {
-          p.lastw[id0[j]] = cts;
-          p.lastw[id1[j]] = cts;
-          rt_record<CL>(c, bk0[j], q0.way, id0[j], cts);
-          rt_record<CL>(c, bk1[j], q1.way, id1[j], cts);
-        } else {  // the paper's ATR: the write-set of commit `cts` at entry cts
-          c.rt[cts & ((uint32_t)(kRtWays << (p.rt_log2 - p.clog2)) - 1)] = ((uint64_t)id1[j] << 32) | id0[j];
-        }
-      }
-      __syncwarp();  // batch j's records precede batch j+1's probes
     }
     const long long ta = clock64();
     if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) done_ring_room(p, c, t, t_begin);
@@ -756,6 +836,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   c.cw_hi = min(c.cw_lo + per, p.n_cw);
   c.qn_log2 = queue_log2(per);
   c.rt = reinterpret_cast<uint64_t*>(smem);
+  c.rt32 = (uint32_t)__cvta_generic_to_shared(c.rt);
   const uint32_t rt_words = (uint32_t)kRtWays << local_log2;
   c.queue = c.rt + rt_words;
   c.evmax = reinterpret_cast<uint32_t*>(c.queue + (1u << c.qn_log2));
@@ -764,7 +845,8 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   c.sh = reinterpret_cast<SrvShared*>(c.last_seen + ls_words);
   if constexpr (CL) c.sh0 = cg::this_cluster().map_shared_rank(c.sh, 0);
   else c.sh0 = c.sh;
-  for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) c.rt[i] = 0xFFFFFFFFull;  // cts 0, no item
+  const uint64_t rt_init = (KIND == CSMV_KIND_BANK && p.atr_mode == CSMV_ATR_HASH) ? 0ull : 0xFFFFFFFFull;
+  for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) c.rt[i] = rt_init;  // table: cts 0, no item; filter: 0
   for (uint32_t i = threadIdx.x; i < (1u << local_log2); i += blockDim.x) c.evmax[i] = 0;
   for (uint32_t i = threadIdx.x; i < (1u << c.qn_log2); i += blockDim.x) c.queue[i] = 0;
   for (uint32_t i = threadIdx.x; i < ls_words; i += blockDim.x) c.last_seen[i] = 0;

@@ -219,9 +219,9 @@ def test_ro_adaptive_parity(preset, streak):
 
 @pytest.mark.parametrize("cap", [256, 1024])
 def test_small_atr_bucket_races(cap):
-    """Few buckets: lanes of one batch often race for the same way of a
-    bucket, so displaced entries are re-inserted (server.cuh rt_record) or
-    fold into the irregular-eviction watermark -- never lost."""
+    """A small recent-write filter (server.cuh filt_idx): lanes of one batch
+    often share slots and the window saturates it, so many updates abort
+    OVERFLOW -- but a write inside the window is never missed."""
     cfg = W.c2(n_items=1 << 14, n_tx=1 << 17, atr_capacity=cap, server_combine=4, server_workers=6,
                client_warps=256, ro_streak=4, publish=csmv.PUBLISH_SERVER)
     rep, stats, log, rings, descs = check(cfg)
