@@ -1,10 +1,10 @@
 // Micro-benchmark of the commit critical section's building blocks, using
-// the real device code (server.cuh): random item ids, a 4K-bucket
-// recent-commit table, 29 of 32 lanes committing 2 items each, one warp.
-//  mode 0: ballot only          mode 1: + bucket loads/eval (probe)
-//  mode 2: + atomic record       mode 3: + store record (rt_record_batch)
-//  mode 4: mode 3 + lastw STGs   mode 5: mode 2 + lastw STGs
-//  mode 6: mode 4 through the ticket lock, W warps (cycles per batch of the chain)
+// the real device code (server.cuh): random item ids, a 16K-bucket
+// recent-commit table, 29 of 32 lanes committing 2 items each.
+//  modes 0-3: one warp, no lock: ballot / +probe / +record / +lastw stores
+//  mode 4   : W warps contending through the real ticket lock (cs_enter /
+//             cs_leave), full probe+record+lastw body -> cycles per batch
+//             of the whole serial chain (handoff included)
 #include <cstdio>
 #include <cuda_runtime.h>
 #include "../../paper_conf_ipps_nunesc022_b200/csrc/kernel.cuh"
@@ -20,12 +20,10 @@ using namespace csmvd;
 __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int iters, int nw) {
   extern __shared__ uint8_t smem[];
   __shared__ SrvShared sh;
-  __shared__ uint8_t own[1 << kOwnLog2];
   SrvCtx c;
   c.clog2 = 0;
   c.rt = reinterpret_cast<uint64_t*>(smem);
   c.evmax = reinterpret_cast<uint32_t*>(c.rt + 4 * 4096);
-  c.own = own;
   c.sh = c.sh0 = &sh;
   for (int i = threadIdx.x; i < 4 * 4096; i += blockDim.x) c.rt[i] = 0xFFFFFFFFull;
   for (int i = threadIdx.x; i < 4096; i += blockDim.x) c.evmax[i] = 0;
@@ -44,7 +42,7 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
     const uint32_t b0 = rt_bucket(id0, 12), b1 = rt_bucket(id1, 12);
     const bool mine = lane < 29;
     uint32_t ticket = 0;
-    const bool locked = mode >= 6;
+    const bool locked = mode >= 4;
     if (locked) {
       ticket = cs_enter<false>(c);
       t = *(volatile uint32_t*)&sh.tail;
@@ -52,30 +50,22 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
     const long long a = clock64();
     const uint32_t s = t > 50 ? t - 50 : 0, e_pre = t;
     RtProbe q0{0, false, false}, q1{0, false, false};
-    RtBucket qb[2];
     if (mode >= 1 && mine) {
-      qb[0] = rt_load<false>(c, b0);
-      qb[1] = rt_load<false>(c, b1);
-      q0 = rt_eval(qb[0], id0, s, e_pre, 0);
-      q1 = rt_eval(qb[1], id1, s, e_pre, 0);
+      q0 = rt_probe<false>(c, b0, id0, s, e_pre, 0);
+      q1 = rt_probe<false>(c, b1, id1, s, e_pre, 0);
+      if (b1 == b0 && q1.way == q0.way) q1.way = (q1.way + 1) & 3;
     }
     const bool commit = mine && !q0.conflict && !q1.conflict && !q0.unknown && !q1.unknown;
     const uint32_t cm = __ballot_sync(0xFFFFFFFFu, commit);
     const uint32_t cts = t + 1 + __popc(cm & lt);
     t += __popc(cm);
-    if (commit && (mode == 4 || mode == 5 || mode == 6)) {
+    if (commit && mode >= 3 && mode != 5) {
       lastw[id0 & 0xFFFFF] = cts;
       lastw[id1 & 0xFFFFF] = cts;
     }
-    if (mode == 2 || mode == 5) {
-      if (commit) {
-        if (b1 == b0 && q1.way == q0.way) q1.way = (q1.way + 1) & 3;
-        rt_record<false>(c, b0, q0.way, id0, cts);
-        rt_record<false>(c, b1, q1.way, id1, cts);
-      }
-    } else if (mode == 3 || mode == 4 || mode == 6) {
-      const uint32_t k2[2] = {id0, id1}, bk2[2] = {b0, b1};
-      rt_record_batch<false, 2>(c, commit, k2, bk2, qb, cts);
+    if (commit && mode >= 2) {
+      rt_record<false>(c, b0, q0.way, id0, cts);
+      rt_record<false>(c, b1, q1.way, id1, cts);
     }
     __syncwarp();
     acc += clock64() - a;
@@ -84,7 +74,7 @@ __global__ void bench(uint32_t* lastw, unsigned long long* out, int mode, int it
   }
   const long long a1 = clock64();
   if (lane == 0 && warp == 0) {
-    out[0] = mode >= 6 ? (a1 - a0) / ((long long)iters * nw) : acc / iters;
+    out[0] = mode >= 4 ? (a1 - a0) / ((long long)iters * nw) : acc / iters;
     out[1] = acc / iters;
     out[2] = sink;
   }
@@ -97,17 +87,19 @@ int main() {
   cudaMallocManaged(&o, 64);
   const int smem = 4 * 4096 * 8 + 4096 * 4;
   cudaFuncSetAttribute(bench, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  const char* names[] = {"ballot only", "probe", "probe+atomic record", "probe+store record",
-                         "store record+lastw", "atomic record+lastw"};
-  for (int m = 0; m < 6; ++m) {
+  const char* names[] = {"ballot only", "probe", "probe+record", "probe+record+lastw"};
+  for (int m = 0; m < 4; ++m) {
     bench<<<1, 256, smem>>>(lw, o, m, 20000, 1);
     cudaDeviceSynchronize();
-    printf("%-24s %llu cycles/batch\n", names[m], o[0]);
+    printf("%-22s %llu cycles/batch\n", names[m], o[0]);
   }
   for (int nw = 1; nw <= 8; nw *= 2) {
-    bench<<<1, 256, smem>>>(lw, o, 6, 20000, nw);
+    bench<<<1, 256, smem>>>(lw, o, 4, 20000, nw);
     cudaDeviceSynchronize();
     printf("locked chain, %d warps: %llu cycles/batch (body %llu)\n", nw, o[0], o[1]);
+    bench<<<1, 256, smem>>>(lw, o, 5, 20000, nw);
+    cudaDeviceSynchronize();
+    printf("locked chain, no lastw stores, %d warps: %llu cycles/batch (body %llu)\n", nw, o[0], o[1]);
   }
   printf("err=%s\n", cudaGetErrorString(cudaGetLastError()));
 }
