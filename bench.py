@@ -37,7 +37,7 @@ METRIC = "committed tx/sec and abort rate at 1 B200 (+partitioned 2/4/8)"
 UNIT = "tx/s"
 
 # tuned launch configuration of the C2 workload
-TUNED = dict(client_warps_per_sm=2, server_workers=6, server_combine=4, ro_streak=8, publish=1)
+TUNED = dict(client_warps_per_sm=2, server_workers=6, server_combine=4, ro_streak=8, publish=1, ro_adaptive=1)
 
 # algorithmic bytes (paper VBox layout P:289): a read moves the
 # VBox head, the visited version's ts and the value (4+4+4); a write-back the
@@ -169,7 +169,8 @@ def make_cfg(args, world: int, rank: int):
     cfg = workloads.PRESETS[args.config]()
     n_tx = args.n_tx or cfg.n_tx
     cfg = cfg.with_(n_tx=n_tx, log_mode=0, ro_streak=TUNED["ro_streak"], publish=TUNED["publish"],
-                    server_workers=TUNED["server_workers"], server_combine=TUNED["server_combine"])
+                    server_workers=TUNED["server_workers"], server_combine=TUNED["server_combine"],
+                    ro_adaptive=TUNED["ro_adaptive"])
     part = partition.partition(cfg.n_items, n_tx, cfg.seed, rank, world)
     lcfg = partition.local_config(cfg, part)
     if cfg.workload.kind == 1:   # KV: the partition is a smaller cache with its own key space
@@ -331,7 +332,7 @@ def bench_ours(args):
                    "n_items": cfg.n_items, "n_versions": cfg.n_versions, "n_tx_per_step": cfg.n_tx,
                    "client_warps_per_gpu": n_cw, "server_workers": w.server_workers,
                    "server_combine": w.server_combine,
-                   "ro_streak": w.ro_streak, "publish": ["client", "server"][w.publish],
+                   "ro_streak": w.ro_streak, "ro_adaptive": w.ro_adaptive, "publish": ["client", "server"][w.publish],
                    "parallelism": "partitioned" if world > 1 else "single-gpu",
                    "multi_gpu": "independent key-range partitions, no cross-GPU transactions, NCCL stats only",
                    "l2": "flushed (512 MiB write) before every timed step"},

@@ -219,28 +219,45 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
       pc.mark(PH_SUBMIT);
     }
 
-    // ---- C: read-only transactions at s
-    if (streak || cu == kNoTx) {
-      uint32_t n_ro = 0;
-      while (cr < p.n_tx) {
-        const BankTx r = gen_bank(p.gen, cr);
-        if (r.is_update) break;
-        if (streak ? n_ro >= streak : n_ro >= 1) break;
-        ++att_r;
-        ++n_ro;
+    // ---- C: read-only transactions at s.  A lane runs
+    // its next read-only transactions up to the next update (at most
+    // ro_streak; one if 0, and only without a pending update); a version
+    // miss ends its run (retried next round).  The warp runs them depth by
+    // depth -- every lane's first, then every lane's second, ... -- each one
+    // scanned by the whole warp (rot_coop), so a round is not as long as
+    // its longest lane's run.
+    {
+      const uint32_t lim = streak ? streak : 1u;
+      bool run = streak || cu == kNoTx;
+      for (uint32_t n_ro = 0; n_ro < lim; ++n_ro) {
+        BankTx r{};
+        bool has = false;
+        if (run && cr < p.n_tx) {
+          r = gen_bank(p.gen, cr);
+          has = !r.is_update;
+        }
+        const uint32_t act = __ballot_sync(FULL, has);
+        if (!act) break;
+        if (has) ++att_r;
+        bool ok;
         int64_t rsum;
         uint64_t rdig;
-        if (!rot_scan<NS>(p, r.start, r.len, s, cr, rsum, rdig)) {
-          cc.abort(CSMV_AB_VERSION, false);  // retried next round
-          break;
+        rot_coop<NS>(p, act, r.start, r.len, s, cr, ok, rsum, rdig);
+        if (has) {
+          if (ok) {
+            if (p.log_mode) log_commit(p, cr, s, 0, att_r, rdig, (uint64_t)rsum);
+            ++cc.c_ro;
+            cc.ro_ck ^= (uint64_t)rsum;
+            cr += T;
+            att_r = 0;
+          } else {
+            cc.abort(CSMV_AB_VERSION, false);  // retried next round
+            run = false;
+          }
         }
-        if (p.log_mode) log_commit(p, cr, s, 0, att_r, rdig, (uint64_t)rsum);
-        ++cc.c_ro;
-        cc.ro_ck ^= (uint64_t)rsum;
-        cr += T;
-        att_r = 0;
+        run = run && has;
         // ro_adaptive: the batch has been answered -> finish the round
-        if (p.ro_adaptive && kept && (uint32_t)(ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
+        if (p.ro_adaptive && kept && (uint32_t)(warp_ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
       }
     }
     __syncwarp();

@@ -149,46 +149,95 @@ __device__ __forceinline__ bool watchdog(const KParams& p, uint64_t t0, uint32_t
 // --------------------------------------------------------------------------
 // Read-only transaction: L consecutive accounts (or all)
 // --------------------------------------------------------------------------
+// Exact warp sums by redux.sync: an int32 per lane as two 16-bit-wide
+// halves (no 32-bit wrap), a u64 per lane (mod 2^64) as four 16-bit chunks.
+__device__ __forceinline__ int64_t warp_sum_i32(int32_t v) {
+  const int hi = __reduce_add_sync(0xFFFFFFFFu, v >> 16);
+  const unsigned lo = __reduce_add_sync(0xFFFFFFFFu, (unsigned)v & 0xFFFFu);
+  return (int64_t)hi * 65536 + (int64_t)lo;
+}
+__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
+  uint64_t r = 0;
+#pragma unroll
+  for (int k = 0; k < 4; ++k)
+    r += (uint64_t)__reduce_add_sync(0xFFFFFFFFu, (unsigned)(v >> (16 * k)) & 0xFFFFu) << (16 * k);
+  return r;
+}
+
+// Warp-cooperative read-only transactions: the lanes in
+// `act` each own one read-only transaction at snapshot s -- tx, a scan of
+// `len` accounts from `start` -- and the whole warp runs them one after
+// another, 32 consecutive accounts per row (one coalesced 1 KiB load of
+// 32-byte VBoxes), U rows in flight.  Each row is reduced across the warp
+// (exact int64 sum, digest, any-miss) and added into its owner lane.  Same
+// per-transaction result as one lane scanning alone; no lane waits for another lane's
+// longer read-only run.
 template <int NS>
-__device__ __forceinline__ bool rot_scan(const KParams& p, uint32_t start, uint32_t len, uint32_t s,
-                                         uint64_t tx, int64_t& sum, uint64_t& dg) {
-  constexpr int U = NS <= 4 ? 8 : (NS == 8 ? 4 : 2);  // rings in flight per lane (memory-level parallelism)
+__device__ __forceinline__ void rot_coop(const KParams& p, uint32_t act, uint32_t start, uint32_t len, uint32_t s,
+                                         uint64_t tx, bool& ok, int64_t& sum, uint64_t& dg) {
+  constexpr int U = NS <= 4 ? 8 : (NS == 8 ? 4 : 2);
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t N = p.n_items;
+  ok = true;
   sum = 0;
   dg = 0;
-  const uint32_t N = p.n_items;
-  uint32_t x = start;
-  for (uint32_t j = 0; j < len; j += U) {
+  const uint32_t L = __shfl_sync(FULL, len, act ? __ffs(act) - 1 : 0);  // the same for every transaction
+  const uint32_t rows = (L + 31) / 32;
+  const uint32_t total = (uint32_t)__popc(act) * rows;
+  for (uint32_t g = 0; g < total; g += U) {
     Ring<NS> r[U];
-    uint32_t xs[U];
+    uint32_t xs[U], own[U], ev[U];
+    uint64_t txo[U];
+    uint32_t so[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
+      const uint32_t idx = g + u;
+      const uint32_t i = idx / rows, k = idx - i * rows;
+      own[u] = idx < total ? __fns(act, 0, i + 1) : 0u;
+      so[u] = __shfl_sync(FULL, start, own[u]);
+      txo[u] = __shfl_sync(FULL, tx, own[u]);
+      ev[u] = k * 32 + lane;
+      uint32_t x = so[u] + ev[u];
+      if (x >= N) x -= N;
+      if (x >= N) x %= N;
       xs[u] = x;
-      if (j + u < len) r[u] = ld_ring<NS>(p.rings + (size_t)x * NS);
-      x = (x + 1 == N) ? 0u : x + 1;
+      if (idx < total && ev[u] < L) r[u] = ld_ring<NS>(p.rings + (size_t)x * NS);
     }
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      if (j + u >= len) break;
-      Sel q = select_version<NS>(r[u], s);
-      if (q.best < 0) return false;  // version recycled
-      uint64_t v = slot_at<NS>(r[u], q.best);
-      if (q.newest > s) {
-        // A newer version exists, so write-backs may have overwritten slots
-        // while we read.  Versions are evicted oldest first, so if the chosen
-        // slot still holds the same version, no version in (best_ts, s] was
-        // missed; otherwise the snapshot's version is gone.
-        if (ld_relaxed64(p.rings + (size_t)xs[u] * NS + q.best) != v) return false;
+      if (g + u >= total) break;  // warp-uniform
+      const bool valid = ev[u] < L;
+      bool miss = false;
+      uint32_t val = 0;
+      if (valid) {
+        const Sel q = select_version<NS>(r[u], s);
+        if (q.best < 0) {
+          miss = true;  // version recycled
+        } else {
+          const uint64_t v = slot_at<NS>(r[u], q.best);
+          // A newer version exists, so write-backs may have overwritten slots
+          // while we read.  Versions are evicted oldest first, so if the chosen
+          // slot still holds the same version, no version in (best_ts, s] was
+          // missed; otherwise the snapshot's version is gone.
+          if (q.newest > s && ld_relaxed64(p.rings + (size_t)xs[u] * NS + q.best) != v) miss = true;
+          val = (uint32_t)v;
+        }
       }
-      int32_t val = (int32_t)(uint32_t)v;
-      sum += val;
+      const bool rmiss = __any_sync(FULL, miss);
+      const int64_t rs = warp_sum_i32(miss ? 0 : (int32_t)val);
+      uint64_t rd = 0;
       if (p.log_mode) {
-        dg += dig1(xs[u], (uint32_t)val);
-        if (p.log_mode == CSMV_LOG_FULL && j + u < p.max_vals)
-          p.vals[tx * p.max_vals + j + u] = (uint32_t)val;
+        rd = warp_sum_u64(valid && !miss ? dig1(xs[u], val) : 0ull);
+        if (p.log_mode == CSMV_LOG_FULL && valid && ev[u] < p.max_vals) p.vals[txo[u] * p.max_vals + ev[u]] = val;
+      }
+      if (lane == own[u]) {
+        ok = ok && !rmiss;
+        sum += rs;
+        dg += rd;
       }
     }
   }
-  return true;
 }
 
 // --------------------------------------------------------------------------

@@ -100,7 +100,7 @@ __device__ __forceinline__ int kv_read_mw(const uint64_t* ring, uint32_t K, uint
 // the read a miss.  When a version newer than s is present the chosen slot
 // is re-read (address-dependent on the first loads, so ordered after them):
 // still intact means no version in (cts, s] was recycled meanwhile (oldest-
-// first recycling) -- the argument of rot_scan.
+// first recycling) -- the argument of rot_coop (kernel.cu).
 // rot = false (a PUT's read): any version newer than s -> RD_NEWER, as in
 // kv_read_mw (a torn slot carries a newer ts, so it is covered too).
 template <int NS>

@@ -790,15 +790,38 @@ __device__ void server_publisher(const KParams& p, const SrvCtx& c, uint64_t t_b
   const uint32_t dmask = (1u << kDoneLog2) - 1;
   uint32_t g = *(volatile uint32_t*)&c.sh->tail;
   uint32_t spins = 0;
+  // one sweep looks at the next 32 * 4 * W flags: W 16-byte loads per lane in
+  // flight, lane l of row k covering CTS g+1 + 4(32k + l) .. +3 (a sweep is
+  // one L2 round trip, so this bounds GTS's advance rate)
+  constexpr int W = 8;
   for (;;) {
-    uint32_t v[4];
+    const uint32_t g0 = g + 1;
+    const uint32_t a0 = g0 & 3u;  // 16-byte loads need a 4-aligned first CTS: start at g0 - a0
+    uint4 v[W];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) v[k] = ld_relaxed(p.done_ring + ((g + 1 + k * 32 + lane) & dmask));
+    for (int k = 0; k < W; ++k)
+      v[k] = ld_relaxed_v4(p.done_ring + ((g0 - a0 + 4u * (k * 32 + lane)) & dmask));
     uint32_t adv = 0;
+    bool open = true;
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const uint32_t bad = __ballot_sync(FULL, v[k] != g + 1 + k * 32 + lane);
-      if (adv == (uint32_t)k * 32) adv += bad ? (uint32_t)(__ffs(bad) - 1) : 32u;
+    for (int k = 0; k < W; ++k) {
+      const uint32_t e0 = g0 - a0 + 4u * (k * 32 + lane);
+      const uint32_t w[4] = {v[k].x, v[k].y, v[k].z, v[k].w};
+      int first_bad = 4;
+#pragma unroll
+      for (int i = 3; i >= 0; --i)
+        if (w[i] != e0 + i && e0 + i >= g0) first_bad = i;  // flags before g0 are not looked at
+      const uint32_t bad = __ballot_sync(FULL, first_bad < 4);
+      if (open) {
+        if (bad) {
+          const int l = __ffs(bad) - 1;
+          const uint32_t fb = __shfl_sync(FULL, (uint32_t)first_bad, l);
+          adv = 4u * (k * 32 + l) + fb - a0;
+          open = false;
+        } else {
+          adv = 4u * (k * 32 + 32) - a0;
+        }
+      }
     }
     if (adv) {
       fence_gpu();
