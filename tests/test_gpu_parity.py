@@ -75,7 +75,10 @@ def test_c1_full_parity(publish):
 
 
 @pytest.mark.parametrize("k,streak,ro_reads", [(1, 0, 0), (2, 0, 0), (4, 0, 0), (8, 0, 0), (16, 0, 0),
-                                               (4, 4, 0), (4, 8, 16), (2, 1, 16)])
+                                               (4, 4, 0), (4, 8, 16), (2, 1, 16),
+                                               # ragged warp-cooperative scans: 2-3 rows with a
+                                               # partial last row, more rows than fit in flight
+                                               (2, 4, 70), (4, 8, 33), (4, 2, 300)])
 def test_one_warp_is_deterministic(k, streak, ro_reads):
     """with one client warp the oracle predicts every snapshot,
     CTS, attempt count and ring exactly."""
@@ -226,3 +229,13 @@ def test_small_atr_bucket_races(cap):
                client_warps=256, ro_streak=4, publish=csmv.PUBLISH_SERVER)
     rep, stats, log, rings, descs = check(cfg)
     assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions), closed_form(cfg, descs, cfg.init_values()))
+
+
+@pytest.mark.parametrize("ro_reads,k", [(40, 4), (97, 2), (1, 4)])
+def test_ragged_read_only_scans(ro_reads, k):
+    """Warp-cooperative read-only scans (kernel.cu rot_coop) with lengths that
+    are not a multiple of the 32-account row, wrapping past the last account,
+    with version misses at K = 2, many warps, FULL log (every value read)."""
+    cfg = W.c2(n_items=1 << 12, n_tx=1 << 15, ro_reads=ro_reads, n_versions=k, log_mode=csmv.LOG_FULL,
+               client_warps=64, ro_streak=8, p_update_ppm=300_000)
+    check(cfg)
