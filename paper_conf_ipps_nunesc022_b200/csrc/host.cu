@@ -416,7 +416,9 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   // bank + CSMV_ATR_HASH reads the same smem as a recent-write filter of
   // 8 << rt_log2 slots (server.cuh); below ~1K slots a window of a few
   // batches saturates it and nearly every update would abort OVERFLOW
-  if (h->kind == CSMV_KIND_BANK && w->atr_mode == CSMV_ATR_HASH && rt_log2 < 7 + clog2) rt_log2 = 7 + clog2;
+  const bool filt = h->kind == CSMV_KIND_BANK ? w->atr_mode == CSMV_ATR_HASH
+                                              : (h->kv_A > kKvFullWays || !(w->debug_flags & CSMV_DBG_KV_ITEMSETS));
+  if (filt && rt_log2 < 7 + clog2) rt_log2 = 7 + clog2;
   const uint32_t per_srv = n_srv ? (n_cw + n_srv - 1) / n_srv : 0u;
   size_t smem = server_smem_bytes(rt_log2 - clog2, per_srv);
   if (h->kind == CSMV_KIND_KV && smem < kv_client_smem_bytes()) smem = kv_client_smem_bytes();

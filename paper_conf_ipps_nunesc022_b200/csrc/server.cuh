@@ -171,6 +171,11 @@ __device__ __forceinline__ void rt_record(const SrvCtx& c, uint32_t bucket, int 
 // ---------------------------------------------------------------------------
 constexpr int kFiltK = 3;
 
+// KV requests in the compact {set clock} u WS form use the filter
+__device__ __forceinline__ bool kv_filter_mode(const KParams& p) {
+  return p.kv_A > kKvFullWays || !(p.debug & CSMV_DBG_KV_ITEMSETS);
+}
+
 // slot k of item x: multiplicative hashes with three odd constants
 __device__ __forceinline__ uint32_t filt_slot(uint32_t x, int k, uint32_t slots_log2) {
   const uint32_t C[3] = {0x9E3779B1u, 0x85EBCA77u, 0xC2B2AE3Du};
@@ -682,6 +687,101 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
 }
 
 // ---------------------------------------------------------------------------
+// KV worker for {set clock} u WS requests (the default, client_kv.cuh):
+// validation is decided by clock[t] alone (DESIGN.md readings), so each PUT
+// validates one item -- exactly against lastw (every CTS <= e_pre, before
+// the lock) and against the recent-write filter for the commits after e_pre
+// (as the bank worker).  Only clocks enter the filter: nothing else is ever
+// validated in this mode; lastw is written for all four written items.
+// ---------------------------------------------------------------------------
+template <bool CL>
+__device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t lt = lanemask_lt();
+  const bool novalid = (p.debug & CSMV_DBG_NO_VALIDATE) != 0;
+  const uint32_t fl2 = p.rt_log2 + 3;
+  unsigned long long busy = 0, locked = 0, batches = 0;
+  unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  for (;;) {
+    uint32_t cw;
+    const long long tq = clock64();
+    if (!claim_request(c, cw)) break;
+    const long long t0 = clock64();
+    fence_cta();  // after the receiver's acquire (see server_receiver)
+    const uint32_t sq = ld_relaxed(&p.req_hdr[cw].round);
+    const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
+    const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
+    uint32_t ids[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) ids[k] = ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + k) * 32 + lane) & ~kWriteBit;
+    const bool mine = (mask >> lane) & 1u;
+    const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
+    srv_fence<CL>();
+    const uint32_t lw = mine ? ld_relaxed(p.lastw + ids[0]) : 0u;
+    const bool chk = mine && (novalid || lw <= s);
+    uint32_t fa[kFiltK];
+#pragma unroll
+    for (int k = 0; k < kFiltK; ++k) fa[k] = filt_addr<CL>(c, filt_slot(ids[0], k, fl2));
+    const uint32_t e_chk = novalid ? 0xFFFFFFFFu : e_pre;
+    if (__ballot_sync(FULL, (s ^ lw ^ ids[1] ^ ids[2] ^ ids[3]) == 0x12345679u) == FULL) __nanosleep(1);
+    const long long tl = clock64();
+    // ---- critical section
+    const uint32_t ticket = cs_enter<CL>(c);
+    const long long t1 = clock64();
+    const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
+    uint32_t v[kFiltK] = {0u, 0u, 0u};
+    if (chk) {
+#pragma unroll
+      for (int k = 0; k < kFiltK; ++k) v[k] = filt_ld<CL>(fa[k]);
+    }
+    const bool ovf = chk && min(v[0], min(v[1], v[2])) > e_chk;
+    const bool commit = chk && !ovf;
+    const uint32_t cm = __ballot_sync(FULL, commit);
+    const uint32_t om = __ballot_sync(FULL, ovf);
+    const uint32_t n = __popc(cm);
+    const long long tv = clock64();
+    if (p.publish == CSMV_PUBLISH_SERVER && n) done_ring_room(p, c, t0c + n, t_begin);
+    if (commit) {
+      const uint32_t cts = t0c + 1 + __popc(cm & lt);
+#pragma unroll
+      for (int k = 0; k < kFiltK; ++k) filt_st<CL>(fa[k], t0c + n);  // the batch's last CTS
+#pragma unroll
+      for (int k = 0; k < 4; ++k) p.lastw[ids[k]] = cts;
+    }
+    const long long tr = clock64();
+    cs_leave<CL>(c, ticket, t0c + n);
+    const long long t2 = clock64();
+    if (lane == 0) {  // round-tagged words, no fence (kernel.cuh Resp)
+      const uint64_t tag = (uint64_t)sq << 32;
+      st_relaxed64(&p.resp[cw].base, tag | (t0c + 1));
+      st_relaxed64(&p.resp[cw].commit, tag | cm);
+      st_relaxed64(&p.resp[cw].ovf, tag | om);
+    }
+    __syncwarp();
+    const long long t3 = clock64();
+    busy += (unsigned long long)(t3 - t0);
+    locked += (unsigned long long)(t2 - t1);
+    ph[0] += (unsigned long long)(t0 - tq);
+    ph[1] += (unsigned long long)(tl - t0);
+    ph[2] += (unsigned long long)(t1 - tl);
+    ph[3] += (unsigned long long)(t2 - t1);
+    ph[4] += (unsigned long long)(t3 - t2);
+    ph[5] += (unsigned long long)(tv - t1);
+    ph[6] += (unsigned long long)(tr - tv);
+    ph[7] += (unsigned long long)(t2 - tr);
+    ++batches;
+  }
+  if (lane == 0) {
+    for (int i = 0; i < 8; ++i) atomicAdd(&p.stats->phase[i], ph[i]);
+    atomicAdd(&p.stats->batches, batches);
+    atomicAdd(&p.stats->groups, batches);
+    atomicAdd(&p.stats->busy_cycles, busy);
+    atomicAdd(&p.stats->lock_cycles, locked);
+  }
+}
+
+// ---------------------------------------------------------------------------
 // CSMV-onlyCS worker: the client-server design with the paper's
 // complementary mechanisms removed -- no collaborative validation (the lane
 // of the transaction scans the list ATR alone), no batched ATR insert
@@ -868,7 +968,8 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   c.sh = reinterpret_cast<SrvShared*>(c.last_seen + ls_words);
   if constexpr (CL) c.sh0 = cg::this_cluster().map_shared_rank(c.sh, 0);
   else c.sh0 = c.sh;
-  const uint64_t rt_init = (KIND == CSMV_KIND_BANK && p.atr_mode == CSMV_ATR_HASH) ? 0ull : 0xFFFFFFFFull;
+  const bool filt = KIND == CSMV_KIND_BANK ? p.atr_mode == CSMV_ATR_HASH : kv_filter_mode(p);
+  const uint64_t rt_init = filt ? 0ull : 0xFFFFFFFFull;
   for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) c.rt[i] = rt_init;  // table: cts 0, no item; filter: 0
   for (uint32_t i = threadIdx.x; i < (1u << local_log2); i += blockDim.x) c.evmax[i] = 0;
   for (uint32_t i = threadIdx.x; i < (1u << c.qn_log2); i += blockDim.x) c.queue[i] = 0;
@@ -888,7 +989,10 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   if (warp == 0) {
     server_receiver(p, c, t_begin);
   } else if (warp <= p.n_workers) {
-    if constexpr (KIND == CSMV_KIND_KV) server_worker_generic<CL>(p, c, t_begin);
+    if constexpr (KIND == CSMV_KIND_KV) {
+      if (kv_filter_mode(p)) server_worker_kv_filter<CL>(p, c, t_begin);
+      else server_worker_generic<CL>(p, c, t_begin);
+    }
     else if (!CL && p.commit == CSMV_COMMIT_ONLYCS) server_worker_onlycs<NS>(p, c, t_begin);
     else server_worker<CL>(p, c, t_begin);
   } else if (warp == p.n_workers + 1 && rank == 0 && p.publish == CSMV_PUBLISH_SERVER) {

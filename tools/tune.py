@@ -24,8 +24,12 @@ def main(argv):
             k, v = kv.split("=")
             kw[k] = int(v)
         cfg = workloads.PRESETS[name](**kw)
-        st = csmv.Store(cfg.n_items, cfg.n_versions)
-        st.load(cfg.init_values())
+        if cfg.workload.kind == csmv.KIND_KV:
+            st = csmv.KvStore(cfg.n_items, cfg.workload.kv_ways, cfg.n_versions)
+            st.load(cfg.workload.kv_keys)
+        else:
+            st = csmv.Store(cfg.n_items, cfg.n_versions)
+            st.load(cfg.init_values())
         with st:
             for r in range(reps):
                 x = st.run(cfg.workload, cfg.n_tx, cfg.seed + r)
