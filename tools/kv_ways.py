@@ -17,7 +17,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
 
 WAYS = (4, 8, 16, 32, 64, 128, 256)
-TUNED = dict(server_workers=6, ro_streak=8, publish=csmv.PUBLISH_SERVER)
+TUNED = dict(server_workers=6, ro_streak=8, ro_adaptive=1, publish=csmv.PUBLISH_SERVER)
 
 
 def cfg_for(ways: int, n_tx: int, slots: int, **kw):
