@@ -79,6 +79,10 @@ extern "C" {
 #define CSMV_DBG_PHASES 8u     /* per-phase client clocks (csmv_stats_t.client_phase_cycles) */
 #define CSMV_DBG_KV_ITEMSETS 16u /* KV, A <= 16: ship PUT read/write sets item by item (the paper's literal
                                     form); default {set clock} u WS, which decides identically */
+#define CSMV_DBG_ALT_COMMIT 32u /* bank, atr_mode HASH: swap the commit path -- the single-CTA server
+                                   commits through the commit ring and one committer warp instead of the
+                                   ticket-locked critical section, the cluster server the other way
+                                   round; A/B only */
 
 typedef struct csmv_workload {
     uint32_t kind;             /* CSMV_KIND_* */

@@ -404,6 +404,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   // server CTA: warp 0 receiver, warps 1..n_workers workers, last warp publisher
   uint32_t n_workers = w->server_workers ? w->server_workers : 4u;
   if (n_workers > kWarps - 2) n_workers = kWarps - 2;
+  // bank + filter: the last warp of CTA 0 is the committer (server.cuh commit ring)
+  const bool cmring = h->kind == CSMV_KIND_BANK && w->atr_mode == CSMV_ATR_HASH && w->commit == CSMV_COMMIT_CSMV &&
+                      ((w->server == CSMV_SERVER_CLUSTER) != ((w->debug_flags & CSMV_DBG_ALT_COMMIT) != 0));
+  if (cmring && n_workers > kWarps - 3) n_workers = kWarps - 3;
   uint32_t n_cw = w->client_warps ? w->client_warps : h->max_cw;
   if (n_cw > h->max_cw) n_cw = h->max_cw;
   if (n_cw == 0) return set_err(CSMV_EINVAL, "csmv_run: no client warps");
@@ -419,7 +423,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   const bool filt = h->kind == CSMV_KIND_BANK ? w->atr_mode == CSMV_ATR_HASH
                                               : (h->kv_A > kKvFullWays || !(w->debug_flags & CSMV_DBG_KV_ITEMSETS));
   if (filt && rt_log2 < 7 + clog2) rt_log2 = 7 + clog2;
-  const uint32_t per_srv = n_srv ? (n_cw + n_srv - 1) / n_srv : 0u;
+  // cluster + commit ring: CTA 0 runs only the committer and the publisher,
+  // CTAs 1..C-1 receive (server.cuh server_cta)
+  const uint32_t n_serve = (cmring && n_srv > 1) ? n_srv - 1 : n_srv;
+  const uint32_t per_srv = n_serve ? (n_cw + n_serve - 1) / n_serve : 0u;
   size_t smem = server_smem_bytes(rt_log2 - clog2, per_srv);
   if (h->kind == CSMV_KIND_KV && smem < kv_client_smem_bytes()) smem = kv_client_smem_bytes();
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");

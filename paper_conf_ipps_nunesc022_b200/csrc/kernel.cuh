@@ -31,6 +31,20 @@ constexpr int kBlock = 256;            // threads per CTA (8 warps)
 constexpr int kWarps = kBlock / 32;
 constexpr uint32_t kDoneLog2 = 20;     // done ring entries (CSMV_PUBLISH_SERVER)
 constexpr int kMaxCombine = 4;         // batches a server worker commits per critical section
+constexpr uint32_t kCmRingLog2 = 5;    // commit-ring slots (worker warps -> committer warp, bank)
+
+// One commit-ring slot: a batch a worker warp has prepared for the committer
+// (server.cuh).  Lane l's words: {fa0, fa1, fa2, fb0}, {fb1, fb2, id0, id1}
+// -- the shared-memory addresses of its items' filter slots and the items.
+struct alignas(16) CmSlot {
+  uint32_t flag;   // = slot sequence number + 1 once the payload is written
+  uint32_t cw;     // client warp
+  uint32_t round;  // request round (tags the response)
+  uint32_t e_pre;  // tail the worker's lastw prefetch covers
+  uint32_t chk;    // lanes whose exact lastw check passed
+  uint32_t pad[3];
+  uint4 w[2][32];
+};
 
 struct Ctl {
   uint32_t error;       // 0 ok, 1 watchdog, 2 protocol
@@ -137,9 +151,11 @@ __host__ __device__ inline uint32_t queue_log2(uint32_t n_cw) {
 // smem the server CTA needs (every CTA of the fused grid gets the same):
 // recent-commit table, dispatch queue, receiver's last-seen doorbells, control words
 // (per server CTA: its stripe of 2^local_log2 buckets and its slice of n_cw)
+// rt stripe | dispatch queue | evmax stripe | last-seen doorbells | control
+// block (64 B) | commit ring
 inline size_t server_smem_bytes(uint32_t local_log2, uint32_t n_cw) {
   return ((size_t)(32 + 4) << local_log2) + ((size_t)8 << queue_log2(n_cw)) +
-         (((size_t)n_cw + 31) / 32 * 32) * 4 + 64;
+         (((size_t)n_cw + 31) / 32 * 32) * 4 + 64 + (sizeof(CmSlot) << kCmRingLog2);
 }
 
 // host-callable launchers (kernel.cu)

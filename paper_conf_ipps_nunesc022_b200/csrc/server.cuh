@@ -26,7 +26,12 @@ struct SrvShared {
   uint32_t gts_seen;     // publisher progress seen by workers (back-pressure) [CTA 0]
   uint32_t q_head;       // next dispatch-queue slot a worker claims          [per CTA]
   uint32_t exit;         // receiver: all clients finished                    [per CTA]
+  uint32_t ring_head;    // commit ring: next slot a worker claims            [CTA 0]
+  uint32_t ring_done;    // commit ring: slots the committer has finished     [CTA 0]
+  uint32_t workers_left; // commit ring: worker warps still running          [CTA 0]
+  uint32_t pad[7];
 };
+static_assert(sizeof(SrvShared) == 64, "control block is 64 B (server_smem_bytes)");
 
 // ---------------------------------------------------------------------------
 // The ATR, item-indexed and split in two levels:
@@ -60,7 +65,30 @@ struct SrvCtx {
   uint32_t qn_log2;
   uint32_t* last_seen;
   uint32_t cw_lo, cw_hi;  // client warps this CTA's receiver serves
+  uint32_t ring32;     // CTA 0's commit ring: shared (::cluster in a cluster) window address
 };
+
+// shared-memory stores/loads of the commit ring (explicit shared::cluster
+// forms in a cluster: the payload goes to CTA 0 through DSMEM)
+template <bool CL>
+__device__ __forceinline__ void ring_st_v4(uint32_t a, uint4 v) {
+  if constexpr (CL)
+    asm volatile("st.shared::cluster.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+                 : "memory");
+  else
+    asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+                 : "memory");
+}
+// acquire load of a flag in this CTA's shared memory written (after a
+// release fence) by a warp of this CTA (CL = false: a plain LDS) or of any
+// CTA of the cluster
+template <bool CL>
+__device__ __forceinline__ uint32_t ring_ld_acquire(uint32_t a) {
+  uint32_t v;
+  if constexpr (CL) asm volatile("ld.acquire.cluster.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  else asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
 
 template <bool CL>
 __device__ __forceinline__ uint64_t* rt_at(const SrvCtx& c, uint32_t b) {
@@ -565,6 +593,276 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
   }
 }
 
+// bank + recent-write filter: the cluster server commits through the commit
+// ring (below), the single-CTA server under the ticket lock (server_worker);
+// CSMV_DBG_ALT_COMMIT swaps them
+__device__ __forceinline__ bool server_uses_ring(const KParams& p) {
+  return p.kind == CSMV_KIND_BANK && p.atr_mode == CSMV_ATR_HASH && p.commit == CSMV_COMMIT_CSMV &&
+         ((p.n_server_ctas > 1) != ((p.debug & CSMV_DBG_ALT_COMMIT) != 0));
+}
+
+// ---------------------------------------------------------------------------
+// Bank commit through the commit ring (atr_mode HASH, the default).
+// The order-dependent part of a commit -- filter probe, CTS assignment,
+// filter update, lastw, respond -- is run by ONE committer warp
+// in CTA 0, which owns the recent-write filter and the CTS counter outright:
+// no lock, no lock handoff, and its filter accesses are local shared memory
+// even in a cluster.  Worker warps (every server CTA) do everything that needs
+// no order: claim dispatched batches, load them, prefetch lastw and settle the
+// exact part of the validation (lastw[x] <= s for every CTS <= e_pre), compute
+// the filter-slot addresses, and push the prepared batches into the ring in
+// CTA 0's shared memory (DSMEM stores from the other CTAs of a cluster).  The
+// committer takes the slots in ring order, so every batch is validated after
+// the write-sets of all batches before it were recorded and receives the next
+// consecutive CTS range -- as if each had held the lock in that order.
+// ---------------------------------------------------------------------------
+template <bool CL>
+__device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+  constexpr int M = kMaxCombine;
+  constexpr uint32_t R = 1u << kCmRingLog2;
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t qmask = (1u << c.qn_log2) - 1;
+  const uint32_t m_max = p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine);
+  const uint32_t fl2 = p.rt_log2 - p.clog2 + 3;  // the filter: CTA 0's stripe, 8 << local_log2 slots
+  const bool novalid = (p.debug & CSMV_DBG_NO_VALIDATE) != 0;
+  unsigned long long busy = 0, batches = 0, groups = 0, ph0 = 0, ph1 = 0, ph4 = 0;
+  for (;;) {
+    const long long tq = clock64();
+    uint32_t cwv[M];
+    if (!claim_request(c, cwv[0])) break;
+    uint32_t m = 1;
+#pragma unroll
+    for (int j = 1; j < M; ++j) {
+      uint32_t got = 0xFFFFFFFFu;
+      if (m == (uint32_t)j && m < m_max && lane == 0) {
+        const uint32_t h = *(volatile uint32_t*)&c.sh->q_head;
+        const uint64_t e = *(volatile uint64_t*)&c.queue[h & qmask];
+        if ((uint32_t)(e >> 32) == (h >> c.qn_log2) + 1 && atomicCAS(&c.sh->q_head, h, h + 1) == h) got = (uint32_t)e;
+      }
+      got = __shfl_sync(FULL, got, 0);
+      cwv[j] = got;
+      if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
+    }
+    const long long t0 = clock64();
+    fence_cta();  // payload loads after the queue entries (the receiver fenced after the doorbells)
+    uint32_t sq[M], sn[M], msk[M], id0[M], id1[M];
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      sq[j] = sn[j] = msk[j] = id0[j] = id1[j] = 0;
+      if (j < (int)m) {
+        sn[j] = ld_relaxed(&p.req_hdr[cwv[j]].snapshot);
+        msk[j] = ld_relaxed(&p.req_hdr[cwv[j]].mask);
+        sq[j] = ld_relaxed(&p.req_hdr[cwv[j]].round);
+        id0[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + lane) & ~kWriteBit;
+        id1[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + 32 + lane) & ~kWriteBit;
+      }
+    }
+    bool mine[M];
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      mine[j] = (msk[j] >> lane) & 1u;
+      if (!mine[j]) id0[j] = id1[j] = 0;
+    }
+    // m consecutive ring slots, in claim order
+    uint32_t s0 = 0;
+    if (lane == 0) s0 = atomicAdd(&c.sh0->ring_head, m);
+    s0 = __shfl_sync(FULL, s0, 0);
+    const long long tl = clock64();
+    {  // room: slot s0+m-1 is free once the committer finished s0+m-1-R
+      uint32_t it = 0;
+      while ((int)(s0 + m - *(volatile uint32_t*)&c.sh0->ring_done) > (int)R) {
+        if ((++it & 1023u) == 0 && (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 8))) break;
+        __nanosleep(32);
+      }
+      __syncwarp();
+      srv_fence<CL>();  // the committer's reads of the slot's previous use precede our stores
+    }
+    // lastw prefetched only now: the window the filter must cover is then
+    // the ring's depth, not the wait for room as well
+    const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
+    srv_fence<CL>();
+    uint32_t chkm[M];
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      uint32_t lw0 = 0, lw1 = 0;
+      if (mine[j]) {
+        lw0 = ld_relaxed(p.lastw + id0[j]);
+        lw1 = ld_relaxed(p.lastw + id1[j]);
+      }
+      chkm[j] = __ballot_sync(FULL, mine[j] && (novalid || (lw0 <= sn[j] && lw1 <= sn[j])));
+    }
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      if (j < (int)m) {
+        const uint32_t sl = c.ring32 + (uint32_t)sizeof(CmSlot) * ((s0 + j) & (R - 1));
+        uint4 a, b;  // filter slots as byte offsets (the committer adds CTA 0's base)
+        a.x = 4u * filt_slot(id0[j], 0, fl2);
+        a.y = 4u * filt_slot(id0[j], 1, fl2);
+        a.z = 4u * filt_slot(id0[j], 2, fl2);
+        a.w = 4u * filt_slot(id1[j], 0, fl2);
+        b.x = 4u * filt_slot(id1[j], 1, fl2);
+        b.y = 4u * filt_slot(id1[j], 2, fl2);
+        b.z = id0[j];
+        b.w = id1[j];
+        ring_st_v4<CL>(sl + (uint32_t)offsetof(CmSlot, w) + 16u * lane, a);
+        ring_st_v4<CL>(sl + (uint32_t)offsetof(CmSlot, w) + 16u * (32 + lane), b);
+        if (lane == 0) ring_st_v4<CL>(sl + 16u, make_uint4(chkm[j], 0u, 0u, 0u));
+        if (lane == 0) filt_st<CL>(sl + 4u, cwv[j]);
+        if (lane == 0) filt_st<CL>(sl + 8u, sq[j]);
+        if (lane == 0) filt_st<CL>(sl + 12u, novalid ? 0xFFFFFFFFu : e_pre);
+      }
+    }
+    __syncwarp();
+    srv_fence<CL>();  // payloads before flags
+    if (lane < m) filt_st<CL>(c.ring32 + (uint32_t)sizeof(CmSlot) * ((s0 + lane) & (R - 1)), s0 + lane + 1);
+    __syncwarp();
+    const long long t3 = clock64();
+    busy += (unsigned long long)(t3 - t0);
+    ph0 += (unsigned long long)(t0 - tq);
+    ph1 += (unsigned long long)(tl - t0);
+    ph4 += (unsigned long long)(t3 - tl);
+    batches += m;
+    ++groups;
+  }
+  __syncwarp();
+  if (lane == 0) {
+    srv_fence<CL>();  // every flag we wrote precedes the count
+    atomicSub(&c.sh0->workers_left, 1u);
+    atomicAdd(&p.stats->phase[0], ph0);
+    atomicAdd(&p.stats->phase[1], ph1);
+    atomicAdd(&p.stats->phase[4], ph4);
+    atomicAdd(&p.stats->batches, batches);
+    atomicAdd(&p.stats->groups, groups);
+    atomicAdd(&p.stats->busy_cycles, busy);
+  }
+}
+
+// The committer warp (CTA 0).  `ring` is CTA 0's commit ring (local).  The
+// next slot's flag and payload are loaded while the current batch is being
+// committed, so the serial chain per batch is: filter loads -> commit mask
+// -> CTS -> filter stores.
+struct CmPayload {
+  uint4 w0, w1;
+  uint32_t cw, round, e_chk, chkm;
+};
+
+template <bool CL>
+__device__ __forceinline__ bool cm_try(CmSlot* sl, uint32_t seq, CmPayload& q) {
+  const uint32_t f = ring_ld_acquire<CL>((uint32_t)__cvta_generic_to_shared(&sl->flag));
+  const uint32_t lane = threadIdx.x & 31;
+  q.w0 = sl->w[0][lane];
+  q.w1 = sl->w[1][lane];
+  const uint4 h = *reinterpret_cast<const uint4*>(sl);
+  q.cw = h.y;
+  q.round = h.z;
+  q.e_chk = h.w;
+  q.chkm = sl->chk;
+  return __shfl_sync(0xFFFFFFFFu, f, 0) == seq + 1;  // lane 0's view decides
+}
+
+template <bool CL>
+__device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring, uint64_t t_begin) {
+  constexpr uint32_t R = 1u << kCmRingLog2;
+  constexpr uint32_t kTailEvery = CL ? 32u : 4u;  // the cluster fence is a gpu-scope MEMBAR
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t lt = lanemask_lt();
+  const uint32_t dmask = (1u << kDoneLog2) - 1;
+  const bool srv_pub = p.publish == CSMV_PUBLISH_SERVER;
+  const uint32_t fbase = c.rt32;  // the filter (this CTA's rt stripe); slots arrive as byte offsets
+  uint32_t t = *(volatile uint32_t*)&c.sh->tail;
+  uint32_t tpub = t;
+  uint32_t gseen = t;
+  unsigned long long cs = 0, wait = 0;
+  CmPayload q;
+  bool have = false;
+  for (uint32_t next = 0;; ++next) {
+    const long long tw = clock64();
+    // wait for slot `next` (unless the prefetch already found it ready)
+    for (uint32_t it = 0; !have;) {
+      have = cm_try<CL>(ring + (next & (R - 1)), next, q);
+      if (have) break;
+      // idle: publish the tail now (a later e_pre only widens the filter's window)
+      if (t != tpub) {
+        srv_fence<CL>();
+        if (lane == 0) *(volatile uint32_t*)&c.sh->tail = t;
+        tpub = t;
+      }
+      uint32_t done = 0;
+      if (lane == 0 && *(volatile uint32_t*)&c.sh->workers_left == 0 &&
+          *(volatile uint32_t*)&c.sh->ring_head == next)
+        done = 1;
+      if (lane == 0 && (++it & 4095u) == 0 && (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 9))) done = 1;
+      if (__shfl_sync(FULL, done, 0)) break;
+    }
+    if (!have) break;
+    const long long t1 = clock64();
+    const CmPayload cur = q;
+    const bool chk = (cur.chkm >> lane) & 1u;
+    uint32_t v0 = 0, v1 = 0, v2 = 0, v3 = 0, v4 = 0, v5 = 0;
+    if (chk) {
+      v0 = filt_ld<false>(fbase + cur.w0.x);
+      v1 = filt_ld<false>(fbase + cur.w0.y);
+      v2 = filt_ld<false>(fbase + cur.w0.z);
+      v3 = filt_ld<false>(fbase + cur.w0.w);
+      v4 = filt_ld<false>(fbase + cur.w1.x);
+      v5 = filt_ld<false>(fbase + cur.w1.y);
+    }
+    // prefetch slot next+1 (its payload is only used if its flag was set)
+    have = cm_try<CL>(ring + ((next + 1) & (R - 1)), next + 1, q);
+    // a write after e_pre to one of the items raised all of its slots above
+    // e_pre (every earlier batch of the ring included)
+    const uint32_t lo = max(min(v0, min(v1, v2)), min(v3, min(v4, v5)));
+    const bool ovf = chk && lo > cur.e_chk;
+    const bool commit = chk && !ovf;
+    const uint32_t cm = __ballot_sync(FULL, commit), om = __ballot_sync(FULL, ovf);
+    const uint32_t base = t + 1;
+    const uint32_t cts = base + __popc(cm & lt);
+    t += __popc(cm);
+    if (srv_pub && t > gseen + dmask) {  // done-ring back-pressure: CTS t may reuse slot t & mask once GTS >= t - 2^20
+      for (uint32_t it = 0; t > gseen + dmask;) {
+        gseen = __shfl_sync(FULL, ld_relaxed(p.gts), 0);
+        if ((++it & 255u) == 0 && __shfl_sync(FULL, (uint32_t)(lane == 0 && watchdog(p, t_begin, 4)), 0)) break;
+      }
+    }
+    if (commit) {  // the batch's last CTS: equal values for shared slots, race-free
+      filt_st<false>(fbase + cur.w0.x, t);
+      filt_st<false>(fbase + cur.w0.y, t);
+      filt_st<false>(fbase + cur.w0.z, t);
+      filt_st<false>(fbase + cur.w0.w, t);
+      filt_st<false>(fbase + cur.w1.x, t);
+      filt_st<false>(fbase + cur.w1.y, t);
+      p.lastw[cur.w1.z] = cts;
+      p.lastw[cur.w1.w] = cts;
+    }
+    if (lane == 0) {  // respond: round-tagged words, no fence (kernel.cuh Resp); slot release
+      const uint64_t tag = (uint64_t)cur.round << 32;
+      st_relaxed64x2(&p.resp[cur.cw].base, tag | base, tag | cm);
+      st_relaxed64(&p.resp[cur.cw].ovf, tag | om);
+      *(volatile uint32_t*)&c.sh->ring_done = next + 1;
+    }
+    __syncwarp();  // this batch's filter stores precede the next batch's loads
+    // tail (the e_pre workers prefetch lastw under) needs a fence ordering the
+    // lastw stores before it: every kTailEvery batches under load, else when idle
+    if (((next + 1) & (kTailEvery - 1)) == 0 && t != tpub) {
+      srv_fence<CL>();
+      if (lane == 0) *(volatile uint32_t*)&c.sh->tail = t;
+      tpub = t;
+    }
+    const long long t2 = clock64();
+    wait += (unsigned long long)(t1 - tw);
+    cs += (unsigned long long)(t2 - t1);
+  }
+  srv_fence<CL>();
+  if (lane == 0) *(volatile uint32_t*)&c.sh->tail = t;
+  if (lane == 0) {
+    atomicAdd(&p.stats->phase[2], wait);
+    atomicAdd(&p.stats->phase[3], cs);
+    atomicAdd(&p.stats->lock_cycles, cs);
+  }
+}
+
 // ---------------------------------------------------------------------------
 // Generic worker (variable-length read/write sets, the KV workload): one
 // batch per critical section, validated against the two-level ATR exactly
@@ -952,10 +1250,14 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   const uint32_t C = p.n_server_ctas;
   const uint32_t rank = CL ? cg::this_cluster().block_rank() : 0u;
   const uint32_t local_log2 = p.rt_log2 - p.clog2;
-  const uint32_t per = (p.n_cw + C - 1) / C;
+  // cluster + commit ring: CTA 0 is left to the committer (and publisher);
+  // the client doorbells are sliced over CTAs 1..C-1
+  const bool ring_cl = CL && server_uses_ring(p);
+  const uint32_t nserve = ring_cl ? C - 1 : C, srank = ring_cl ? rank - 1 : rank;
+  const uint32_t per = (p.n_cw + nserve - 1) / nserve;
   SrvCtx c;
   c.clog2 = p.clog2;
-  c.cw_lo = min(rank * per, p.n_cw);
+  c.cw_lo = (ring_cl && rank == 0) ? p.n_cw : min(srank * per, p.n_cw);
   c.cw_hi = min(c.cw_lo + per, p.n_cw);
   c.qn_log2 = queue_log2(per);
   c.rt = reinterpret_cast<uint64_t*>(smem);
@@ -966,14 +1268,23 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   c.last_seen = c.evmax + (1u << local_log2);
   const uint32_t ls_words = (per + 31) / 32 * 32;
   c.sh = reinterpret_cast<SrvShared*>(c.last_seen + ls_words);
-  if constexpr (CL) c.sh0 = cg::this_cluster().map_shared_rank(c.sh, 0);
-  else c.sh0 = c.sh;
+  CmSlot* ring = reinterpret_cast<CmSlot*>(reinterpret_cast<uint8_t*>(c.sh) + sizeof(SrvShared));
+  c.ring32 = (uint32_t)__cvta_generic_to_shared(ring);
+  if constexpr (CL) {
+    c.sh0 = cg::this_cluster().map_shared_rank(c.sh, 0);
+    asm("mapa.shared::cluster.u32 %0, %1, 0;" : "=r"(c.ring32) : "r"(c.ring32));
+  } else {
+    c.sh0 = c.sh;
+  }
+  // bank + filter: the commit ring and one committer warp (unless the A/B flag asks for the lock)
+  const bool cmring = server_uses_ring(p);
   const bool filt = KIND == CSMV_KIND_BANK ? p.atr_mode == CSMV_ATR_HASH : kv_filter_mode(p);
   const uint64_t rt_init = filt ? 0ull : 0xFFFFFFFFull;
   for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) c.rt[i] = rt_init;  // table: cts 0, no item; filter: 0
   for (uint32_t i = threadIdx.x; i < (1u << local_log2); i += blockDim.x) c.evmax[i] = 0;
   for (uint32_t i = threadIdx.x; i < (1u << c.qn_log2); i += blockDim.x) c.queue[i] = 0;
   for (uint32_t i = threadIdx.x; i < ls_words; i += blockDim.x) c.last_seen[i] = 0;
+  for (uint32_t i = threadIdx.x; i < (1u << kCmRingLog2); i += blockDim.x) ring[i].flag = 0;
   if (threadIdx.x == 0) {
     const uint32_t g0 = *p.gts;
     c.sh->tail = g0;
@@ -982,11 +1293,17 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     c.sh->gts_seen = g0;
     c.sh->q_head = 0;
     c.sh->exit = 0;
+    c.sh->ring_head = 0;
+    c.sh->ring_done = 0;
+    c.sh->workers_left = p.n_workers * nserve;
   }
   if constexpr (CL) cg::this_cluster().sync();
   else __syncthreads();
   const uint32_t warp = threadIdx.x >> 5;
-  if (warp == 0) {
+  const bool serving = !(ring_cl && rank == 0);
+  if (!serving && warp <= p.n_workers) {
+    // CTA 0 of a ring cluster: no receiver, no workers
+  } else if (warp == 0) {
     server_receiver(p, c, t_begin);
   } else if (warp <= p.n_workers) {
     if constexpr (KIND == CSMV_KIND_KV) {
@@ -994,9 +1311,12 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
       else server_worker_generic<CL>(p, c, t_begin);
     }
     else if (!CL && p.commit == CSMV_COMMIT_ONLYCS) server_worker_onlycs<NS>(p, c, t_begin);
+    else if (cmring) server_worker_cm<CL>(p, c, t_begin);
     else server_worker<CL>(p, c, t_begin);
   } else if (warp == p.n_workers + 1 && rank == 0 && p.publish == CSMV_PUBLISH_SERVER) {
     server_publisher(p, c, t_begin);
+  } else if (warp == kWarps - 1 && rank == 0 && cmring) {
+    server_committer<CL>(p, c, ring, t_begin);
   }
   if constexpr (CL) cg::this_cluster().sync();
   else __syncthreads();

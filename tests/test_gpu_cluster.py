@@ -1,5 +1,7 @@
-"""GPU parity of the thread-block-cluster server (the recent-commit table
-striped over C CTAs' shared memory through DSMEM, CTS counter in CTA 0) and
+"""GPU parity of the thread-block-cluster server (receivers and workers in
+every CTA of the cluster, the bank commit through the commit ring to one
+committer warp in CTA 0; KV and the A/B flag: the recent-commit table striped
+over the CTAs' shared memory through DSMEM under a ticket lock in CTA 0) and
 of the single-CTA server on the same workloads (C5's server axis)."""
 import numpy as np
 import pytest
@@ -14,11 +16,12 @@ from tests.test_gpu_parity import check, closed_form, newest  # noqa: E402
 from tests.test_gpu_kv import ocfg_of, as_state, run as run_kv  # noqa: E402
 
 
-@pytest.mark.parametrize("cs", [2, 4, 8, 16])
-def test_bank_cluster_parity(cs):
+@pytest.mark.parametrize("cs,flags", [(2, 0), (4, 0), (8, 0), (16, 0), (2, csmv.DBG_ALT_COMMIT),
+                                      (16, csmv.DBG_ALT_COMMIT)])
+def test_bank_cluster_parity(cs, flags):
     cfg = W.c2(n_items=1 << 16, n_tx=1 << 18, server=csmv.SERVER_CLUSTER, cluster_size=cs,
                publish=csmv.PUBLISH_SERVER, ro_streak=8, server_workers=6, server_combine=4,
-               client_warps=256)
+               client_warps=256, debug_flags=flags)
     rep, stats, log, rings, descs = check(cfg)
     assert stats["server_ctas"] == cs
     assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions), closed_form(cfg, descs, cfg.init_values()))
@@ -54,6 +57,29 @@ def test_kv_cluster_parity():
 def test_cluster_one_client_warp_is_deterministic():
     """P7 holds with the cluster server too (the server's shape is invisible)."""
     cfg = W.c1(client_warps=1, n_tx=2000, server=csmv.SERVER_CLUSTER, cluster_size=2, ro_streak=4)
+    from tests.test_gpu_parity import run_gpu, oracle_cfg
+    stats, log, (vals, mv), rings = run_gpu(cfg)
+    ocfg = oracle_cfg(cfg)
+    descs = oracle.bank_gen(ocfg, cfg.seed, cfg.n_tx)
+    plog, pvals, prings, pst = oracle.bank_predict(ocfg, cfg.init_values(), descs, 32, max_vals=mv)
+    assert np.array_equal(log, plog) and np.array_equal(rings, prings)
+
+
+@pytest.mark.parametrize("publish", [0, 1])
+def test_bank_commit_ring_single_cta(publish):
+    """The commit ring on the single-CTA server (CSMV_DBG_ALT_COMMIT): same
+    history checks, closed-form final store."""
+    cfg = W.c2(n_items=1 << 14, n_tx=1 << 18, publish=publish, ro_streak=8, server_workers=6,
+               server_combine=4, client_warps=256, debug_flags=csmv.DBG_ALT_COMMIT)
+    rep, stats, log, rings, descs = check(cfg)
+    assert stats["server_workers"] == 5  # the last warp of CTA 0 is the committer
+    assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions), closed_form(cfg, descs, cfg.init_values()))
+
+
+@pytest.mark.parametrize("server,flags", [(0, 32), (1, 0), (1, 32)])
+def test_commit_designs_one_client_warp_deterministic(server, flags):
+    """P7 through every commit design: ring or lock, one CTA or a cluster."""
+    cfg = W.c1(client_warps=1, n_tx=2000, server=server, cluster_size=4, ro_streak=4, debug_flags=flags)
     from tests.test_gpu_parity import run_gpu, oracle_cfg
     stats, log, (vals, mv), rings = run_gpu(cfg)
     ocfg = oracle_cfg(cfg)

@@ -161,6 +161,11 @@ def test_no_validate_is_caught():
                debug_flags=csmv.DBG_NO_VALIDATE)
     rep, *_ = check(cfg, expect_ok=False)
     assert not rep["ok"]
+    # the same through the commit ring (one CTA, then a cluster)
+    for srv, fl in ((csmv.SERVER_CTA, csmv.DBG_ALT_COMMIT), (csmv.SERVER_CLUSTER, 0)):
+        rep, *_ = check(cfg.with_(server=srv, cluster_size=4, debug_flags=csmv.DBG_NO_VALIDATE | fl),
+                        expect_ok=False)
+        assert not rep["ok"]
 
 
 def test_generator_parity():
