@@ -98,7 +98,7 @@ typedef struct csmv_workload {
     uint32_t server;           /* CSMV_SERVER_* */
     uint32_t cluster_size;     /* cluster server CTAs (2..16) */
     uint32_t server_workers;   /* worker warps per server CTA (0 = default) */
-    uint32_t server_combine;   /* batches a worker commits per critical section (1..4; 0 = 1) */
+    uint32_t server_combine;   /* batches a worker commits per critical section (1..8; 0 = 1) */
     uint32_t atr_capacity;     /* ATR entries (0 = default); rounded to the layout */
     uint32_t atr_mode;         /* CSMV_ATR_* */
     uint32_t publish;          /* CSMV_PUBLISH_* */

@@ -184,46 +184,66 @@ __device__ __forceinline__ void rot_coop(const KParams& p, uint32_t act, uint32_
   dg = 0;
   const uint32_t L = __shfl_sync(FULL, len, act ? __ffs(act) - 1 : 0);  // the same for every transaction
   const uint32_t rows = (L + 31) / 32;
-  const uint32_t total = (uint32_t)__popc(act) * rows;
-  for (uint32_t g = 0; g < total; g += U) {
+  const bool full_log = p.log_mode == CSMV_LOG_FULL;
+  const bool long_scan = L > N;  // a scan longer than the store wraps more than once
+  // owners are taken lowest lane first, `rows` rows each; (rem, cur, k) are
+  // warp-uniform, so the shuffles below run under uniform branches
+  uint32_t rem = act, cur = 0, k = rows, cur_start = 0;
+  uint64_t cur_tx = 0;
+  while (rem || k < rows) {
     Ring<NS> r[U];
     uint32_t xs[U], own[U], ev[U];
     uint64_t txo[U];
-    uint32_t so[U];
+    bool on[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      const uint32_t idx = g + u;
-      const uint32_t i = idx / rows, k = idx - i * rows;
-      own[u] = idx < total ? __fns(act, 0, i + 1) : 0u;
-      so[u] = __shfl_sync(FULL, start, own[u]);
-      txo[u] = __shfl_sync(FULL, tx, own[u]);
+      if (k >= rows && rem) {  // next owner
+        cur = __ffs(rem) - 1;
+        rem &= rem - 1;
+        k = 0;
+        cur_start = __shfl_sync(FULL, start, cur);
+        if (full_log) cur_tx = __shfl_sync(FULL, tx, cur);
+      }
+      on[u] = k < rows;
+      own[u] = cur;
+      txo[u] = cur_tx;
       ev[u] = k * 32 + lane;
-      uint32_t x = so[u] + ev[u];
+      uint32_t x = cur_start + ev[u];  // start < N; ev < L
       if (x >= N) x -= N;
-      if (x >= N) x %= N;
+      if (long_scan && x >= N) x %= N;
       xs[u] = x;
-      if (idx < total && ev[u] < L) r[u] = ld_ring<NS>(p.rings + (size_t)x * NS);
+      if (on[u] && ev[u] < L) r[u] = ld_ring<NS>(p.rings + (size_t)x * NS);
+      if (on[u]) ++k;
     }
+    // version selection for every row first, so that the re-reads a newer
+    // version calls for are in flight together (one L2 round trip per group)
+    uint64_t vv[U], rv[U];
+    bool miss_[U], re[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      if (g + u >= total) break;  // warp-uniform
-      const bool valid = ev[u] < L;
-      bool miss = false;
-      uint32_t val = 0;
-      if (valid) {
+      vv[u] = rv[u] = 0;
+      miss_[u] = re[u] = false;
+      if (on[u] && ev[u] < L) {
         const Sel q = select_version<NS>(r[u], s);
         if (q.best < 0) {
-          miss = true;  // version recycled
+          miss_[u] = true;  // version recycled
         } else {
-          const uint64_t v = slot_at<NS>(r[u], q.best);
+          vv[u] = slot_at<NS>(r[u], q.best);
           // A newer version exists, so write-backs may have overwritten slots
           // while we read.  Versions are evicted oldest first, so if the chosen
           // slot still holds the same version, no version in (best_ts, s] was
           // missed; otherwise the snapshot's version is gone.
-          if (q.newest > s && ld_relaxed64(p.rings + (size_t)xs[u] * NS + q.best) != v) miss = true;
-          val = (uint32_t)v;
+          re[u] = q.newest > s;
+          if (re[u]) rv[u] = ld_relaxed64(p.rings + (size_t)xs[u] * NS + q.best);
         }
       }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (!on[u]) break;  // warp-uniform
+      const bool valid = ev[u] < L;
+      const bool miss = miss_[u] || (re[u] && rv[u] != vv[u]);
+      const uint32_t val = (uint32_t)vv[u];
       const bool rmiss = __any_sync(FULL, miss);
       const int64_t rs = warp_sum_i32(miss ? 0 : (int32_t)val);
       uint64_t rd = 0;

@@ -30,7 +30,7 @@ constexpr uint32_t kWriteBit = 0x80000000u;
 constexpr int kBlock = 256;            // threads per CTA (8 warps)
 constexpr int kWarps = kBlock / 32;
 constexpr uint32_t kDoneLog2 = 20;     // done ring entries (CSMV_PUBLISH_SERVER)
-constexpr int kMaxCombine = 4;         // batches a server worker commits per critical section
+constexpr int kMaxCombine = 8;         // batches a server worker commits per critical section
 constexpr uint32_t kCmRingLog2 = 5;    // commit-ring slots (worker warps -> committer warp, bank)
 
 // One commit-ring slot: a batch a worker warp has prepared for the committer

@@ -29,7 +29,8 @@ struct SrvShared {
   uint32_t ring_head;    // commit ring: next slot a worker claims            [CTA 0]
   uint32_t ring_done;    // commit ring: slots the committer has finished     [CTA 0]
   uint32_t workers_left; // commit ring: worker warps still running          [CTA 0]
-  uint32_t pad[7];
+  uint32_t lw_done;      // locked bank worker: lastw written for every CTS <= lw_done [CTA 0]
+  uint32_t pad[6];
 };
 static_assert(sizeof(SrvShared) == 64, "control block is 64 B (server_smem_bytes)");
 
@@ -198,6 +199,10 @@ __device__ __forceinline__ void rt_record(const SrvCtx& c, uint32_t bucket, int 
 // Per item: k loads and k stores, no atomics, no eviction.
 // ---------------------------------------------------------------------------
 constexpr int kFiltK = 3;
+#ifndef CSMV_BANK_FILT_K
+#define CSMV_BANK_FILT_K 3
+#endif
+constexpr int kBankFiltK = CSMV_BANK_FILT_K;  // hashes the locked bank worker uses (<= kFiltK)
 
 // KV requests in the compact {set clock} u WS form use the filter
 __device__ __forceinline__ bool kv_filter_mode(const KParams& p) {
@@ -465,9 +470,11 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       mine[j] = (msk[j] >> lane) & 1u;
       if (!mine[j]) id0[j] = id1[j] = 0;
     }
-    const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
-    srv_fence<CL>();
     const bool hash = p.atr_mode == CSMV_ATR_HASH;
+    // lastw covers every CTS <= e_pre (HASH: lastw is written after the
+    // critical section and lw_done advanced in CTS order, below)
+    const uint32_t e_pre = hash ? *(volatile uint32_t*)&c.sh0->lw_done : *(volatile uint32_t*)&c.sh0->tail;
+    srv_fence<CL>();
     const bool novalid = (p.debug & CSMV_DBG_NO_VALIDATE) != 0;
     // HASH: the exact part of the validation (lastw, every CTS <= e_pre) and
     // the filter slot addresses are settled before the lock
@@ -500,38 +507,42 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     const long long t1 = clock64();
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
     uint32_t t = t0c;
-    uint32_t cm[M], om[M], base[M];
+    uint32_t cm[M], om[M], base[M], cts_of[M];
     if (hash) {
       // batch j: a write after e_pre to one of its items raised all of that
       // item's slots above e_pre (earlier batches of this section included)
 #pragma unroll
       for (int j = 0; j < M; ++j) {
-        cm[j] = om[j] = 0;
+        cm[j] = om[j] = cts_of[j] = 0;
         base[j] = t + 1;
         if (j < (int)m) {
           uint32_t va[kFiltK] = {0u, 0u, 0u}, vb[kFiltK] = {0u, 0u, 0u};
           if (chk[j]) {
 #pragma unroll
-            for (int k = 0; k < kFiltK; ++k) {
+            for (int k = 0; k < kBankFiltK; ++k) {
               va[k] = filt_ld<CL>(fa[j][k]);
               vb[k] = filt_ld<CL>(fb[j][k]);
             }
           }
-          const uint32_t lo = max(min(va[0], min(va[1], va[2])), min(vb[0], min(vb[1], vb[2])));
+          uint32_t la = va[0], lb = vb[0];
+#pragma unroll
+          for (int k = 1; k < kBankFiltK; ++k) {
+            la = min(la, va[k]);
+            lb = min(lb, vb[k]);
+          }
+          const uint32_t lo = max(la, lb);
           const bool ovf = chk[j] && lo > e_chk;
           const bool commit = chk[j] && !ovf;
           cm[j] = __ballot_sync(FULL, commit);
           om[j] = __ballot_sync(FULL, ovf);
-          const uint32_t cts = t + 1 + __popc(cm[j] & lt);
+          cts_of[j] = t + 1 + __popc(cm[j] & lt);
           t += __popc(cm[j]);
           if (commit) {
 #pragma unroll
-            for (int k = 0; k < kFiltK; ++k) {  // the batch's last CTS: equal values, race-free
+            for (int k = 0; k < kBankFiltK; ++k) {  // the batch's last CTS: equal values, race-free
               filt_st<CL>(fa[j][k], t);
               filt_st<CL>(fb[j][k], t);
             }
-            p.lastw[id0[j]] = cts;
-            p.lastw[id1[j]] = cts;
           }
           __syncwarp();  // batch j's records precede batch j+1's probes
         }
@@ -559,6 +570,26 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) done_ring_room(p, c, t, t_begin);
     cs_leave<CL>(c, ticket, t);
     const long long t2 = clock64();
+    if (hash && t != t0c) {
+      // lastw for this group's commits, outside the lock; then lw_done moves
+      // from t0c to t once every earlier group has published (CTS order),
+      // so a worker that reads lw_done = e sees lastw of every CTS <= e
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        if (j < (int)m && ((cm[j] >> lane) & 1u)) {
+          p.lastw[id0[j]] = cts_of[j];
+          p.lastw[id1[j]] = cts_of[j];
+        }
+      }
+      if (lane == 0) {
+        uint32_t it = 0;
+        while (*(volatile uint32_t*)&c.sh0->lw_done != t0c)
+          if ((++it & 1023u) == 0 && watchdog(p, t_begin, 10)) break;
+      }
+      __syncwarp();
+      srv_fence<CL>();
+      if (lane == 0) *(volatile uint32_t*)&c.sh0->lw_done = t;
+    }
     // ---- respond: round-tagged words, no fence (kernel.cuh Resp)
     if (lane < (uint32_t)m) {
 #pragma unroll
@@ -1296,6 +1327,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     c.sh->ring_head = 0;
     c.sh->ring_done = 0;
     c.sh->workers_left = p.n_workers * nserve;
+    c.sh->lw_done = g0;
   }
   if constexpr (CL) cg::this_cluster().sync();
   else __syncthreads();

@@ -8,7 +8,7 @@ import sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
 
-BASE = dict(client_warps=294, publish=1, server_workers=6, server_combine=4, ro_streak=8)
+BASE = dict(client_warps=294, publish=1, server_workers=6, server_combine=8, ro_streak=8, ro_adaptive=1, log_mode=0)
 
 
 def main(argv):
