@@ -17,7 +17,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
 
-TUNED = dict(client_warps=294, server_workers=6, server_combine=4, ro_streak=8, ro_adaptive=1, publish=csmv.PUBLISH_SERVER)
+TUNED = dict(client_warps=294, server_workers=6, server_combine=8, ro_streak=8, ro_adaptive=1, publish=csmv.PUBLISH_SERVER)
 
 
 def run_point(cfg, check: bool):
