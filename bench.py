@@ -37,7 +37,7 @@ METRIC = "committed tx/sec and abort rate at 1 B200 (+partitioned 2/4/8)"
 UNIT = "tx/s"
 
 # tuned launch configuration of the C2 workload
-TUNED = dict(client_warps_per_sm=2, server_workers=6, server_combine=8, ro_streak=8, publish=1, ro_adaptive=1)
+TUNED = dict(client_warps_per_sm=2, server_workers=7, server_combine=8, ro_streak=8, publish=1, ro_adaptive=1)
 
 # algorithmic bytes (paper VBox layout P:289): a read moves the
 # VBox head, the visited version's ts and the value (4+4+4); a write-back the

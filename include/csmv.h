@@ -83,6 +83,8 @@ extern "C" {
                                    commits through the commit ring and one committer warp instead of the
                                    ticket-locked critical section, the cluster server the other way
                                    round; A/B only */
+#define CSMV_DBG_RECEIVER 64u  /* bank, single-CTA locked commit: keep the receiver warp and dispatch
+                                  queue instead of self-receiving worker warps; A/B only */
 
 typedef struct csmv_workload {
     uint32_t kind;             /* CSMV_KIND_* */

@@ -23,7 +23,7 @@ SERVER_CTA, SERVER_CLUSTER = 0, 1
 PUBLISH_CLIENT, PUBLISH_SERVER = 0, 1
 ATR_HASH, ATR_LIST, ATR_LIST_NOCV = 0, 1, 2
 COMMIT_CSMV, COMMIT_ONLYCS, COMMIT_JVSTM = 0, 1, 2
-DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER, DBG_PHASES, DBG_KV_ITEMSETS, DBG_ALT_COMMIT = 1, 2, 4, 8, 16, 32
+DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER, DBG_PHASES, DBG_KV_ITEMSETS, DBG_ALT_COMMIT, DBG_RECEIVER = 1, 2, 4, 8, 16, 32, 64
 CLIENT_PHASES = ("read", "preval", "submit", "rot", "wait_server", "writeback", "publish", "divergence")
 ABORT_REASONS = ("preval", "conflict", "early", "overflow", "version")
 

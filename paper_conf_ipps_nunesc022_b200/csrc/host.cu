@@ -408,6 +408,13 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   const bool cmring = h->kind == CSMV_KIND_BANK && w->atr_mode == CSMV_ATR_HASH && w->commit == CSMV_COMMIT_CSMV &&
                       ((w->server == CSMV_SERVER_CLUSTER) != ((w->debug_flags & CSMV_DBG_ALT_COMMIT) != 0));
   if (cmring && n_workers > kWarps - 3) n_workers = kWarps - 3;
+  // bank, one CTA, locked commit: self-receiving workers (no receiver warp)
+  const bool selfrecv = h->kind == CSMV_KIND_BANK && w->server == CSMV_SERVER_CTA && w->atr_mode == CSMV_ATR_HASH &&
+                        w->commit == CSMV_COMMIT_CSMV && !(w->debug_flags & (CSMV_DBG_ALT_COMMIT | CSMV_DBG_RECEIVER));
+  if (selfrecv) {  // warps 0..n_workers-1 workers, warp n_workers the publisher
+    n_workers = w->server_workers ? w->server_workers : 4u;
+    if (n_workers > kWarps - 1) n_workers = kWarps - 1;
+  }
   uint32_t n_cw = w->client_warps ? w->client_warps : h->max_cw;
   if (n_cw > h->max_cw) n_cw = h->max_cw;
   if (n_cw == 0) return set_err(CSMV_EINVAL, "csmv_run: no client warps");

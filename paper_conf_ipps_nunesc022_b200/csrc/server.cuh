@@ -411,6 +411,58 @@ __device__ __forceinline__ void atr_list_validate(const KParams& p, const SrvCtx
   }
 }
 
+// bank, one CTA, ticket-locked commit: the worker warps receive for
+// themselves (no receiver warp, no dispatch queue); CSMV_DBG_RECEIVER keeps
+// the receiver for A/B runs
+__device__ __forceinline__ bool server_self_recv(const KParams& p) {
+  return p.kind == CSMV_KIND_BANK && p.n_server_ctas == 1 && p.atr_mode == CSMV_ATR_HASH &&
+         p.commit == CSMV_COMMIT_CSMV && !(p.debug & (CSMV_DBG_ALT_COMMIT | CSMV_DBG_RECEIVER));
+}
+
+// Self-receiving worker: sweep this worker's slice [lo, hi) of the client
+// doorbells with coalesced loads and claim up to m_max new requests, lowest
+// client warp first (P:103's receiver, folded into the worker).  Returns the
+// number claimed; 0 once every client has finished (or on error).  At most
+// one request per client warp is outstanding, and only this warp reads or
+// writes last_seen[lo, hi).
+template <int M>
+__device__ __forceinline__ uint32_t self_claim(const KParams& p, const SrvCtx& c, uint32_t lo, uint32_t hi,
+                                               uint32_t m_max, uint32_t (&cwv)[M], uint64_t t_begin) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t n = hi - lo, rows = (n + 31) / 32;
+  for (uint32_t idle = 1;; ++idle) {
+    uint32_t m = 0;
+    for (uint32_t r = 0; r < rows && m < m_max; ++r) {
+      const uint32_t i = r * 32 + lane;
+      const uint32_t seq = i < n ? ld_relaxed(p.req_seq + lo + i) : 0u;
+      uint32_t pm = __ballot_sync(FULL, i < n && seq != c.last_seen[lo - c.cw_lo + i]);
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        if ((uint32_t)j == m && pm && m < m_max) {
+          const uint32_t l = __ffs(pm) - 1;
+          pm &= pm - 1;
+          if (lane == l) c.last_seen[lo - c.cw_lo + i] = seq;
+          cwv[j] = lo + r * 32 + l;
+          m = j + 1;
+        }
+      }
+    }
+    if (m) {
+      fence_gpu();  // acquire: the payloads of the doorbells just seen precede our loads of them
+      return m;
+    }
+    if ((idle & 15u) == 0) {
+      uint32_t fin = 0;
+      if (lane == 0) {
+        const uint32_t er = ld_relaxed(&p.ctl->error);
+        fin = er || ld_relaxed(&p.ctl->done_warps) >= p.n_cw || watchdog(p, t_begin, 3);
+      }
+      if (__shfl_sync(FULL, fin, 0)) return 0;
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------
 // Bank worker warp.  Claims up to kMaxCombine dispatched batches (the first
 // blocking, the rest only if already queued), loads them outside the lock,
@@ -430,20 +482,29 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
   const uint32_t m_max = p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine);
   unsigned long long busy = 0, locked = 0, batches = 0, groups = 0;
   unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  const bool self = server_self_recv(p);
+  const uint32_t w = threadIdx.x >> 5, per = (c.cw_hi - c.cw_lo + p.n_workers - 1) / p.n_workers;
+  const uint32_t my_lo = min(c.cw_lo + w * per, c.cw_hi), my_hi = min(my_lo + per, c.cw_hi);
   for (;;) {
     const long long tq = clock64();
     uint32_t cwv[M];
-    if (!claim_request(c, cwv[0])) break;
-    // ---- combine: grab further requests that are already queued
     uint32_t m = 1;
+    if (self) {
+      m = self_claim<M>(p, c, my_lo, my_hi, m_max, cwv, t_begin);
+      if (!m) break;
+    } else if (!claim_request(c, cwv[0])) {
+      break;
+    }
+    // ---- combine: grab further requests that are already queued
 #pragma unroll
     for (int j = 1; j < M; ++j) {
       uint32_t got = 0xFFFFFFFFu;
-      if (m == (uint32_t)j && m < m_max && lane == 0) {
+      if (!self && m == (uint32_t)j && m < m_max && lane == 0) {
         const uint32_t h = *(volatile uint32_t*)&c.sh->q_head;
         const uint64_t e = *(volatile uint64_t*)&c.queue[h & qmask];
         if ((uint32_t)(e >> 32) == (h >> c.qn_log2) + 1 && atomicCAS(&c.sh->q_head, h, h + 1) == h) got = (uint32_t)e;
       }
+      if (self) continue;
       got = __shfl_sync(FULL, got, 0);
       cwv[j] = got;
       if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
@@ -451,7 +512,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     const long long t0 = clock64();
     // ---- load the batches: header and ids together (the receiver's fence
     // ordered them after the doorbells; ours orders them after the queue)
-    fence_cta();
+    if (!self) fence_cta();
     uint32_t sq[M], sn[M], msk[M], id0[M], id1[M];
 #pragma unroll
     for (int j = 0; j < M; ++j) {
@@ -1333,7 +1394,11 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   else __syncthreads();
   const uint32_t warp = threadIdx.x >> 5;
   const bool serving = !(ring_cl && rank == 0);
-  if (!serving && warp <= p.n_workers) {
+  if (!CL && server_self_recv(p)) {
+    // warps 0..n_workers-1 self-receiving workers, then the publisher
+    if (warp < p.n_workers) server_worker<CL>(p, c, t_begin);
+    else if (warp == p.n_workers && p.publish == CSMV_PUBLISH_SERVER) server_publisher(p, c, t_begin);
+  } else if (!serving && warp <= p.n_workers) {
     // CTA 0 of a ring cluster: no receiver, no workers
   } else if (warp == 0) {
     server_receiver(p, c, t_begin);

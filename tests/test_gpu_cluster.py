@@ -86,3 +86,16 @@ def test_commit_designs_one_client_warp_deterministic(server, flags):
     descs = oracle.bank_gen(ocfg, cfg.seed, cfg.n_tx)
     plog, pvals, prings, pst = oracle.bank_predict(ocfg, cfg.init_values(), descs, 32, max_vals=mv)
     assert np.array_equal(log, plog) and np.array_equal(rings, prings)
+
+
+@pytest.mark.parametrize("workers", [1, 3, 7])
+def test_bank_self_receiving_workers(workers):
+    """Self-receiving worker warps (the default single-CTA bank server) with
+    1, 3 and 7 workers, against the receiver-warp design (CSMV_DBG_RECEIVER)."""
+    for flags in (0, csmv.DBG_RECEIVER):
+        cfg = W.c2(n_items=1 << 14, n_tx=1 << 17, publish=1, ro_streak=8, server_workers=workers,
+                   server_combine=8, client_warps=200, debug_flags=flags)
+        rep, stats, log, rings, descs = check(cfg)
+        assert stats["server_workers"] == (workers if not flags else min(workers, 6))
+        assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions),
+                              closed_form(cfg, descs, cfg.init_values()))
