@@ -37,7 +37,12 @@ METRIC = "committed tx/sec and abort rate at 1 B200 (+partitioned 2/4/8)"
 UNIT = "tx/s"
 
 # tuned launch configuration of the C2 workload
-TUNED = dict(client_warps_per_sm=2, server_workers=7, server_combine=8, ro_streak=8, publish=1, ro_adaptive=1)
+TUNED = dict(client_warps_per_sm=2, server_workers=6, server_combine=8, ro_streak=8, publish=1, ro_adaptive=1,
+             server_recv=0)
+# per-workload overrides of the tuned launch (tools/tune.py on B200): the hot-item
+# chains of C3 want the lower-latency self-receiving server, the PUT convoys of
+# C4 longer read-only runs ahead of a blocked PUT
+TUNED_PER_CONFIG = {"C3": dict(server_recv=1, server_workers=7), "C4": dict(ro_streak=32)}
 
 # algorithmic bytes (paper VBox layout P:289): a read moves the
 # VBox head, the visited version's ts and the value (4+4+4); a write-back the
@@ -168,9 +173,10 @@ def make_cfg(args, world: int, rank: int):
     from paper_conf_ipps_nunesc022_b200 import partition, workloads
     cfg = workloads.PRESETS[args.config]()
     n_tx = args.n_tx or cfg.n_tx
-    cfg = cfg.with_(n_tx=n_tx, log_mode=0, ro_streak=TUNED["ro_streak"], publish=TUNED["publish"],
-                    server_workers=TUNED["server_workers"], server_combine=TUNED["server_combine"],
-                    ro_adaptive=TUNED["ro_adaptive"])
+    t = dict(TUNED, **TUNED_PER_CONFIG.get(args.config, {}))
+    cfg = cfg.with_(n_tx=n_tx, log_mode=0, ro_streak=t["ro_streak"], publish=t["publish"],
+                    server_workers=t["server_workers"], server_combine=t["server_combine"],
+                    ro_adaptive=t["ro_adaptive"], server_recv=t["server_recv"])
     part = partition.partition(cfg.n_items, n_tx, cfg.seed, rank, world)
     lcfg = partition.local_config(cfg, part)
     if cfg.workload.kind == 1:   # KV: the partition is a smaller cache with its own key space
@@ -333,6 +339,7 @@ def bench_ours(args):
                    "client_warps_per_gpu": n_cw, "server_workers": w.server_workers,
                    "server_combine": w.server_combine,
                    "ro_streak": w.ro_streak, "ro_adaptive": w.ro_adaptive, "publish": ["client", "server"][w.publish],
+                   "server_recv": ["receiver warp", "self-receiving workers"][w.server_recv],
                    "parallelism": "partitioned" if world > 1 else "single-gpu",
                    "multi_gpu": "independent key-range partitions, no cross-GPU transactions, NCCL stats only",
                    "l2": "flushed (512 MiB write) before every timed step"},

@@ -83,8 +83,12 @@ extern "C" {
                                    commits through the commit ring and one committer warp instead of the
                                    ticket-locked critical section, the cluster server the other way
                                    round; A/B only */
-#define CSMV_DBG_RECEIVER 64u  /* bank, single-CTA locked commit: keep the receiver warp and dispatch
-                                  queue instead of self-receiving worker warps; A/B only */
+
+#define CSMV_RECV_WARP 0u       /* a receiver warp sweeps the doorbells into a shared-memory dispatch
+                                   queue; combining fills larger batches */
+#define CSMV_RECV_SELF 1u       /* bank, single-CTA locked commit: every worker warp sweeps its own
+                                   slice of the doorbells (no receiver warp, one more worker, no queue);
+                                   lower latency -- helps hot-item chains (C3); other servers ignore it */
 
 typedef struct csmv_workload {
     uint32_t kind;             /* CSMV_KIND_* */
@@ -115,6 +119,7 @@ typedef struct csmv_workload {
     uint32_t ro_adaptive;      /* 1: a lane stops its read-only run (at most ro_streak) as soon as the
                                   server has answered the warp's batch -- rounds track the server
                                   round trip (timing-dependent schedule; 0 = fixed, deterministic) */
+    uint32_t server_recv;      /* CSMV_RECV_*: how the server's worker warps get requests */
 } csmv_workload;
 
 /* ---- statistics ---- */

@@ -23,7 +23,8 @@ SERVER_CTA, SERVER_CLUSTER = 0, 1
 PUBLISH_CLIENT, PUBLISH_SERVER = 0, 1
 ATR_HASH, ATR_LIST, ATR_LIST_NOCV = 0, 1, 2
 COMMIT_CSMV, COMMIT_ONLYCS, COMMIT_JVSTM = 0, 1, 2
-DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER, DBG_PHASES, DBG_KV_ITEMSETS, DBG_ALT_COMMIT, DBG_RECEIVER = 1, 2, 4, 8, 16, 32, 64
+DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER, DBG_PHASES, DBG_KV_ITEMSETS, DBG_ALT_COMMIT = 1, 2, 4, 8, 16, 32
+RECV_WARP, RECV_SELF = 0, 1
 CLIENT_PHASES = ("read", "preval", "submit", "rot", "wait_server", "writeback", "publish", "divergence")
 ABORT_REASONS = ("preval", "conflict", "early", "overflow", "version")
 
@@ -42,7 +43,7 @@ class _Workload(C.Structure):
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
         "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers", "server_combine",
         "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms", "commit",
-        "ro_adaptive")]
+        "ro_adaptive", "server_recv")]
 
 
 class _Stats(C.Structure):
@@ -87,6 +88,7 @@ class Workload:
     watchdog_ms: int = 0
     commit: int = COMMIT_CSMV
     ro_adaptive: int = 0
+    server_recv: int = 0
 
     def to_c(self) -> _Workload:
         return _Workload(*[getattr(self, f.name) for f in fields(self)])

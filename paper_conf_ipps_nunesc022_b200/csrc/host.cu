@@ -409,8 +409,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
                       ((w->server == CSMV_SERVER_CLUSTER) != ((w->debug_flags & CSMV_DBG_ALT_COMMIT) != 0));
   if (cmring && n_workers > kWarps - 3) n_workers = kWarps - 3;
   // bank, one CTA, locked commit: self-receiving workers (no receiver warp)
-  const bool selfrecv = h->kind == CSMV_KIND_BANK && w->server == CSMV_SERVER_CTA && w->atr_mode == CSMV_ATR_HASH &&
-                        w->commit == CSMV_COMMIT_CSMV && !(w->debug_flags & (CSMV_DBG_ALT_COMMIT | CSMV_DBG_RECEIVER));
+  if (w->server_recv > CSMV_RECV_SELF) return set_err(CSMV_EINVAL, "csmv_run: unknown server_recv %u", w->server_recv);
+  const bool selfrecv = w->server_recv == CSMV_RECV_SELF && h->kind == CSMV_KIND_BANK && w->server == CSMV_SERVER_CTA &&
+                        w->atr_mode == CSMV_ATR_HASH && w->commit == CSMV_COMMIT_CSMV &&
+                        !(w->debug_flags & CSMV_DBG_ALT_COMMIT);
   if (selfrecv) {  // warps 0..n_workers-1 workers, warp n_workers the publisher
     n_workers = w->server_workers ? w->server_workers : 4u;
     if (n_workers > kWarps - 1) n_workers = kWarps - 1;
@@ -517,6 +519,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.debug = w->debug_flags;
   p.commit = w->commit;
   p.ro_adaptive = w->ro_adaptive;
+  p.server_recv = w->server_recv;
   p.req_vals = h->d_req_vals;
   p.jv_ws = h->d_jv_ws;
   p.jv_tag = h->d_jv_tag;

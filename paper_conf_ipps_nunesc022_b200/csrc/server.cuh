@@ -411,12 +411,11 @@ __device__ __forceinline__ void atr_list_validate(const KParams& p, const SrvCtx
   }
 }
 
-// bank, one CTA, ticket-locked commit: the worker warps receive for
-// themselves (no receiver warp, no dispatch queue); CSMV_DBG_RECEIVER keeps
-// the receiver for A/B runs
+// CSMV_RECV_SELF (bank, one CTA, ticket-locked commit): the worker warps
+// receive for themselves -- no receiver warp, no dispatch queue
 __device__ __forceinline__ bool server_self_recv(const KParams& p) {
-  return p.kind == CSMV_KIND_BANK && p.n_server_ctas == 1 && p.atr_mode == CSMV_ATR_HASH &&
-         p.commit == CSMV_COMMIT_CSMV && !(p.debug & (CSMV_DBG_ALT_COMMIT | CSMV_DBG_RECEIVER));
+  return p.server_recv == CSMV_RECV_SELF && p.kind == CSMV_KIND_BANK && p.n_server_ctas == 1 &&
+         p.atr_mode == CSMV_ATR_HASH && p.commit == CSMV_COMMIT_CSMV && !(p.debug & CSMV_DBG_ALT_COMMIT);
 }
 
 // Self-receiving worker: sweep this worker's slice [lo, hi) of the client
@@ -472,7 +471,7 @@ __device__ __forceinline__ uint32_t self_claim(const KParams& p, const SrvCtx& c
 // consecutive CTS range.  A batch is validated by the whole warp,
 // one lane per transaction, __ballot_sync for the commit mask.
 // ---------------------------------------------------------------------------
-template <bool CL>
+template <bool CL, bool SELF>
 __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
   constexpr int M = kMaxCombine;
   const uint32_t FULL = 0xFFFFFFFFu;
@@ -482,18 +481,22 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
   const uint32_t m_max = p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine);
   unsigned long long busy = 0, locked = 0, batches = 0, groups = 0;
   unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-  const bool self = server_self_recv(p);
-  const uint32_t w = threadIdx.x >> 5, per = (c.cw_hi - c.cw_lo + p.n_workers - 1) / p.n_workers;
-  const uint32_t my_lo = min(c.cw_lo + w * per, c.cw_hi), my_hi = min(my_lo + per, c.cw_hi);
+  constexpr bool self = SELF;
+  uint32_t my_lo = 0, my_hi = 0;
+  if constexpr (SELF) {
+    const uint32_t w = threadIdx.x >> 5, per = (c.cw_hi - c.cw_lo + p.n_workers - 1) / p.n_workers;
+    my_lo = min(c.cw_lo + w * per, c.cw_hi);
+    my_hi = min(my_lo + per, c.cw_hi);
+  }
   for (;;) {
     const long long tq = clock64();
     uint32_t cwv[M];
     uint32_t m = 1;
-    if (self) {
+    if constexpr (SELF) {
       m = self_claim<M>(p, c, my_lo, my_hi, m_max, cwv, t_begin);
       if (!m) break;
-    } else if (!claim_request(c, cwv[0])) {
-      break;
+    } else {
+      if (!claim_request(c, cwv[0])) break;
     }
     // ---- combine: grab further requests that are already queued
 #pragma unroll
@@ -1396,7 +1399,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   const bool serving = !(ring_cl && rank == 0);
   if (!CL && server_self_recv(p)) {
     // warps 0..n_workers-1 self-receiving workers, then the publisher
-    if (warp < p.n_workers) server_worker<CL>(p, c, t_begin);
+    if (warp < p.n_workers) server_worker<CL, !CL>(p, c, t_begin);
     else if (warp == p.n_workers && p.publish == CSMV_PUBLISH_SERVER) server_publisher(p, c, t_begin);
   } else if (!serving && warp <= p.n_workers) {
     // CTA 0 of a ring cluster: no receiver, no workers
@@ -1409,7 +1412,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     }
     else if (!CL && p.commit == CSMV_COMMIT_ONLYCS) server_worker_onlycs<NS>(p, c, t_begin);
     else if (cmring) server_worker_cm<CL>(p, c, t_begin);
-    else server_worker<CL>(p, c, t_begin);
+    else server_worker<CL, false>(p, c, t_begin);
   } else if (warp == p.n_workers + 1 && rank == 0 && p.publish == CSMV_PUBLISH_SERVER) {
     server_publisher(p, c, t_begin);
   } else if (warp == kWarps - 1 && rank == 0 && cmring) {

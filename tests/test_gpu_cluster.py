@@ -90,12 +90,25 @@ def test_commit_designs_one_client_warp_deterministic(server, flags):
 
 @pytest.mark.parametrize("workers", [1, 3, 7])
 def test_bank_self_receiving_workers(workers):
-    """Self-receiving worker warps (the default single-CTA bank server) with
-    1, 3 and 7 workers, against the receiver-warp design (CSMV_DBG_RECEIVER)."""
-    for flags in (0, csmv.DBG_RECEIVER):
+    """Self-receiving worker warps (CSMV_RECV_SELF) with 1, 3 and 7 workers,
+    and the receiver-warp design on the same workload."""
+    for recv in (csmv.RECV_SELF, csmv.RECV_WARP):
         cfg = W.c2(n_items=1 << 14, n_tx=1 << 17, publish=1, ro_streak=8, server_workers=workers,
-                   server_combine=8, client_warps=200, debug_flags=flags)
+                   server_combine=8, client_warps=200, server_recv=recv)
         rep, stats, log, rings, descs = check(cfg)
-        assert stats["server_workers"] == (workers if not flags else min(workers, 6))
+        assert stats["server_workers"] == (workers if recv == csmv.RECV_SELF else min(workers, 6))
         assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions),
                               closed_form(cfg, descs, cfg.init_values()))
+
+
+def test_self_receiving_one_warp_deterministic_and_c3():
+    """P7 and a contended C3 run through the self-receiving server."""
+    cfg = W.c1(client_warps=1, n_tx=2000, ro_streak=4, server_recv=csmv.RECV_SELF)
+    from tests.test_gpu_parity import run_gpu, oracle_cfg
+    stats, log, (vals, mv), rings = run_gpu(cfg)
+    ocfg = oracle_cfg(cfg)
+    descs = oracle.bank_gen(ocfg, cfg.seed, cfg.n_tx)
+    plog, pvals, prings, pst = oracle.bank_predict(ocfg, cfg.init_values(), descs, 32, max_vals=mv)
+    assert np.array_equal(log, plog) and np.array_equal(rings, prings)
+    check(W.c3(n_tx=1 << 17, client_warps=128, ro_streak=8, server_combine=8, server_workers=7,
+               server_recv=csmv.RECV_SELF, publish=1, ro_adaptive=1))
