@@ -278,6 +278,13 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         if (p.commit != CSMV_COMMIT_ONLYCS) {
           write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
           write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
+          // lastw (the item-indexed ATR's exact level, server.cuh): written
+          // here, before this commit is published, so GTS = g implies lastw
+          // of every commit <= g.  Two commits writing one item are ordered
+          // (the later one's snapshot covers the earlier one), so plain
+          // stores leave lastw at the latest.
+          st_relaxed(p.lastw + d.src, cts);
+          st_relaxed(p.lastw + d.dst, cts);
         }
         if (p.log_mode) {
           log_commit(p, cu, s, cts, att_u, dig1(d.src, vs) + dig1(d.dst, vd), dig1(d.src, ns) + dig1(d.dst, nd));

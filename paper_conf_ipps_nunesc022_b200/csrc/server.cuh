@@ -29,8 +29,7 @@ struct SrvShared {
   uint32_t ring_head;    // commit ring: next slot a worker claims            [CTA 0]
   uint32_t ring_done;    // commit ring: slots the committer has finished     [CTA 0]
   uint32_t workers_left; // commit ring: worker warps still running          [CTA 0]
-  uint32_t lw_done;      // locked bank worker: lastw written for every CTS <= lw_done [CTA 0]
-  uint32_t pad[6];
+  uint32_t pad[7];
 };
 static_assert(sizeof(SrvShared) == 64, "control block is 64 B (server_smem_bytes)");
 
@@ -535,9 +534,9 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       if (!mine[j]) id0[j] = id1[j] = 0;
     }
     const bool hash = p.atr_mode == CSMV_ATR_HASH;
-    // lastw covers every CTS <= e_pre (HASH: lastw is written after the
-    // critical section and lw_done advanced in CTS order, below)
-    const uint32_t e_pre = hash ? *(volatile uint32_t*)&c.sh0->lw_done : *(volatile uint32_t*)&c.sh0->tail;
+    // lastw covers every CTS <= e_pre: clients write lastw with their
+    // write-back, before the commit is published, so e_pre = GTS (acquire)
+    const uint32_t e_pre = hash ? ld_acquire(p.gts) : *(volatile uint32_t*)&c.sh0->tail;
     srv_fence<CL>();
     const bool novalid = (p.debug & CSMV_DBG_NO_VALIDATE) != 0;
     // HASH: the exact part of the validation (lastw, every CTS <= e_pre) and
@@ -571,13 +570,13 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     const long long t1 = clock64();
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
     uint32_t t = t0c;
-    uint32_t cm[M], om[M], base[M], cts_of[M];
+    uint32_t cm[M], om[M], base[M];
     if (hash) {
       // batch j: a write after e_pre to one of its items raised all of that
       // item's slots above e_pre (earlier batches of this section included)
 #pragma unroll
       for (int j = 0; j < M; ++j) {
-        cm[j] = om[j] = cts_of[j] = 0;
+        cm[j] = om[j] = 0;
         base[j] = t + 1;
         if (j < (int)m) {
           uint32_t va[kFiltK] = {0u, 0u, 0u}, vb[kFiltK] = {0u, 0u, 0u};
@@ -599,7 +598,6 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
           const bool commit = chk[j] && !ovf;
           cm[j] = __ballot_sync(FULL, commit);
           om[j] = __ballot_sync(FULL, ovf);
-          cts_of[j] = t + 1 + __popc(cm[j] & lt);
           t += __popc(cm[j]);
           if (commit) {
 #pragma unroll
@@ -634,26 +632,6 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) done_ring_room(p, c, t, t_begin);
     cs_leave<CL>(c, ticket, t);
     const long long t2 = clock64();
-    if (hash && t != t0c) {
-      // lastw for this group's commits, outside the lock; then lw_done moves
-      // from t0c to t once every earlier group has published (CTS order),
-      // so a worker that reads lw_done = e sees lastw of every CTS <= e
-#pragma unroll
-      for (int j = 0; j < M; ++j) {
-        if (j < (int)m && ((cm[j] >> lane) & 1u)) {
-          p.lastw[id0[j]] = cts_of[j];
-          p.lastw[id1[j]] = cts_of[j];
-        }
-      }
-      if (lane == 0) {
-        uint32_t it = 0;
-        while (*(volatile uint32_t*)&c.sh0->lw_done != t0c)
-          if ((++it & 1023u) == 0 && watchdog(p, t_begin, 10)) break;
-      }
-      __syncwarp();
-      srv_fence<CL>();
-      if (lane == 0) *(volatile uint32_t*)&c.sh0->lw_done = t;
-    }
     // ---- respond: round-tagged words, no fence (kernel.cuh Resp)
     if (lane < (uint32_t)m) {
 #pragma unroll
@@ -775,7 +753,7 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
     }
     // lastw prefetched only now: the window the filter must cover is then
     // the ring's depth, not the wait for room as well
-    const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
+    const uint32_t e_pre = ld_acquire(p.gts);  // lastw covers every CTS <= GTS (client write-back)
     srv_fence<CL>();
     uint32_t chkm[M];
 #pragma unroll
@@ -859,7 +837,6 @@ __device__ __forceinline__ bool cm_try(CmSlot* sl, uint32_t seq, CmPayload& q) {
 template <bool CL>
 __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring, uint64_t t_begin) {
   constexpr uint32_t R = 1u << kCmRingLog2;
-  constexpr uint32_t kTailEvery = CL ? 32u : 4u;  // the cluster fence is a gpu-scope MEMBAR
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t lt = lanemask_lt();
@@ -867,7 +844,6 @@ __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring
   const bool srv_pub = p.publish == CSMV_PUBLISH_SERVER;
   const uint32_t fbase = c.rt32;  // the filter (this CTA's rt stripe); slots arrive as byte offsets
   uint32_t t = *(volatile uint32_t*)&c.sh->tail;
-  uint32_t tpub = t;
   uint32_t gseen = t;
   unsigned long long cs = 0, wait = 0;
   CmPayload q;
@@ -878,12 +854,6 @@ __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring
     for (uint32_t it = 0; !have;) {
       have = cm_try<CL>(ring + (next & (R - 1)), next, q);
       if (have) break;
-      // idle: publish the tail now (a later e_pre only widens the filter's window)
-      if (t != tpub) {
-        srv_fence<CL>();
-        if (lane == 0) *(volatile uint32_t*)&c.sh->tail = t;
-        tpub = t;
-      }
       uint32_t done = 0;
       if (lane == 0 && *(volatile uint32_t*)&c.sh->workers_left == 0 &&
           *(volatile uint32_t*)&c.sh->ring_head == next)
@@ -913,7 +883,6 @@ __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring
     const bool commit = chk && !ovf;
     const uint32_t cm = __ballot_sync(FULL, commit), om = __ballot_sync(FULL, ovf);
     const uint32_t base = t + 1;
-    const uint32_t cts = base + __popc(cm & lt);
     t += __popc(cm);
     if (srv_pub && t > gseen + dmask) {  // done-ring back-pressure: CTS t may reuse slot t & mask once GTS >= t - 2^20
       for (uint32_t it = 0; t > gseen + dmask;) {
@@ -928,8 +897,6 @@ __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring
       filt_st<false>(fbase + cur.w0.w, t);
       filt_st<false>(fbase + cur.w1.x, t);
       filt_st<false>(fbase + cur.w1.y, t);
-      p.lastw[cur.w1.z] = cts;
-      p.lastw[cur.w1.w] = cts;
     }
     if (lane == 0) {  // respond: round-tagged words, no fence (kernel.cuh Resp); slot release
       const uint64_t tag = (uint64_t)cur.round << 32;
@@ -937,14 +904,8 @@ __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring
       st_relaxed64(&p.resp[cur.cw].ovf, tag | om);
       *(volatile uint32_t*)&c.sh->ring_done = next + 1;
     }
+    if (lane == 0) *(volatile uint32_t*)&c.sh->tail = t;  // the CTS counter (read at exit)
     __syncwarp();  // this batch's filter stores precede the next batch's loads
-    // tail (the e_pre workers prefetch lastw under) needs a fence ordering the
-    // lastw stores before it: every kTailEvery batches under load, else when idle
-    if (((next + 1) & (kTailEvery - 1)) == 0 && t != tpub) {
-      srv_fence<CL>();
-      if (lane == 0) *(volatile uint32_t*)&c.sh->tail = t;
-      tpub = t;
-    }
     const long long t2 = clock64();
     wait += (unsigned long long)(t1 - tw);
     cs += (unsigned long long)(t2 - t1);
@@ -1391,7 +1352,6 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     c.sh->ring_head = 0;
     c.sh->ring_done = 0;
     c.sh->workers_left = p.n_workers * nserve;
-    c.sh->lw_done = g0;
   }
   if constexpr (CL) cg::this_cluster().sync();
   else __syncthreads();
