@@ -240,6 +240,42 @@ __device__ __forceinline__ void filt_st(uint32_t a, uint32_t v) {
   else asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
 
+// The bank filter keeps 16-bit slots (twice the slots in the same shared
+// memory, so far fewer false positives): slot i holds the low 16 bits of the
+// last CTS stored into it, and slots are written in CTS order (by the
+// critical-section holder / the committer).  With tail t and a window
+// W = t - e_pre < 2^16, a slot written at c in (e_pre, t] has age
+// (t - v) mod 2^16 = t - c < W; an older slot may alias into the window
+// (probability ~W / 2^16), which is only a false positive.  So
+//    unknown(x)  iff  W >= 2^16  or  max_k age(F[h_k(x)]) < W
+// never misses a write of x after e_pre.
+__device__ __forceinline__ uint32_t filt16_age(uint32_t t, uint32_t v) { return (t - v) & 0xFFFFu; }
+
+template <bool CL>
+__device__ __forceinline__ uint32_t filt16_addr(const SrvCtx& c, uint32_t i) {
+  if constexpr (!CL) {
+    return c.rt32 + 2u * i;
+  } else {
+    const uint32_t owner = i & ((1u << c.clog2) - 1), local = c.rt32 + 2u * (i >> c.clog2);
+    uint32_t a;
+    asm("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(a) : "r"(local), "r"(owner));
+    return a;
+  }
+}
+template <bool CL>
+__device__ __forceinline__ uint32_t filt16_ld(uint32_t a) {
+  uint16_t v;
+  if constexpr (CL) asm volatile("ld.shared::cluster.u16 %0, [%1];" : "=h"(v) : "r"(a) : "memory");
+  else asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a) : "memory");
+  return v;
+}
+template <bool CL>
+__device__ __forceinline__ void filt16_st(uint32_t a, uint32_t v) {
+  const uint16_t h = (uint16_t)v;
+  if constexpr (CL) asm volatile("st.shared::cluster.u16 [%0], %1;" ::"r"(a), "h"(h) : "memory");
+  else asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"(h) : "memory");
+}
+
 // ---------------------------------------------------------------------------
 // Receiver warp: sweeps its slice of the client doorbells with
 // coalesced loads and dispatches new requests to this CTA's workers through
@@ -544,7 +580,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     bool chk[M];
     uint32_t fa[M][kFiltK], fb[M][kFiltK];
     uint32_t xor_all = e_pre;
-    const uint32_t fl2 = p.rt_log2 + 3;
+    const uint32_t fl2 = p.rt_log2 + 4;  // 16-bit filter slots
 #pragma unroll
     for (int j = 0; j < M; ++j) {
       uint32_t lw0 = 0, lw1 = 0;
@@ -555,12 +591,11 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       chk[j] = mine[j] && (novalid || (lw0 <= sn[j] && lw1 <= sn[j]));
 #pragma unroll
       for (int k = 0; k < kFiltK; ++k) {
-        fa[j][k] = filt_addr<CL>(c, filt_slot(id0[j], k, fl2));
-        fb[j][k] = filt_addr<CL>(c, filt_slot(id1[j], k, fl2));
+        fa[j][k] = filt16_addr<CL>(c, filt_slot(id0[j], k, fl2));
+        fb[j][k] = filt16_addr<CL>(c, filt_slot(id1[j], k, fl2));
       }
       xor_all ^= lw0 ^ lw1 ^ sn[j];
     }
-    const uint32_t e_chk = novalid ? 0xFFFFFFFFu : e_pre;
     // The payload must have arrived before the lock is taken: a warp vote on
     // values derived from it makes the loads complete here.
     if (__ballot_sync(FULL, xor_all == 0x12345679u) == FULL) __nanosleep(1);
@@ -583,18 +618,18 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
           if (chk[j]) {
 #pragma unroll
             for (int k = 0; k < kBankFiltK; ++k) {
-              va[k] = filt_ld<CL>(fa[j][k]);
-              vb[k] = filt_ld<CL>(fb[j][k]);
+              va[k] = filt16_ld<CL>(fa[j][k]);
+              vb[k] = filt16_ld<CL>(fb[j][k]);
             }
           }
-          uint32_t la = va[0], lb = vb[0];
+          uint32_t aa = filt16_age(t, va[0]), ab = filt16_age(t, vb[0]);
 #pragma unroll
           for (int k = 1; k < kBankFiltK; ++k) {
-            la = min(la, va[k]);
-            lb = min(lb, vb[k]);
+            aa = max(aa, filt16_age(t, va[k]));
+            ab = max(ab, filt16_age(t, vb[k]));
           }
-          const uint32_t lo = max(la, lb);
-          const bool ovf = chk[j] && lo > e_chk;
+          const uint32_t win = t - e_pre;  // commits the exact lastw check did not cover
+          const bool ovf = chk[j] && !novalid && (win > 0xFFFFu || min(aa, ab) < win);
           const bool commit = chk[j] && !ovf;
           cm[j] = __ballot_sync(FULL, commit);
           om[j] = __ballot_sync(FULL, ovf);
@@ -602,8 +637,8 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
           if (commit) {
 #pragma unroll
             for (int k = 0; k < kBankFiltK; ++k) {  // the batch's last CTS: equal values, race-free
-              filt_st<CL>(fa[j][k], t);
-              filt_st<CL>(fb[j][k], t);
+              filt16_st<CL>(fa[j][k], t);
+              filt16_st<CL>(fb[j][k], t);
             }
           }
           __syncwarp();  // batch j's records precede batch j+1's probes
@@ -697,7 +732,7 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t qmask = (1u << c.qn_log2) - 1;
   const uint32_t m_max = p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine);
-  const uint32_t fl2 = p.rt_log2 - p.clog2 + 3;  // the filter: CTA 0's stripe, 8 << local_log2 slots
+  const uint32_t fl2 = p.rt_log2 - p.clog2 + 3;  // the filter: CTA 0's stripe, 8 << local_log2 32-bit slots
   const bool novalid = (p.debug & CSMV_DBG_NO_VALIDATE) != 0;
   unsigned long long busy = 0, batches = 0, groups = 0, ph0 = 0, ph1 = 0, ph4 = 0;
   for (;;) {
@@ -878,6 +913,8 @@ __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring
     have = cm_try<CL>(ring + ((next + 1) & (R - 1)), next + 1, q);
     // a write after e_pre to one of the items raised all of its slots above
     // e_pre (every earlier batch of the ring included)
+    // (32-bit slots here: the committer's chain is the cluster server's bound,
+    // and the 16-bit age test costs more than its fewer false positives gain)
     const uint32_t lo = max(min(v0, min(v1, v2)), min(v3, min(v4, v5)));
     const bool ovf = chk && lo > cur.e_chk;
     const bool commit = chk && !ovf;
