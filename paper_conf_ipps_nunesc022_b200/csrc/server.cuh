@@ -202,6 +202,7 @@ constexpr int kFiltK = 3;
 #define CSMV_BANK_FILT_K 3
 #endif
 constexpr int kBankFiltK = CSMV_BANK_FILT_K;  // hashes the locked bank worker uses (<= kFiltK)
+static_assert(kBankFiltK >= 1 && kBankFiltK <= kFiltK, "CSMV_BANK_FILT_K must be 1..kFiltK");
 
 // KV requests in the compact {set clock} u WS form use the filter
 __device__ __forceinline__ bool kv_filter_mode(const KParams& p) {

@@ -244,3 +244,16 @@ def test_ragged_read_only_scans(ro_reads, k):
     cfg = W.c2(n_items=1 << 12, n_tx=1 << 15, ro_reads=ro_reads, n_versions=k, log_mode=csmv.LOG_FULL,
                client_warps=64, ro_streak=8, p_update_ppm=300_000)
     check(cfg)
+
+
+@pytest.mark.parametrize("publish", [0, 1])
+def test_filter16_wraps(publish):
+    """The 16-bit filter slots (server.cuh) wrap several times: > 4 x 2^16
+    commits through the smallest filter (2K slots, so slots alias often) on a
+    contended store.  Aliasing may only add OVERFLOW aborts -- a missed
+    conflict would be a history the oracle rejects."""
+    cfg = W.c2(n_items=1 << 12, n_tx=1 << 19, p_update_ppm=700_000, atr_capacity=16, server_combine=8,
+               server_workers=6, client_warps=256, publish=publish, ro_streak=8, ro_adaptive=1)
+    rep, stats, *_ = check(cfg)
+    assert stats["gts_final"] - stats["gts_start"] > 4 * 65536
+    assert stats["aborts"]["overflow"]["update"] > 0
