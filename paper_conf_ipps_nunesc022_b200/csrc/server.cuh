@@ -365,25 +365,45 @@ __device__ __forceinline__ bool claim_request(const SrvCtx& c, uint32_t& cw) {
 }
 
 // Ticket lock around the commit critical section, in CTA 0's shared memory.
+// One CTA: acquire = ld.acquire.cta of now_serving (a plain LDS), release =
+// st.release.cta (one MEMBAR.CTA) -- no fences beyond that.  Cluster: the
+// DSMEM words with cluster-scope fences.
 template <bool CL>
 __device__ __forceinline__ uint32_t cs_enter(const SrvCtx& c) {
   uint32_t ticket = 0;
   if ((threadIdx.x & 31) == 0) ticket = atomicAdd(&c.sh0->next_ticket, 1u);
   ticket = __shfl_sync(0xFFFFFFFFu, ticket, 0);
-  while (*(volatile uint32_t*)&c.sh0->now_serving != ticket) __nanosleep(16);
-  __syncwarp();
-  srv_fence<CL>();
+  if constexpr (CL) {
+    while (*(volatile uint32_t*)&c.sh0->now_serving != ticket) __nanosleep(16);
+    __syncwarp();
+    srv_fence<CL>();
+  } else {
+    const uint32_t a = (uint32_t)__cvta_generic_to_shared(&c.sh0->now_serving);
+    for (;;) {
+      uint32_t v;
+      asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+      if (v == ticket) break;
+      __nanosleep(16);
+    }
+    __syncwarp();
+  }
   return ticket;
 }
 
 template <bool CL>
 __device__ __forceinline__ void cs_leave(const SrvCtx& c, uint32_t ticket, uint32_t new_tail) {
   __syncwarp();
-  srv_fence<CL>();
-  if ((threadIdx.x & 31) == 0) {
-    *(volatile uint32_t*)&c.sh0->tail = new_tail;
+  if constexpr (CL) {
     srv_fence<CL>();
-    *(volatile uint32_t*)&c.sh0->now_serving = ticket + 1;
+    if ((threadIdx.x & 31) == 0) {
+      *(volatile uint32_t*)&c.sh0->tail = new_tail;
+      srv_fence<CL>();
+      *(volatile uint32_t*)&c.sh0->now_serving = ticket + 1;
+    }
+  } else if ((threadIdx.x & 31) == 0) {
+    *(volatile uint32_t*)&c.sh0->tail = new_tail;
+    const uint32_t a = (uint32_t)__cvta_generic_to_shared(&c.sh0->now_serving);
+    asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" ::"r"(a), "r"(ticket + 1) : "memory");
   }
 }
 
@@ -607,12 +627,14 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     const uint32_t t0c = *(volatile uint32_t*)&c.sh0->tail;
     uint32_t t = t0c;
     uint32_t cm[M], om[M], base[M];
+    bool ovfl[M];
     if (hash) {
       // batch j: a write after e_pre to one of its items raised all of that
       // item's slots above e_pre (earlier batches of this section included)
 #pragma unroll
       for (int j = 0; j < M; ++j) {
         cm[j] = om[j] = 0;
+        ovfl[j] = false;
         base[j] = t + 1;
         if (j < (int)m) {
           uint32_t va[kFiltK] = {0u, 0u, 0u}, vb[kFiltK] = {0u, 0u, 0u};
@@ -623,17 +645,18 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
               vb[k] = filt16_ld<CL>(fb[j][k]);
             }
           }
-          uint32_t aa = filt16_age(t, va[0]), ab = filt16_age(t, vb[0]);
-#pragma unroll
-          for (int k = 1; k < kBankFiltK; ++k) {
-            aa = max(aa, filt16_age(t, va[k]));
-            ab = max(ab, filt16_age(t, vb[k]));
-          }
+          // slot v is recent iff its CTS lies in (e_pre, t]: (v - e_pre - 1) mod 2^16 < t - e_pre
           const uint32_t win = t - e_pre;  // commits the exact lastw check did not cover
-          const bool ovf = chk[j] && !novalid && (win > 0xFFFFu || min(aa, ab) < win);
+          bool ra = true, rb = true;
+#pragma unroll
+          for (int k = 0; k < kBankFiltK; ++k) {
+            ra = ra && ((va[k] - e_pre - 1u) & 0xFFFFu) < win;
+            rb = rb && ((vb[k] - e_pre - 1u) & 0xFFFFu) < win;
+          }
+          const bool ovf = chk[j] && !novalid && (win > 0xFFFFu || ra || rb);
           const bool commit = chk[j] && !ovf;
           cm[j] = __ballot_sync(FULL, commit);
-          om[j] = __ballot_sync(FULL, ovf);
+          ovfl[j] = ovf;  // the overflow mask is voted after the lock
           t += __popc(cm[j]);
           if (commit) {
 #pragma unroll
@@ -668,6 +691,10 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) done_ring_room(p, c, t, t_begin);
     cs_leave<CL>(c, ticket, t);
     const long long t2 = clock64();
+    if (hash) {
+#pragma unroll
+      for (int j = 0; j < M; ++j) om[j] = __ballot_sync(FULL, ovfl[j]);
+    }
     // ---- respond: round-tagged words, no fence (kernel.cuh Resp)
     if (lane < (uint32_t)m) {
 #pragma unroll
