@@ -71,6 +71,7 @@ struct csmv {
   bool loaded = false;
   // bank store
   uint64_t* d_rings = nullptr;
+  int32_t* d_init = nullptr;  // csmv_load staging (allocated once: no pool growth inside a timed load)
   // KV store
   uint32_t kv_S = 0, kv_A = 0, kv_T = 0, kv_keys = 0;
   uint64_t *d_key = nullptr, *d_val = nullptr, *d_lru = nullptr, *d_clk = nullptr;
@@ -108,7 +109,7 @@ struct csmv {
 static void free_all(csmv* h) {
   void* ps[] = {h->d_rings, h->d_key, h->d_val, h->d_lru, h->d_clk, h->d_lastw, h->d_gts, h->d_ctl,
                 h->d_stats, h->d_done, h->d_req_seq, h->d_req_hdr, h->d_req_ids, h->d_req_cnt,
-                h->d_resp, h->d_log, h->d_vals, h->d_zipf, h->d_req_vals, h->d_jv_ws, h->d_jv_tag};
+                h->d_resp, h->d_log, h->d_vals, h->d_zipf, h->d_req_vals, h->d_jv_ws, h->d_jv_tag, h->d_init};
   for (void* q : ps) cudaFree(q);
   if (h->ev0) cudaEventDestroy(h->ev0);
   if (h->ev1) cudaEventDestroy(h->ev1);
@@ -182,6 +183,7 @@ csmv_t* csmv_create(uint64_t n_items, uint32_t n_versions) {
   h->sm_count = sms;
   h->maxid = 2;
   if (cudaMalloc(&h->d_rings, n_items * h->nslot * sizeof(uint64_t)) != cudaSuccess) return create_fail(h, "rings");
+  if (cudaMalloc(&h->d_init, n_items * sizeof(int32_t)) != cudaSuccess) return create_fail(h, "init staging");
   if (!alloc_common(h)) return create_fail(h, "control buffers");
   if (cudaMalloc(&h->d_req_vals, (size_t)h->max_cw * 64 * sizeof(uint32_t)) != cudaSuccess)
     return create_fail(h, "request values");
@@ -237,14 +239,12 @@ int csmv_load(csmv_t* h, const int32_t* init, uint64_t n) {
   if (n != h->n_items)
     return set_err(CSMV_EINVAL, "csmv_load: n=%llu != n_items=%llu", (unsigned long long)n,
                    (unsigned long long)h->n_items);
-  int32_t* d_init = nullptr;
-  CK(cudaMallocAsync((void**)&d_init, n * sizeof(int32_t), h->stream));
+  int32_t* d_init = h->d_init;
   CK(cudaMemcpyAsync(d_init, init, n * sizeof(int32_t), cudaMemcpyHostToDevice, h->stream));
   CK(launch_init_rings(h->d_rings, h->nslot, d_init, n, h->d_gts, h->stream));
   CK(cudaMemsetAsync(h->d_lastw, 0, n * sizeof(uint32_t), h->stream));
   // CTS restart at 1: stale done flags of an earlier run would publish GTS early
   CK(cudaMemsetAsync(h->d_done, 0, sizeof(uint32_t) << kDoneLog2, h->stream));
-  CK(cudaFreeAsync(d_init, h->stream));
   CK(cudaStreamSynchronize(h->stream));
   h->loaded = true;
   return CSMV_OK;
