@@ -293,7 +293,8 @@ def bench_ours(args):
     kmean = sum(kern_ns) / len(kern_ns)
     achieved = algo / (kmean * 1e-9) / 1e9
     peak, peak_kind = peaks()
-    traffic = traffic_per_launch()
+    # the committed capture is of the C2 bench step: other workloads have none
+    traffic = traffic_per_launch() if args.config == "C2" and world == 1 else None
     last = steps[-1][2]
     # serial commit chain: batches/s against the critical section's own bound
     cs_cycles = last["server_phase_cycles"]["critical"] / max(1, last["batches"])
