@@ -67,6 +67,19 @@ def peaks():
     return 6650.0, "fallback"
 
 
+def serial_chain(batches_per_s, cs_cycles, upd_per_batch, clocks):
+    """The commit critical section is one serial chain on the server SM: its
+    own roofline is one batch per `cs_cycles` at the SM clock; `frac` is the
+    share of that bound the run reached (how busy the chain was)."""
+    d = {"batches_per_s": batches_per_s, "critical_section_cycles_per_batch": cs_cycles,
+         "updates_per_batch": upd_per_batch}
+    mhz = clocks.get("sm_mhz") or clocks.get("sm_max_mhz")
+    if mhz and cs_cycles > 0:
+        bound = mhz * 1e6 / cs_cycles
+        d.update({"bound_batches_per_s": bound, "frac": batches_per_s / bound})
+    return d
+
+
 def traffic_per_launch():
     """dram bytes per launch of csmv_fused from the committed ncu capture."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
@@ -109,6 +122,12 @@ class Clocks:
                 self.proc.kill()
 
     def summary(self):
+        if getattr(self, "_summary", None) is not None:
+            return self._summary
+        self._summary = self._read()
+        return self._summary
+
+    def _read(self):
         if not self.path or not os.path.exists(self.path):
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         sm, smax, reasons = [], None, set()
@@ -348,9 +367,8 @@ def bench_ours(args):
                      "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                      "kernel": "csmv_fused", "algorithmic_bytes_per_launch": algo,
                      "note": "latency/serialisation-bound: see serial_chain"},
-        "serial_chain": {"batches_per_s": red["batches"] / (total_ms_max * 1e-3),
-                         "critical_section_cycles_per_batch": cs_cycles,
-                         "updates_per_batch": red["committed_update"] / max(1, red["batches"])},
+        "serial_chain": serial_chain(red["batches"] / (total_ms_max * 1e-3), cs_cycles,
+                                     red["committed_update"] / max(1, red["batches"]), clk.summary()),
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(init.nbytes),
                 "d2h_bytes_per_step": 400, "steps": e2e_steps,
                 "load_ms_per_step": 1e3 * t_load / e2e_steps, "wall_ms_per_step": 1e3 * e2e_s / e2e_steps},
