@@ -86,6 +86,8 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
   if (cw >= p.n_cw) return;
   const uint64_t T = (uint64_t)p.n_cw * 32;
   uint64_t cu = kNoTx;                       // pending update
+  uint64_t du_id = kNoTx;                    // cu's descriptor, drawn once (not every retry round)
+  BankTx du{};
   uint64_t cr = (uint64_t)cw * 32 + lane;    // read cursor
   uint32_t att_u = 0, att_r = 0, hold = 0, n_srv_ab = 0;
   ClientCounters cc;
@@ -123,7 +125,11 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         --hold;
         status = ST_ABORT;  // sitting out (backoff)
       } else {
-        d = gen_bank(p.gen, cu);
+        if (du_id != cu) {
+          du = gen_bank(p.gen, cu);
+          du_id = cu;
+        }
+        d = du;
         ++att_u;
         rs = ld_ring<NS>(p.rings + (size_t)d.src * NS);
         rd = ld_ring<NS>(p.rings + (size_t)d.dst * NS);
@@ -232,10 +238,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
       for (uint32_t n_ro = 0; n_ro < lim; ++n_ro) {
         BankTx r{};
         bool has = false;
-        if (run && cr < p.n_tx) {
-          r = gen_bank(p.gen, cr);
-          has = !r.is_update;
-        }
+        if (run && cr < p.n_tx) has = gen_bank_ro(p.gen, cr, r.start, r.len);
         const uint32_t act = __ballot_sync(FULL, has);
         if (!act) break;
         if (has) ++att_r;

@@ -72,6 +72,8 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
   if (cw >= p.n_cw) return;
   const uint64_t T = (uint64_t)p.n_cw * 32;
   uint64_t cu = kNoTx;
+  uint64_t dk_id = kNoTx;  // cu whose key dk_key holds
+  uint32_t dk_key = 0;
   uint64_t cr = (uint64_t)cw * 32 + lane;
   uint32_t att_u = 0, att_r = 0, hold = 0, n_srv_ab = 0;
   ClientCounters cc;
@@ -115,7 +117,11 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         --hold;
         status = ST_ABORT;
       } else {
-        d = gen_kv(p.gen, cu);
+        if (dk_id != cu) {  // the pending PUT's key, drawn once (not every retry round)
+          dk_key = gen_kv_key(p.gen, cu);
+          dk_id = cu;
+        }
+        d = gen_kv_k(p.gen, cu, dk_key);
         kv_key16(d.key, kk);
         tset = kv_set(d.key, Tn);
         ++att_u;
@@ -289,9 +295,9 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     if (streak || cu == kNoTx) {
       uint32_t n_ro = 0;
       while (cr < p.n_tx) {
-        const KvTx g = gen_kv(p.gen, cr);
-        if (g.is_update) break;
+        if (gen_kv_is_update(p.gen, cr)) break;  // before the key draw: the next round adopts it
         if (streak ? n_ro >= streak : n_ro >= 1) break;
+        const KvTx g = gen_kv(p.gen, cr);
         ++att_r;
         ++n_ro;
         uint64_t dg;

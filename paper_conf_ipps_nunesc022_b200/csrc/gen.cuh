@@ -77,6 +77,20 @@ __device__ __forceinline__ BankTx gen_bank(const GenParams& g, uint64_t tx) {
   return d;
 }
 
+// the read-only fields of transaction tx without the update's endpoint
+// draws (zipf picks are a binary search): false if tx is an update
+__device__ __forceinline__ bool gen_bank_ro(const GenParams& g, uint64_t tx, uint32_t& start, uint32_t& len) {
+  start = len = 0;
+  if (gen_is_update(g, tx)) return false;
+  if (g.ro_reads == 0) {
+    len = g.n_items;
+  } else {
+    start = (uint32_t)uniform(draw(g.seed, tx, 1), g.n_items);
+    len = g.ro_reads;
+  }
+  return true;
+}
+
 // digest contribution of one 4-byte item (docs/GENERATOR.md section 5)
 __device__ __forceinline__ uint64_t dig1(uint32_t item, uint32_t val) {
   return mix64(((uint64_t)item << 32) ^ (uint64_t)val);

@@ -272,12 +272,19 @@ int csmv_load_kv(csmv_t* h, uint64_t n_keys) {
   if (n_keys == 0 || n_keys >= (1ull << 32)) return set_err(CSMV_EINVAL, "csmv_load_kv: bad n_keys");
   const uint32_t S = h->kv_S, A = h->kv_A, T = h->kv_T;
   std::vector<uint32_t> keys((size_t)S * 4, 0), vals((size_t)S * 8, 0), lru(S, 0), clocks(T, 0);
-  // PUT semantics per key, in key order (docs/GENERATOR.md 4)
+  // PUT semantics per key, in key order (docs/GENERATOR.md 4).  The preload
+  // keys are pairwise distinct (a = mix64(k) is a bijection of k), so while
+  // no key is all-zero (an all-zero key would read as an empty way) a set's
+  // c-th insertion lands in way (c-1) mod A: the first A fill the empty ways
+  // in order, every later one evicts the way with the smallest LRU clock,
+  // i.e. the oldest insertion.  That O(1) form is used when it applies.
+  bool fifo = true;
+  for (uint64_t k = 0; k < n_keys && fifo; ++k) fifo = mix64(k) != 0 || mix64(k ^ 0x5555555555555555ull) != 0;
   for (uint64_t k = 0; k < n_keys; ++k) {
     const uint64_t a = mix64(k), b = mix64(k ^ 0x5555555555555555ull);
     const uint32_t kk[4] = {(uint32_t)a, (uint32_t)(a >> 32), (uint32_t)b, (uint32_t)(b >> 32)};
     const uint32_t t = (uint32_t)umulhi(mix64(k ^ 0xA5A5A5A5A5A5A5A5ull), T);
-    uint32_t victim = UINT32_MAX;
+    uint32_t victim = fifo ? t * A + clocks[t] % A : UINT32_MAX;
     for (uint32_t w = 0; w < A && victim == UINT32_MAX; ++w) {
       const uint32_t* q = &keys[((size_t)t * A + w) * 4];
       if ((q[0] == kk[0] && q[1] == kk[1] && q[2] == kk[2] && q[3] == kk[3]) || !(q[0] | q[1] | q[2] | q[3]))

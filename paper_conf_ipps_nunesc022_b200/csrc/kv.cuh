@@ -36,10 +36,17 @@ struct KvTx {
   uint32_t val[8];
 };
 
-__device__ __forceinline__ KvTx gen_kv(const GenParams& g, uint64_t tx) {
+__device__ __forceinline__ bool gen_kv_is_update(const GenParams& g, uint64_t tx) {
+  return (draw(g.seed, tx, 0) >> 32) < g.upd_thresh;
+}
+__device__ __forceinline__ uint32_t gen_kv_key(const GenParams& g, uint64_t tx) {
+  return gen_pick(g, draw(g.seed, tx, 1));  // a zipf pick is a binary search over the key CDF
+}
+// transaction tx with its key already drawn (gen_kv_key)
+__device__ __forceinline__ KvTx gen_kv_k(const GenParams& g, uint64_t tx, uint32_t key) {
   KvTx d;
-  d.is_update = (draw(g.seed, tx, 0) >> 32) < g.upd_thresh;
-  d.key = gen_pick(g, draw(g.seed, tx, 1));
+  d.is_update = gen_kv_is_update(g, tx);
+  d.key = key;
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
     const uint64_t v = d.is_update ? draw(g.seed, tx, 4 + j) : 0ull;
@@ -48,6 +55,7 @@ __device__ __forceinline__ KvTx gen_kv(const GenParams& g, uint64_t tx) {
   }
   return d;
 }
+__device__ __forceinline__ KvTx gen_kv(const GenParams& g, uint64_t tx) { return gen_kv_k(g, tx, gen_kv_key(g, tx)); }
 
 __device__ __forceinline__ uint64_t dig_word(uint32_t item, uint32_t w, uint32_t word) {
   return mix64(((uint64_t)item << 35) ^ ((uint64_t)w << 32) ^ (uint64_t)word);

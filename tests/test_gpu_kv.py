@@ -36,9 +36,13 @@ def run(cfg):
     return pre, stats, log, fin
 
 
-@pytest.mark.parametrize("S,A", [(1 << 12, 16), (1 << 10, 4)])
-def test_preload_parity(S, A):
-    cfg = W.c4(n_items=S, kv_ways=A, n_tx=0)
+@pytest.mark.parametrize("S,A,keys", [(1 << 12, 16, 0), (1 << 10, 4, 0), (1 << 12, 16, 3 << 12),
+                                      (1 << 12, 16, 1000), (1 << 10, 1, 0), (1 << 12, 256, 5 << 12)])
+def test_preload_parity(S, A, keys):
+    """The library's preload (O(1) per key: a set's c-th insertion takes way
+    (c-1) mod A) against the oracle's literal PUT-by-PUT preload, with fewer,
+    as many and more keys than slots."""
+    cfg = W.c4(n_items=S, kv_ways=A, n_tx=0, **({"kv_keys": keys} if keys else {}))
     pre, *_ = run(cfg)
     ref = oracle.kv_preload(ocfg_of(cfg))
     for a, b in zip(pre, (ref.keys, ref.vals, ref.lru, ref.clocks)):
