@@ -602,10 +602,24 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     uint32_t fa[M][kFiltK], fb[M][kFiltK];
     uint32_t xor_all = e_pre;
     const uint32_t fl2 = p.rt_log2 + 4;  // 16-bit filter slots
+    // Self-receiving workers (latency-bound hot-item chains, C3): all 2M
+    // lastw loads in one L2 round trip (idle lanes read lastw[0]).  With a
+    // receiver (C2) they stay one round trip per batch: that latency is the
+    // window in which further batches queue up to be combined
+    // (profiles/r01/ab_late.md).
+    uint32_t lwa[M], lwb[M];
 #pragma unroll
     for (int j = 0; j < M; ++j) {
-      uint32_t lw0 = 0, lw1 = 0;
-      if (mine[j] && hash) {
+      lwa[j] = lwb[j] = 0;
+      if (SELF && hash) {
+        lwa[j] = ld_relaxed(p.lastw + id0[j]);
+        lwb[j] = ld_relaxed(p.lastw + id1[j]);
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < M; ++j) {
+      uint32_t lw0 = lwa[j], lw1 = lwb[j];
+      if (!SELF && mine[j] && hash) {
         lw0 = ld_relaxed(p.lastw + id0[j]);
         lw1 = ld_relaxed(p.lastw + id1[j]);
       }
