@@ -185,7 +185,12 @@ csmv_t *csmv_create_kv(uint64_t n_slots, uint32_t ways, uint32_t n_versions);
 int csmv_load(csmv_t *h, const int32_t *init_values, uint64_t n);
 
 /* KV: preload keys 0..n_keys-1 with PUT semantics (docs/GENERATOR.md
- * section 4) as version ts = 0 and reset GTS to 0. */
+ * section 4) as version ts = 0 and reset GTS to 0.  Computed on the device
+ * (count keys per set, bucket them, keep each set's A largest keys: a set's
+ * r-th insertion takes way r mod A) in a device staging buffer of about
+ * (13*S + 4*T + n_keys) * 4 bytes that the handle keeps for later loads
+ * (grown when n_keys grows, freed by csmv_destroy).  EINVAL if n_keys is 0 or
+ * >= 2^32; ECUDA on an allocation or launch failure. */
 int csmv_load_kv(csmv_t *h, uint64_t n_keys);
 
 /* Run on the given CUDA stream (a cudaStream_t, e.g. torch's current

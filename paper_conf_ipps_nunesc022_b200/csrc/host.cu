@@ -3,8 +3,8 @@
 // Every transaction step runs in the fused kernel (kernel.cu); the host only
 // allocates, initialises, launches and copies results.  Nothing here falls
 // back to the CPU: without an sm_100a device csmv_create fails.  The one
-// host-side computation is the KV preload (setup, not timed): keys
-// 0..n_keys-1 inserted serially with PUT semantics (docs/GENERATOR.md 4).
+// host-side computation is the zipf CDF (setup); the KV preload runs on the
+// device (launch_kv_preload).
 #include <cuda_runtime.h>
 
 #include <cmath>
@@ -74,6 +74,8 @@ struct csmv {
   int32_t* d_init = nullptr;  // csmv_load staging (allocated once: no pool growth inside a timed load)
   // KV store
   uint32_t kv_S = 0, kv_A = 0, kv_T = 0, kv_keys = 0;
+  uint32_t* d_kvstage = nullptr;  // csmv_load_kv staging + scratch (kept: no allocation inside a timed load)
+  size_t kvstage_bytes = 0;
   uint64_t *d_key = nullptr, *d_val = nullptr, *d_lru = nullptr, *d_clk = nullptr;
   // shared
   uint32_t* d_lastw = nullptr;
@@ -109,7 +111,8 @@ struct csmv {
 static void free_all(csmv* h) {
   void* ps[] = {h->d_rings, h->d_key, h->d_val, h->d_lru, h->d_clk, h->d_lastw, h->d_gts, h->d_ctl,
                 h->d_stats, h->d_done, h->d_req_seq, h->d_req_hdr, h->d_req_ids, h->d_req_cnt,
-                h->d_resp, h->d_log, h->d_vals, h->d_zipf, h->d_req_vals, h->d_jv_ws, h->d_jv_tag, h->d_init};
+                h->d_resp, h->d_log, h->d_vals, h->d_zipf, h->d_req_vals, h->d_jv_ws, h->d_jv_tag, h->d_init,
+                h->d_kvstage};
   for (void* q : ps) cudaFree(q);
   if (h->ev0) cudaEventDestroy(h->ev0);
   if (h->ev1) cudaEventDestroy(h->ev1);
@@ -271,54 +274,35 @@ int csmv_load_kv(csmv_t* h, uint64_t n_keys) {
   if (h->kind != CSMV_KIND_KV) return set_err(CSMV_EINVAL, "csmv_load_kv: not a KV store");
   if (n_keys == 0 || n_keys >= (1ull << 32)) return set_err(CSMV_EINVAL, "csmv_load_kv: bad n_keys");
   const uint32_t S = h->kv_S, A = h->kv_A, T = h->kv_T;
-  std::vector<uint32_t> keys((size_t)S * 4, 0), vals((size_t)S * 8, 0), lru(S, 0), clocks(T, 0);
-  // PUT semantics per key, in key order (docs/GENERATOR.md 4).  The preload
-  // keys are pairwise distinct (a = mix64(k) is a bijection of k), so while
-  // no key is all-zero (an all-zero key would read as an empty way) a set's
-  // c-th insertion lands in way (c-1) mod A: the first A fill the empty ways
-  // in order, every later one evicts the way with the smallest LRU clock,
-  // i.e. the oldest insertion.  That O(1) form is used when it applies.
-  bool fifo = true;
-  for (uint64_t k = 0; k < n_keys && fifo; ++k) fifo = mix64(k) != 0 || mix64(k ^ 0x5555555555555555ull) != 0;
-  for (uint64_t k = 0; k < n_keys; ++k) {
-    const uint64_t a = mix64(k), b = mix64(k ^ 0x5555555555555555ull);
-    const uint32_t kk[4] = {(uint32_t)a, (uint32_t)(a >> 32), (uint32_t)b, (uint32_t)(b >> 32)};
-    const uint32_t t = (uint32_t)umulhi(mix64(k ^ 0xA5A5A5A5A5A5A5A5ull), T);
-    uint32_t victim = fifo ? t * A + clocks[t] % A : UINT32_MAX;
-    for (uint32_t w = 0; w < A && victim == UINT32_MAX; ++w) {
-      const uint32_t* q = &keys[((size_t)t * A + w) * 4];
-      if ((q[0] == kk[0] && q[1] == kk[1] && q[2] == kk[2] && q[3] == kk[3]) || !(q[0] | q[1] | q[2] | q[3]))
-        victim = t * A + w;
-    }
-    if (victim == UINT32_MAX) {
-      victim = t * A;
-      for (uint32_t w = 1; w < A; ++w)
-        if (lru[t * A + w] < lru[victim]) victim = t * A + w;
-    }
-    const uint32_t c = clocks[t] + 1;
-    memcpy(&keys[(size_t)victim * 4], kk, 16);
-    for (uint32_t j = 0; j < 4; ++j) {
-      const uint64_t x = mix64(((k << 2) | j) ^ 0x3C3C3C3C3C3C3C3Cull);
-      vals[(size_t)victim * 8 + 2 * j] = (uint32_t)x;
-      vals[(size_t)victim * 8 + 2 * j + 1] = (uint32_t)(x >> 32);
-    }
-    lru[victim] = c;
-    clocks[t] = c;
-  }
+  // PUT semantics per key, in key order (docs/GENERATOR.md 4), computed on
+  // the device: a set's r-th insertion takes way r mod A (launch_kv_preload).
   uint32_t* d = nullptr;
   const size_t words = (size_t)S * 13 + T;
-  CK(cudaMalloc(&d, words * 4));
-  cudaError_t e = cudaMemcpy(d, keys.data(), (size_t)S * 16, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(d + (size_t)S * 4, vals.data(), (size_t)S * 32, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(d + (size_t)S * 12, lru.data(), (size_t)S * 4, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(d + (size_t)S * 13, clocks.data(), (size_t)T * 4, cudaMemcpyHostToDevice);
+  const size_t scratch_words = 3 * (size_t)T + n_keys;
+  size_t cub_bytes = 0;
+  cudaError_t e = launch_kv_preload((uint32_t)n_keys, T, A, nullptr, nullptr, &cub_bytes, nullptr, nullptr, nullptr,
+                                    nullptr, h->stream);
+  if (e != cudaSuccess) return set_err(CSMV_ECUDA, "csmv_load_kv: %s", cudaGetErrorString(e));
+  const size_t need = (words + scratch_words) * 4 + cub_bytes;
+  if (h->kvstage_bytes < need) {
+    cudaFree(h->d_kvstage);
+    h->d_kvstage = nullptr;
+    h->kvstage_bytes = 0;
+    CK(cudaMalloc(&h->d_kvstage, need));
+    h->kvstage_bytes = need;
+  }
+  d = h->d_kvstage;
+  uint32_t* scratch = d + words;
+  e = cudaMemsetAsync(d, 0, words * 4, h->stream);
+  if (e == cudaSuccess)
+    e = launch_kv_preload((uint32_t)n_keys, T, A, scratch, scratch + scratch_words, &cub_bytes, d,
+                          d + (size_t)S * 4, d + (size_t)S * 12, d + (size_t)S * 13, h->stream);
   if (e == cudaSuccess)
     e = launch_init_kv(kv_params(h), h->nslot, d, d + (size_t)S * 4, d + (size_t)S * 12, d + (size_t)S * 13,
                        h->stream);
   if (e == cudaSuccess) e = cudaMemsetAsync(h->d_lastw, 0, h->n_items * 4, h->stream);
   if (e == cudaSuccess) e = cudaMemsetAsync(h->d_done, 0, sizeof(uint32_t) << kDoneLog2, h->stream);
   if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
-  cudaFree(d);
   if (e != cudaSuccess) return set_err(CSMV_ECUDA, "csmv_load_kv: %s", cudaGetErrorString(e));
   h->kv_keys = (uint32_t)n_keys;
   h->loaded = true;

@@ -27,6 +27,8 @@
 // the commit path.
 #include <cuda_runtime.h>
 
+#include <cub/device/device_scan.cuh>
+
 #include "kernel.cuh"
 #include "ptx.cuh"
 
@@ -489,7 +491,7 @@ cudaError_t fused_capacity(const KParams& p, uint32_t nslot, size_t smem, int* c
 
 cudaError_t launch_init_kv(const KParams& p, uint32_t nslot, const uint32_t* keys, const uint32_t* vals,
                            const uint32_t* lru, const uint32_t* clocks, cudaStream_t st) {
-  const uint32_t blocks = (uint32_t)((p.kv_S + 255) / 256);
+  const uint32_t blocks = 148 * 8;
   switch (nslot) {
     case 2: init_kv_rings<2><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
     case 4: init_kv_rings<4><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
@@ -497,6 +499,24 @@ cudaError_t launch_init_kv(const KParams& p, uint32_t nslot, const uint32_t* key
     case 16: init_kv_rings<16><<<blocks, 256, 0, st>>>(p, keys, vals, lru, clocks); break;
     default: return cudaErrorInvalidValue;
   }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_kv_preload(uint32_t n_keys, uint32_t T, uint32_t A, uint32_t* scratch, void* cub_tmp,
+                              size_t* cub_bytes, uint32_t* keys, uint32_t* vals, uint32_t* lru, uint32_t* clocks,
+                              cudaStream_t st) {
+  uint32_t *cnt = scratch, *off = scratch + T, *fill = scratch + 2 * (size_t)T, *bucket = scratch + 3 * (size_t)T;
+  if (!cub_tmp) return cub::DeviceScan::ExclusiveSum(nullptr, *cub_bytes, cnt, off, (int)T, st);
+  if (A == 0 || A > kMaxWays) return cudaErrorInvalidValue;
+  cudaError_t e = cudaMemsetAsync(cnt, 0, (size_t)T * 4, st);
+  if (e == cudaSuccess) e = cudaMemsetAsync(fill, 0, (size_t)T * 4, st);
+  if (e != cudaSuccess) return e;
+  const uint32_t grid = 148 * 8;
+  kv_preload_count<<<grid, 256, 0, st>>>(n_keys, T, cnt);
+  e = cub::DeviceScan::ExclusiveSum(cub_tmp, *cub_bytes, cnt, off, (int)T, st);
+  if (e != cudaSuccess) return e;
+  kv_preload_scatter<<<grid, 256, 0, st>>>(n_keys, T, off, fill, bucket);
+  kv_preload_place<<<(T + 127) / 128, 128, 0, st>>>(T, A, off, cnt, bucket, keys, vals, lru, clocks);
   return cudaGetLastError();
 }
 

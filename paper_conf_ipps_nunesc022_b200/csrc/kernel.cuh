@@ -172,6 +172,13 @@ cudaError_t launch_gen_descs(GenParams g, uint64_t tx0, uint64_t n, uint32_t* ou
 cudaError_t fused_capacity(const KParams& p, uint32_t nslot, size_t smem, int* ctas);
 cudaError_t launch_init_kv(const KParams& p, uint32_t nslot, const uint32_t* keys, const uint32_t* vals,
                            const uint32_t* lru, const uint32_t* clocks, cudaStream_t st);
+// Device preload of keys 0..n_keys-1 (kv_kernels.cuh) into the plain-word
+// layout launch_init_kv installs (keys/vals/lru/clocks zeroed by the
+// caller).  scratch: 3*T + n_keys words.  With cub_tmp == nullptr only sets
+// *cub_bytes (the scan's temporary storage size).
+cudaError_t launch_kv_preload(uint32_t n_keys, uint32_t T, uint32_t A, uint32_t* scratch, void* cub_tmp,
+                              size_t* cub_bytes, uint32_t* keys, uint32_t* vals, uint32_t* lru, uint32_t* clocks,
+                              cudaStream_t st);
 cudaError_t launch_kv_newest(const KParams& p, uint32_t nslot, uint32_t* keys, uint32_t* vals, uint32_t* lru,
                              uint32_t* clocks, cudaStream_t st);
 cudaError_t launch_gen_kv_descs(GenParams g, uint64_t tx0, uint64_t n, uint32_t* out, cudaStream_t st);

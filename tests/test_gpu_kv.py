@@ -37,11 +37,13 @@ def run(cfg):
 
 
 @pytest.mark.parametrize("S,A,keys", [(1 << 12, 16, 0), (1 << 10, 4, 0), (1 << 12, 16, 3 << 12),
-                                      (1 << 12, 16, 1000), (1 << 10, 1, 0), (1 << 12, 256, 5 << 12)])
+                                      (1 << 12, 16, 1000), (1 << 10, 1, 0), (1 << 12, 256, 5 << 12),
+                                      (256, 256, 3000), (1 << 22, 16, 0), (1 << 22, 16, 3 << 21)])
 def test_preload_parity(S, A, keys):
-    """The library's preload (O(1) per key: a set's c-th insertion takes way
-    (c-1) mod A) against the oracle's literal PUT-by-PUT preload, with fewer,
-    as many and more keys than slots."""
+    """The library's device preload (count, bucket, keep each set's A largest
+    keys: a set's r-th insertion takes way r mod A) against the oracle's
+    literal PUT-by-PUT preload, with fewer, as many and more keys than slots,
+    one set (T = 1) and C4's full 4M slots."""
     cfg = W.c4(n_items=S, kv_ways=A, n_tx=0, **({"kv_keys": keys} if keys else {}))
     pre, *_ = run(cfg)
     ref = oracle.kv_preload(ocfg_of(cfg))
