@@ -322,7 +322,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
             if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 2);
             if (__shfl_sync(FULL, bad, 0)) break;
           }
-          __nanosleep(32);
+          __nanosleep(CSMV_SLEEP_PUB);
         }
         if (lane == 0) st_release(p.gts, base + n - 1);  // release also orders the write-backs
       } else if (cts && p.commit != CSMV_COMMIT_ONLYCS) {

@@ -132,7 +132,7 @@ __device__ __forceinline__ bool wait_response(const KParams& p, uint32_t cw, uin
       if ((threadIdx.x & 31) == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);
       if (__shfl_sync(FULL, bad, 0)) return false;
     }
-    __nanosleep(64);
+    __nanosleep(CSMV_SLEEP_RESP);
   }
   base = (uint32_t)b;
   cmask = (uint32_t)c;

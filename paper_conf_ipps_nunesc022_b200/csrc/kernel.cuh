@@ -23,6 +23,19 @@
 #include "../../include/csmv.h"
 #include "gen.cuh"
 
+// back-off (ns) of three spin waits: a client warp polling its response, the
+// client GTS publish chain, a server worker polling its dispatch queue
+// (build-time knobs for A/B: CSMV_NVCC_EXTRA="-DCSMV_SLEEP_RESP=..")
+#ifndef CSMV_SLEEP_RESP
+#define CSMV_SLEEP_RESP 64
+#endif
+#ifndef CSMV_SLEEP_PUB
+#define CSMV_SLEEP_PUB 32
+#endif
+#ifndef CSMV_SLEEP_QUEUE
+#define CSMV_SLEEP_QUEUE 64
+#endif
+
 namespace csmvd {
 
 constexpr uint32_t kEmptyTs = 0xFFFFFFFFu;

@@ -360,7 +360,7 @@ __device__ __forceinline__ bool claim_request(const SrvCtx& c, uint32_t& cw) {
       return true;
     }
     if (*(volatile uint32_t*)&c.sh->exit) return false;
-    __nanosleep(64);
+    __nanosleep(CSMV_SLEEP_QUEUE);
   }
 }
 
