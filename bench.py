@@ -5,18 +5,28 @@ configs[1] = C2: bank, 1M accounts, K=4 versions, full-GPU client grid, 50%
 update, uniform access, read-only = 64-read scans.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                  [--config C2|C3|C4|C1]
 
 A step is one csmv_run over n_tx = 2^24 freshly generated transactions
 (every one commits exactly once; aborted attempts are retried inside the
 step).  The store and GTS persist across steps.  L2 is flushed (a 512 MiB
-write) before every timed step.  N > 1 runs one process per GPU under
-torchrun as independent key-range-partitioned instances (no cross-GPU
-transactions; NCCL only reduces statistics), scaling "weak"-ish: the job's
-n_tx and accounts are split across ranks.
+write) before every timed step.
+
+--gpus N > 1 runs one process per GPU (torchrun; bench.py spawns it itself
+when started without one) as independent key-range-partitioned instances:
+rank g runs the full per-GPU workload on its own key range of an N x larger
+job (weak scaling), its own server and GTS, no cross-GPU transactions; NCCL
+only reduces the statistics.
 
 --impl reference times the CPU oracle (the deterministic 1-warp schedule of
 oracle/, single-threaded C) on bounded samples of the same workload: the
 tier's reference arm is the oracle, there is no GPU reference to install.
+
+Roofs: the measured L2 / cross-SM / shared-atomic roofs of
+tools/ubench/roofs.cu and the critical-section chain floor of
+tools/ubench/filt16_ubench.cu are read from profiles/roofs_b200.json; the
+per-launch DRAM / L2 bytes and shared atomics from profiles/ncu_summary.json
+(tools/ncu_extract.py over the committed ncu captures).
 """
 from __future__ import annotations
 
@@ -61,36 +71,59 @@ def algorithmic_bytes(stats: dict, ro_reads: int, n_items: int) -> float:
     return stats["committed_update"] * BYTES_TRANSFER + stats["committed_ro"] * BYTES_READ * L
 
 
-def peaks():
-    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
-    if os.path.exists(p):
-        with open(p) as f:
-            d = json.load(f)
-        return float(d["hbm_gbs"]), "measured"
-    return 6650.0, "fallback"
+def _load_json(*parts):
+    p = os.path.join(ROOT, *parts)
+    if not os.path.exists(p):
+        return {}
+    with open(p) as f:
+        return json.load(f)
 
 
-def serial_chain(batches_per_s, cs_cycles, upd_per_batch, clocks):
-    """The commit critical section is one serial chain on the server SM: its
-    own roofline is one batch per `cs_cycles` at the SM clock; `frac` is the
-    share of that bound the run reached (how busy the chain was)."""
+def hbm_peak():
+    d = _load_json("MEASURED_PEAKS.json")
+    if "hbm_gbs" in d:
+        return float(d["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs (copy bandwidth, driver-measured)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def roofs():
+    """Measured roofs of this B200 (tools/ubench/roofs.cu, filt16_ubench.cu)."""
+    return _load_json("profiles", "roofs_b200.json")
+
+
+def ncu_entry(config: str):
+    """Per-launch counters of csmv_fused for this config's bench step."""
+    return _load_json("profiles", "ncu_summary.json").get(config.lower(), {})
+
+
+def serial_chain(batches_per_s, cs_cycles, upd_per_batch, clocks, floor_cycles):
+    """The commit critical section is one serial chain on the server SM.  Its
+    floor is the same chain (filter loads -> recency test -> ballot -> CTS ->
+    filter stores) timed alone on an idle SM (filt16_ubench): one batch per
+    `floor_cycles` at the SM clock.  `frac` = batches/s reached / that bound;
+    `occupancy` = the chain's measured cycles per batch over the floor."""
     d = {"batches_per_s": batches_per_s, "critical_section_cycles_per_batch": cs_cycles,
-         "updates_per_batch": upd_per_batch}
+         "updates_per_batch": upd_per_batch,
+         "critical_section_cycles_per_update": cs_cycles / upd_per_batch if upd_per_batch else None}
     mhz = clocks.get("sm_mhz") or clocks.get("sm_max_mhz")
-    if mhz and cs_cycles > 0:
-        bound = mhz * 1e6 / cs_cycles
-        d.update({"bound_batches_per_s": bound, "frac": batches_per_s / bound})
+    if mhz and floor_cycles:
+        bound = mhz * 1e6 / floor_cycles
+        d.update({"floor_cycles_per_batch": floor_cycles, "floor_source": "profiles/roofs_b200.json cs_floor_cycles",
+                  "bound_batches_per_s": bound, "frac": batches_per_s / bound,
+                  "updates_bound_per_s": bound * upd_per_batch})
     return d
 
 
-def traffic_per_launch():
-    """dram bytes per launch of csmv_fused from the committed ncu capture."""
-    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
-    if not os.path.exists(p):
-        return None
-    with open(p) as f:
-        d = json.load(f)
-    return d.get("c2_bench", {}).get("dram_bytes_per_launch")
+def cpu_info():
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
 
 
 class Clocks:
@@ -192,6 +225,9 @@ def oracle_sample_rate(cfg, budget_s: float, chunk: int, tx_start: int = 0):
 
 
 def make_cfg(args, world: int, rank: int):
+    """The preset with the tuned launch; for world > 1 this rank's weak
+    partition: the full per-GPU workload on key range [rank*N, (rank+1)*N)
+    of the job, seed mix64(seed ^ rank) (partition.py)."""
     from paper_conf_ipps_nunesc022_b200 import partition, workloads
     cfg = workloads.PRESETS[args.config]()
     n_tx = args.n_tx or cfg.n_tx
@@ -199,11 +235,8 @@ def make_cfg(args, world: int, rank: int):
     cfg = cfg.with_(n_tx=n_tx, log_mode=0, ro_streak=t["ro_streak"], publish=t["publish"],
                     server_workers=t["server_workers"], server_combine=t["server_combine"],
                     ro_adaptive=t["ro_adaptive"], server_recv=t["server_recv"])
-    part = partition.partition(cfg.n_items, n_tx, cfg.seed, rank, world)
+    part = partition.partition(cfg.n_items, n_tx, cfg.seed, rank, world, mode="weak")
     lcfg = partition.local_config(cfg, part)
-    if cfg.workload.kind == 1:   # KV: the partition is a smaller cache with its own key space
-        lcfg = lcfg.with_(kv_keys=lcfg.n_items - lcfg.n_items % cfg.workload.kv_ways,
-                          n_items=lcfg.n_items - lcfg.n_items % cfg.workload.kv_ways)
     return cfg, lcfg, part
 
 
@@ -237,10 +270,70 @@ def bench_reference(args):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
             "data": "synthetic", "config": {"workload": DESCR.get(cfg.name, cfg.name), "n_items": cfg.n_items,
                                             "n_versions": cfg.n_versions, "sample": sample},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                             **cpu_info()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
+
+
+def roofline_block(args, cfg, lcfg, steps, kern_ns, is_kv, world):
+    """Roofline of the dominant (only) kernel csmv_fused against the roof
+    that binds its configuration (SURVEY 8(d) rooflines 1-3):
+      C2 / C3 (store L2-resident): L2 bandwidth -- algorithmic bytes per
+        launch / launch time against the measured L2 read roof;
+      C4 (store 1.7 GB, HBM-resident): HBM bandwidth against MEASURED_PEAKS;
+    plus the sector-granular L2 traffic and the server SM's shared-memory
+    atomics from the committed ncu capture of the same bench step."""
+    w = lcfg.workload
+    algo = sum(kv_bytes(s, w.kv_ways) if is_kv else algorithmic_bytes(s, w.ro_reads, lcfg.n_items)
+               for _, _, s in steps) / len(steps)
+    kmean_s = sum(kern_ns) / len(kern_ns) * 1e-9
+    achieved = algo / kmean_s / 1e9
+    rf = roofs()
+    nc = ncu_entry(args.config) if world == 1 else {}
+    store_bytes = steps[-1][2]["store_bytes"]
+    l2_resident = store_bytes < 64 << 20
+    if l2_resident and rf.get("l2_read_gbs"):
+        bound, peak = "l2", rf["l2_read_gbs"]
+        peak_src = "profiles/roofs_b200.json l2_read_gbs (tools/ubench/roofs.cu, all SMs, 256-bit loads, L2-resident)"
+    else:
+        bound = "hbm"
+        peak, peak_src = hbm_peak()
+    out = {"bound": bound, "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+           "traffic": nc.get("dram_bytes_per_launch"), "peak_source": peak_src, "kernel": "csmv_fused",
+           "algorithmic_bytes_per_launch": algo, "kernel_ms": kmean_s * 1e3,
+           "store_bytes": store_bytes}
+    if nc:
+        out["ncu"] = {k: nc[k] for k in ("capture", "n_tx_per_launch", "duration_ms", "dram_bytes_per_launch",
+                                          "l2_bytes_per_launch", "shared_atomics_per_launch") if k in nc}
+        scale = lcfg.n_tx / nc.get("n_tx_per_launch", lcfg.n_tx)
+        if nc.get("l2_bytes_per_launch"):
+            l2b = nc["l2_bytes_per_launch"] * scale
+            out["l2_traffic"] = {"bytes_per_launch": l2b, "achieved_gbs": l2b / kmean_s / 1e9,
+                                 "peak_gbs": rf.get("l2_read_gbs"),
+                                 "frac": (l2b / kmean_s / 1e9) / rf["l2_read_gbs"] if rf.get("l2_read_gbs") else None,
+                                 "x_algorithmic": l2b / algo if algo else None}
+        if nc.get("shared_atomics_per_launch") and rf.get("smem_atom_per_s_sm"):
+            a = nc["shared_atomics_per_launch"] * scale / kmean_s
+            out["server_smem_atomics"] = {"per_s": a, "peak_per_s_one_sm": rf["smem_atom_per_s_sm"],
+                                          "frac": a / rf["smem_atom_per_s_sm"],
+                                          "note": "all shared atomics of the launch (server dispatch-queue claims,"
+                                                  " lock tickets) against one SM's measured atomic throughput"}
+    return out
+
+
+def spawn_ranks(args):
+    """--gpus N > 1 without a launcher: re-run this command under torchrun
+    (one process per GPU, 127.0.0.1 rendezvous); rank 0 prints the line."""
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
 
 
 def bench_ours(args):
@@ -253,6 +346,9 @@ def bench_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        sys.stderr.write(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}\n")
+        return 2
     if world > 1:
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
@@ -308,17 +404,8 @@ def bench_ours(args):
     red = partition.reduce_stats(agg, device=dev if world > 1 else None)
     total_ms_max = red["elapsed_ns"] / 1e6
     value = red["committed"] / (total_ms_max * 1e-3)
-
-    # roofline of the dominant (only) kernel, csmv_fused
-    algo = sum(kv_bytes(s, w.kv_ways) if is_kv else algorithmic_bytes(s, w.ro_reads, lcfg.n_items)
-               for _, _, s in steps) / len(steps)
-    kmean = sum(kern_ns) / len(kern_ns)
-    achieved = algo / (kmean * 1e-9) / 1e9
-    peak, peak_kind = peaks()
-    # the committed capture is of the C2 bench step: other workloads have none
-    traffic = traffic_per_launch() if args.config == "C2" and world == 1 else None
+    roof = roofline_block(args, cfg, lcfg, steps, kern_ns, is_kv, world)
     last = steps[-1][2]
-    # serial commit chain: batches/s against the critical section's own bound
     cs_cycles = last["server_phase_cycles"]["critical"] / max(1, last["batches"])
 
     # end to end through the public API with host buffers: load (H2D of the
@@ -326,6 +413,7 @@ def bench_ours(args):
     e2e_steps = max(1, min(3, args.steps))
     init_pinned = None if is_kv else torch.from_numpy(init).pin_memory()
     torch.cuda.synchronize()
+    barrier()
     t0 = time.perf_counter()
     e2e_committed = 0
     t_load = 0.0
@@ -350,28 +438,29 @@ def bench_ours(args):
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         r, n, s = oracle_sample_rate(cfg, args.cpu_budget, 1 << 18)
-        cpu = {"value": r, "unit": UNIT, "cores": 1, "kind": "oracle",
+        cpu = {"value": r, "unit": UNIT, "cores": 1, "kind": "oracle", **cpu_info(),
                "sample": f"{n} consecutive {cfg.name} transactions ({s:.1f} s, 1-warp schedule, {cfg.n_items} items)"}
+    rf = roofs()
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": total_ms_max / args.steps, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
         "abort_rate": red["abort_rate"],
         "config": {"workload": DESCR.get(cfg.name, cfg.name),
-                   "n_items": cfg.n_items, "n_versions": cfg.n_versions, "n_tx_per_step": cfg.n_tx,
+                   "n_items_per_gpu": lcfg.n_items, "n_items_job": lcfg.n_items * world,
+                   "n_versions": cfg.n_versions, "n_tx_per_step_per_gpu": lcfg.n_tx,
                    "client_warps_per_gpu": n_cw, "server_workers": w.server_workers,
                    "server_combine": w.server_combine,
                    "ro_streak": w.ro_streak, "ro_adaptive": w.ro_adaptive, "publish": ["client", "server"][w.publish],
                    "server_recv": ["receiver warp", "self-receiving workers"][w.server_recv],
-                   "parallelism": "partitioned" if world > 1 else "single-gpu",
-                   "multi_gpu": "independent key-range partitions, no cross-GPU transactions, NCCL stats only",
+                   "parallelism": f"partitioned x{world}" if world > 1 else "single-gpu",
+                   "multi_gpu": "independent key-range partitions (rank g: keys [g*N, (g+1)*N), full per-GPU "
+                                "workload), no cross-GPU transactions, NCCL stats only",
                    "l2": "flushed (512 MiB write) before every timed step"},
-        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
-                     "kernel": "csmv_fused", "algorithmic_bytes_per_launch": algo,
-                     "note": "latency/serialisation-bound: see serial_chain"},
+        "roofline": roof,
         "serial_chain": serial_chain(red["batches"] / (total_ms_max * 1e-3), cs_cycles,
-                                     red["committed_update"] / max(1, red["batches"]), clk.summary()),
+                                     red["committed_update"] / max(1, red["batches"]), clk.summary(),
+                                     rf.get("cs_floor_cycles")),
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 0 if is_kv else int(init.nbytes),
                 "d2h_bytes_per_step": 400, "steps": e2e_steps,
                 "load_ms_per_step": 1e3 * t_load / e2e_steps, "wall_ms_per_step": 1e3 * e2e_s / e2e_steps},
@@ -380,12 +469,36 @@ def bench_ours(args):
         "kernel_ms_per_step": statistics.mean(kern_ns) / 1e6,
         "aborts": last["aborts"],
     }
+    if args.config == "C3" and rf.get("xsm_roundtrip_ns"):
+        line["hot_chain"] = hot_chain(last, lcfg, rf, statistics.mean(kern_ns))
     if cpu:
         line["cpu_baseline"] = cpu
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def hot_chain(st, lcfg, rf, kern_ns):
+    """C3: every committed transfer touching the hottest account must see the
+    previous one in its snapshot, so those commits form a chain
+    whose link is at least publish -> snapshot -> read -> request -> server
+    -> response: two cross-SM round trips (client->server->client, and the
+    GTS publish -> next client's acquire) plus the ring read.  Floor per link
+    = 2 x xsm_roundtrip + l2_load (tools/ubench/roofs.cu)."""
+    import numpy as np
+    n = lcfg.n_items
+    theta = lcfg.workload.zipf_theta_milli / 1000.0
+    r = np.arange(1, n + 1, dtype=np.float64) ** -theta
+    p0 = r[0] / r.sum()
+    # a transfer touches account 0 if src or dst is 0 (dst = src+1 on a collision)
+    p_touch = 1 - (1 - p0) ** 2
+    links = st["committed_update"] * p_touch
+    floor_ns = 2 * rf["xsm_roundtrip_ns"] + rf["l2_load_ns"]
+    link_ns = kern_ns / links if links else None
+    return {"hot_commits": links, "link_ns": link_ns, "floor_link_ns": floor_ns,
+            "frac": floor_ns / link_ns if link_ns else None,
+            "floor": "2 x xsm_roundtrip_ns + l2_load_ns (profiles/roofs_b200.json)"}
 
 
 def main():
@@ -401,6 +514,8 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=10.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return spawn_ranks(args)
     if args.impl == "reference":
         return bench_reference(args)
     return bench_ours(args)

@@ -75,7 +75,9 @@ extern "C" {
 
 #define CSMV_DBG_NO_PREVAL 1u  /* negative control: skip client pre-validation */
 #define CSMV_DBG_NO_VALIDATE 2u/* negative control: server commits without validating */
-#define CSMV_DBG_JITTER 4u     /* random __nanosleep in client and server */
+#define CSMV_DBG_JITTER 4u     /* race widening: every client and server warp sleeps a seeded 0..2047 ns
+                                  at each cross-warp protocol step (doorbell, response poll, write-back,
+                                  publish, receiver sweep, payload load, lock entry, e_pre -> lastw) */
 #define CSMV_DBG_PHASES 8u     /* per-phase client clocks (csmv_stats_t.client_phase_cycles) */
 #define CSMV_DBG_KV_ITEMSETS 16u /* KV, A <= 16: ship PUT read/write sets item by item (the paper's literal
                                     form); default {set clock} u WS, which decides identically */

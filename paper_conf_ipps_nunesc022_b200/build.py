@@ -34,27 +34,61 @@ def deps():
     return sources() + sorted(glob.glob(os.path.join(CSRC, "*.cuh"))) + [HEADER]
 
 
+STAMP = LIB + ".flags"
+
+
+def extra_flags() -> str:
+    """Build-time A/B knobs (CSMV_NVCC_EXTRA, e.g. -DCSMV_SLEEP_RESP=..)."""
+    return " ".join(os.environ.get("CSMV_NVCC_EXTRA", "").split())
+
+
 def stale() -> bool:
-    if not os.path.exists(LIB):
+    """Rebuild when a source is newer than the library or the library was
+    built with other CSMV_NVCC_EXTRA flags (recorded in a stamp file), so an
+    A/B build is never silently reused as the default one."""
+    if not os.path.exists(LIB) or not os.path.exists(STAMP):
         return True
+    with open(STAMP) as f:
+        if f.read() != extra_flags():
+            return True
     t = os.path.getmtime(LIB)
     return any(os.path.getmtime(p) > t for p in deps())
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    """Compile every csrc/*.cu to an object in parallel (the four fused-kernel
+    instantiations dominate), then link libcsmv.so."""
     if not force and not stale():
         return LIB
+    from concurrent.futures import ThreadPoolExecutor
+
     os.makedirs(LIBDIR, exist_ok=True)
-    cmd = [nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
-           "-Xptxas", "-v" if verbose else "-O3", "-I", os.path.join(ROOT, "include"),
-           *os.environ.get("CSMV_NVCC_EXTRA", "").split(), "-o", LIB + ".tmp", *sources()]
-    r = subprocess.run(cmd, capture_output=True, text=True)
+    objdir = os.path.join(LIBDIR, "obj")
+    os.makedirs(objdir, exist_ok=True)
+    common = [nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
+              "-I", os.path.join(ROOT, "include"), *extra_flags().split()]
+
+    def compile_one(src):
+        obj = os.path.join(objdir, os.path.basename(src)[:-3] + ".o")
+        cmd = [*common, "-Xptxas", "-v" if verbose else "-O3", "-c", "-o", obj, src]
+        return obj, subprocess.run(cmd, capture_output=True, text=True)
+
+    with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 4)) as ex:
+        results = list(ex.map(compile_one, sources()))
+    for obj, r in results:
+        if r.returncode != 0:
+            sys.stderr.write(r.stdout + r.stderr)
+            raise RuntimeError(f"nvcc failed compiling {os.path.basename(obj)}")
+        if verbose:
+            sys.stderr.write(f"== {os.path.basename(obj)}\n" + r.stderr)
+    r = subprocess.run([nvcc(), *ARCH, "-shared", "-o", LIB + ".tmp", *[o for o, _ in results]],
+                       capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
-        raise RuntimeError("nvcc failed building libcsmv.so")
-    if verbose:
-        sys.stderr.write(r.stderr)
+        raise RuntimeError("nvcc failed linking libcsmv.so")
     os.replace(LIB + ".tmp", LIB)
+    with open(STAMP, "w") as f:
+        f.write(extra_flags())
     return LIB
 
 

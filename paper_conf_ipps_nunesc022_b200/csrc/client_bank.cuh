@@ -97,6 +97,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
   const uint32_t lt = lanemask_lt();
   const uint32_t streak = p.ro_streak;
   PhaseClock pc((p.debug & CSMV_DBG_PHASES) != 0);
+  Jitter jit(p, 1);
 
   for (;;) {
     if (!__any_sync(FULL, cu != kNoTx || cr < p.n_tx)) break;
@@ -150,6 +151,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
     }
 
     pc.mark(PH_READ);
+    jit();  // versions read, not yet validated
     if (p.commit == CSMV_COMMIT_JVSTM) {
       // ---- B': decentralized commit, every lane on its own
       if (status == ST_CAND) {
@@ -221,6 +223,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
       }
       __syncwarp();
       fence_gpu();
+      jit();  // payload written, doorbell not yet
       if (lane == 0) st_relaxed(&p.req_seq[cw], round);
       pc.mark(PH_SUBMIT);
     }
@@ -269,10 +272,11 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
 
     // ---- D: the server's answer, write-back, GTS
     uint32_t base = 0, cmask = 0, omask = 0;
-    wait_response(p, cw, round, t_begin, base, cmask, omask);
+    wait_response(p, cw, round, t_begin, base, cmask, omask, jit);
     if (p.commit == CSMV_COMMIT_ONLYCS) fence_gpu();  // acquire: the server's write-backs
     pc.mark(PH_WAIT);
     uint32_t cts = 0;
+    jit();  // committed, versions not yet written back
     if (mine) {
       if ((cmask >> lane) & 1u) {
         // Client-side write-back with CTS = base + rank.
@@ -310,6 +314,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
     pc.mark(PH_WRITEBACK);
     const uint32_t n = __popc(cmask);
     if (n) {
+      jit();  // write-backs done, commit not yet published
       if (p.publish == CSMV_PUBLISH_CLIENT) {
         // Advance GTS by n once every earlier commit is visible:
         // spin until GTS == first CTS - 1 ("GTS 1" = GTS+1).

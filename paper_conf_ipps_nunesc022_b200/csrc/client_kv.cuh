@@ -83,6 +83,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
   const uint32_t streak = p.ro_streak;
   const bool compact = A > kKvFullWays || !(p.debug & CSMV_DBG_KV_ITEMSETS);
   PhaseClock pc((p.debug & CSMV_DBG_PHASES) != 0);
+  Jitter jit(p, 1);
   // per-warp smem scratch, lane-minor: RS[kKvMaxRs][32], WS[4][32], NRS[32]
   uint32_t* RS = scratch + (size_t)wib * 32 * (kKvMaxRs + 5);
   uint32_t* WS = RS + kKvMaxRs * 32;
@@ -215,6 +216,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     }
     __syncwarp();
     pc.mark(PH_READ);
+    jit();  // versions read, not yet validated
 
     // ---- B: pre-validation: lane j is dropped if WS_i n (RS_j u WS_j)
     // or WS_j n RS_i is non-empty for an earlier kept lane i
@@ -287,6 +289,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       }
       __syncwarp();
       fence_gpu();
+      jit();  // payload written, doorbell not yet
       if (lane == 0) st_relaxed(&p.req_seq[cw], round);
       pc.mark(PH_SUBMIT);
     }
@@ -320,10 +323,11 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
 
     // ---- D: response, write-back, GTS
     uint32_t base = 0, cmask = 0, omask = 0;
-    wait_response(p, cw, round, t_begin, base, cmask, omask);
+    wait_response(p, cw, round, t_begin, base, cmask, omask, jit);
     if (p.commit == CSMV_COMMIT_ONLYCS) fence_gpu();  // acquire: the server's write-backs
     pc.mark(PH_WAIT);
     uint32_t cts = 0;
+    jit();  // committed, versions not yet written back
     if (mine) {
       if ((cmask >> lane) & 1u) {
         // Client-side write-back: the paper's 4 writes.
@@ -355,6 +359,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     pc.mark(PH_WRITEBACK);
     const uint32_t n = __popc(cmask);
     if (n) {
+      jit();  // write-backs done, commit not yet published
       if (p.publish == CSMV_PUBLISH_CLIENT) {
         __syncwarp();
         fence_gpu();

@@ -444,6 +444,9 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   uint32_t n_ctas = n_cw < max_client_ctas ? n_cw : max_client_ctas;
   if (n_srv > 1) n_ctas = (n_ctas + n_srv - 1) / n_srv * n_srv;  // grid a multiple of the cluster
   if (n_srv > 1 && n_ctas > max_client_ctas) n_ctas = max_client_ctas / n_srv * n_srv;
+  if (n_ctas == 0) return set_err(CSMV_EINVAL, "csmv_run: no client CTA fits beside the server");
+  // client warp cw runs on CTA cw mod n_ctas, warp cw / n_ctas: never more than the grid holds
+  if (n_cw > n_ctas * kWarps) n_cw = n_ctas * kWarps;
 
   // logs
   uint32_t max_vals = 0;

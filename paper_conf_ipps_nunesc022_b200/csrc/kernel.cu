@@ -1,396 +1,13 @@
-// kernel.cu -- the fused persistent CSMV kernel for sm_100a.
-//
-// One cooperative grid holds both roles of the paper's client-server split
-// (P:99-105): CTAs 0..C-1 are the server (C = 1, the paper's one SM, or a
-// thread-block cluster), the rest are client SMs.  Fusing the roles into one
-// launch guarantees co-residency of a server that spins on its clients (the
-// paper launches two kernels; separate kernels deadlock when a profiler
-// serialises them).  CSMV_COMMIT_JVSTM launches clients only.
-//
-// Client warp, one round (client_bank.cuh / client_kv.cuh):
-//   TXBegin     s <- GTS (one acquire load per warp round)
-//   TXRead      newest version with ts <= s from the VBox ring
-//   pre-validation of the warp's update lanes (shuffle/ballot)
-//   submit the batch (request slot + doorbell)
-//   read-only transactions at s while the batch is at the server
-//   the response, client write-back of the new versions
-//   ordered GTS advance by n (CSMV_PUBLISH_CLIENT) or a done
-//   flag per CTS for the server publisher (CSMV_PUBLISH_SERVER)
-//   aborted transactions retry with a fresh snapshot next round
-//
-// Server (server.cuh): a receiver warp per server CTA dispatches doorbells to
-// worker warps; a worker validates whole batches (one lane per transaction,
-// __ballot_sync) against the two-level item-indexed ATR (HBM lastw + smem
-// recent-commit table; or the paper's list ATR), reserves consecutive CTS
-// and records the write-sets inside a shared-memory ticket-locked critical
-// section.  No global atomics on
-// the commit path.
+// kernel.cu -- host-side launchers: the fused kernel (instantiated in
+// fused_*.cu) and the small setup, dump and generator kernels.
 #include <cuda_runtime.h>
 
 #include <cub/device/device_scan.cuh>
 
-#include "kernel.cuh"
-#include "ptx.cuh"
-
-namespace csmvd {
-
-enum : int { ST_NONE = 0, ST_RO_OK, ST_CAND, ST_UPD_OK, ST_ABORT };
-
-// --------------------------------------------------------------------------
-// VBox read (TXRead) and write-back
-// --------------------------------------------------------------------------
-struct Sel {
-  int best;          // slot of the newest version with ts <= s, -1 if none
-  uint32_t best_ts;
-  uint32_t newest;   // largest ts present
-};
-
-template <int NS>
-__device__ __forceinline__ Sel select_version(const Ring<NS>& r, uint32_t s) {
-  Sel q{-1, 0u, 0u};
-#pragma unroll
-  for (int j = 0; j < NS; ++j) {
-    uint32_t ts = (uint32_t)(r.s[j] >> 32);
-    if (ts != kEmptyTs) {
-      q.newest = max(q.newest, ts);
-      if (ts <= s && (q.best < 0 || ts > q.best_ts)) {
-        q.best = j;
-        q.best_ts = ts;
-      }
-    }
-  }
-  return q;
-}
-
-template <int NS>
-__device__ __forceinline__ uint64_t slot_at(const Ring<NS>& r, int j) {
-  uint64_t v = r.s[0];
-#pragma unroll
-  for (int i = 1; i < NS; ++i) v = (j == i) ? r.s[i] : v;
-  return v;
-}
-
-// Replace the first unused slot, else the oldest version.  The
-// writer owns the item: the WW check orders all writers of an item
-// and the ring is unchanged since this transaction read it.
-template <int NS>
-__device__ __forceinline__ void write_back(uint64_t* ring, const Ring<NS>& r, uint32_t K,
-                                           uint32_t cts, uint32_t val) {
-  int victim = -1;
-  uint32_t vts = kEmptyTs;
-#pragma unroll
-  for (int j = 0; j < NS; ++j) {
-    uint32_t ts = (uint32_t)(r.s[j] >> 32);
-    if ((uint32_t)j < K && victim < 0 && ts == kEmptyTs) victim = j;
-  }
-  if (victim < 0) {
-    victim = 0;
-    vts = (uint32_t)(r.s[0] >> 32);
-#pragma unroll
-    for (int j = 1; j < NS; ++j) {
-      uint32_t ts = (uint32_t)(r.s[j] >> 32);
-      if ((uint32_t)j < K && ts < vts) {
-        victim = j;
-        vts = ts;
-      }
-    }
-  }
-  st_relaxed64(ring + victim, ((uint64_t)cts << 32) | val);
-}
-
-// one relaxed load by lane 0, broadcast: keeps spin loops warp-uniform
-__device__ __forceinline__ uint32_t warp_ld_relaxed(const uint32_t* p) {
-  uint32_t v = 0;
-  if ((threadIdx.x & 31) == 0) v = ld_relaxed(p);
-  return __shfl_sync(0xFFFFFFFFu, v, 0);
-}
-
-__device__ __forceinline__ uint64_t warp_ld_relaxed64(const uint64_t* p) {
-  uint64_t v = 0;
-  if ((threadIdx.x & 31) == 0) v = ld_relaxed64(p);
-  return __shfl_sync(0xFFFFFFFFu, v, 0);
-}
-
-__device__ __forceinline__ bool watchdog(const KParams& p, uint64_t t0, uint32_t where);
-
-// Wait for the server's answer to request `round` of client warp cw (all
-// three words tagged with round).  false if the run is being torn down.
-__device__ __forceinline__ bool wait_response(const KParams& p, uint32_t cw, uint32_t round, uint64_t t_begin,
-                                              uint32_t& base, uint32_t& cmask, uint32_t& omask) {
-  const uint32_t FULL = 0xFFFFFFFFu;
-  uint32_t it = 0;
-  uint64_t b, c, o;
-  for (;;) {
-    b = warp_ld_relaxed64(&p.resp[cw].base);
-    if ((uint32_t)(b >> 32) == round) {
-      c = warp_ld_relaxed64(&p.resp[cw].commit);
-      o = warp_ld_relaxed64(&p.resp[cw].ovf);
-      if ((uint32_t)(c >> 32) == round && (uint32_t)(o >> 32) == round) break;
-    }
-    if ((++it & 255u) == 0) {
-      uint32_t bad = 0;
-      if ((threadIdx.x & 31) == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);
-      if (__shfl_sync(FULL, bad, 0)) return false;
-    }
-    __nanosleep(CSMV_SLEEP_RESP);
-  }
-  base = (uint32_t)b;
-  cmask = (uint32_t)c;
-  omask = (uint32_t)o;
-  return true;
-}
-
-__device__ __forceinline__ bool watchdog(const KParams& p, uint64_t t0, uint32_t where) {
-  if (globaltimer() - t0 > p.watchdog_ns) {
-    if (atomicCAS(&p.ctl->error, 0u, 1u) == 0u) p.ctl->where = where;
-    return true;
-  }
-  return false;
-}
-
-// --------------------------------------------------------------------------
-// Read-only transaction: L consecutive accounts (or all)
-// --------------------------------------------------------------------------
-// Exact warp sums by redux.sync: an int32 per lane as two 16-bit-wide
-// halves (no 32-bit wrap), a u64 per lane (mod 2^64) as four 16-bit chunks.
-__device__ __forceinline__ int64_t warp_sum_i32(int32_t v) {
-  const int hi = __reduce_add_sync(0xFFFFFFFFu, v >> 16);
-  const unsigned lo = __reduce_add_sync(0xFFFFFFFFu, (unsigned)v & 0xFFFFu);
-  return (int64_t)hi * 65536 + (int64_t)lo;
-}
-__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
-  uint64_t r = 0;
-#pragma unroll
-  for (int k = 0; k < 4; ++k)
-    r += (uint64_t)__reduce_add_sync(0xFFFFFFFFu, (unsigned)(v >> (16 * k)) & 0xFFFFu) << (16 * k);
-  return r;
-}
-
-// Warp-cooperative read-only transactions: the lanes in
-// `act` each own one read-only transaction at snapshot s -- tx, a scan of
-// `len` accounts from `start` -- and the whole warp runs them one after
-// another, 32 consecutive accounts per row (one coalesced 1 KiB load of
-// 32-byte VBoxes), U rows in flight.  Each row is reduced across the warp
-// (exact int64 sum, digest, any-miss) and added into its owner lane.  Same
-// per-transaction result as one lane scanning alone; no lane waits for another lane's
-// longer read-only run.
-template <int NS>
-__device__ __forceinline__ void rot_coop(const KParams& p, uint32_t act, uint32_t start, uint32_t len, uint32_t s,
-                                         uint64_t tx, bool& ok, int64_t& sum, uint64_t& dg) {
-  constexpr int U = NS <= 4 ? 8 : (NS == 8 ? 4 : 2);
-  const uint32_t FULL = 0xFFFFFFFFu;
-  const uint32_t lane = threadIdx.x & 31;
-  const uint32_t N = p.n_items;
-  ok = true;
-  sum = 0;
-  dg = 0;
-  const uint32_t L = __shfl_sync(FULL, len, act ? __ffs(act) - 1 : 0);  // the same for every transaction
-  const uint32_t rows = (L + 31) / 32;
-  const bool full_log = p.log_mode == CSMV_LOG_FULL;
-  const bool long_scan = L > N;  // a scan longer than the store wraps more than once
-  // owners are taken lowest lane first, `rows` rows each; (rem, cur, k) are
-  // warp-uniform, so the shuffles below run under uniform branches
-  uint32_t rem = act, cur = 0, k = rows, cur_start = 0;
-  uint64_t cur_tx = 0;
-  while (rem || k < rows) {
-    Ring<NS> r[U];
-    uint32_t xs[U], own[U], ev[U];
-    uint64_t txo[U];
-    bool on[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      if (k >= rows && rem) {  // next owner
-        cur = __ffs(rem) - 1;
-        rem &= rem - 1;
-        k = 0;
-        cur_start = __shfl_sync(FULL, start, cur);
-        if (full_log) cur_tx = __shfl_sync(FULL, tx, cur);
-      }
-      on[u] = k < rows;
-      own[u] = cur;
-      txo[u] = cur_tx;
-      ev[u] = k * 32 + lane;
-      uint32_t x = cur_start + ev[u];  // start < N; ev < L
-      if (x >= N) x -= N;
-      if (long_scan && x >= N) x %= N;
-      xs[u] = x;
-      if (on[u] && ev[u] < L) r[u] = ld_ring<NS>(p.rings + (size_t)x * NS);
-      if (on[u]) ++k;
-    }
-    // version selection for every row first, so that the re-reads a newer
-    // version calls for are in flight together (one L2 round trip per group)
-    uint64_t vv[U], rv[U];
-    bool miss_[U], re[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      vv[u] = rv[u] = 0;
-      miss_[u] = re[u] = false;
-      if (on[u] && ev[u] < L) {
-        const Sel q = select_version<NS>(r[u], s);
-        if (q.best < 0) {
-          miss_[u] = true;  // version recycled
-        } else {
-          vv[u] = slot_at<NS>(r[u], q.best);
-          // A newer version exists, so write-backs may have overwritten slots
-          // while we read.  Versions are evicted oldest first, so if the chosen
-          // slot still holds the same version, no version in (best_ts, s] was
-          // missed; otherwise the snapshot's version is gone.
-          re[u] = q.newest > s;
-          if (re[u]) rv[u] = ld_relaxed64(p.rings + (size_t)xs[u] * NS + q.best);
-        }
-      }
-    }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      if (!on[u]) break;  // warp-uniform
-      const bool valid = ev[u] < L;
-      const bool miss = miss_[u] || (re[u] && rv[u] != vv[u]);
-      const uint32_t val = (uint32_t)vv[u];
-      const bool rmiss = __any_sync(FULL, miss);
-      const int64_t rs = warp_sum_i32(miss ? 0 : (int32_t)val);
-      uint64_t rd = 0;
-      if (p.log_mode) {
-        rd = warp_sum_u64(valid && !miss ? dig1(xs[u], val) : 0ull);
-        if (p.log_mode == CSMV_LOG_FULL && valid && ev[u] < p.max_vals) p.vals[txo[u] * p.max_vals + ev[u]] = val;
-      }
-      if (lane == own[u]) {
-        ok = ok && !rmiss;
-        sum += rs;
-        dg += rd;
-      }
-    }
-  }
-}
-
-// --------------------------------------------------------------------------
-// Client warp
-// --------------------------------------------------------------------------
-struct ClientCounters {
-  uint32_t c_upd = 0, c_ro = 0, n_rounds = 0, cas_fail = 0;
-  uint32_t ab[CSMV_N_ABORT][2];
-  uint64_t ro_ck = 0;
-  __device__ ClientCounters() {
-#pragma unroll
-    for (int i = 0; i < (int)CSMV_N_ABORT; ++i) ab[i][0] = ab[i][1] = 0;
-  }
-  __device__ __forceinline__ void abort(int reason, bool upd) {
-#pragma unroll
-    for (int i = 0; i < (int)CSMV_N_ABORT; ++i)
-      if (reason == i) ++ab[i][upd ? 1 : 0];
-  }
-};
-
-// Per-phase client clocks (CSMV_DBG_PHASES; the shape of Tables I and III,
-// P:136-147).  Every lane accumulates; the flush reports the
-// mean over lanes, so warp-convergent phases read as the warp's time and
-// lane-divergent ones (JVSTM-GPU) as the mean lane's.
-enum : int {
-  PH_READ = 0,     // A: snapshot + update reads
-  PH_PREVAL,       // B: pre-validation          | JVSTM: validation + CTS CAS
-  PH_SUBMIT,       // B: request + doorbell      | JVSTM: ATR record insert
-  PH_ROT,          // C: read-only transactions
-  PH_WAIT,         // D: waiting for the server
-  PH_WRITEBACK,    // D: write-back
-  PH_PUBLISH,      // D: GTS advance / done flag
-  PH_DIVERGENCE,   // JVSTM: a lane's wait from its own commit end to reconvergence
-};
-
-struct PhaseClock {
-  unsigned long long ph[8];
-  long long t;
-  bool on;
-  __device__ explicit PhaseClock(bool enabled) : t(0), on(enabled) {
-#pragma unroll
-    for (int i = 0; i < 8; ++i) ph[i] = 0;
-  }
-  __device__ __forceinline__ void start() {
-    if (on) t = clock64();
-  }
-  __device__ __forceinline__ void mark(int k) {
-    if (on) {
-      const long long n = clock64();
-#pragma unroll
-      for (int i = 0; i < 8; ++i)
-        if (i == k) ph[i] += (unsigned long long)(n - t);
-      t = n;
-    }
-  }
-  __device__ __forceinline__ void flush(const KParams& p) const {
-    if (!on) return;
-#pragma unroll
-    for (int i = 0; i < 8; ++i) {
-      unsigned long long v = ph[i];
-#pragma unroll
-      for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, o);
-      if ((threadIdx.x & 31) == 0 && v) atomicAdd(&p.stats->client_phase[i], v / 32);
-    }
-  }
-};
-
-__device__ __forceinline__ void log_commit(const KParams& p, uint64_t tx, uint32_t s, uint32_t cts,
-                                           uint32_t att, uint64_t rdig, uint64_t aux) {
-  csmv_log_rec rec;
-  rec.tx = (uint32_t)tx;
-  rec.snapshot = s;
-  rec.cts = cts;
-  rec.attempts = att;
-  rec.read_digest = rdig;
-  rec.aux = aux;
-  p.log[tx] = rec;
-}
-
-// flush per-warp counters once (no global atomics on the commit path)
-__device__ __forceinline__ void client_flush(const KParams& p, const ClientCounters& cc) {
-  const uint32_t FULL = 0xFFFFFFFFu;
-  const uint32_t lane = threadIdx.x & 31;
-  const uint32_t s_upd = __reduce_add_sync(FULL, cc.c_upd), s_ro = __reduce_add_sync(FULL, cc.c_ro);
-  const uint32_t s_cf = __reduce_add_sync(FULL, cc.cas_fail);
-  uint32_t s_ab[CSMV_N_ABORT][2];
-#pragma unroll
-  for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
-    s_ab[i][0] = __reduce_add_sync(FULL, cc.ab[i][0]);
-    s_ab[i][1] = __reduce_add_sync(FULL, cc.ab[i][1]);
-  }
-  uint64_t ro_ck = cc.ro_ck;
-#pragma unroll
-  for (int o = 16; o; o >>= 1) ro_ck ^= __shfl_xor_sync(FULL, ro_ck, o);
-  if (lane == 0) {
-    atomicAdd(&p.stats->committed_update, (unsigned long long)s_upd);
-    atomicAdd(&p.stats->committed_ro, (unsigned long long)s_ro);
-    for (int i = 0; i < (int)CSMV_N_ABORT; ++i) {
-      if (s_ab[i][0]) atomicAdd(&p.stats->aborts[i][0], (unsigned long long)s_ab[i][0]);
-      if (s_ab[i][1]) atomicAdd(&p.stats->aborts[i][1], (unsigned long long)s_ab[i][1]);
-    }
-    atomicAdd(&p.stats->rounds, (unsigned long long)cc.n_rounds);
-    if (s_cf) atomicAdd(&p.stats->cas_fail, (unsigned long long)s_cf);
-    atomicXor(&p.stats->ro_checksum, (unsigned long long)ro_ck);
-    __threadfence();
-    atomicAdd(&p.ctl->done_warps, 1u);
-  }
-}
-
-}  // namespace csmvd
-
-#include "client_bank.cuh"
-
-namespace csmvd {
-
-}  // namespace csmvd
-
-#include "kv.cuh"
-#include "server.cuh"
+#include "fused.cuh"
 #include "kv_kernels.cuh"
 
 namespace csmvd {
-
-template <int NS, int KIND, bool CL>
-__global__ void __launch_bounds__(kBlock, 1) csmv_fused(const KParams p) {
-  extern __shared__ __align__(16) uint8_t smem[];
-  const uint64_t t_begin = globaltimer();
-  if (blockIdx.x < p.n_server_ctas) server_cta<NS, KIND, CL>(p, smem, t_begin);
-  else if constexpr (KIND == CSMV_KIND_KV) client_warp_kv<NS>(p, t_begin, reinterpret_cast<uint32_t*>(smem));
-  else client_warp<NS>(p, t_begin);
-}
 
 template <int NS>
 __global__ void init_rings(uint64_t* rings, const int32_t* init, uint64_t n, uint32_t* gts) {
@@ -417,68 +34,12 @@ __global__ void gen_descs_kernel(GenParams g, uint64_t tx0, uint64_t n, uint32_t
   o[5] = d.len;
 }
 
-template <int NS, int KIND, bool CL>
-static cudaError_t launch_ns(const KParams& p, uint32_t grid, size_t smem, cudaStream_t st, int* occ) {
-  auto kern = csmv_fused<NS, KIND, CL>;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  if (CL) {
-    e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-    if (e != cudaSuccess) return e;
-  }
-  cudaLaunchConfig_t cfg = {};
-  cudaLaunchAttribute at[2];
-  at[0].id = cudaLaunchAttributeCooperative;
-  at[0].val.cooperative = 1;
-  at[1].id = cudaLaunchAttributeClusterDimension;
-  at[1].val.clusterDim.x = CL ? p.n_server_ctas : 1;
-  at[1].val.clusterDim.y = 1;
-  at[1].val.clusterDim.z = 1;
-  cfg.blockDim = dim3(kBlock);
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = st;
-  cfg.attrs = at;
-  cfg.numAttrs = CL ? 2 : 1;
-  if (occ) {  // query: co-resident CTAs of this configuration
-    if (CL) {
-      cfg.gridDim = dim3(p.n_server_ctas);
-      int ncl = 0;
-      e = cudaOccupancyMaxActiveClusters(&ncl, kern, &cfg);
-      *occ = ncl * (int)p.n_server_ctas;
-      return e;
-    }
-    int b = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kern, kBlock, smem);
-    int dev = 0, sms = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    *occ = b * sms;
-    return e;
-  }
-  cfg.gridDim = dim3(grid);
-  return cudaLaunchKernelEx(&cfg, kern, p);
-}
-
-template <int KIND, bool CL>
-static cudaError_t launch_kind(const KParams& p, uint32_t nslot, uint32_t grid, size_t smem, cudaStream_t st,
-                               int* occ) {
-  switch (nslot) {
-    case 2: return launch_ns<2, KIND, CL>(p, grid, smem, st, occ);
-    case 4: return launch_ns<4, KIND, CL>(p, grid, smem, st, occ);
-    case 8: return launch_ns<8, KIND, CL>(p, grid, smem, st, occ);
-    case 16: return launch_ns<16, KIND, CL>(p, grid, smem, st, occ);
-  }
-  return cudaErrorInvalidValue;
-}
-
 static cudaError_t launch_any(const KParams& p, uint32_t nslot, uint32_t grid, size_t smem, cudaStream_t st,
                               int* occ) {
   const bool cl = p.n_server_ctas > 1;
   if (p.kind == CSMV_KIND_KV)
-    return cl ? launch_kind<CSMV_KIND_KV, true>(p, nslot, grid, smem, st, occ)
-              : launch_kind<CSMV_KIND_KV, false>(p, nslot, grid, smem, st, occ);
-  return cl ? launch_kind<CSMV_KIND_BANK, true>(p, nslot, grid, smem, st, occ)
-            : launch_kind<CSMV_KIND_BANK, false>(p, nslot, grid, smem, st, occ);
+    return cl ? launch_fused_kv_cl(p, nslot, grid, smem, st, occ) : launch_fused_kv_cta(p, nslot, grid, smem, st, occ);
+  return cl ? launch_fused_bank_cl(p, nslot, grid, smem, st, occ) : launch_fused_bank_cta(p, nslot, grid, smem, st, occ);
 }
 
 cudaError_t launch_fused(const KParams& p, uint32_t nslot, uint32_t grid, size_t smem, cudaStream_t st) {

@@ -1,5 +1,5 @@
-// kv_kernels.cuh -- client warp and server worker for the MemcachedGPU
-// workload.  Included by kernel.cu after the shared helpers.
+// kv_kernels.cuh -- setup, dump and generator kernels of the MemcachedGPU
+// workload; its client warp is client_kv.cuh.  Included by kernel.cu.
 //
 // GET(k) is a read-only transaction: scan the ways of set(k), stop at the
 // matching key (then read its value) or at the first empty way; never
@@ -10,12 +10,7 @@
 // so the request carries per-lane id lists and the server validates them
 // with the generic worker below.
 #pragma once
-
-namespace csmvd {
-
-}  // namespace csmvd
-
-#include "client_kv.cuh"
+#include "fused.cuh"
 
 namespace csmvd {
 

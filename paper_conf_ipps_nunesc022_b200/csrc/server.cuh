@@ -285,7 +285,7 @@ __device__ __forceinline__ void filt16_st(uint32_t a, uint32_t v) {
 // warp is outstanding, so QN >= slice slots never wrap onto an unconsumed
 // entry.
 // ---------------------------------------------------------------------------
-__device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+static __device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t n = c.cw_hi - c.cw_lo;
@@ -294,9 +294,12 @@ __device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64_t t_be
   const uint32_t qmask = (1u << c.qn_log2) - 1;
   uint32_t tail = 0;
   uint32_t idle = 0;
+  Jitter jit(p, 3);
   for (;;) {
-    bool found = false, fenced = false;
+    jit();
+    bool found = false;
     for (uint32_t r0 = 0; r0 < rows; r0 += 8) {
+      bool fenced = false;  // per group of 8 rows: each group's doorbells are loaded after the last fence
       uint32_t seq[8];
 #pragma unroll
       for (int k = 0; k < 8; ++k) {
@@ -310,7 +313,7 @@ __device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64_t t_be
         const uint32_t pm = __ballot_sync(FULL, pend);
         if (pm) {
           found = true;
-          if (!fenced) {  // acquire: the payloads of the doorbells just seen precede
+          if (!fenced) {  // acquire: the payloads of this group's doorbells precede
             fence_gpu();  // every worker's reads of them (queue -> fence.cta -> loads)
             fenced = true;
           }
@@ -401,9 +404,13 @@ __device__ __forceinline__ void cs_leave(const SrvCtx& c, uint32_t ticket, uint3
       *(volatile uint32_t*)&c.sh0->now_serving = ticket + 1;
     }
   } else if ((threadIdx.x & 31) == 0) {
+    // one fence orders every store of the section (the warp's, through the
+    // __syncwarp above: filter slots, and the KV workers' lastw) before BOTH
+    // the tail -- which KV workers read outside the lock as e_pre and then
+    // load lastw under it -- and the lock handoff
+    fence_cta();
     *(volatile uint32_t*)&c.sh0->tail = new_tail;
-    const uint32_t a = (uint32_t)__cvta_generic_to_shared(&c.sh0->now_serving);
-    asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" ::"r"(a), "r"(ticket + 1) : "memory");
+    *(volatile uint32_t*)&c.sh0->now_serving = ticket + 1;
   }
 }
 
@@ -538,6 +545,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
   unsigned long long busy = 0, locked = 0, batches = 0, groups = 0;
   unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   constexpr bool self = SELF;
+  Jitter jit(p, 4);
   uint32_t my_lo = 0, my_hi = 0;
   if constexpr (SELF) {
     const uint32_t w = threadIdx.x >> 5, per = (c.cw_hi - c.cw_lo + p.n_workers - 1) / p.n_workers;
@@ -569,6 +577,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
     }
     const long long t0 = clock64();
+    jit();  // claimed, payload not yet loaded
     // ---- load the batches: header and ids together (the receiver's fence
     // ordered them after the doorbells; ours orders them after the queue)
     if (!self) fence_cta();
@@ -634,6 +643,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     // The payload must have arrived before the lock is taken: a warp vote on
     // values derived from it makes the loads complete here.
     if (__ballot_sync(FULL, xor_all == 0x12345679u) == FULL) __nanosleep(1);
+    jit();  // lastw checked against e_pre, lock not yet taken
     const long long tl = clock64();
     // ---- critical section: validate, reserve CTS, record
     const uint32_t ticket = cs_enter<CL>(c);
@@ -777,6 +787,7 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
   const uint32_t fl2 = p.rt_log2 - p.clog2 + 3;  // the filter: CTA 0's stripe, 8 << local_log2 32-bit slots
   const bool novalid = (p.debug & CSMV_DBG_NO_VALIDATE) != 0;
   unsigned long long busy = 0, batches = 0, groups = 0, ph0 = 0, ph1 = 0, ph4 = 0;
+  Jitter jit(p, 5);
   for (;;) {
     const long long tq = clock64();
     uint32_t cwv[M];
@@ -832,6 +843,7 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
     // the ring's depth, not the wait for room as well
     const uint32_t e_pre = ld_acquire(p.gts);  // lastw covers every CTS <= GTS (client write-back)
     srv_fence<CL>();
+    jit();  // e_pre read, lastw not yet
     uint32_t chkm[M];
 #pragma unroll
     for (int j = 0; j < M; ++j) {
@@ -925,6 +937,7 @@ __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring
   unsigned long long cs = 0, wait = 0;
   CmPayload q;
   bool have = false;
+  Jitter jit(p, 6);
   for (uint32_t next = 0;; ++next) {
     const long long tw = clock64();
     // wait for slot `next` (unless the prefetch already found it ready)
@@ -939,6 +952,7 @@ __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring
       if (__shfl_sync(FULL, done, 0)) break;
     }
     if (!have) break;
+    jit();
     const long long t1 = clock64();
     const CmPayload cur = q;
     const bool chk = (cur.chkm >> lane) & 1u;
@@ -1015,6 +1029,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
   // PUT's set, read and written by every PUT of that set while nothing else
   // writes the set -- it alone decides validation (DESIGN.md readings)
   const bool compact = p.kv_A > kKvFullWays || !(p.debug & CSMV_DBG_KV_ITEMSETS);
+  Jitter jit(p, 7);
   for (;;) {
     uint32_t cw;
     const long long tq = clock64();
@@ -1034,6 +1049,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     const uint32_t nval = compact ? min(cnt, 1u) : cnt;  // ids to validate
     const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
     srv_fence<CL>();
+    jit();  // e_pre read, lastw not yet (the window cs_leave's fence covers)
     uint32_t lw[kKvMaxId];
     uint32_t x = s ^ e_pre;
 #pragma unroll
@@ -1042,6 +1058,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
       x ^= ids[k] ^ lw[k];
     }
     if (__ballot_sync(FULL, x == 0x12345679u) == FULL) __nanosleep(1);  // payload complete before the lock
+    jit();
     const long long tl = clock64();
     // ---- critical section
     const uint32_t ticket = cs_enter<CL>(c);
@@ -1079,7 +1096,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
       for (uint32_t k = 0; k < kKvMaxId; ++k) {
         if (k < cnt && (ids[k] & kWriteBit)) {
           const uint32_t id = ids[k] & ~kWriteBit, b = rt_bucket(id, p.rt_log2);
-          p.lastw[id] = cts;  // every written item, so lastw stays exact for any later run
+          st_relaxed(p.lastw + id, cts);  // every written item, so lastw stays exact for any later run
           if (k < nval || !compact) {
             const RtProbe q = rt_probe<CL>(c, b, id, 0u, 0u, 0u);  // the way to (re)use
             rt_record<CL>(c, b, q.way, id, cts);
@@ -1136,6 +1153,7 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
   const uint32_t fl2 = p.rt_log2 + 3;
   unsigned long long busy = 0, locked = 0, batches = 0;
   unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  Jitter jit(p, 8);
   for (;;) {
     uint32_t cw;
     const long long tq = clock64();
@@ -1151,6 +1169,7 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
     const bool mine = (mask >> lane) & 1u;
     const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
     srv_fence<CL>();
+    jit();  // e_pre read, lastw not yet (the window cs_leave's fence covers)
     const uint32_t lw = mine ? ld_relaxed(p.lastw + ids[0]) : 0u;
     const bool chk = mine && (novalid || lw <= s);
     uint32_t fa[kFiltK];
@@ -1158,6 +1177,7 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
     for (int k = 0; k < kFiltK; ++k) fa[k] = filt_addr<CL>(c, filt_slot(ids[0], k, fl2));
     const uint32_t e_chk = novalid ? 0xFFFFFFFFu : e_pre;
     if (__ballot_sync(FULL, (s ^ lw ^ ids[1] ^ ids[2] ^ ids[3]) == 0x12345679u) == FULL) __nanosleep(1);
+    jit();
     const long long tl = clock64();
     // ---- critical section
     const uint32_t ticket = cs_enter<CL>(c);
@@ -1180,7 +1200,7 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
 #pragma unroll
       for (int k = 0; k < kFiltK; ++k) filt_st<CL>(fa[k], t0c + n);  // the batch's last CTS
 #pragma unroll
-      for (int k = 0; k < 4; ++k) p.lastw[ids[k]] = cts;
+      for (int k = 0; k < 4; ++k) st_relaxed(p.lastw + ids[k], cts);
     }
     const long long tr = clock64();
     cs_leave<CL>(c, ticket, t0c + n);
@@ -1232,6 +1252,7 @@ __device__ void server_worker_onlycs(const KParams& p, const SrvCtx& c, uint64_t
   const uint32_t R = (uint32_t)kRtWays << p.rt_log2;
   const uint32_t dmask = (1u << kDoneLog2) - 1;
   unsigned long long busy = 0, locked = 0, batches = 0;
+  Jitter jit(p, 9);
   for (;;) {
     uint32_t cw;
     if (!claim_request(c, cw)) break;
@@ -1249,6 +1270,7 @@ __device__ void server_worker_onlycs(const KParams& p, const SrvCtx& c, uint64_t
       nb = ld_relaxed(p.req_vals + (size_t)cw * 64 + 32 + lane);
     }
     if (__ballot_sync(FULL, (a ^ b ^ na ^ nb ^ s) == 0x12345679u) == FULL) __nanosleep(1);
+    jit();
     const uint32_t ticket = cs_enter<false>(c);
     const long long t1 = clock64();
     const uint32_t base = *(volatile uint32_t*)&c.sh0->tail + 1;
@@ -1317,17 +1339,19 @@ __device__ void server_worker_onlycs(const KParams& p, const SrvCtx& c, uint64_t
 // are done.  Same invariant as P:116 (GTS = c only once every commit <= c
 // has written back), without a client-side serial chain.  CTA 0 only.
 // ---------------------------------------------------------------------------
-__device__ void server_publisher(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+static __device__ void server_publisher(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t dmask = (1u << kDoneLog2) - 1;
   uint32_t g = *(volatile uint32_t*)&c.sh->tail;
   uint32_t spins = 0;
+  Jitter jit(p, 10);
   // one sweep looks at the next 32 * 4 * W flags: W 16-byte loads per lane in
   // flight, lane l of row k covering CTS g+1 + 4(32k + l) .. +3 (a sweep is
   // one L2 round trip, so this bounds GTS's advance rate)
   constexpr int W = 8;
   for (;;) {
+    jit();
     const uint32_t g0 = g + 1;
     const uint32_t a0 = g0 & 3u;  // 16-byte loads need a 4-aligned first CTS: start at g0 - a0
     uint4 v[W];

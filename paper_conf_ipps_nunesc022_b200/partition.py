@@ -2,13 +2,20 @@
 
 CSMV serialises every update through one CTS sequence and one GTS (P:65,
 P:101), so a single store does not shard.  For G GPUs the framework
-runs G *independent key-range-partitioned instances*: rank g owns accounts
-[g*N/G, (g+1)*N/G) as its own store (local ids 0..N_g-1), runs its own
-server and GTS, generates its n_tx/G transactions with seed_g = mix64(seed ^ g)
-inside its partition, and never exchanges data with another rank.  The only
-collective is the end-of-run statistics reduction (SUM of counters, MAX of
-elapsed time) -- every figure is labelled "partitioned, no cross-GPU
+runs G *independent key-range-partitioned instances*: rank g owns its own
+key range of the job's accounts as its own store (local ids 0..N_g-1), runs
+its own server and GTS, generates its transactions with seed_g = mix64(seed ^
+g) inside its partition, and never exchanges data with another rank.  The
+only collective is the end-of-run statistics reduction (SUM of counters, MAX
+of elapsed time) -- every figure is labelled "partitioned, no cross-GPU
 transactions".
+
+Two ways to split a job (``mode``):
+  * "weak" (bench.py's): every rank runs the full per-GPU workload -- n_items
+    accounts and n_tx transactions -- on key range [g*n_items, (g+1)*n_items)
+    of a G*n_items-account job; per-GPU work is fixed as G grows;
+  * "strong": a fixed job of n_items accounts and n_tx transactions is split
+    into G near-equal key and transaction ranges.
 """
 from __future__ import annotations
 
@@ -39,14 +46,18 @@ class Part:
     seed: int
 
 
-def partition(n_items: int, n_tx: int, seed: int, rank: int, world: int) -> Part:
+def partition(n_items: int, n_tx: int, seed: int, rank: int, world: int, mode: str = "strong") -> Part:
     if not 0 <= rank < world:
         raise ValueError("rank out of range")
+    s = seed if world == 1 else mix64(seed ^ rank)
+    if mode == "weak":
+        return Part(rank, world, n_items * rank, n_items, n_tx * rank, n_tx, s)
+    if mode != "strong":
+        raise ValueError(f"unknown partition mode {mode!r}")
     lo = n_items * rank // world
     hi = n_items * (rank + 1) // world
     t_lo = n_tx * rank // world
     t_hi = n_tx * (rank + 1) // world
-    s = seed if world == 1 else mix64(seed ^ rank)
     return Part(rank, world, lo, hi - lo, t_lo, t_hi - t_lo, s)
 
 

@@ -24,6 +24,17 @@ def test_partition_tiles_everything():
         P.partition(10, 10, 1, 2, 2)
 
 
+def test_weak_partition_fixes_per_rank_work():
+    for world in (1, 2, 4, 8):
+        parts = [P.partition(1 << 20, 1 << 24, 1, r, world, mode="weak") for r in range(world)]
+        assert all(p.n_items == 1 << 20 and p.n_tx == 1 << 24 for p in parts)
+        assert [p.item_lo for p in parts] == [r << 20 for r in range(world)]   # disjoint key ranges
+        assert len({p.seed for p in parts}) == world
+    assert P.partition(10, 10, 7, 0, 1, mode="weak").seed == 7
+    with pytest.raises(ValueError):
+        P.partition(10, 10, 1, 0, 1, mode="diagonal")
+
+
 def test_mix64_vector():
     assert P.mix64(0) == 0xE220A8397B1DCDAF
 
