@@ -122,6 +122,12 @@ typedef struct csmv_workload {
                                   server has answered the warp's batch -- rounds track the server
                                   round trip (timing-dependent schedule; 0 = fixed, deterministic) */
     uint32_t server_recv;      /* CSMV_RECV_*: how the server's worker warps get requests */
+    uint32_t client_group;     /* 0/1: one request per client warp (the paper's batch); G = 2, 4, 8:
+                                  the G client warps of a group (same CTA) pre-validate against each other
+                                  in shared memory (P:118 extended across warps) and submit ONE request of
+                                  up to 32G conflict-free transactions, committed in one step of the
+                                  critical section (CTA-level batch).  Bank, single-CTA ticket-locked
+                                  server with a receiver warp, item-indexed ATR, CSMV commit */
 } csmv_workload;
 
 /* ---- statistics ---- */

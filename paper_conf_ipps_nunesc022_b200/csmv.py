@@ -43,7 +43,7 @@ class _Workload(C.Structure):
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
         "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers", "server_combine",
         "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms", "commit",
-        "ro_adaptive", "server_recv")]
+        "ro_adaptive", "server_recv", "client_group")]
 
 
 class _Stats(C.Structure):
@@ -89,6 +89,7 @@ class Workload:
     commit: int = COMMIT_CSMV
     ro_adaptive: int = 0
     server_recv: int = 0
+    client_group: int = 0
 
     def to_c(self) -> _Workload:
         return _Workload(*[getattr(self, f.name) for f in fields(self)])

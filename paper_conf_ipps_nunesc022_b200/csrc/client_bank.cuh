@@ -78,12 +78,71 @@ __device__ __forceinline__ uint32_t jv_commit(const KParams& p, uint32_t s, uint
   return cts;
 }
 
+// ---------------------------------------------------------------------------
+// CTA-level batches (csmv_workload.client_group = G > 1).  The active client
+// warps of a CTA form groups of up to G warps (warps gG .. gG+G-1).  Each
+// round, after its own pre-validation, a warp publishes the kept
+// lanes' (src, dst) in shared memory; after a group barrier every lane that
+// is still kept checks them against the kept lanes of every lower warp of
+// its group and drops out (PREVAL) on any overlap -- a conservative greedy in
+// (warp, lane) order: the lower warps' sets are their own kept sets, so a
+// transaction may be dropped for a conflict with one that is itself dropped
+// (only an extra abort; the submitted batch is conflict-free either way).
+// Each warp still writes its own request slot; the group's first warp rings
+// ONE doorbell for all of them, and the server commits the whole group in
+// one step of its critical section (server_worker, G sub-batches probed
+// together) and answers each warp in its own response slot.  Group rounds
+// are lock-step: a named barrier (id 1 + g) at the top of the round (the
+// group continues while any warp has work, and stops on an error seen by
+// any), one after the kept sets are published, one after the payloads are
+// fenced.  Everything after that (read-only transactions, the response,
+// write-back, publish) is per warp as before.
+// ---------------------------------------------------------------------------
+struct Group {
+  uint32_t size = 1;     // warps in this warp's group (1: per-warp batches)
+  uint32_t pos = 0;      // this warp's position in it
+  uint32_t bar = 0;      // named barrier id
+  uint32_t* flags = nullptr;  // [size] per-warp words (top-of-round vote / kept masks)
+  uint2* ids = nullptr;       // [size][32] kept lanes' (src, dst)
+  __device__ __forceinline__ void sync() const {
+    asm volatile("bar.sync %0, %1;" ::"r"(bar), "r"(size * 32) : "memory");
+  }
+  // OR of `v` over the group's warps (lane 0 of each contributes)
+  __device__ __forceinline__ uint32_t vote_or(uint32_t v, uint32_t slot) const {
+    if ((threadIdx.x & 31) == 0) flags[slot * 8 + pos] = v;
+    sync();
+    uint32_t r = 0;
+    for (uint32_t k = 0; k < size; ++k) r |= ((volatile uint32_t*)flags)[slot * 8 + k];
+    return r;
+  }
+};
+
+__device__ __forceinline__ Group make_group(const KParams& p, uint8_t* smem) {
+  Group g;
+  const uint32_t G = p.group > 1 ? p.group : 1u;
+  if (G == 1) return g;
+  const uint32_t wib = threadIdx.x >> 5, cta = blockIdx.x - p.n_server_ctas;
+  // active warps of this CTA: w with w * n_client_ctas + cta < n_cw
+  uint32_t n_act = cta < p.n_cw ? (p.n_cw - cta + p.n_client_ctas - 1) / p.n_client_ctas : 0u;
+  if (n_act > (uint32_t)kWarps) n_act = kWarps;
+  const uint32_t gi = wib / G;
+  g.size = min(G, n_act - gi * G);
+  g.pos = wib % G;
+  g.bar = 1 + gi;
+  uint8_t* base = smem + (size_t)gi * (G * 32 * sizeof(uint2) + 3 * 8 * sizeof(uint32_t));
+  g.ids = reinterpret_cast<uint2*>(base);
+  g.flags = reinterpret_cast<uint32_t*>(base + G * 32 * sizeof(uint2));
+  return g;
+}
+
 template <int NS>
-__device__ void client_warp(const KParams& p, uint64_t t_begin) {
+__device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t cw = (threadIdx.x >> 5) * p.n_client_ctas + (blockIdx.x - p.n_server_ctas);
   if (cw >= p.n_cw) return;
+  const Group grp = make_group(p, smem);
+  const bool grouped = grp.size > 1;
   const uint64_t T = (uint64_t)p.n_cw * 32;
   uint64_t cu = kNoTx;                       // pending update
   uint64_t du_id = kNoTx;                    // cu's descriptor, drawn once (not every retry round)
@@ -100,7 +159,16 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
   Jitter jit(p, 1);
 
   for (;;) {
-    if (!__any_sync(FULL, cu != kNoTx || cr < p.n_tx)) break;
+    const bool work = __any_sync(FULL, cu != kNoTx || cr < p.n_tx);
+    if (grouped) {  // lock-step group round: go on while any warp has work, stop on any error
+      uint32_t e = 0;
+      if (lane == 0) e = ld_relaxed(&p.ctl->error);
+      e = __shfl_sync(FULL, e, 0);
+      const uint32_t v = grp.vote_or((work ? 1u : 0u) | (e ? 2u : 0u), 0);
+      if (v != 1u) break;
+    } else if (!work) {
+      break;
+    }
     pc.start();
     ++round;
     ++cc.n_rounds;
@@ -110,7 +178,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
       err = ld_relaxed(&p.ctl->error);
     }
     s = __shfl_sync(FULL, s, 0);
-    if (__shfl_sync(FULL, err, 0)) break;
+    if (!grouped && __shfl_sync(FULL, err, 0)) break;
 
     // ---- A: the pending update reads at s
     int status = ST_NONE;
@@ -204,10 +272,56 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         rem &= ~__ballot_sync(FULL, conf) & ~(1u << i);
       }
     }
+    uint32_t gkept = kept;  // grouped: the group submits iff any of its warps kept a lane
+    uint32_t watch = cw;    // the response slot that tells the read-only run the batch is answered
+    if (grouped) {
+      // cross-warp pre-validation against the kept lanes of the lower warps
+      grp.ids[grp.pos * 32 + lane] = make_uint2(d.src, d.dst);
+      grp.vote_or(kept, 1);  // publishes `kept` in flags[8 + pos]; the barrier orders the ids too
+      bool conf = false;
+      if ((kept >> lane) & 1u) {
+        for (uint32_t w = 0; w < grp.pos; ++w) {
+          uint32_t mk = ((volatile uint32_t*)grp.flags)[8 + w];
+          while (mk) {
+            const uint32_t j = __ffs(mk) - 1;
+            mk &= mk - 1;
+            const uint2 o = grp.ids[w * 32 + j];
+            conf |= d.src == o.x || d.src == o.y || d.dst == o.x || d.dst == o.y;
+          }
+        }
+      }
+      kept &= ~__ballot_sync(FULL, conf);
+    }
     const bool mine = (kept >> lane) & 1u;
     if (status == ST_CAND && !mine) cc.abort(CSMV_AB_PREVAL, true);
     if (p.commit != CSMV_COMMIT_JVSTM) pc.mark(PH_PREVAL);
-    if (kept) {
+    if (grouped) {
+      // every warp writes its header (mask possibly 0: the server reads all G
+      // slots of a group); the first warp rings the group's doorbell after
+      // every payload is fenced
+      if (mine) {
+        my_ids[lane] = d.src | kWriteBit;
+        my_ids[32 + lane] = d.dst | kWriteBit;
+      }
+      if (lane == 0) {
+        p.req_hdr[cw].snapshot = s;
+        p.req_hdr[cw].mask = kept;
+        p.req_hdr[cw].round = round;
+      }
+      __syncwarp();
+      fence_gpu();
+      gkept = grp.vote_or(kept, 2);
+      // the server answers the warps that submitted something; all warps of
+      // the group watch the first of them, so their rounds stay aligned
+      for (uint32_t k = 0; k < grp.size; ++k)
+        if (((volatile uint32_t*)grp.flags)[16 + k]) {
+          watch = cw + (k - grp.pos) * p.n_client_ctas;
+          break;
+        }
+      jit();  // payloads written, doorbell not yet
+      if (gkept && grp.pos == 0 && lane == 0) st_relaxed(&p.req_seq[cw], round);
+      pc.mark(PH_SUBMIT);
+    } else if (kept) {
       if (mine) {
         my_ids[lane] = d.src | kWriteBit;
         my_ids[32 + lane] = d.dst | kWriteBit;
@@ -263,12 +377,12 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin) {
         }
         run = run && has;
         // ro_adaptive: the batch has been answered -> finish the round
-        if (p.ro_adaptive && kept && (uint32_t)(warp_ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
+        if (p.ro_adaptive && gkept && (uint32_t)(warp_ld_relaxed64(&p.resp[watch].base) >> 32) == round) break;
       }
     }
     __syncwarp();
     pc.mark(PH_ROT);
-    if (!kept) continue;
+    if (!kept) continue;  // grouped: the server answers only the warps that submitted something
 
     // ---- D: the server's answer, write-back, GTS
     uint32_t base = 0, cmask = 0, omask = 0;

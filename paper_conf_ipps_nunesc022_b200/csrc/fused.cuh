@@ -408,7 +408,7 @@ __global__ void __launch_bounds__(kBlock, 1) csmv_fused(const KParams p) {
   const uint64_t t_begin = globaltimer();
   if (blockIdx.x < p.n_server_ctas) server_cta<NS, KIND, CL>(p, smem, t_begin);
   else if constexpr (KIND == CSMV_KIND_KV) client_warp_kv<NS>(p, t_begin, reinterpret_cast<uint32_t*>(smem));
-  else client_warp<NS>(p, t_begin);
+  else client_warp<NS>(p, t_begin, smem);
 }
 
 template <int NS, int KIND, bool CL>

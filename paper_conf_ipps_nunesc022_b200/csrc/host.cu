@@ -58,8 +58,6 @@ std::vector<uint64_t> build_zipf(uint32_t n, uint32_t theta_milli) {
 
 uint32_t nslot_for(uint32_t k) { return k <= 2 ? 2 : k <= 4 ? 4 : k <= 8 ? 8 : 16; }
 
-uint64_t umulhi(uint64_t a, uint64_t b) { return (uint64_t)(((unsigned __int128)a * b) >> 64); }
-
 }  // namespace
 
 struct csmv {
@@ -408,6 +406,14 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
     n_workers = w->server_workers ? w->server_workers : 4u;
     if (n_workers > kWarps - 1) n_workers = kWarps - 1;
   }
+  // CTA-level batches: G client warps of one CTA per request
+  const uint32_t group = w->client_group ? w->client_group : 1u;
+  if (group != 1 && group != 2 && group != 4 && group != 8)
+    return set_err(CSMV_EINVAL, "csmv_run: client_group must be 1, 2, 4 or 8");
+  if (group > 1 && (h->kind != CSMV_KIND_BANK || w->server != CSMV_SERVER_CTA || w->atr_mode != CSMV_ATR_HASH ||
+                    w->commit != CSMV_COMMIT_CSMV || selfrecv || cmring))
+    return set_err(CSMV_EINVAL, "csmv_run: client_group > 1 needs the bank workload on the single-CTA "
+                                "ticket-locked server with a receiver warp (atr_mode HASH, CSMV commit)");
   uint32_t n_cw = w->client_warps ? w->client_warps : h->max_cw;
   if (n_cw > h->max_cw) n_cw = h->max_cw;
   if (n_cw == 0) return set_err(CSMV_EINVAL, "csmv_run: no client warps");
@@ -514,6 +520,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.commit = w->commit;
   p.ro_adaptive = w->ro_adaptive;
   p.server_recv = w->server_recv;
+  p.group = group;
   p.req_vals = h->d_req_vals;
   p.jv_ws = h->d_jv_ws;
   p.jv_tag = h->d_jv_tag;

@@ -141,6 +141,7 @@ struct KParams {
   uint32_t commit;
   uint32_t ro_adaptive;       // stop a read-only run once the server has answered
   uint32_t server_recv;       // CSMV_RECV_*
+  uint32_t group;             // client warps per request (1 = per-warp batches; 2/4/8 = CTA-level batches)
   uint32_t* req_vals;         // ONLYCS: new values [n_cw][2][32] for the server-side write-back
   uint64_t* jv_ws;            // JVSTM: global ATR, write-set of CTS c at c & (2^jv_log2 - 1)
   uint32_t* jv_tag;           //        entry tag = c once the record of c is written

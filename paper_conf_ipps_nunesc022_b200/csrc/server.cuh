@@ -533,15 +533,27 @@ __device__ __forceinline__ uint32_t self_claim(const KParams& p, const SrvCtx& c
 // validated after batch j-1's write-set was recorded, and receives the next
 // consecutive CTS range.  A batch is validated by the whole warp,
 // one lane per transaction, __ballot_sync for the commit mask.
+//
+// G > 1 (csmv_workload.client_group, CTA-level batches): a request is the
+// G sub-batches of a client group (client_bank.cuh), mutually conflict-free
+// by the clients' cross-warp pre-validation.  Up to M/G requests are combined;
+// within one, the G sub-batches' filter probes are issued together and
+// evaluated against the same window (none can conflict with another), their
+// CTS ranges follow one another in warp order, and their filter slots are
+// stored once with the request's last CTS: one step of the serial chain per
+// request instead of one per sub-batch.
 // ---------------------------------------------------------------------------
-template <bool CL, bool SELF>
+template <bool CL, bool SELF, int G = 1>
 __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
   constexpr int M = kMaxCombine;
+  constexpr int MR = M / G;  // requests per critical section
+  static_assert(!SELF || G == 1, "self-receiving workers take per-warp batches");
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t lt = lanemask_lt();
   const uint32_t qmask = (1u << c.qn_log2) - 1;
-  const uint32_t m_max = p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine);
+  const uint32_t m_max = G > 1 ? max(1u, min(p.combine, (uint32_t)M) / G)
+                              : (p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine));
   unsigned long long busy = 0, locked = 0, batches = 0, groups = 0;
   unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   constexpr bool self = SELF;
@@ -564,7 +576,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     }
     // ---- combine: grab further requests that are already queued
 #pragma unroll
-    for (int j = 1; j < M; ++j) {
+    for (int j = 1; j < MR; ++j) {
       uint32_t got = 0xFFFFFFFFu;
       if (!self && m == (uint32_t)j && m < m_max && lane == 0) {
         const uint32_t h = *(volatile uint32_t*)&c.sh->q_head;
@@ -576,6 +588,21 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       cwv[j] = got;
       if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
     }
+    const uint32_t m_req = m;
+    if constexpr (G > 1) {
+      // expand request r (its group's first warp) into sub-batches r*G + k:
+      // the group's warps lead + k * n_client_ctas, as many as the CTA has
+#pragma unroll
+      for (int r = MR - 1; r >= 0; --r) {
+        const uint32_t lead = cwv[r], cta = lead % p.n_client_ctas, w0 = lead / p.n_client_ctas;
+        const uint32_t n_act = min((uint32_t)kWarps, (p.n_cw - cta + p.n_client_ctas - 1) / p.n_client_ctas);
+        const uint32_t gs = min((uint32_t)G, n_act - w0);
+#pragma unroll
+        for (int k = 0; k < G; ++k)
+          cwv[r * G + k] = ((uint32_t)r < m_req && (uint32_t)k < gs) ? lead + k * p.n_client_ctas : 0xFFFFFFFFu;
+      }
+      m = m_req * G;
+    }
     const long long t0 = clock64();
     jit();  // claimed, payload not yet loaded
     // ---- load the batches: header and ids together (the receiver's fence
@@ -585,7 +612,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
 #pragma unroll
     for (int j = 0; j < M; ++j) {
       sq[j] = sn[j] = msk[j] = id0[j] = id1[j] = 0;
-      if (j < (int)m) {
+      if (j < (int)m && (G == 1 || cwv[j] != 0xFFFFFFFFu)) {
         sn[j] = ld_relaxed(&p.req_hdr[cwv[j]].snapshot);
         msk[j] = ld_relaxed(&p.req_hdr[cwv[j]].mask);
         sq[j] = ld_relaxed(&p.req_hdr[cwv[j]].round);
@@ -599,7 +626,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       mine[j] = (msk[j] >> lane) & 1u;
       if (!mine[j]) id0[j] = id1[j] = 0;
     }
-    const bool hash = p.atr_mode == CSMV_ATR_HASH;
+    const bool hash = G > 1 || p.atr_mode == CSMV_ATR_HASH;
     // lastw covers every CTS <= e_pre: clients write lastw with their
     // write-back, before the commit is published, so e_pre = GTS (acquire)
     const uint32_t e_pre = hash ? ld_acquire(p.gts) : *(volatile uint32_t*)&c.sh0->tail;
@@ -653,43 +680,62 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     uint32_t cm[M], om[M], base[M];
     bool ovfl[M];
     if (hash) {
-      // batch j: a write after e_pre to one of its items raised all of that
-      // item's slots above e_pre (earlier batches of this section included)
+      // request r (sub-batches r*G .. r*G+G-1): a write after e_pre to one of
+      // its items raised all of that item's slots above e_pre (earlier
+      // requests of this section included; the sub-batches of one request
+      // are conflict-free, so they need not see each other's stores)
 #pragma unroll
-      for (int j = 0; j < M; ++j) {
-        cm[j] = om[j] = 0;
-        ovfl[j] = false;
-        base[j] = t + 1;
-        if (j < (int)m) {
-          uint32_t va[kFiltK] = {0u, 0u, 0u}, vb[kFiltK] = {0u, 0u, 0u};
-          if (chk[j]) {
+      for (int r = 0; r < MR; ++r) {
+        uint32_t va[G][kFiltK], vb[G][kFiltK];
+        bool cmt[G];
 #pragma unroll
-            for (int k = 0; k < kBankFiltK; ++k) {
-              va[k] = filt16_ld<CL>(fa[j][k]);
-              vb[k] = filt16_ld<CL>(fb[j][k]);
+        for (int k = 0; k < G; ++k) {
+          const int j = r * G + k;
+          cm[j] = om[j] = 0;
+          ovfl[j] = false;
+          base[j] = t + 1;
+          cmt[k] = false;
+#pragma unroll
+          for (int q = 0; q < kFiltK; ++q) va[k][q] = vb[k][q] = 0u;
+          if ((uint32_t)r < m_req && chk[j]) {
+#pragma unroll
+            for (int q = 0; q < kBankFiltK; ++q) {
+              va[k][q] = filt16_ld<CL>(fa[j][q]);
+              vb[k][q] = filt16_ld<CL>(fb[j][q]);
             }
           }
+        }
+        if ((uint32_t)r < m_req) {
           // slot v is recent iff its CTS lies in (e_pre, t]: (v - e_pre - 1) mod 2^16 < t - e_pre
           const uint32_t win = t - e_pre;  // commits the exact lastw check did not cover
-          bool ra = true, rb = true;
 #pragma unroll
-          for (int k = 0; k < kBankFiltK; ++k) {
-            ra = ra && ((va[k] - e_pre - 1u) & 0xFFFFu) < win;
-            rb = rb && ((vb[k] - e_pre - 1u) & 0xFFFFu) < win;
+          for (int k = 0; k < G; ++k) {
+            const int j = r * G + k;
+            bool ra = true, rb = true;
+#pragma unroll
+            for (int q = 0; q < kBankFiltK; ++q) {
+              ra = ra && ((va[k][q] - e_pre - 1u) & 0xFFFFu) < win;
+              rb = rb && ((vb[k][q] - e_pre - 1u) & 0xFFFFu) < win;
+            }
+            const bool ovf = chk[j] && !novalid && (win > 0xFFFFu || ra || rb);
+            cmt[k] = chk[j] && !ovf;
+            cm[j] = __ballot_sync(FULL, cmt[k]);
+            ovfl[j] = ovf;  // the overflow mask is voted after the lock
+            base[j] = t + 1;
+            t += __popc(cm[j]);
           }
-          const bool ovf = chk[j] && !novalid && (win > 0xFFFFu || ra || rb);
-          const bool commit = chk[j] && !ovf;
-          cm[j] = __ballot_sync(FULL, commit);
-          ovfl[j] = ovf;  // the overflow mask is voted after the lock
-          t += __popc(cm[j]);
-          if (commit) {
 #pragma unroll
-            for (int k = 0; k < kBankFiltK; ++k) {  // the batch's last CTS: equal values, race-free
-              filt16_st<CL>(fa[j][k], t);
-              filt16_st<CL>(fb[j][k], t);
+          for (int k = 0; k < G; ++k) {
+            const int j = r * G + k;
+            if (cmt[k]) {
+#pragma unroll
+              for (int q = 0; q < kBankFiltK; ++q) {  // the request's last CTS: equal values, race-free
+                filt16_st<CL>(fa[j][q], t);
+                filt16_st<CL>(fb[j][q], t);
+              }
             }
           }
-          __syncwarp();  // batch j's records precede batch j+1's probes
+          __syncwarp();  // request r's records precede request r+1's probes
         }
       }
     } else {
@@ -719,11 +765,13 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
 #pragma unroll
       for (int j = 0; j < M; ++j) om[j] = __ballot_sync(FULL, ovfl[j]);
     }
-    // ---- respond: round-tagged words, no fence (kernel.cuh Resp)
+    // ---- respond: round-tagged words, no fence (kernel.cuh Resp);
+    // only to warps that submitted something (a grouped warp with mask 0
+    // waits for nothing, and a late word could land on its next request)
     if (lane < (uint32_t)m) {
 #pragma unroll
       for (int j = 0; j < M; ++j) {
-        if ((uint32_t)j == lane) {
+        if ((uint32_t)j == lane && msk[j] != 0) {
           const uint64_t tag = (uint64_t)sq[j] << 32;
           st_relaxed64(&p.resp[cwv[j]].base, tag | base[j]);
           st_relaxed64(&p.resp[cwv[j]].commit, tag | cm[j]);
@@ -741,7 +789,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     ph[3] += (unsigned long long)(t2 - t1);
     ph[4] += (unsigned long long)(t3 - t2);
     ph[5] += (unsigned long long)(ta - t1);
-    batches += m;
+    batches += m_req;
     ++groups;
   }
   if (lane == 0) {
@@ -1475,6 +1523,9 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     }
     else if (!CL && p.commit == CSMV_COMMIT_ONLYCS) server_worker_onlycs<NS>(p, c, t_begin);
     else if (cmring) server_worker_cm<CL>(p, c, t_begin);
+    else if (!CL && p.group == 2) server_worker<CL, false, 2>(p, c, t_begin);
+    else if (!CL && p.group == 4) server_worker<CL, false, 4>(p, c, t_begin);
+    else if (!CL && p.group == 8) server_worker<CL, false, 8>(p, c, t_begin);
     else server_worker<CL, false>(p, c, t_begin);
   } else if (warp == p.n_workers + 1 && rank == 0 && p.publish == CSMV_PUBLISH_SERVER) {
     server_publisher(p, c, t_begin);
