@@ -46,16 +46,30 @@ if ROOT not in sys.path:
 METRIC = "committed tx/sec and abort rate at 1 B200 (+partitioned 2/4/8)"
 UNIT = "tx/s"
 
-# tuned launch configuration of the C2 workload
-TUNED = dict(client_warps_per_sm=2, server_workers=6, server_combine=8, ro_streak=8, publish=1, ro_adaptive=1,
-             server_recv=0)
+# tuned launch configuration of the C2 workload: 4 client warps
+# per SM submitting CTA-level batches of 4 warps (client_group, 355 -> 490 M
+# tx/s with the 2-hash filter, profiles/r02/tune_group.md)
+TUNED = dict(client_warps_per_sm=4, client_group=4, server_workers=6, server_combine=8, ro_streak=8, publish=1,
+             ro_adaptive=1, server_recv=0)
 # per-workload overrides of the tuned launch (tools/tune.py on B200): the hot-item
 # chains of C3 want the lower-latency self-receiving server combining at most 2
 # batches per critical section (3.3M -> 4.5M tx/s against 8) and the clients'
 # own ordered GTS publish (no publisher hop on the chain: 4.4M -> 5.0M), the PUT
-# convoys of C4 longer read-only runs ahead of a blocked PUT
-TUNED_PER_CONFIG = {"C3": dict(server_recv=1, server_workers=7, server_combine=2, publish=0),
-                    "C4": dict(ro_streak=32)}
+# convoys of C4 longer read-only runs ahead of a blocked PUT; both keep per-warp
+# batches (the self-receiving server and the KV workload take no groups)
+TUNED_PER_CONFIG = {"C3": dict(server_recv=1, server_workers=7, server_combine=2, publish=0, client_warps_per_sm=2,
+                               client_group=1),
+                    "C4": dict(ro_streak=32, client_warps_per_sm=2, client_group=1)}
+
+
+def tuned(config: str) -> dict:
+    return dict(TUNED, **TUNED_PER_CONFIG.get(config, {}))
+
+
+def tuned_client_warps(config: str, sms: int) -> int:
+    """client warps of the tuned launch: every SM but the server's hosts
+    client_warps_per_sm of them."""
+    return tuned(config)["client_warps_per_sm"] * (sms - 1)
 
 # algorithmic bytes (SURVEY 8(d), paper VBox layout P:289): a read moves the
 # VBox head, the visited version's ts and the value (4+4+4); a write-back the
@@ -231,10 +245,10 @@ def make_cfg(args, world: int, rank: int):
     from paper_conf_ipps_nunesc022_b200 import partition, workloads
     cfg = workloads.PRESETS[args.config]()
     n_tx = args.n_tx or cfg.n_tx
-    t = dict(TUNED, **TUNED_PER_CONFIG.get(args.config, {}))
+    t = tuned(args.config)
     cfg = cfg.with_(n_tx=n_tx, log_mode=0, ro_streak=t["ro_streak"], publish=t["publish"],
                     server_workers=t["server_workers"], server_combine=t["server_combine"],
-                    ro_adaptive=t["ro_adaptive"], server_recv=t["server_recv"])
+                    ro_adaptive=t["ro_adaptive"], server_recv=t["server_recv"], client_group=t["client_group"])
     part = partition.partition(cfg.n_items, n_tx, cfg.seed, rank, world, mode="weak")
     lcfg = partition.local_config(cfg, part)
     return cfg, lcfg, part
@@ -358,7 +372,7 @@ def bench_ours(args):
     cfg, lcfg, part = make_cfg(args, world, rank)
     props = torch.cuda.get_device_properties(dev)
     n_cw = args.client_warps or lcfg.workload.client_warps or \
-        TUNED["client_warps_per_sm"] * (props.multi_processor_count - 1)
+        tuned_client_warps(args.config, props.multi_processor_count)
     lcfg = lcfg.with_(client_warps=n_cw)
     w = lcfg.workload
     is_kv = w.kind == csmv.KIND_KV
@@ -449,7 +463,7 @@ def bench_ours(args):
         "config": {"workload": DESCR.get(cfg.name, cfg.name),
                    "n_items_per_gpu": lcfg.n_items, "n_items_job": lcfg.n_items * world,
                    "n_versions": cfg.n_versions, "n_tx_per_step_per_gpu": lcfg.n_tx,
-                   "client_warps_per_gpu": n_cw, "server_workers": w.server_workers,
+                   "client_warps_per_gpu": n_cw, "client_group": w.client_group, "server_workers": w.server_workers,
                    "server_combine": w.server_combine,
                    "ro_streak": w.ro_streak, "ro_adaptive": w.ro_adaptive, "publish": ["client", "server"][w.publish],
                    "server_recv": ["receiver warp", "self-receiving workers"][w.server_recv],

@@ -199,7 +199,7 @@ __device__ __forceinline__ void rt_record(const SrvCtx& c, uint32_t bucket, int 
 // ---------------------------------------------------------------------------
 constexpr int kFiltK = 3;
 #ifndef CSMV_BANK_FILT_K
-#define CSMV_BANK_FILT_K 3
+#define CSMV_BANK_FILT_K 2
 #endif
 constexpr int kBankFiltK = CSMV_BANK_FILT_K;  // hashes the locked bank worker uses (<= kFiltK)
 static_assert(kBankFiltK >= 1 && kBankFiltK <= kFiltK, "CSMV_BANK_FILT_K must be 1..kFiltK");
@@ -543,6 +543,11 @@ __device__ __forceinline__ uint32_t self_claim(const KParams& p, const SrvCtx& c
 // stored once with the request's last CTS: one step of the serial chain per
 // request instead of one per sub-batch.
 // ---------------------------------------------------------------------------
+#ifndef CSMV_LASTW_ONE_TRIP
+#define CSMV_LASTW_ONE_TRIP 1
+#endif
+constexpr bool kLastwOneTrip = CSMV_LASTW_ONE_TRIP;  // grouped requests: every lastw load of a group in flight at once
+
 template <bool CL, bool SELF, int G = 1>
 __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
   constexpr int M = kMaxCombine;
@@ -647,7 +652,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
 #pragma unroll
     for (int j = 0; j < M; ++j) {
       lwa[j] = lwb[j] = 0;
-      if (SELF && hash) {
+      if ((SELF || (G > 1 && kLastwOneTrip)) && hash) {
         lwa[j] = ld_relaxed(p.lastw + id0[j]);
         lwb[j] = ld_relaxed(p.lastw + id1[j]);
       }
@@ -655,7 +660,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
 #pragma unroll
     for (int j = 0; j < M; ++j) {
       uint32_t lw0 = lwa[j], lw1 = lwb[j];
-      if (!SELF && mine[j] && hash) {
+      if (!(SELF || (G > 1 && kLastwOneTrip)) && mine[j] && hash) {
         lw0 = ld_relaxed(p.lastw + id0[j]);
         lw1 = ld_relaxed(p.lastw + id1[j]);
       }

@@ -26,7 +26,7 @@ from tests.test_gpu_parity import oracle_cfg  # noqa: E402
 def bench_cfg(name, n_tx=0):
     _, lcfg, _ = bench.make_cfg(types.SimpleNamespace(config=name, n_tx=n_tx), 1, 0)
     sms = torch.cuda.get_device_properties(0).multi_processor_count
-    return lcfg.with_(client_warps=bench.TUNED["client_warps_per_sm"] * (sms - 1), log_mode=csmv.LOG_DIGEST)
+    return lcfg.with_(client_warps=bench.tuned_client_warps(name, sms), log_mode=csmv.LOG_DIGEST)
 
 
 @pytest.mark.parametrize("name", ["C2", "C3"])
