@@ -86,6 +86,10 @@ extern "C" {
                                    ticket-locked critical section, the cluster server the other way
                                    round; A/B only */
 
+#define CSMV_DBG_TRACE 64u     /* hot-chain trace: every committed update that writes csmv_workload.
+                                   trace_item (bank: an account; KV: a set) logs a csmv_trace_rec with
+                                   device-wide timestamps (globaltimer) -- csmv_get_trace */
+
 #define CSMV_RECV_WARP 0u       /* a receiver warp sweeps the doorbells into a shared-memory dispatch
                                    queue; combining fills larger batches */
 #define CSMV_RECV_SELF 1u       /* bank, single-CTA locked commit: every worker warp sweeps its own
@@ -120,7 +124,9 @@ typedef struct csmv_workload {
     uint32_t commit;           /* CSMV_COMMIT_* (0 = the paper's CSMV) */
     uint32_t ro_adaptive;      /* 1: a lane stops its read-only run (at most ro_streak) as soon as the
                                   server has answered the warp's batch -- rounds track the server
-                                  round trip (timing-dependent schedule; 0 = fixed, deterministic) */
+                                  round trip (timing-dependent schedule; 0 = fixed, deterministic);
+                                  2 (KV): also when the warp submitted nothing because its PUTs met
+                                  versions newer than the snapshot, once GTS covers them */
     uint32_t server_recv;      /* CSMV_RECV_*: how the server's worker warps get requests */
     uint32_t client_group;     /* 0/1: one request per client warp (the paper's batch); G = 2, 4, 8:
                                   the G client warps of a group (same CTA) pre-validate against each other
@@ -128,6 +134,8 @@ typedef struct csmv_workload {
                                   up to 32G conflict-free transactions, committed in one step of the
                                   critical section (CTA-level batch).  Bank, single-CTA ticket-locked
                                   server with a receiver warp, item-indexed ATR, CSMV commit */
+    uint32_t trace_item;       /* CSMV_DBG_TRACE: bank account / KV set whose committed writers are traced;
+                                  0xFFFFFFFF = the hottest (account 0 / the set of key 0: zipf rank 0) */
 } csmv_workload;
 
 /* ---- statistics ---- */
@@ -172,6 +180,15 @@ typedef struct csmv_log_rec {
     uint32_t tx, snapshot, cts, attempts;
     uint64_t read_digest, aux;
 } csmv_log_rec;
+
+/* CSMV_DBG_TRACE record of one committed update writing the traced item:
+ * its commit timestamp and snapshot, and globaltimer (ns, device-wide) at
+ * the start of the client round (TXBegin), the doorbell, the response and
+ * the end of its publish step (GTS advanced, or done flag stored). */
+typedef struct csmv_trace_rec {
+    uint32_t cts, snapshot;
+    uint64_t t_begin, t_submit, t_response, t_publish;
+} csmv_trace_rec;
 
 typedef struct csmv csmv_t;
 
@@ -237,6 +254,13 @@ int csmv_dump_kv(const csmv_t *h, uint32_t *keys, uint32_t *vals, uint32_t *lru,
  * generator parity check. */
 int csmv_gen_descs(csmv_t *h, const csmv_workload *w, uint64_t seed, uint64_t tx0,
                    uint64_t n, uint32_t *out);
+
+/* CSMV_DBG_TRACE records of the last csmv_run (in completion order, at
+ * most 2^18): copies min(cap, recorded) into buf; *n_out = records
+ * recorded (may exceed cap).  ESTATE if the last run was not traced.
+ * Diagnostic of the hot-item commit chain (every writer of
+ * an item commits and publishes after the previous one). */
+int csmv_get_trace(const csmv_t *h, csmv_trace_rec *buf, uint64_t cap, uint64_t *n_out);
 
 /* The zipf CDF table the library built for (n, theta_milli). */
 int csmv_zipf_table(uint32_t n, uint32_t theta_milli, uint64_t *out);

@@ -23,11 +23,13 @@ SERVER_CTA, SERVER_CLUSTER = 0, 1
 PUBLISH_CLIENT, PUBLISH_SERVER = 0, 1
 ATR_HASH, ATR_LIST, ATR_LIST_NOCV = 0, 1, 2
 COMMIT_CSMV, COMMIT_ONLYCS, COMMIT_JVSTM = 0, 1, 2
-DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER, DBG_PHASES, DBG_KV_ITEMSETS, DBG_ALT_COMMIT = 1, 2, 4, 8, 16, 32
+DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER, DBG_PHASES, DBG_KV_ITEMSETS, DBG_ALT_COMMIT, DBG_TRACE = 1, 2, 4, 8, 16, 32, 64
 RECV_WARP, RECV_SELF = 0, 1
 CLIENT_PHASES = ("read", "preval", "submit", "rot", "wait_server", "writeback", "publish", "divergence")
 ABORT_REASONS = ("preval", "conflict", "early", "overflow", "version")
 
+TRACE_DTYPE = np.dtype([("cts", "<u4"), ("snapshot", "<u4"), ("t_begin", "<u8"), ("t_submit", "<u8"),
+                        ("t_response", "<u8"), ("t_publish", "<u8")])
 LOG_DTYPE = np.dtype([("tx", "<u4"), ("snapshot", "<u4"), ("cts", "<u4"),
                       ("attempts", "<u4"), ("read_digest", "<u8"), ("aux", "<u8")])
 
@@ -43,7 +45,7 @@ class _Workload(C.Structure):
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
         "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers", "server_combine",
         "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms", "commit",
-        "ro_adaptive", "server_recv", "client_group")]
+        "ro_adaptive", "server_recv", "client_group", "trace_item")]
 
 
 class _Stats(C.Structure):
@@ -90,6 +92,7 @@ class Workload:
     ro_adaptive: int = 0
     server_recv: int = 0
     client_group: int = 0
+    trace_item: int = 0xFFFFFFFF
 
     def to_c(self) -> _Workload:
         return _Workload(*[getattr(self, f.name) for f in fields(self)])
@@ -125,6 +128,7 @@ def lib() -> C.CDLL:
     L.csmv_dump_kv.argtypes = [vp, vp, vp, vp, vp]
     L.csmv_gen_descs.argtypes = [vp, C.POINTER(_Workload), u64, u64, u64, vp]
     L.csmv_zipf_table.argtypes = [u32, u32, vp]
+    L.csmv_get_trace.argtypes = [vp, vp, u64, C.POINTER(u64)]
     L.csmv_destroy.argtypes = [vp]
     L.csmv_destroy.restype = None
     _lib = L
@@ -213,6 +217,13 @@ class Store:
         out = np.zeros(n * mv.value, dtype=np.uint32)
         _check(lib().csmv_get_vals(self.h, _ptr(out), out.size, C.byref(mv)))
         return out, mv.value
+
+    def trace(self, cap: int = 1 << 18) -> np.ndarray:
+        """CSMV_DBG_TRACE records of the last run (csmv_get_trace)."""
+        out = np.zeros(cap, dtype=TRACE_DTYPE)
+        n = C.c_uint64()
+        _check(lib().csmv_get_trace(self.h, _ptr(out), cap, C.byref(n)))
+        return out[: min(cap, n.value)]
 
     def dump(self) -> np.ndarray:
         out = np.zeros(self.n_items * self.n_versions, dtype=np.uint64)

@@ -157,6 +157,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
   const uint32_t streak = p.ro_streak;
   PhaseClock pc((p.debug & CSMV_DBG_PHASES) != 0);
   Jitter jit(p, 1);
+  const bool tracing = (p.debug & CSMV_DBG_TRACE) != 0;
 
   for (;;) {
     const bool work = __any_sync(FULL, cu != kNoTx || cr < p.n_tx);
@@ -172,6 +173,8 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
     pc.start();
     ++round;
     ++cc.n_rounds;
+    const uint64_t t_rb = tracing ? globaltimer() : 0;
+    uint64_t t_sub = 0;
     uint32_t s = 0, err = 0;
     if (lane == 0) {
       s = ld_acquire(p.gts);  // TXBegin: snapshot
@@ -320,6 +323,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
         }
       jit();  // payloads written, doorbell not yet
       if (gkept && grp.pos == 0 && lane == 0) st_relaxed(&p.req_seq[cw], round);
+      if (tracing) t_sub = globaltimer();
       pc.mark(PH_SUBMIT);
     } else if (kept) {
       if (mine) {
@@ -339,8 +343,97 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       fence_gpu();
       jit();  // payload written, doorbell not yet
       if (lane == 0) st_relaxed(&p.req_seq[cw], round);
+      if (tracing) t_sub = globaltimer();
       pc.mark(PH_SUBMIT);
     }
+
+    // ---- D (as a step callable from inside C): the server's answer
+    // (P:101), client write-back, GTS.  With ro_adaptive the read-only
+    // phase polls for the answer at every row group and runs D right away,
+    // so a commit is written back and published about one L2 round trip
+    // after its answer instead of after the whole read-only phase -- the
+    // step every hot-item chain link waits for (tools/chain.py).  Not in
+    // the deterministic (fixed) mode: there D stays after C.
+    uint32_t cts = 0;
+    uint64_t t_resp = 0;
+    bool d_done = false;
+    auto phase_d = [&](uint32_t base, uint32_t cmask, uint32_t omask) {
+      t_resp = tracing ? globaltimer() : 0;
+      if (p.commit == CSMV_COMMIT_ONLYCS) fence_gpu();  // acquire: the server's write-backs
+      pc.mark(PH_WAIT);
+      jit();  // committed, versions not yet written back
+      if (mine) {
+        if ((cmask >> lane) & 1u) {
+          // Client-side write-back with CTS = base + rank.
+          cts = base + __popc(cmask & lt);
+          const uint32_t ns = vs - (uint32_t)d.amt, nd = vd + (uint32_t)d.amt;
+          if (p.commit != CSMV_COMMIT_ONLYCS) {
+            write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
+            write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
+            // lastw (the item-indexed ATR's exact level, server.cuh): written
+            // here, before this commit is published, so GTS = g implies lastw
+            // of every commit <= g.  Two commits writing one item are ordered
+            // (the later one's snapshot covers the earlier one), so plain
+            // stores leave lastw at the latest.
+            st_relaxed(p.lastw + d.src, cts);
+            st_relaxed(p.lastw + d.dst, cts);
+          }
+          if (p.log_mode) {
+            log_commit(p, cu, s, cts, att_u, dig1(d.src, vs) + dig1(d.dst, vd), dig1(d.src, ns) + dig1(d.dst, nd));
+            if (p.log_mode == CSMV_LOG_FULL && p.max_vals >= 2) {
+              p.vals[cu * p.max_vals] = vs;
+              p.vals[cu * p.max_vals + 1] = vd;
+            }
+          }
+          ++cc.c_upd;
+          cu = kNoTx;
+          att_u = 0;
+          n_srv_ab = 0;
+        } else {
+          const bool ovf = (omask >> lane) & 1u;
+          cc.abort(ovf ? CSMV_AB_OVERFLOW : CSMV_AB_CONFLICT, true);
+          if (!ovf && p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
+        }
+      }
+      __syncwarp();
+      pc.mark(PH_WRITEBACK);
+      const uint32_t n = __popc(cmask);
+      if (n) {
+        jit();  // write-backs done, commit not yet published
+        if (p.publish == CSMV_PUBLISH_CLIENT) {
+          // Advance GTS by n once every earlier commit is visible:
+          // spin until GTS == first CTS - 1 ("GTS 1" = GTS+1).
+          __syncwarp();
+          fence_gpu();
+          uint32_t it = 0;
+          while (warp_ld_relaxed(p.gts) != base - 1) {
+            if ((++it & 255u) == 0) {
+              uint32_t bad = 0;
+              if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 2);
+              if (__shfl_sync(FULL, bad, 0)) break;
+            }
+            __nanosleep(CSMV_SLEEP_PUB);
+          }
+          if (lane == 0) st_release(p.gts, base + n - 1);  // release also orders the write-backs
+        } else if (cts && p.commit != CSMV_COMMIT_ONLYCS) {
+          st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
+        }
+      }
+      pc.mark(PH_PUBLISH);
+      d_done = true;
+    };
+    const bool early_d = p.ro_adaptive && kept && p.commit == CSMV_COMMIT_CSMV;
+    // the response's first word is prefetched by lane 0 one row group ahead
+    // (its latency hides behind the group's own loads)
+    uint64_t pf = 0;
+    auto poll = [&]() {
+      if (!early_d || d_done) return;
+      uint32_t b0, c0, o0;
+      if (__shfl_sync(FULL, (uint32_t)(pf >> 32), 0) == round && try_response(p, cw, round, b0, c0, o0))
+        phase_d(b0, c0, o0);
+      else if (lane == 0)
+        pf = ld_relaxed64(&p.resp[cw].base);
+    };
 
     // ---- C: read-only transactions at s.  A lane runs
     // its next read-only transactions up to the next update (at most
@@ -362,7 +455,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
         bool ok;
         int64_t rsum;
         uint64_t rdig;
-        rot_coop<NS>(p, act, r.start, r.len, s, cr, ok, rsum, rdig);
+        rot_coop<NS>(p, act, r.start, r.len, s, cr, ok, rsum, rdig, poll);
         if (has) {
           if (ok) {
             if (p.log_mode) log_commit(p, cr, s, 0, att_r, rdig, (uint64_t)rsum);
@@ -377,78 +470,21 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
         }
         run = run && has;
         // ro_adaptive: the batch has been answered -> finish the round
-        if (p.ro_adaptive && gkept && (uint32_t)(warp_ld_relaxed64(&p.resp[watch].base) >> 32) == round) break;
+        if (p.ro_adaptive && gkept && (d_done || (uint32_t)(warp_ld_relaxed64(&p.resp[watch].base) >> 32) == round)) break;
       }
     }
     __syncwarp();
     pc.mark(PH_ROT);
     if (!kept) continue;  // grouped: the server answers only the warps that submitted something
 
-    // ---- D: the server's answer, write-back, GTS
-    uint32_t base = 0, cmask = 0, omask = 0;
-    wait_response(p, cw, round, t_begin, base, cmask, omask, jit);
-    if (p.commit == CSMV_COMMIT_ONLYCS) fence_gpu();  // acquire: the server's write-backs
-    pc.mark(PH_WAIT);
-    uint32_t cts = 0;
-    jit();  // committed, versions not yet written back
-    if (mine) {
-      if ((cmask >> lane) & 1u) {
-        // Client-side write-back with CTS = base + rank.
-        cts = base + __popc(cmask & lt);
-        const uint32_t ns = vs - (uint32_t)d.amt, nd = vd + (uint32_t)d.amt;
-        if (p.commit != CSMV_COMMIT_ONLYCS) {
-          write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
-          write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
-          // lastw (the item-indexed ATR's exact level, server.cuh): written
-          // here, before this commit is published, so GTS = g implies lastw
-          // of every commit <= g.  Two commits writing one item are ordered
-          // (the later one's snapshot covers the earlier one), so plain
-          // stores leave lastw at the latest.
-          st_relaxed(p.lastw + d.src, cts);
-          st_relaxed(p.lastw + d.dst, cts);
-        }
-        if (p.log_mode) {
-          log_commit(p, cu, s, cts, att_u, dig1(d.src, vs) + dig1(d.dst, vd), dig1(d.src, ns) + dig1(d.dst, nd));
-          if (p.log_mode == CSMV_LOG_FULL && p.max_vals >= 2) {
-            p.vals[cu * p.max_vals] = vs;
-            p.vals[cu * p.max_vals + 1] = vd;
-          }
-        }
-        ++cc.c_upd;
-        cu = kNoTx;
-        att_u = 0;
-        n_srv_ab = 0;
-      } else {
-        const bool ovf = (omask >> lane) & 1u;
-        cc.abort(ovf ? CSMV_AB_OVERFLOW : CSMV_AB_CONFLICT, true);
-        if (!ovf && p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
-      }
+    // ---- D, unless the read-only phase already ran it
+    if (!d_done) {
+      uint32_t base = 0, cmask = 0, omask = 0;
+      wait_response(p, cw, round, t_begin, base, cmask, omask, jit);
+      phase_d(base, cmask, omask);
     }
-    __syncwarp();
-    pc.mark(PH_WRITEBACK);
-    const uint32_t n = __popc(cmask);
-    if (n) {
-      jit();  // write-backs done, commit not yet published
-      if (p.publish == CSMV_PUBLISH_CLIENT) {
-        // Advance GTS by n once every earlier commit is visible:
-        // spin until GTS == first CTS - 1 ("GTS 1" = GTS+1).
-        __syncwarp();
-        fence_gpu();
-        uint32_t it = 0;
-        while (warp_ld_relaxed(p.gts) != base - 1) {
-          if ((++it & 255u) == 0) {
-            uint32_t bad = 0;
-            if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 2);
-            if (__shfl_sync(FULL, bad, 0)) break;
-          }
-          __nanosleep(CSMV_SLEEP_PUB);
-        }
-        if (lane == 0) st_release(p.gts, base + n - 1);  // release also orders the write-backs
-      } else if (cts && p.commit != CSMV_COMMIT_ONLYCS) {
-        st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
-      }
-    }
-    pc.mark(PH_PUBLISH);
+    if (tracing && cts && (d.src == p.trace_item || d.dst == p.trace_item))
+      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer());
   }
   client_flush(p, cc);
   pc.flush(p);

@@ -84,6 +84,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
   const bool compact = A > kKvFullWays || !(p.debug & CSMV_DBG_KV_ITEMSETS);
   PhaseClock pc((p.debug & CSMV_DBG_PHASES) != 0);
   Jitter jit(p, 1);
+  const bool tracing = (p.debug & CSMV_DBG_TRACE) != 0;
   // per-warp smem scratch, lane-minor: RS[kKvMaxRs][32], WS[4][32], NRS[32]
   uint32_t* RS = scratch + (size_t)wib * 32 * (kKvMaxRs + 5);
   uint32_t* WS = RS + kKvMaxRs * 32;
@@ -95,6 +96,8 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     pc.start();
     ++round;
     ++cc.n_rounds;
+    const uint64_t t_rb = tracing ? globaltimer() : 0;
+    uint64_t t_sub = 0;
     uint32_t s = 0, err = 0;
     if (lane == 0) {
       s = ld_acquire(p.gts);  // TXBegin
@@ -109,10 +112,12 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     uint32_t kk[4] = {0, 0, 0, 0};
     uint32_t victim = 0, tset = 0, clk = 0, nrs = 0;
     uint64_t rdig = 0;
+    uint32_t need = 0;  // a PUT that met a version newer than s retries once GTS >= need
     if (cu == kNoTx && cr < p.n_tx && gen_is_update(p.gen, cr)) {
       cu = cr;
       cr += T;
     }
+    bool pending = false;  // a PUT to read this round
     if (cu != kNoTx) {
       if (hold) {
         --hold;
@@ -126,10 +131,42 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         kv_key16(d.key, kk);
         tset = kv_set(d.key, Tn);
         ++att_u;
+        pending = true;
+      }
+    }
+    // Pre-validation before the reads ({set clock} u WS requests): two PUTs
+    // conflict iff they share a set, and the lowest lane of a set is the one
+    // pre-validation keeps (Q5) -- so the others lose now, without
+    // scanning a set they cannot commit in.  (A lower lane whose read then
+    // fails no longer lets the next lane of its set in: only an extra abort.
+    // With one client warp no read fails, so the deterministic schedule is
+    // the same.)  On a hot set this removes every duplicate scan of its ~80
+    // sectors per warp round.
+    bool reader = pending;
+    if (compact && !(p.debug & CSMV_DBG_NO_PREVAL)) {
+      const uint32_t pm = __ballot_sync(FULL, pending);
+      const uint32_t peers = __match_any_sync(FULL, pending ? tset : 0xFFFFFFFFu);
+      reader = pending && (peers & pm & lt) == 0;
+    }
+    if (pending && !reader) {
+      cc.abort(CSMV_AB_PREVAL, true);
+      status = ST_ABORT;
+    }
+    if (reader) {
+      {
         int r = RD_OK;
+        uint32_t seen = 0;  // newest version timestamp the reads met
         victim = 0xFFFFFFFFu;
-        // key scan, U ways in flight (as in kv_get), stop at match or empty
-        constexpr int U = 1;
+        // the set clock first: every PUT on the set writes it, so a PUT
+        // committed after s on this set shows here after one load and the
+        // scans are skipped (the abort is the same: the clock is in RS)
+        if (compact) {
+          r = kv_read_1<NS>(p.kv_clk + (size_t)tset * NS, K, s, clk, &seen);
+          if (r == RD_OK) rdig += dig1(3 * S + tset, clk);
+        }
+        // key scan, U ways in flight (as in kv_get), stop at match or empty;
+        // the ways loaded past the stop are not read (not in RS)
+        constexpr int U = NS <= 4 ? 4 : (NS == 8 ? 2 : 1);
         for (uint32_t w0 = 0; w0 < A && victim == 0xFFFFFFFFu && r == RD_OK; w0 += U) {
           Ring<4> rk[U][NS];
 #pragma unroll
@@ -145,7 +182,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
             if (w0 + u >= A || victim != 0xFFFFFFFFu || r != RD_OK) break;
             const uint32_t slot = tset * A + w0 + u;
             uint32_t key[4];
-            r = kv_key_pick<NS>(p.kv_key + (size_t)slot * NS * 4, rk[u], K, s, false, key);
+            r = kv_key_pick<NS>(p.kv_key + (size_t)slot * NS * 4, rk[u], K, s, false, key, &seen);
             if (r != RD_OK) break;
             if (!compact) RS[nrs++ * 32 + lane] = slot;
 #pragma unroll
@@ -170,6 +207,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
               if (w0 + u >= A) break;
               const uint32_t slot = tset * A + w0 + u;
               const Sel q = select_version<NS>(rl[u], s);
+              seen = max(seen, q.newest);
               if (q.newest > s) {
                 r = RD_NEWER;
                 break;
@@ -188,18 +226,20 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
             }
           }
         }
-        if (r == RD_OK) {
-          r = kv_read_1<NS>(p.kv_clk + (size_t)tset * NS, K, s, clk);
+        if (r == RD_OK && !compact) {
+          r = kv_read_1<NS>(p.kv_clk + (size_t)tset * NS, K, s, clk, &seen);
           if (r == RD_OK) {
-            if (!compact) RS[nrs++ * 32 + lane] = 3 * S + tset;
+            RS[nrs++ * 32 + lane] = 3 * S + tset;
             rdig += dig1(3 * S + tset, clk);
           }
         }
         if (r == RD_NEWER) {
+          need = seen;  // retry once GTS covers the newer version (its commit is then visible)
           cc.abort(CSMV_AB_EARLY, true);
           status = ST_ABORT;
           if (p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
         } else if (r == RD_MISS) {
+          need = s + 1;  // every version <= s is recycled: only a newer snapshot can read it
           cc.abort(CSMV_AB_VERSION, true);
           status = ST_ABORT;
         } else {
@@ -291,30 +331,45 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       fence_gpu();
       jit();  // payload written, doorbell not yet
       if (lane == 0) st_relaxed(&p.req_seq[cw], round);
+      if (tracing) t_sub = globaltimer();
       pc.mark(PH_SUBMIT);
     }
 
-    // ---- C: GETs at s while the batch is at the server
-    if (streak || cu == kNoTx) {
-      uint32_t n_ro = 0;
-      while (cr < p.n_tx) {
-        if (gen_kv_is_update(p.gen, cr)) break;  // before the key draw: the next round adopts it
-        if (streak ? n_ro >= streak : n_ro >= 1) break;
-        const KvTx g = gen_kv(p.gen, cr);
-        ++att_r;
-        ++n_ro;
-        uint64_t dg;
-        uint32_t hit;
-        if (kv_get<NS>(p, g.key, s, dg, hit) != RD_OK) {
-          cc.abort(CSMV_AB_VERSION, false);  // retried next round
-          break;
+    // ---- C: GETs at s while the batch is at the server, one
+    // per active lane per step.  ro_adaptive ends the run early, warp-wide:
+    // once the server has answered the warp's batch; with ro_adaptive = 2
+    // also -- when the warp submitted nothing because its PUTs read versions
+    // newer than s -- as soon as GTS covers the newest of those versions (a
+    // retry can then read them).
+    {
+      const bool blocked = cu != kNoTx && status == ST_ABORT && need != 0;
+      uint32_t need_min = blocked ? need : 0xFFFFFFFFu;
+      need_min = __reduce_min_sync(FULL, need_min);
+      bool run = streak || cu == kNoTx;
+      const uint32_t lim = streak ? streak : 1u;
+      for (uint32_t n_ro = 0; n_ro < lim; ++n_ro) {
+        bool has = run && cr < p.n_tx && !gen_kv_is_update(p.gen, cr);  // an update: the next round adopts it
+        if (!__any_sync(FULL, has)) break;
+        if (has) {
+          const KvTx g = gen_kv(p.gen, cr);
+          ++att_r;
+          uint64_t dg;
+          uint32_t hit;
+          if (kv_get<NS>(p, g.key, s, dg, hit) != RD_OK) {
+            cc.abort(CSMV_AB_VERSION, false);  // retried next round
+            run = false;
+          } else {
+            if (p.log_mode) log_commit(p, cr, s, 0, att_r, dg, hit);
+            ++cc.c_ro;
+            cc.ro_ck ^= dg;
+            cr += T;
+            att_r = 0;
+          }
         }
-        if (p.log_mode) log_commit(p, cr, s, 0, att_r, dg, hit);
-        ++cc.c_ro;
-        cc.ro_ck ^= dg;
-        cr += T;
-        att_r = 0;
-        if (p.ro_adaptive && kept && (uint32_t)(ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
+        if (p.ro_adaptive) {
+          if (kept && (uint32_t)(warp_ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
+          if (p.ro_adaptive >= 2 && !kept && need_min != 0xFFFFFFFFu && warp_ld_relaxed(p.gts) >= need_min) break;
+        }
       }
     }
     __syncwarp();
@@ -324,6 +379,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     // ---- D: response, write-back, GTS
     uint32_t base = 0, cmask = 0, omask = 0;
     wait_response(p, cw, round, t_begin, base, cmask, omask, jit);
+    const uint64_t t_resp = tracing ? globaltimer() : 0;
     if (p.commit == CSMV_COMMIT_ONLYCS) fence_gpu();  // acquire: the server's write-backs
     pc.mark(PH_WAIT);
     uint32_t cts = 0;
@@ -378,6 +434,8 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       }
     }
     pc.mark(PH_PUBLISH);
+    if (tracing && cts && tset == p.trace_item)
+      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer());
   }
   client_flush(p, cc);
   pc.flush(p);

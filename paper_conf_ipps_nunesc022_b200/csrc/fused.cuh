@@ -135,6 +135,21 @@ struct Jitter {
   }
 };
 
+// Non-blocking: the server's answer to request `round` of client warp cw,
+// if all three words carry the round's tag yet.
+__device__ __forceinline__ bool try_response(const KParams& p, uint32_t cw, uint32_t round, uint32_t& base,
+                                             uint32_t& cmask, uint32_t& omask) {
+  const uint64_t b = warp_ld_relaxed64(&p.resp[cw].base);
+  if ((uint32_t)(b >> 32) != round) return false;
+  const uint64_t c = warp_ld_relaxed64(&p.resp[cw].commit);
+  const uint64_t o = warp_ld_relaxed64(&p.resp[cw].ovf);
+  if ((uint32_t)(c >> 32) != round || (uint32_t)(o >> 32) != round) return false;
+  base = (uint32_t)b;
+  cmask = (uint32_t)c;
+  omask = (uint32_t)o;
+  return true;
+}
+
 // Wait for the server's answer to request `round` of client warp cw (all
 // three words tagged with round).  false if the run is being torn down.
 __device__ __forceinline__ bool wait_response(const KParams& p, uint32_t cw, uint32_t round, uint64_t t_begin,
@@ -197,9 +212,17 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 // (exact int64 sum, digest, any-miss) and added into its owner lane.  Same
 // per-transaction result as one lane scanning alone; no lane waits for another lane's
 // longer read-only run.
-template <int NS>
+//
+// `poll` is called at every row-group boundary (warp-uniform): the client
+// uses it to finish its batch (write-back, publish) as soon as the server's
+// answer is in, instead of after the whole read-only phase.
+struct NoPoll {
+  __device__ __forceinline__ void operator()() const {}
+};
+
+template <int NS, typename Poll = NoPoll>
 __device__ __forceinline__ void rot_coop(const KParams& p, uint32_t act, uint32_t start, uint32_t len, uint32_t s,
-                                         uint64_t tx, bool& ok, int64_t& sum, uint64_t& dg) {
+                                         uint64_t tx, bool& ok, int64_t& sum, uint64_t& dg, Poll poll = Poll()) {
   constexpr int U = NS <= 4 ? 8 : (NS == 8 ? 4 : 2);
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
@@ -282,6 +305,7 @@ __device__ __forceinline__ void rot_coop(const KParams& p, uint32_t act, uint32_
         dg += rd;
       }
     }
+    poll();
   }
 }
 
@@ -349,6 +373,22 @@ struct PhaseClock {
     }
   }
 };
+
+// CSMV_DBG_TRACE: one record per committed writer of the traced item
+__device__ __forceinline__ void trace_commit(const KParams& p, uint32_t cts, uint32_t s, uint64_t tb, uint64_t ts,
+                                             uint64_t tr, uint64_t tp) {
+  const uint32_t i = atomicAdd(&p.ctl->trace_n, 1u);
+  if (i < kTraceCap) {
+    csmv_trace_rec r;
+    r.cts = cts;
+    r.snapshot = s;
+    r.t_begin = tb;
+    r.t_submit = ts;
+    r.t_response = tr;
+    r.t_publish = tp;
+    p.trace[i] = r;
+  }
+}
 
 __device__ __forceinline__ void log_commit(const KParams& p, uint64_t tx, uint32_t s, uint32_t cts,
                                            uint32_t att, uint64_t rdig, uint64_t aux) {

@@ -90,6 +90,8 @@ struct csmv {
   Resp* d_resp = nullptr;
   uint32_t* d_req_vals = nullptr;  // CSMV_COMMIT_ONLYCS (bank)
   uint64_t* d_jv_ws = nullptr;     // CSMV_COMMIT_JVSTM global ATR (allocated on first use)
+  csmv_trace_rec* d_trace = nullptr;  // CSMV_DBG_TRACE (allocated on first use)
+  bool last_traced = false;
   uint32_t* d_jv_tag = nullptr;
   // logs
   csmv_log_rec* d_log = nullptr;
@@ -110,7 +112,7 @@ static void free_all(csmv* h) {
   void* ps[] = {h->d_rings, h->d_key, h->d_val, h->d_lru, h->d_clk, h->d_lastw, h->d_gts, h->d_ctl,
                 h->d_stats, h->d_done, h->d_req_seq, h->d_req_hdr, h->d_req_ids, h->d_req_cnt,
                 h->d_resp, h->d_log, h->d_vals, h->d_zipf, h->d_req_vals, h->d_jv_ws, h->d_jv_tag, h->d_init,
-                h->d_kvstage};
+                h->d_kvstage, h->d_trace};
   for (void* q : ps) cudaFree(q);
   if (h->ev0) cudaEventDestroy(h->ev0);
   if (h->ev1) cudaEventDestroy(h->ev1);
@@ -521,6 +523,14 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.ro_adaptive = w->ro_adaptive;
   p.server_recv = w->server_recv;
   p.group = group;
+  const bool traced = (w->debug_flags & CSMV_DBG_TRACE) != 0;
+  if (traced && !h->d_trace) CK(cudaMalloc(&h->d_trace, sizeof(csmv_trace_rec) * kTraceCap));
+  p.trace = h->d_trace;
+  p.trace_item = w->trace_item;
+  if (w->trace_item == 0xFFFFFFFFu)  // the hottest: zipf rank 0 (bank account 0, KV the set of key 0)
+    p.trace_item = h->kind == CSMV_KIND_KV
+                       ? (uint32_t)(((unsigned __int128)mix64(0ull ^ 0xA5A5A5A5A5A5A5A5ull) * h->kv_T) >> 64)
+                       : 0u;
   p.req_vals = h->d_req_vals;
   p.jv_ws = h->d_jv_ws;
   p.jv_tag = h->d_jv_tag;
@@ -585,6 +595,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   h->last_n_tx = n_tx;
   h->last_log_mode = w->log_mode;
   h->last_max_vals = max_vals;
+  h->last_traced = traced;
   if (ctl.error) {
     h->loaded = false;
     return set_err(CSMV_ETIMEOUT, "csmv_run: device watchdog fired (loop %u); store state undefined", ctl.where);
@@ -667,6 +678,18 @@ int csmv_gen_descs(csmv_t* h, const csmv_workload* w, uint64_t seed, uint64_t tx
   if (e == cudaSuccess) e = cudaMemcpy(out, d, n * per * sizeof(uint32_t), cudaMemcpyDeviceToHost);
   cudaFree(d);
   if (e != cudaSuccess) return set_err(CSMV_ECUDA, "csmv_gen_descs: %s", cudaGetErrorString(e));
+  return CSMV_OK;
+}
+
+int csmv_get_trace(const csmv_t* h, csmv_trace_rec* buf, uint64_t cap, uint64_t* n_out) {
+  if (!h || !buf || !n_out) return set_err(CSMV_EINVAL, "csmv_get_trace: null argument");
+  if (!h->last_traced || !h->d_trace) return set_err(CSMV_ESTATE, "csmv_get_trace: last run was not traced");
+  Ctl ctl;
+  CK(cudaMemcpy(&ctl, h->d_ctl, sizeof ctl, cudaMemcpyDeviceToHost));
+  const uint64_t n = ctl.trace_n < kTraceCap ? ctl.trace_n : kTraceCap;
+  const uint64_t m = n < cap ? n : cap;
+  if (m) CK(cudaMemcpy(buf, h->d_trace, m * sizeof(csmv_trace_rec), cudaMemcpyDeviceToHost));
+  *n_out = ctl.trace_n;
   return CSMV_OK;
 }
 

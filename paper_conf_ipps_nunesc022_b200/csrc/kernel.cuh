@@ -65,7 +65,9 @@ struct Ctl {
   uint32_t tail_final;  // server: last CTS assigned
   uint32_t where;       // which spin loop fired the watchdog
   uint32_t jv_tail;     // CSMV_COMMIT_JVSTM: last CTS reserved (global CAS target)
+  uint32_t trace_n;     // CSMV_DBG_TRACE: records claimed
 };
+constexpr uint32_t kTraceCap = 1u << 18;
 
 struct ReqHdr {        // written before the doorbell
   uint32_t snapshot;
@@ -142,6 +144,8 @@ struct KParams {
   uint32_t ro_adaptive;       // stop a read-only run once the server has answered
   uint32_t server_recv;       // CSMV_RECV_*
   uint32_t group;             // client warps per request (1 = per-warp batches; 2/4/8 = CTA-level batches)
+  csmv_trace_rec* trace;      // CSMV_DBG_TRACE buffer (kTraceCap records)
+  uint32_t trace_item;        // bank account / KV set traced
   uint32_t* req_vals;         // ONLYCS: new values [n_cw][2][32] for the server-side write-back
   uint64_t* jv_ws;            // JVSTM: global ATR, write-set of CTS c at c & (2^jv_log2 - 1)
   uint32_t* jv_tag;           //        entry tag = c once the record of c is written

@@ -64,9 +64,10 @@ __device__ __forceinline__ uint64_t dig_word(uint32_t item, uint32_t w, uint32_t
 // Read a W-word item at snapshot s.  rot: a read-only transaction (a newer
 // version is fine); otherwise any version newer than s means
 // validation must fail (RD_NEWER).
+// `seen` (optional) is raised to the newest version timestamp present.
 template <int NS, int W>
 __device__ __forceinline__ int kv_read_mw(const uint64_t* ring, uint32_t K, uint32_t s, bool rot,
-                                          uint32_t (&out)[W]) {
+                                          uint32_t (&out)[W], uint32_t* seen = nullptr) {
   uint32_t ts[NS];
 #pragma unroll
   for (int j = 0; j < NS; ++j) ts[j] = ((uint32_t)j < K) ? (uint32_t)(ld_relaxed64(ring + j * W) >> 32) : kEmptyTs;
@@ -81,6 +82,7 @@ __device__ __forceinline__ int kv_read_mw(const uint64_t* ring, uint32_t K, uint
       cts = ts[j];
     }
   }
+  if (seen) *seen = max(*seen, newest);
   if (!rot && newest > s) return RD_NEWER;
   if (cand < 0) return RD_MISS;
   // the payload read is the re-check: every word still tagged cts means the
@@ -113,7 +115,7 @@ __device__ __forceinline__ int kv_read_mw(const uint64_t* ring, uint32_t K, uint
 // kv_read_mw (a torn slot carries a newer ts, so it is covered too).
 template <int NS>
 __device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (&r)[NS], uint32_t K, uint32_t s,
-                                           bool rot, uint32_t (&out)[4]) {
+                                           bool rot, uint32_t (&out)[4], uint32_t* seen = nullptr) {
   int cand = -1;
   uint32_t cts = 0, newest = 0, torn_max = 0;
   bool torn = false;
@@ -138,6 +140,7 @@ __device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (
       cts = t0;
     }
   }
+  if (seen) *seen = max(*seen, newest);
   if (!rot && newest > s) return RD_NEWER;
   if (cand < 0 || (torn && torn_max > cts)) return RD_MISS;
   if (newest > s) {
@@ -195,9 +198,10 @@ __device__ __forceinline__ void kv_write_mw(uint64_t* ring, uint32_t K, uint32_t
 
 // Single-word item (LRU stamp, set clock): only update transactions read them.
 template <int NS>
-__device__ __forceinline__ int kv_read_1(const uint64_t* ring, uint32_t K, uint32_t s, uint32_t& out) {
+__device__ __forceinline__ int kv_read_1(const uint64_t* ring, uint32_t K, uint32_t s, uint32_t& out,
+                                         uint32_t* seen = nullptr) {
   uint32_t o[1];
-  const int r = kv_read_mw<NS, 1>(ring, K, s, false, o);
+  const int r = kv_read_mw<NS, 1>(ring, K, s, false, o, seen);
   out = o[0];
   return r;
 }

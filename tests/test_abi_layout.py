@@ -49,3 +49,9 @@ def test_stats_mirror():
 def test_log_record_is_32_bytes():
     assert csmv.LOG_DTYPE.itemsize == 32
     assert [n for n, _, _ in c_struct_fields("csmv_log_rec")] == list(csmv.LOG_DTYPE.names)
+
+
+def test_trace_record_mirror():
+    c = c_struct_fields("csmv_trace_rec")
+    assert [n for n, _, _ in c] == list(csmv.TRACE_DTYPE.names)
+    assert sum(s * n for _, s, n in c) == csmv.TRACE_DTYPE.itemsize == 40

@@ -1,0 +1,61 @@
+"""Hot-item commit chain (CSMV_DBG_TRACE): every committed writer of the
+traced item (bank account 0 / the KV set of key 0, zipf rank 0) logs its
+CTS, snapshot and device-wide timestamps.  Consecutive writers form the
+chain the paper's ordering implies (the next writer's
+snapshot must include the previous commit).  Per link i -> i+1 this prints
+the median of
+  link      t_response(i+1) - t_response(i)
+  publish   t_publish(i) - t_response(i)          write-back + publish of i
+  restart   t_begin(i+1) - t_publish(i)           until the next winner's round starts
+  read      t_submit(i+1) - t_begin(i+1)          its snapshot + reads + pre-validation
+  server    t_response(i+1) - t_submit(i+1)       request -> response
+(restart can be negative: the winner's round began before i was
+published, e.g. when GTS was advanced by the server publisher meanwhile).
+
+usage: python tools/chain.py C3|C4 [key=value ...]
+"""
+import json
+import os
+import sys
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
+
+BASE = {"C3": dict(client_warps=294, server_recv=1, server_workers=7, server_combine=2, publish=0, ro_streak=8,
+                   ro_adaptive=1),
+        "C4": dict(client_warps=294, server_workers=6, server_combine=8, publish=1, ro_streak=32, ro_adaptive=1),
+        "C2": dict(client_warps=588, client_group=4, server_workers=6, server_combine=8, publish=1, ro_streak=8,
+                   ro_adaptive=1)}
+
+
+def main(argv):
+    kw = dict(BASE.get(argv[0], {}))
+    kw.update({k: int(v) for k, v in (a.split("=") for a in argv[1:])})
+    kw["debug_flags"] = kw.get("debug_flags", 0) | csmv.DBG_TRACE
+    cfg = workloads.PRESETS[argv[0]](**kw)
+    if cfg.workload.kind == csmv.KIND_KV:
+        st = csmv.KvStore(cfg.n_items, cfg.workload.kv_ways, cfg.n_versions)
+        st.load(cfg.workload.kv_keys)
+    else:
+        st = csmv.Store(cfg.n_items, cfg.n_versions)
+        st.load(cfg.init_values())
+    with st:
+        s = st.run(cfg.workload, cfg.n_tx, cfg.seed)
+        tr = st.trace()
+    tr = np.sort(tr, order="cts")
+    f = lambda a: float(np.median(a)) / 1e3 if len(a) else None  # noqa: E731
+    r, p, b, sub = (tr[k].astype(np.int64) for k in ("t_response", "t_publish", "t_begin", "t_submit"))
+    out = {"cfg": argv, "tx_per_s_M": round(s["tx_per_s"] / 1e6, 2), "kernel_ms": s["elapsed_ns"] / 1e6,
+           "hot_commits": int(len(tr)), "span_ms": float((r[-1] - r[0]) / 1e6) if len(tr) > 1 else None,
+           "median_us": {"link": f(np.diff(r)), "publish": f(p - r), "restart": f(b[1:] - p[:-1]),
+                         "read": f(sub - b), "server": f(r - sub)},
+           "mean_link_us": float(np.mean(np.diff(r))) / 1e3 if len(tr) > 1 else None,
+           "snapshot_lag_median": float(np.median(tr["cts"][1:].astype(np.int64) - tr["snapshot"][1:]))
+           if len(tr) > 1 else None}
+    print(json.dumps(out), flush=True)
+
+
+if __name__ == "__main__":
+    main(sys.argv[1:])
