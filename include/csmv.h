@@ -136,6 +136,10 @@ typedef struct csmv_workload {
                                   server with a receiver warp, item-indexed ATR, CSMV commit */
     uint32_t trace_item;       /* CSMV_DBG_TRACE: bank account / KV set whose committed writers are traced;
                                   0xFFFFFFFF = the hottest (account 0 / the set of key 0: zipf rank 0) */
+    uint32_t elide_ww;         /* 1: blind-write elision -- validate the read-set only, no separate
+                                  write-write check; allowed only for workloads without blind writes: the
+                                  bank (every transfer reads what it writes: RS = WS, so validating RS is
+                                  the whole check); EINVAL for KV, whose PUTs write the value blindly */
 } csmv_workload;
 
 /* ---- statistics ---- */

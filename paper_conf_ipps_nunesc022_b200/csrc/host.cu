@@ -360,6 +360,14 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (w->atr_mode != CSMV_ATR_HASH && (h->kind != CSMV_KIND_BANK || w->server != CSMV_SERVER_CTA))
     return set_err(CSMV_EINVAL, "csmv_run: the list ATR is built for the bank workload on the single-CTA server");
   if (n_tx >= (1ull << 32)) return set_err(CSMV_EINVAL, "csmv_run: n_tx must be < 2^32");
+  // blind-write elision is safe only without blind writes: a bank
+  // transfer reads both accounts it writes (RS = WS, so the validated
+  // read-set already is RS u WS); a KV PUT writes its value (and, on a key
+  // match or empty way, its LRU stamp) without reading it
+  if (w->elide_ww > 1) return set_err(CSMV_EINVAL, "csmv_run: elide_ww must be 0 or 1");
+  if (w->elide_ww && h->kind == CSMV_KIND_KV)
+    return set_err(CSMV_EINVAL, "csmv_run: elide_ww refused: KV PUTs write blindly (value, LRU), so the "
+                                "write-write check of P:115 cannot be omitted");
   if (w->commit > CSMV_COMMIT_JVSTM) return set_err(CSMV_EINVAL, "csmv_run: unknown commit %u", w->commit);
   const bool jvstm = w->commit == CSMV_COMMIT_JVSTM;
   if (w->commit != CSMV_COMMIT_CSMV && (h->kind != CSMV_KIND_BANK || w->server != CSMV_SERVER_CTA))

@@ -257,3 +257,22 @@ def test_filter16_wraps(publish):
     rep, stats, *_ = check(cfg)
     assert stats["gts_final"] - stats["gts_start"] > 4 * 65536
     assert stats["aborts"]["overflow"]["update"] > 0
+
+
+def test_blind_write_elision():
+    """without blind writes the write-write check can be omitted.
+    The bank qualifies (RS = WS): with elide_ww the history is still
+    opaque, and with one client warp it is the very same history; the KV
+    workload (blind value/LRU writes) is refused."""
+    cfg = W.c2(n_items=1 << 14, n_tx=1 << 16, client_warps=256, elide_ww=1, ro_streak=4)
+    check(cfg)
+    one = W.c1(client_warps=1, n_tx=3000, log_mode=csmv.LOG_FULL)
+    a = run_gpu(one)
+    b = run_gpu(one.with_(elide_ww=1))
+    assert np.array_equal(a[1], b[1]) and np.array_equal(a[3], b[3])
+    kv = W.c4(n_items=1 << 12, n_tx=1 << 10, elide_ww=1)
+    with csmv.KvStore(kv.n_items, kv.workload.kv_ways, kv.n_versions) as st:
+        st.load(kv.workload.kv_keys)
+        with pytest.raises(csmv.CsmvError) as e:
+            st.run(kv.workload, kv.n_tx, kv.seed)
+        assert e.value.code == csmv.EINVAL
