@@ -154,8 +154,9 @@ typedef struct csmv_stats {
     uint64_t committed_update;
     uint64_t committed_ro;
     uint64_t aborts[CSMV_N_ABORT][2]; /* [reason][0 = read-only, 1 = update] */
-    uint64_t batches;          /* requests the server processed */
-    uint64_t server_groups;    /* critical sections (each commits 1..4 batches) */
+    uint64_t batches;          /* requests the server processed (a request = one warp's batch, or one
+                                  client group's batches with client_group > 1) */
+    uint64_t server_groups;    /* critical sections (each commits up to server_combine batches) */
     uint64_t rounds;           /* client warp rounds */
     uint64_t gts_start;
     uint64_t gts_final;
@@ -196,7 +197,7 @@ typedef struct csmv_trace_rec {
 
 typedef struct csmv csmv_t;
 
-/* Version of this ABI (CSMV_ABI_VERSION). */
+/* Version of this ABI (CSMV_ABI_VERSION); never fails. */
 int csmv_abi_version(void);
 
 /* Create a store of n_items 4-byte items (bank accounts), each a VBox of
@@ -210,11 +211,17 @@ csmv_t *csmv_create(uint64_t n_items, uint32_t n_versions);
 csmv_t *csmv_create_kv(uint64_t n_slots, uint32_t ways, uint32_t n_versions);
 
 /* Bank: install init_values[0..n) (host memory) as version ts = 0 of every
- * item and reset GTS to 0.  EINVAL if n != n_items. */
+ * item and reset GTS to 0 -- the VBoxes' initial versions before any
+ * transaction ("GTS ... keeps track of how many update
+ * transactions committed so far").  The host buffer is copied during the
+ * call (caller keeps ownership).  EINVAL if n != n_items or a null
+ * argument; ECUDA on a copy/launch failure.  Also clears lastw and the
+ * done flags, so runs restart at CTS 1. */
 int csmv_load(csmv_t *h, const int32_t *init_values, uint64_t n);
 
 /* KV: preload keys 0..n_keys-1 with PUT semantics (docs/GENERATOR.md
- * section 4) as version ts = 0 and reset GTS to 0.  Computed on the device
+ * section 4; MemcachedGPU's set-associative cache) as version ts = 0
+ * and reset GTS to 0.  Computed on the device
  * (count keys per set, bucket them, keep each set's A largest keys: a set's
  * r-th insertion takes way r mod A) in a device staging buffer of about
  * (13*S + 4*T + n_keys) * 4 bytes that the handle keeps for later loads
@@ -223,7 +230,10 @@ int csmv_load(csmv_t *h, const int32_t *init_values, uint64_t n);
 int csmv_load_kv(csmv_t *h, uint64_t n_keys);
 
 /* Run on the given CUDA stream (a cudaStream_t, e.g. torch's current
- * stream); NULL = the legacy default stream. */
+ * stream); NULL = the legacy default stream.  Not from the paper: the
+ * library activates its server and client kernel on the caller's stream
+ * ("activating the (server) kernel").  The handle does not own the
+ * stream.  EINVAL on a null handle; never fails otherwise. */
 int csmv_set_stream(csmv_t *h, void *cuda_stream);
 
 /* Run transactions 0..n_tx-1 of the workload to completion: every
@@ -233,29 +243,43 @@ int csmv_set_stream(csmv_t *h, void *cuda_stream);
  * reloaded); EOVERFLOW if GTS + n_tx would exceed 2^32 - 2. */
 int csmv_run(csmv_t *h, const csmv_workload *w, uint64_t n_tx, uint64_t seed);
 
-/* Statistics of the last csmv_run. */
+/* Statistics of the last csmv_run: committed transactions, aborted attempts
+ * by reason, elapsed time -- the paper's measures: throughput (TXs/sec) and
+ * abort rate (Table V), and the store's memory next to the paper's
+ * VBox size formula.  Copied into caller memory.  EINVAL on a null
+ * argument. */
 int csmv_stats(const csmv_t *h, csmv_stats_t *out);
 
 /* Log of the last csmv_run (needs log_mode != NONE): n_tx records into buf
- * (cap records).  EOVERFLOW if cap < n_tx; *n_out = records written. */
+ * (cap records), one per transaction: its snapshot, CTS
+ * and digests of what it read and wrote -- what the replaying oracle needs
+ * to check opacity in CTS order.  ESTATE if the last run had no log;
+ * EOVERFLOW if cap < n_tx; *n_out = records written. */
 int csmv_get_log(const csmv_t *h, csmv_log_rec *buf, uint64_t cap, uint64_t *n_out);
 
 /* FULL log values of the last run: n_tx * (*max_vals) u32 words, transaction
- * t's reads at [t * max_vals, ...).  Pass buf = NULL to query the size. */
+ * t's reads at [t * max_vals, ...) -- every value it observed.
+ * Pass buf = NULL to query the size.  ESTATE if the last run was not FULL;
+ * EOVERFLOW if cap_words is too small. */
 int csmv_get_vals(const csmv_t *h, uint32_t *buf, uint64_t cap_words, uint32_t *max_vals);
 
 /* Bank: copy the version store out as n_items * n_versions packed slots
- * (ts << 32) | (uint32_t)value, ts = 0xFFFFFFFF for an unused slot. */
+ * (ts << 32) | (uint32_t)value, ts = 0xFFFFFFFF for an unused slot -- the
+ * K versions each VBox keeps.  EINVAL on a KV store or a
+ * null argument; EOVERFLOW if cap < n_items * n_versions. */
 int csmv_dump_store(const csmv_t *h, uint64_t *rings_out, uint64_t cap);
 
-/* KV: newest value of every item: keys (n_slots*4 words), values
- * (n_slots*8), lru (n_slots), clocks (n_slots/ways).  Any may be NULL. */
+/* KV: newest value of every item (P:185's key, value, LRU stamp and set
+ * clock items): keys (n_slots*4 words), values (n_slots*8), lru (n_slots),
+ * clocks (n_slots/ways).  Any may be NULL.  EINVAL on a bank store; ESTATE
+ * if not loaded. */
 int csmv_dump_kv(const csmv_t *h, uint32_t *keys, uint32_t *vals, uint32_t *lru,
                  uint32_t *clocks);
 
 /* Copy transaction descriptors tx0..tx0+n-1 as the device generator sees
- * them (6 u32 per bank tx: is_update, src, dst, amt, start, len), for the
- * generator parity check. */
+ * them (6 u32 per bank tx: is_update, src, dst, amt, start, len -- the
+ * Bank's transfers and balance scans; 10 per KV tx), for the
+ * generator parity check.  EINVAL on a bad workload. */
 int csmv_gen_descs(csmv_t *h, const csmv_workload *w, uint64_t seed, uint64_t tx0,
                    uint64_t n, uint32_t *out);
 
@@ -266,13 +290,17 @@ int csmv_gen_descs(csmv_t *h, const csmv_workload *w, uint64_t seed, uint64_t tx
  * an item commits and publishes after the previous one). */
 int csmv_get_trace(const csmv_t *h, csmv_trace_rec *buf, uint64_t cap, uint64_t *n_out);
 
-/* The zipf CDF table the library built for (n, theta_milli). */
+/* The zipf CDF table the library built for (n, theta_milli) (the
+ * skewed key popularity of the MemcachedGPU workload).  EINVAL on
+ * n = 0 or a null buffer. */
 int csmv_zipf_table(uint32_t n, uint32_t theta_milli, uint64_t *out);
 
-/* Release everything; accepts NULL. */
+/* Release everything the handle owns (device memory, events); accepts
+ * NULL.  Waits for the handle's stream first. */
 void csmv_destroy(csmv_t *h);
 
-/* Message of the last error on this thread ("" if none). */
+/* Message of the last error on this thread ("" if none); owned by the
+ * library, valid until the thread's next failing call. */
 const char *csmv_last_error(void);
 
 #ifdef __cplusplus

@@ -56,16 +56,29 @@ def kv_ways(path):
 
 def c5(path):
     rs = rows(path)
-    print("| point | items | K | update % | server | tx/s | abort rate | parity |")
-    print("|---|---|---|---|---|---|---|---|")
+    ok = [r for r in rs if "error" not in r]
+    n_par = sum(1 for r in ok if r.get("parity") is True)
+    print(f"{len(rs)} points, {n_par} parity-ok, {len(rs) - len(ok)} errors\n")
+    pairs = {}
+    for r in ok:
+        pairs.setdefault(r["name"][:-3], {})[r["server"]] = r.get("tx_per_s_mean", r["tx_per_s"])
+    ratios = sorted(v["cluster"] / v["cta"] for v in pairs.values() if "cta" in v and "cluster" in v)
+    if ratios:
+        print(f"cluster/CTA throughput ratio over {len(ratios)} pairs: median {ratios[len(ratios) // 2]:.2f}, "
+              f"min {ratios[0]:.2f}, max {ratios[-1]:.2f}\n")
+    print("| point | items | K | update % | server | group | tx/s mean (min-max, seeds) | abort rate | parity |")
+    print("|---|---|---|---|---|---|---|---|---|")
     for r in rs:
         if "error" in r:
-            print(f"| {r['name']} | | | | | error: {r['error'][:50]} | | |")
+            print(f"| {r['name']} | | | | | | error: {r['error'][:50]} | | |")
             continue
         par = {True: "ok", False: "FAIL"}.get(r.get("parity"), "-")
+        mean = r.get("tx_per_s_mean", r["tx_per_s"])
+        rng = f" ({fmt_rate(r['tx_per_s_min'])}-{fmt_rate(r['tx_per_s_max'])}, {len(r['seeds_timed'])})" \
+            if "tx_per_s_min" in r else ""
         print(f"| {r['name']} | {r['n_items']} | {r['K']} | {r['p_update_ppm'] / 1e4:.0f} | "
-              f"{r['server']}{'' if r['server'] == 'cta' else r['cluster_size']} | {fmt_rate(r['tx_per_s'])} | "
-              f"{r['abort_rate']:.3f} | {par} |")
+              f"{r['server']}{'' if r['server'] == 'cta' else r['cluster_size']} | {r.get('client_group', 1)} | "
+              f"{fmt_rate(mean)}{rng} | {r['abort_rate']:.3f} | {par} |")
 
 
 if __name__ == "__main__":

@@ -1,11 +1,16 @@
 """C5 sweep (BASELINE.json configs[4]): update rate 10-90% x contention
 (1K-16M items) x K = 2/4/8 versions x single-SM vs cluster server.
 
-For every point: one DIGEST-logged run (seed 1) checked element by element
-against the CPU oracle (--check), then one timed run without logging
-(seed 2).  Writes one JSON line per point.
+For every point (SURVEY 8(d) protocol): one DIGEST-logged run (seed 1)
+checked element by element against the CPU oracle (--check), then timed runs
+without logging for seeds 1..--seeds (mean, min, max of tx/s).  The launch
+is bench.py's tuned one scaled to the point: client warps = max(16,
+min(W, N/64)) so that in-flight updates stay well below the item count
+(Q29), W = 588 in CTA-level groups of 4 for the single-CTA server (when a
+CTA hosts at least two client warps), 294 per-warp batches for the cluster
+server.  Writes one JSON line per point.
 
-usage: python tools/sweep_c5.py [--n-tx N] [--check] [--out FILE] [--servers 0,1]
+usage: python tools/sweep_c5.py [--n-tx N] [--check] [--seeds 3] [--out FILE] [--servers 0,1]
 """
 import argparse
 import json
@@ -17,10 +22,10 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
 
-TUNED = dict(client_warps=294, server_workers=6, server_combine=8, ro_streak=8, ro_adaptive=1, publish=csmv.PUBLISH_SERVER)
+TUNED = dict(server_workers=6, server_combine=8, ro_streak=8, ro_adaptive=1, publish=csmv.PUBLISH_SERVER)
 
 
-def run_point(cfg, check: bool):
+def run_point(cfg, check: bool, seeds: int):
     import numpy as np
     w = cfg.workload
     out = {"name": cfg.name, "n_items": cfg.n_items, "K": cfg.n_versions, "p_update_ppm": w.p_update_ppm,
@@ -43,11 +48,15 @@ def run_point(cfg, check: bool):
             out["oracle_s"] = rep["seconds"]
             if not rep["ok"]:
                 out["parity_msg"] = rep["msg"]
-        st.load(init)
-        wt = workloads.Config(cfg.name, cfg.n_items, cfg.n_versions, cfg.workload, cfg.n_tx, cfg.seed).with_(log_mode=0)
-        t = time.time()
-        s = st.run(wt.workload, cfg.n_tx, cfg.seed + 1)
-        out["wall_s"] = time.time() - t
+        rates, last = [], None
+        for sd in range(1, seeds + 1):
+            st.load(init)
+            wt = workloads.Config(cfg.name, cfg.n_items, cfg.n_versions, cfg.workload, cfg.n_tx, sd).with_(log_mode=0)
+            last = st.run(wt.workload, cfg.n_tx, sd)
+            rates.append(last["tx_per_s"])
+    s = last
+    out["tx_per_s_mean"], out["tx_per_s_min"], out["tx_per_s_max"] = sum(rates) / len(rates), min(rates), max(rates)
+    out["seeds_timed"] = list(range(1, seeds + 1))
     for k in ("tx_per_s", "abort_rate", "committed_update", "committed_ro", "batches", "server_ctas", "client_warps",
               "elapsed_ns"):
         out[k] = s[k]
@@ -57,7 +66,8 @@ def run_point(cfg, check: bool):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--n-tx", type=int, default=1 << 21)
+    ap.add_argument("--n-tx", type=int, default=1 << 22)
+    ap.add_argument("--seeds", type=int, default=3)
     ap.add_argument("--check", action="store_true")
     ap.add_argument("--out", default="")
     ap.add_argument("--servers", default="0,1")
@@ -66,10 +76,14 @@ def main():
     servers = tuple(int(x) for x in args.servers.split(","))
     f = open(args.out, "w") if args.out else None
     for cfg in workloads.c5_points(args.n_tx, servers=servers):
-        cw = max(16, min(TUNED["client_warps"], cfg.n_items // 64))  # in-flight updates << items (Q29)
-        cfg = cfg.with_(cluster_size=args.cluster_size, watchdog_ms=60_000, **dict(TUNED, client_warps=cw))
+        single = cfg.workload.server == csmv.SERVER_CTA
+        cw = max(16, min(588 if single else 294, cfg.n_items // 64))  # in-flight updates << items (Q29)
+        group = 4 if single and cw >= 296 else 1
+        cfg = cfg.with_(cluster_size=args.cluster_size, watchdog_ms=60_000, client_group=group,
+                        **dict(TUNED, client_warps=cw))
         try:
-            r = run_point(cfg, args.check)
+            r = run_point(cfg, args.check, args.seeds)
+            r["client_group"] = group
         except Exception as e:  # report and continue the sweep
             r = {"name": cfg.name, "error": str(e)}
         line = json.dumps(r)
