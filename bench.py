@@ -55,11 +55,14 @@ TUNED = dict(client_warps_per_sm=4, client_group=4, server_workers=6, server_com
 # chains of C3 want the lower-latency self-receiving server combining at most 2
 # batches per critical section (3.3M -> 4.5M tx/s against 8) and the clients'
 # own ordered GTS publish (no publisher hop on the chain: 4.4M -> 5.0M), the PUT
-# convoys of C4 longer read-only runs ahead of a blocked PUT; both keep per-warp
-# batches (the self-receiving server and the KV workload take no groups)
+# convoys of C4 longer read-only runs ahead of a blocked PUT, and a PUT that met
+# a newer version of its set sits out up to 16 rounds but its warp's GET run
+# ends once GTS covers that version (ro_adaptive 2: 52 -> 55 M tx/s, abort rate
+# 54 % -> 13 %); both keep per-warp batches (the self-receiving server and the
+# KV workload take no groups)
 TUNED_PER_CONFIG = {"C3": dict(server_recv=1, server_workers=7, server_combine=2, publish=0, client_warps_per_sm=2,
                                client_group=1),
-                    "C4": dict(ro_streak=32, client_warps_per_sm=2, client_group=1)}
+                    "C4": dict(ro_streak=32, client_warps_per_sm=2, client_group=1, ro_adaptive=2, backoff_max=16)}
 
 
 def tuned(config: str) -> dict:
@@ -248,7 +251,8 @@ def make_cfg(args, world: int, rank: int):
     t = tuned(args.config)
     cfg = cfg.with_(n_tx=n_tx, log_mode=0, ro_streak=t["ro_streak"], publish=t["publish"],
                     server_workers=t["server_workers"], server_combine=t["server_combine"],
-                    ro_adaptive=t["ro_adaptive"], server_recv=t["server_recv"], client_group=t["client_group"])
+                    ro_adaptive=t["ro_adaptive"], server_recv=t["server_recv"], client_group=t["client_group"],
+                    backoff_max=t.get("backoff_max", 0))
     part = partition.partition(cfg.n_items, n_tx, cfg.seed, rank, world, mode="weak")
     lcfg = partition.local_config(cfg, part)
     return cfg, lcfg, part
@@ -465,7 +469,8 @@ def bench_ours(args):
                    "n_versions": cfg.n_versions, "n_tx_per_step_per_gpu": lcfg.n_tx,
                    "client_warps_per_gpu": n_cw, "client_group": w.client_group, "server_workers": w.server_workers,
                    "server_combine": w.server_combine,
-                   "ro_streak": w.ro_streak, "ro_adaptive": w.ro_adaptive, "publish": ["client", "server"][w.publish],
+                   "ro_streak": w.ro_streak, "ro_adaptive": w.ro_adaptive, "backoff_max": w.backoff_max,
+                   "publish": ["client", "server"][w.publish],
                    "server_recv": ["receiver warp", "self-receiving workers"][w.server_recv],
                    "parallelism": f"partitioned x{world}" if world > 1 else "single-gpu",
                    "multi_gpu": "independent key-range partitions (rank g: keys [g*N, (g+1)*N), full per-GPU "

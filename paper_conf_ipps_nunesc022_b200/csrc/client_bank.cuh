@@ -423,16 +423,22 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       d_done = true;
     };
     const bool early_d = p.ro_adaptive && kept && p.commit == CSMV_COMMIT_CSMV;
-    // the response's first word is prefetched by lane 0 one row group ahead
-    // (its latency hides behind the group's own loads)
+    // ro_adaptive: the watched response slot's first word is prefetched by
+    // lane 0 one row group ahead (its latency hides behind the group's own
+    // loads; a blocking poll would add an L2 round trip to every group);
+    // `answered` once it carries this round's tag
     uint64_t pf = 0;
+    bool answered = false;
+    const uint32_t wslot = kept ? cw : watch;
     auto poll = [&]() {
-      if (!early_d || d_done) return;
-      uint32_t b0, c0, o0;
-      if (__shfl_sync(FULL, (uint32_t)(pf >> 32), 0) == round && try_response(p, cw, round, b0, c0, o0))
-        phase_d(b0, c0, o0);
-      else if (lane == 0)
-        pf = ld_relaxed64(&p.resp[cw].base);
+      if (!p.ro_adaptive || !gkept || d_done || answered) return;
+      if (__shfl_sync(FULL, (uint32_t)(pf >> 32), 0) == round) {
+        answered = true;
+        uint32_t b0, c0, o0;
+        if (early_d && try_response(p, cw, round, b0, c0, o0)) phase_d(b0, c0, o0);
+      } else if (lane == 0) {
+        pf = ld_relaxed64(&p.resp[wslot].base);
+      }
     };
 
     // ---- C: read-only transactions at s.  A lane runs
@@ -470,7 +476,8 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
         }
         run = run && has;
         // ro_adaptive: the batch has been answered -> finish the round
-        if (p.ro_adaptive && gkept && (d_done || (uint32_t)(warp_ld_relaxed64(&p.resp[watch].base) >> 32) == round)) break;
+        poll();
+        if (p.ro_adaptive && gkept && (d_done || answered)) break;
       }
     }
     __syncwarp();

@@ -1,4 +1,13 @@
 // client_kv.cuh -- the client warp of the MemcachedGPU workload.
+//
+// CSMV_KV_POLL_PREFETCH (A/B, default 0): poll the response with a load
+// issued one GET step ahead instead of a blocking load per step.  It
+// answers ~5 us sooner, yet C4 loses ~20 %: warps whose batch returns early
+// start their next round (and re-scan the hot sets) sooner, and the herd on
+// a hot set grows (tools/chain.py: restart 6.6 -> 16.9 us per link).
+#ifndef CSMV_KV_POLL_PREFETCH
+#define CSMV_KV_POLL_PREFETCH 0
+#endif
 // Same lane state machine and round phases as client_bank.cuh; GET is the
 // read-only transaction, PUT the update transaction (docs/GENERATOR.md 4).
 //
@@ -347,6 +356,8 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       need_min = __reduce_min_sync(FULL, need_min);
       bool run = streak || cu == kNoTx;
       const uint32_t lim = streak ? streak : 1u;
+      uint64_t pf = 0;  // CSMV_KV_POLL_PREFETCH: the response's first word, prefetched one GET step ahead
+      (void)pf;
       for (uint32_t n_ro = 0; n_ro < lim; ++n_ro) {
         bool has = run && cr < p.n_tx && !gen_kv_is_update(p.gen, cr);  // an update: the next round adopts it
         if (!__any_sync(FULL, has)) break;
@@ -367,7 +378,14 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           }
         }
         if (p.ro_adaptive) {
-          if (kept && (uint32_t)(warp_ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
+          if (kept) {
+#if CSMV_KV_POLL_PREFETCH
+            if (__shfl_sync(FULL, (uint32_t)(pf >> 32), 0) == round) break;
+            if (lane == 0) pf = ld_relaxed64(&p.resp[cw].base);
+#else
+            if ((uint32_t)(warp_ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
+#endif
+          }
           if (p.ro_adaptive >= 2 && !kept && need_min != 0xFFFFFFFFu && warp_ld_relaxed(p.gts) >= need_min) break;
         }
       }
@@ -389,10 +407,21 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         // Client-side write-back: the paper's 4 writes.
         cts = base + __popc(cmask & lt);
         const uint32_t cn = clk + 1;
-        kv_write_mw<NS, 4>(p.kv_key + (size_t)victim * NS * 4, K, cts, kk);
-        kv_write_mw<NS, 8>(p.kv_val + (size_t)victim * NS * 8, K, cts, d.val);
-        kv_write_1<NS>(p.kv_lru + (size_t)victim * NS, K, cts, cn);
-        kv_write_1<NS>(p.kv_clk + (size_t)tset * NS, K, cts, cn);
+        // the four rings' slot timestamps in one round trip, then the stores
+        uint64_t* rk = p.kv_key + (size_t)victim * NS * 4;
+        uint64_t* rv = p.kv_val + (size_t)victim * NS * 8;
+        uint64_t* rl = p.kv_lru + (size_t)victim * NS;
+        uint64_t* rc = p.kv_clk + (size_t)tset * NS;
+        uint32_t tk[NS], tv[NS], tl[NS], tc[NS];
+        kv_ring_ts<NS, 4>(rk, K, tk);
+        kv_ring_ts<NS, 8>(rv, K, tv);
+        kv_ring_ts<NS, 1>(rl, K, tl);
+        kv_ring_ts<NS, 1>(rc, K, tc);
+        const uint32_t cn1[1] = {cn};
+        kv_install<NS, 4>(rk, tk, K, cts, kk);
+        kv_install<NS, 8>(rv, tv, K, cts, d.val);
+        kv_install<NS, 1>(rl, tl, K, cts, cn1);
+        kv_install<NS, 1>(rc, tc, K, cts, cn1);
         if (p.log_mode) {
           uint64_t wd = dig1(2 * S + victim, cn) + dig1(3 * S + tset, cn);
 #pragma unroll

@@ -161,13 +161,19 @@ __device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (
   return RD_OK;
 }
 
-// Install version (cts, data) over the first unused slot, else the oldest
-// (P:291).  The writer owns the item (WW check).
+// The version timestamps of a W-word ring (one load per slot).
 template <int NS, int W>
-__device__ __forceinline__ void kv_write_mw(uint64_t* ring, uint32_t K, uint32_t cts, const uint32_t (&data)[W]) {
-  uint32_t ts[NS];
+__device__ __forceinline__ void kv_ring_ts(const uint64_t* ring, uint32_t K, uint32_t (&ts)[NS]) {
 #pragma unroll
   for (int j = 0; j < NS; ++j) ts[j] = ((uint32_t)j < K) ? (uint32_t)(ld_relaxed64(ring + j * W) >> 32) : 0u;
+}
+
+// Install version (cts, data) over the first unused slot, else the oldest
+// (P:291), given the ring's slot timestamps.  The writer owns the item (WW
+// check): nothing else writes it between those loads and the store.
+template <int NS, int W>
+__device__ __forceinline__ void kv_install(uint64_t* ring, const uint32_t (&ts)[NS], uint32_t K, uint32_t cts,
+                                           const uint32_t (&data)[W]) {
   int victim = -1;
 #pragma unroll
   for (int j = 0; j < NS; ++j)
@@ -194,6 +200,13 @@ __device__ __forceinline__ void kv_write_mw(uint64_t* ring, uint32_t K, uint32_t
       st_relaxed64(dst + w, ((uint64_t)cts << 32) | data[w]);
     }
   }
+}
+
+template <int NS, int W>
+__device__ __forceinline__ void kv_write_mw(uint64_t* ring, uint32_t K, uint32_t cts, const uint32_t (&data)[W]) {
+  uint32_t ts[NS];
+  kv_ring_ts<NS, W>(ring, K, ts);
+  kv_install<NS, W>(ring, ts, K, cts, data);
 }
 
 // Single-word item (LRU stamp, set clock): only update transactions read them.
