@@ -116,16 +116,17 @@ def ncu_entry(config: str):
 def serial_chain(batches_per_s, cs_cycles, upd_per_batch, clocks, floor_cycles):
     """The commit critical section is one serial chain on the server SM.  Its
     floor is the same chain (filter loads -> recency test -> ballot -> CTS ->
-    filter stores) timed alone on an idle SM (filt16_ubench): one batch per
-    `floor_cycles` at the SM clock.  `frac` = batches/s reached / that bound;
-    `occupancy` = the chain's measured cycles per batch over the floor."""
+    filter stores) for one request (a batch, or a client group's G batches)
+    timed alone on an idle SM (filt16_ubench): one request per `floor_cycles`
+    at the SM clock.  `frac` = requests/s reached / that bound."""
     d = {"batches_per_s": batches_per_s, "critical_section_cycles_per_batch": cs_cycles,
          "updates_per_batch": upd_per_batch,
          "critical_section_cycles_per_update": cs_cycles / upd_per_batch if upd_per_batch else None}
     mhz = clocks.get("sm_mhz") or clocks.get("sm_max_mhz")
     if mhz and floor_cycles:
         bound = mhz * 1e6 / floor_cycles
-        d.update({"floor_cycles_per_batch": floor_cycles, "floor_source": "profiles/roofs_b200.json cs_floor_cycles",
+        d.update({"floor_cycles_per_batch": floor_cycles,
+                  "floor_source": "profiles/roofs_b200.json cs_floor_cycles_per_request[g<group>k2]",
                   "bound_batches_per_s": bound, "frac": batches_per_s / bound,
                   "updates_bound_per_s": bound * upd_per_batch})
     return d
@@ -479,7 +480,8 @@ def bench_ours(args):
         "roofline": roof,
         "serial_chain": serial_chain(red["batches"] / (total_ms_max * 1e-3), cs_cycles,
                                      red["committed_update"] / max(1, red["batches"]), clk.summary(),
-                                     rf.get("cs_floor_cycles")),
+                                     rf.get("cs_floor_cycles_per_request", {}).get(
+                                         f"g{max(1, w.client_group)}k2", rf.get("cs_floor_cycles"))),
         "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": 0 if is_kv else int(init.nbytes),
                 "d2h_bytes_per_step": 400, "steps": e2e_steps,
                 "load_ms_per_step": 1e3 * t_load / e2e_steps, "wall_ms_per_step": 1e3 * e2e_s / e2e_steps},
