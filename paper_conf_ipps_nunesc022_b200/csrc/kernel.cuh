@@ -35,6 +35,13 @@
 #ifndef CSMV_SLEEP_QUEUE
 #define CSMV_SLEEP_QUEUE 64
 #endif
+// idle back-off (ns) of the server's receiver sweep and publisher sweep (0 = spin)
+#ifndef CSMV_SLEEP_RECV
+#define CSMV_SLEEP_RECV 0
+#endif
+#ifndef CSMV_SLEEP_PUBLISHER
+#define CSMV_SLEEP_PUBLISHER 0
+#endif
 
 namespace csmvd {
 

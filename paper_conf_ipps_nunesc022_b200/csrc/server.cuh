@@ -331,6 +331,9 @@ static __device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64
       idle = 0;
       continue;
     }
+    // an idle sweep backs off briefly: the receiver shares the server SM's
+    // issue slots and load pipe with the critical section
+    if (CSMV_SLEEP_RECV) __nanosleep(CSMV_SLEEP_RECV);
     if ((++idle & 15u) == 0) {
       uint32_t dw = 0, er = 0;
       if (lane == 0) {
@@ -1439,6 +1442,7 @@ static __device__ void server_publisher(const KParams& p, const SrvCtx& c, uint6
       if (lane == 0) st_release(p.gts, g);
       continue;
     }
+    if (CSMV_SLEEP_PUBLISHER) __nanosleep(CSMV_SLEEP_PUBLISHER);
     if ((++spins & 63u) == 0) {
       uint32_t dw = 0, er = 0;
       if (lane == 0) {
