@@ -35,6 +35,10 @@
 #ifndef CSMV_SLEEP_QUEUE
 #define CSMV_SLEEP_QUEUE 64
 #endif
+// back-off (ns) of a worker polling the ticket lock (single-CTA server)
+#ifndef CSMV_SLEEP_LOCK
+#define CSMV_SLEEP_LOCK 16
+#endif
 // idle back-off (ns) of the server's receiver sweep and publisher sweep (0 = spin)
 #ifndef CSMV_SLEEP_RECV
 #define CSMV_SLEEP_RECV 0

@@ -389,7 +389,7 @@ __device__ __forceinline__ uint32_t cs_enter(const SrvCtx& c) {
       uint32_t v;
       asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
       if (v == ticket) break;
-      __nanosleep(16);
+      if (CSMV_SLEEP_LOCK) __nanosleep(CSMV_SLEEP_LOCK);
     }
     __syncwarp();
   }
@@ -694,26 +694,27 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       // are conflict-free, so they need not see each other's stores)
 #pragma unroll
       for (int r = 0; r < MR; ++r) {
-        uint32_t va[G][kFiltK], vb[G][kFiltK];
-        bool cmt[G];
 #pragma unroll
         for (int k = 0; k < G; ++k) {
           const int j = r * G + k;
           cm[j] = om[j] = 0;
           ovfl[j] = false;
           base[j] = t + 1;
-          cmt[k] = false;
-#pragma unroll
-          for (int q = 0; q < kFiltK; ++q) va[k][q] = vb[k][q] = 0u;
-          if ((uint32_t)r < m_req && chk[j]) {
-#pragma unroll
-            for (int q = 0; q < kBankFiltK; ++q) {
-              va[k][q] = filt16_ld<CL>(fa[j][q]);
-              vb[k][q] = filt16_ld<CL>(fb[j][q]);
-            }
-          }
         }
         if ((uint32_t)r < m_req) {
+          // every lane probes (a lane without a live transaction probes the
+          // slots of item 0, a valid address): no predicated loads and no
+          // zero-fill moves in the chain; chk masks the result
+          uint32_t va[G][kFiltK], vb[G][kFiltK];
+          bool cmt[G];
+#pragma unroll
+          for (int k = 0; k < G; ++k) {
+#pragma unroll
+            for (int q = 0; q < kBankFiltK; ++q) {
+              va[k][q] = filt16_ld<CL>(fa[r * G + k][q]);
+              vb[k][q] = filt16_ld<CL>(fb[r * G + k][q]);
+            }
+          }
           // slot v is recent iff its CTS lies in (e_pre, t]: (v - e_pre - 1) mod 2^16 < t - e_pre
           const uint32_t win = t - e_pre;  // commits the exact lastw check did not cover
 #pragma unroll
