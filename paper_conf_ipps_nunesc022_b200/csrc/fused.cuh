@@ -137,13 +137,22 @@ struct Jitter {
 
 // Non-blocking: the server's answer to request `round` of client warp cw,
 // if all three words carry the round's tag yet.
+// The three words of a response, loaded by lanes 0-2 at once (one L2 round
+// trip, not three) and broadcast.
+__device__ __forceinline__ void ld_response(const KParams& p, uint32_t cw, uint64_t& b, uint64_t& c, uint64_t& o) {
+  const uint32_t lane = threadIdx.x & 31;
+  uint64_t v = 0;
+  if (lane < 3) v = ld_relaxed64(&p.resp[cw].base + lane);
+  b = __shfl_sync(0xFFFFFFFFu, v, 0);
+  c = __shfl_sync(0xFFFFFFFFu, v, 1);
+  o = __shfl_sync(0xFFFFFFFFu, v, 2);
+}
+
 __device__ __forceinline__ bool try_response(const KParams& p, uint32_t cw, uint32_t round, uint32_t& base,
                                              uint32_t& cmask, uint32_t& omask) {
-  const uint64_t b = warp_ld_relaxed64(&p.resp[cw].base);
-  if ((uint32_t)(b >> 32) != round) return false;
-  const uint64_t c = warp_ld_relaxed64(&p.resp[cw].commit);
-  const uint64_t o = warp_ld_relaxed64(&p.resp[cw].ovf);
-  if ((uint32_t)(c >> 32) != round || (uint32_t)(o >> 32) != round) return false;
+  uint64_t b, c, o;
+  ld_response(p, cw, b, c, o);
+  if ((uint32_t)(b >> 32) != round || (uint32_t)(c >> 32) != round || (uint32_t)(o >> 32) != round) return false;
   base = (uint32_t)b;
   cmask = (uint32_t)c;
   omask = (uint32_t)o;
@@ -159,12 +168,8 @@ __device__ __forceinline__ bool wait_response(const KParams& p, uint32_t cw, uin
   uint64_t b, c, o;
   for (;;) {
     jit();
-    b = warp_ld_relaxed64(&p.resp[cw].base);
-    if ((uint32_t)(b >> 32) == round) {
-      c = warp_ld_relaxed64(&p.resp[cw].commit);
-      o = warp_ld_relaxed64(&p.resp[cw].ovf);
-      if ((uint32_t)(c >> 32) == round && (uint32_t)(o >> 32) == round) break;
-    }
+    ld_response(p, cw, b, c, o);
+    if ((uint32_t)(b >> 32) == round && (uint32_t)(c >> 32) == round && (uint32_t)(o >> 32) == round) break;
     if ((++it & 255u) == 0) {
       uint32_t bad = 0;
       if ((threadIdx.x & 31) == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 1);

@@ -489,15 +489,20 @@ __device__ __forceinline__ bool server_self_recv(const KParams& p) {
 // client warp first (P:103's receiver, folded into the worker).  Returns the
 // number claimed; 0 once every client has finished (or on error).  At most
 // one request per client warp is outstanding, and only this warp reads or
-// writes last_seen[lo, hi).
+// writes last_seen[lo, hi).  GTS is read (relaxed) with the doorbells of
+// each sweep; the acquire fence after a successful sweep orders it too, so
+// `gts` is an acquired e_pre for the lastw prefetch with no further round
+// trip (ld.relaxed; fence.acq_rel.gpu = acquire).
 template <int M>
 __device__ __forceinline__ uint32_t self_claim(const KParams& p, const SrvCtx& c, uint32_t lo, uint32_t hi,
-                                               uint32_t m_max, uint32_t (&cwv)[M], uint64_t t_begin) {
+                                               uint32_t m_max, uint32_t (&cwv)[M], uint64_t t_begin, uint32_t& gts) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t n = hi - lo, rows = (n + 31) / 32;
   for (uint32_t idle = 1;; ++idle) {
     uint32_t m = 0;
+    uint32_t g = 0;
+    if (lane == 0) g = ld_relaxed(p.gts);
     for (uint32_t r = 0; r < rows && m < m_max; ++r) {
       const uint32_t i = r * 32 + lane;
       const uint32_t seq = i < n ? ld_relaxed(p.req_seq + lo + i) : 0u;
@@ -515,6 +520,7 @@ __device__ __forceinline__ uint32_t self_claim(const KParams& p, const SrvCtx& c
     }
     if (m) {
       fence_gpu();  // acquire: the payloads of the doorbells just seen precede our loads of them
+      gts = __shfl_sync(FULL, g, 0);
       return m;
     }
     if ((idle & 15u) == 0) {
@@ -572,12 +578,13 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     my_lo = min(c.cw_lo + w * per, c.cw_hi);
     my_hi = min(my_lo + per, c.cw_hi);
   }
+  uint32_t gts_claim = 0;  // SELF: GTS read with the doorbells (acquired by the claim's fence)
   for (;;) {
     const long long tq = clock64();
     uint32_t cwv[M];
     uint32_t m = 1;
     if constexpr (SELF) {
-      m = self_claim<M>(p, c, my_lo, my_hi, m_max, cwv, t_begin);
+      m = self_claim<M>(p, c, my_lo, my_hi, m_max, cwv, t_begin, gts_claim);
       if (!m) break;
     } else {
       if (!claim_request(c, cwv[0])) break;
@@ -636,9 +643,10 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     }
     const bool hash = G > 1 || p.atr_mode == CSMV_ATR_HASH;
     // lastw covers every CTS <= e_pre: clients write lastw with their
-    // write-back, before the commit is published, so e_pre = GTS (acquire)
-    const uint32_t e_pre = hash ? ld_acquire(p.gts) : *(volatile uint32_t*)&c.sh0->tail;
-    srv_fence<CL>();
+    // write-back, before the commit is published, so e_pre = GTS (acquire;
+    // self-receiving workers already hold one from their claim)
+    const uint32_t e_pre = SELF ? gts_claim : (hash ? ld_acquire(p.gts) : *(volatile uint32_t*)&c.sh0->tail);
+    if (!SELF) srv_fence<CL>();
     const bool novalid = (p.debug & CSMV_DBG_NO_VALIDATE) != 0;
     // HASH: the exact part of the validation (lastw, every CTS <= e_pre) and
     // the filter slot addresses are settled before the lock
