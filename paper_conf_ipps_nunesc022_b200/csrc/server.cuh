@@ -503,18 +503,28 @@ __device__ __forceinline__ uint32_t self_claim(const KParams& p, const SrvCtx& c
     uint32_t m = 0;
     uint32_t g = 0;
     if (lane == 0) g = ld_relaxed(p.gts);
-    for (uint32_t r = 0; r < rows && m < m_max; ++r) {
-      const uint32_t i = r * 32 + lane;
-      const uint32_t seq = i < n ? ld_relaxed(p.req_seq + lo + i) : 0u;
-      uint32_t pm = __ballot_sync(FULL, i < n && seq != c.last_seen[lo - c.cw_lo + i]);
+    for (uint32_t r0 = 0; r0 < rows && m < m_max; r0 += 4) {
+      // the doorbells of up to 4 rows in flight at once: one L2 round trip
+      uint32_t sqv[4];
 #pragma unroll
-      for (int j = 0; j < M; ++j) {
-        if ((uint32_t)j == m && pm && m < m_max) {
-          const uint32_t l = __ffs(pm) - 1;
-          pm &= pm - 1;
-          if (lane == l) c.last_seen[lo - c.cw_lo + i] = seq;
-          cwv[j] = lo + r * 32 + l;
-          m = j + 1;
+      for (int k = 0; k < 4; ++k) {
+        const uint32_t i = (r0 + k) * 32 + lane;
+        sqv[k] = (r0 + k < rows && i < n) ? ld_relaxed(p.req_seq + lo + i) : 0u;
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const uint32_t r = r0 + k, i = r * 32 + lane;
+        if (r >= rows || m >= m_max) break;
+        uint32_t pm = __ballot_sync(FULL, i < n && sqv[k] != c.last_seen[lo - c.cw_lo + i]);
+#pragma unroll
+        for (int j = 0; j < M; ++j) {
+          if ((uint32_t)j == m && pm && m < m_max) {
+            const uint32_t l = __ffs(pm) - 1;
+            pm &= pm - 1;
+            if (lane == l) c.last_seen[lo - c.cw_lo + i] = sqv[k];
+            cwv[j] = lo + r * 32 + l;
+            m = j + 1;
+          }
         }
       }
     }
