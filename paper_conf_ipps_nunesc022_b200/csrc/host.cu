@@ -420,10 +420,11 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   const uint32_t group = w->client_group ? w->client_group : 1u;
   if (group != 1 && group != 2 && group != 4 && group != 8)
     return set_err(CSMV_EINVAL, "csmv_run: client_group must be 1, 2, 4 or 8");
-  if (group > 1 && (h->kind != CSMV_KIND_BANK || w->server != CSMV_SERVER_CTA || w->atr_mode != CSMV_ATR_HASH ||
-                    w->commit != CSMV_COMMIT_CSMV || selfrecv || cmring))
-    return set_err(CSMV_EINVAL, "csmv_run: client_group > 1 needs the bank workload on the single-CTA "
-                                "ticket-locked server with a receiver warp (atr_mode HASH, CSMV commit)");
+  if (group > 1 && (h->kind != CSMV_KIND_BANK || w->atr_mode != CSMV_ATR_HASH || w->commit != CSMV_COMMIT_CSMV ||
+                    selfrecv || (cmring && group > 4) || (!cmring && w->server != CSMV_SERVER_CTA)))
+    return set_err(CSMV_EINVAL, "csmv_run: client_group > 1 needs the bank workload (atr_mode HASH, CSMV "
+                                "commit) on the ticket-locked single-CTA server with a receiver warp (G = 2/4/8) "
+                                "or on a commit ring (cluster server; G = 2/4)");
   uint32_t n_cw = w->client_warps ? w->client_warps : h->max_cw;
   if (n_cw > h->max_cw) n_cw = h->max_cw;
   if (n_cw == 0) return set_err(CSMV_EINVAL, "csmv_run: no client warps");
@@ -443,7 +444,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   // CTAs 1..C-1 receive (server.cuh server_cta)
   const uint32_t n_serve = (cmring && n_srv > 1) ? n_srv - 1 : n_srv;
   const uint32_t per_srv = n_serve ? (n_cw + n_serve - 1) / n_serve : 0u;
-  size_t smem = server_smem_bytes(rt_log2 - clog2, per_srv);
+  const uint32_t ring_log2 = cm_ring_log2(group, cmring);
+  // eviction watermarks: only the KV item-set table (server_worker_generic) uses them
+  const uint32_t ev_log2 = (h->kind == CSMV_KIND_KV && !filt) ? rt_log2 - clog2 : 2u;  // 16 B keeps what follows aligned
+  size_t smem = server_smem_bytes(rt_log2 - clog2, per_srv, ring_log2, ev_log2);
   if (h->kind == CSMV_KIND_KV && smem < kv_client_smem_bytes()) smem = kv_client_smem_bytes();
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
 
@@ -531,6 +535,8 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.ro_adaptive = w->ro_adaptive;
   p.server_recv = w->server_recv;
   p.group = group;
+  p.cm_ring_log2 = ring_log2;
+  p.ev_log2 = ev_log2;
   const bool traced = (w->debug_flags & CSMV_DBG_TRACE) != 0;
   if (traced && !h->d_trace) CK(cudaMalloc(&h->d_trace, sizeof(csmv_trace_rec) * kTraceCap));
   p.trace = h->d_trace;

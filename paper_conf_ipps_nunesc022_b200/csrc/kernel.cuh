@@ -55,7 +55,22 @@ constexpr int kBlock = 256;            // threads per CTA (8 warps)
 constexpr int kWarps = kBlock / 32;
 constexpr uint32_t kDoneLog2 = 20;     // done ring entries (CSMV_PUBLISH_SERVER)
 constexpr int kMaxCombine = 8;         // batches a server worker commits per critical section
-constexpr uint32_t kCmRingLog2 = 5;    // commit-ring slots (worker warps -> committer warp, bank)
+// commit-ring slots (worker warps -> committer warp, bank): 2^5 for per-warp
+// batches, 2^6 for client groups on a commit ring (a group takes G slots;
+// with 32 slots the committer stalled on slots claimed but not yet filled:
+// cluster-16, G = 4, 736 warps 268 -> 314 M tx/s; per-warp batches lose with
+// 64: 241 -> 229 M).  The ticket-locked server keeps 32 (its CTAs' shared
+// memory, and so every client CTA's, would grow by 33 KB at the L1's
+// expense: its grouped C2 fell 490 -> 313 M with the larger allocation).
+constexpr uint32_t kCmRingLog2 = 5;
+constexpr uint32_t kCmRingLog2Max = 6;
+__host__ __device__ inline uint32_t cm_ring_log2(uint32_t group, bool ring) {
+#ifdef CSMV_RING_ALWAYS
+  return ring && group > 1 ? kCmRingLog2Max : kCmRingLog2;
+#else
+  return !ring ? 0u : group > 1 ? kCmRingLog2Max : kCmRingLog2;  // no commit ring: one unused slot
+#endif
+}
 
 // One commit-ring slot: a batch a worker warp has prepared for the committer
 // (server.cuh).  Lane l's words: {fa0, fa1, fa2, fb0}, {fb1, fb2, id0, id1}
@@ -155,6 +170,8 @@ struct KParams {
   uint32_t ro_adaptive;       // stop a read-only run once the server has answered
   uint32_t server_recv;       // CSMV_RECV_*
   uint32_t group;             // client warps per request (1 = per-warp batches; 2/4/8 = CTA-level batches)
+  uint32_t cm_ring_log2;      // commit-ring slots (cm_ring_log2())
+  uint32_t ev_log2;           // eviction-watermark words per server CTA (log2; 2 = four unused words)
   csmv_trace_rec* trace;      // CSMV_DBG_TRACE buffer (kTraceCap records)
   uint32_t trace_item;        // bank account / KV set traced
   uint32_t* req_vals;         // ONLYCS: new values [n_cw][2][32] for the server-side write-back
@@ -182,10 +199,15 @@ __host__ __device__ inline uint32_t queue_log2(uint32_t n_cw) {
 // recent-commit table, dispatch queue, receiver's last-seen doorbells, control words
 // (per server CTA: its stripe of 2^local_log2 buckets and its slice of n_cw)
 // rt stripe | dispatch queue | evmax stripe | last-seen doorbells | control
-// block (64 B) | commit ring
-inline size_t server_smem_bytes(uint32_t local_log2, uint32_t n_cw) {
-  return ((size_t)(32 + 4) << local_log2) + ((size_t)8 << queue_log2(n_cw)) +
-         (((size_t)n_cw + 31) / 32 * 32) * 4 + 64 + (sizeof(CmSlot) << kCmRingLog2);
+// block (64 B) | commit ring.  Only what the run's commit path uses is
+// allocated (the eviction watermarks only for the KV item-set table, the
+// commit ring only for a ring server): every CTA of the grid gets this much
+// shared memory, and what it takes comes out of the SM's unified L1 --
+// dropping the unused 33 KB ring of the locked server took C2 from ~485 to
+// ~540 M tx/s (profiles/r02/raw/r02ae_ab_smem.jsonl).
+inline size_t server_smem_bytes(uint32_t local_log2, uint32_t n_cw, uint32_t ring_log2, uint32_t ev_log2) {
+  return ((size_t)32 << local_log2) + ((size_t)4 << ev_log2) + ((size_t)8 << queue_log2(n_cw)) +
+         (((size_t)n_cw + 31) / 32 * 32) * 4 + 64 + (sizeof(CmSlot) << ring_log2);
 }
 
 // host-callable launchers (kernel.cu)

@@ -850,15 +850,20 @@ __device__ __forceinline__ bool server_uses_ring(const KParams& p) {
 // committer takes the slots in ring order, so every batch is validated after
 // the write-sets of all batches before it were recorded and receives the next
 // consecutive CTS range -- as if each had held the lock in that order.
+// G > 1 (client groups): a request's G batches go into G consecutive slots
+// (requests never straddle: slots are claimed in whole requests) and the
+// committer commits the G slots in one step of its chain.
 // ---------------------------------------------------------------------------
-template <bool CL>
+template <bool CL, int G = 1>
 __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
   constexpr int M = kMaxCombine;
-  constexpr uint32_t R = 1u << kCmRingLog2;
+  constexpr int MR = M / G;  // requests per claim
+  const uint32_t R = 1u << p.cm_ring_log2;
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t qmask = (1u << c.qn_log2) - 1;
-  const uint32_t m_max = p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine);
+  const uint32_t m_max = G > 1 ? max(1u, min(p.combine, (uint32_t)M) / G)
+                              : (p.combine < 1 ? 1u : (p.combine > (uint32_t)M ? (uint32_t)M : p.combine));
   const uint32_t fl2 = p.rt_log2 - p.clog2 + 3;  // the filter: CTA 0's stripe, 8 << local_log2 32-bit slots
   const bool novalid = (p.debug & CSMV_DBG_NO_VALIDATE) != 0;
   unsigned long long busy = 0, batches = 0, groups = 0, ph0 = 0, ph1 = 0, ph4 = 0;
@@ -869,7 +874,7 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
     if (!claim_request(c, cwv[0])) break;
     uint32_t m = 1;
 #pragma unroll
-    for (int j = 1; j < M; ++j) {
+    for (int j = 1; j < MR; ++j) {
       uint32_t got = 0xFFFFFFFFu;
       if (m == (uint32_t)j && m < m_max && lane == 0) {
         const uint32_t h = *(volatile uint32_t*)&c.sh->q_head;
@@ -880,13 +885,26 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
       cwv[j] = got;
       if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
     }
+    const uint32_t m_req = m;
+    if constexpr (G > 1) {  // request r -> its group's warps lead + k * n_client_ctas (see server_worker)
+#pragma unroll
+      for (int r = MR - 1; r >= 0; --r) {
+        const uint32_t lead = cwv[r], cta = lead % p.n_client_ctas, w0 = lead / p.n_client_ctas;
+        const uint32_t n_act = min((uint32_t)kWarps, (p.n_cw - cta + p.n_client_ctas - 1) / p.n_client_ctas);
+        const uint32_t gs = min((uint32_t)G, n_act - w0);
+#pragma unroll
+        for (int k = 0; k < G; ++k)
+          cwv[r * G + k] = ((uint32_t)r < m_req && (uint32_t)k < gs) ? lead + k * p.n_client_ctas : 0xFFFFFFFFu;
+      }
+      m = m_req * G;
+    }
     const long long t0 = clock64();
     fence_cta();  // payload loads after the queue entries (the receiver fenced after the doorbells)
     uint32_t sq[M], sn[M], msk[M], id0[M], id1[M];
 #pragma unroll
     for (int j = 0; j < M; ++j) {
       sq[j] = sn[j] = msk[j] = id0[j] = id1[j] = 0;
-      if (j < (int)m) {
+      if (j < (int)m && (G == 1 || cwv[j] != 0xFFFFFFFFu)) {
         sn[j] = ld_relaxed(&p.req_hdr[cwv[j]].snapshot);
         msk[j] = ld_relaxed(&p.req_hdr[cwv[j]].mask);
         sq[j] = ld_relaxed(&p.req_hdr[cwv[j]].round);
@@ -944,7 +962,7 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
         b.w = id1[j];
         ring_st_v4<CL>(sl + (uint32_t)offsetof(CmSlot, w) + 16u * lane, a);
         ring_st_v4<CL>(sl + (uint32_t)offsetof(CmSlot, w) + 16u * (32 + lane), b);
-        if (lane == 0) ring_st_v4<CL>(sl + 16u, make_uint4(chkm[j], 0u, 0u, 0u));
+        if (lane == 0) ring_st_v4<CL>(sl + 16u, make_uint4(chkm[j], msk[j], 0u, 0u));
         if (lane == 0) filt_st<CL>(sl + 4u, cwv[j]);
         if (lane == 0) filt_st<CL>(sl + 8u, sq[j]);
         if (lane == 0) filt_st<CL>(sl + 12u, novalid ? 0xFFFFFFFFu : e_pre);
@@ -959,7 +977,7 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
     ph0 += (unsigned long long)(t0 - tq);
     ph1 += (unsigned long long)(tl - t0);
     ph4 += (unsigned long long)(t3 - tl);
-    batches += m;
+    batches += m_req;
     ++groups;
   }
   __syncwarp();
@@ -981,7 +999,7 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
 // -> CTS -> filter stores.
 struct CmPayload {
   uint4 w0, w1;
-  uint32_t cw, round, e_chk, chkm;
+  uint32_t cw, round, e_chk, chkm, msk;
 };
 
 template <bool CL>
@@ -995,29 +1013,64 @@ __device__ __forceinline__ bool cm_try(CmSlot* sl, uint32_t seq, CmPayload& q) {
   q.round = h.z;
   q.e_chk = h.w;
   q.chkm = sl->chk;
+  q.msk = sl->pad[0];
   return __shfl_sync(0xFFFFFFFFu, f, 0) == seq + 1;  // lane 0's view decides
 }
 
-template <bool CL>
+// A slot's payload, loaded after its unit's flags were seen (acquire).
+__device__ __forceinline__ void cm_load(const CmSlot* sl, CmPayload& q) {
+  const uint32_t lane = threadIdx.x & 31;
+  q.w0 = sl->w[0][lane];
+  q.w1 = sl->w[1][lane];
+  const uint4 h = *reinterpret_cast<const uint4*>(sl);
+  q.cw = h.y;
+  q.round = h.z;
+  q.e_chk = h.w;
+  q.chkm = sl->chk;
+  q.msk = sl->pad[0];
+}
+
+template <bool CL, int G = 1>
 __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring, uint64_t t_begin) {
-  constexpr uint32_t R = 1u << kCmRingLog2;
+  const uint32_t R = 1u << p.cm_ring_log2;
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
-  const uint32_t lt = lanemask_lt();
   const uint32_t dmask = (1u << kDoneLog2) - 1;
   const bool srv_pub = p.publish == CSMV_PUBLISH_SERVER;
   const uint32_t fbase = c.rt32;  // the filter (this CTA's rt stripe); slots arrive as byte offsets
   uint32_t t = *(volatile uint32_t*)&c.sh->tail;
   uint32_t gseen = t;
   unsigned long long cs = 0, wait = 0;
-  CmPayload q;
+  CmPayload q[G];  // the next unit: one batch, or a client group's G batches
   bool have = false;
   Jitter jit(p, 6);
-  for (uint32_t next = 0;; ++next) {
+  // A unit is ready when all its G flags are set.  Its G payloads were all
+  // written by one worker warp before one release fence and its flags after
+  // it, so one acquire (of the first flag) orders every payload load; the
+  // other flags are checked relaxed.  (In a cluster the acquire is LDS +
+  // CCTL.IVALL: one per unit instead of one per batch.)
+  auto try_unit = [&](uint32_t first) {
+    if constexpr (G == 1) {
+      return cm_try<CL>(ring + (first & (R - 1)), first, q[0]);
+    } else {
+      uint32_t ok = 1;
+      if (lane == 0) {
+#pragma unroll
+        for (int k = 1; k < G; ++k)
+          ok &= *(volatile uint32_t*)&ring[(first + k) & (R - 1)].flag == first + k + 1;
+        ok &= ring_ld_acquire<CL>((uint32_t)__cvta_generic_to_shared(&ring[first & (R - 1)].flag)) == first + 1;
+      }
+      if (!__shfl_sync(FULL, ok, 0)) return false;
+#pragma unroll
+      for (int k = 0; k < G; ++k) cm_load(ring + ((first + k) & (R - 1)), q[k]);
+      return true;
+    }
+  };
+  for (uint32_t next = 0;; next += G) {
     const long long tw = clock64();
-    // wait for slot `next` (unless the prefetch already found it ready)
+    // wait for the unit starting at slot `next` (unless the prefetch found it ready)
     for (uint32_t it = 0; !have;) {
-      have = cm_try<CL>(ring + (next & (R - 1)), next, q);
+      have = try_unit(next);
       if (have) break;
       uint32_t done = 0;
       if (lane == 0 && *(volatile uint32_t*)&c.sh->workers_left == 0 &&
@@ -1029,51 +1082,71 @@ __device__ void server_committer(const KParams& p, const SrvCtx& c, CmSlot* ring
     if (!have) break;
     jit();
     const long long t1 = clock64();
-    const CmPayload cur = q;
-    const bool chk = (cur.chkm >> lane) & 1u;
-    uint32_t v0 = 0, v1 = 0, v2 = 0, v3 = 0, v4 = 0, v5 = 0;
-    if (chk) {
-      v0 = filt_ld<false>(fbase + cur.w0.x);
-      v1 = filt_ld<false>(fbase + cur.w0.y);
-      v2 = filt_ld<false>(fbase + cur.w0.z);
-      v3 = filt_ld<false>(fbase + cur.w0.w);
-      v4 = filt_ld<false>(fbase + cur.w1.x);
-      v5 = filt_ld<false>(fbase + cur.w1.y);
+    CmPayload cur[G];
+#pragma unroll
+    for (int k = 0; k < G; ++k) cur[k] = q[k];
+    // every lane probes (non-live lanes carry item 0's slots, valid offsets);
+    // chk masks the result -- no predicated loads in the chain
+    uint32_t v[G][6];
+#pragma unroll
+    for (int k = 0; k < G; ++k) {
+      v[k][0] = filt_ld<false>(fbase + cur[k].w0.x);
+      v[k][1] = filt_ld<false>(fbase + cur[k].w0.y);
+      v[k][2] = filt_ld<false>(fbase + cur[k].w0.z);
+      v[k][3] = filt_ld<false>(fbase + cur[k].w0.w);
+      v[k][4] = filt_ld<false>(fbase + cur[k].w1.x);
+      v[k][5] = filt_ld<false>(fbase + cur[k].w1.y);
     }
-    // prefetch slot next+1 (its payload is only used if its flag was set)
-    have = cm_try<CL>(ring + ((next + 1) & (R - 1)), next + 1, q);
+    // prefetch the next unit (its payload is only used if all its flags were set)
+    have = try_unit(next + G);
     // a write after e_pre to one of the items raised all of its slots above
-    // e_pre (every earlier batch of the ring included)
+    // e_pre (every earlier unit of the ring included; the batches of one
+    // unit are conflict-free by the clients' pre-validation)
     // (32-bit slots here: the committer's chain is the cluster server's bound,
     // and the 16-bit age test costs more than its fewer false positives gain)
-    const uint32_t lo = max(min(v0, min(v1, v2)), min(v3, min(v4, v5)));
-    const bool ovf = chk && lo > cur.e_chk;
-    const bool commit = chk && !ovf;
-    const uint32_t cm = __ballot_sync(FULL, commit), om = __ballot_sync(FULL, ovf);
-    const uint32_t base = t + 1;
-    t += __popc(cm);
+    bool commit[G];
+    uint32_t cm[G], om[G], base[G];
+#pragma unroll
+    for (int k = 0; k < G; ++k) {
+      const bool chk = (cur[k].chkm >> lane) & 1u;
+      const uint32_t lo = max(min(v[k][0], min(v[k][1], v[k][2])), min(v[k][3], min(v[k][4], v[k][5])));
+      const bool ovf = chk && lo > cur[k].e_chk;
+      commit[k] = chk && !ovf;
+      cm[k] = __ballot_sync(FULL, commit[k]);
+      om[k] = __ballot_sync(FULL, ovf);
+      base[k] = t + 1;
+      t += __popc(cm[k]);
+    }
     if (srv_pub && t > gseen + dmask) {  // done-ring back-pressure: CTS t may reuse slot t & mask once GTS >= t - 2^20
       for (uint32_t it = 0; t > gseen + dmask;) {
         gseen = __shfl_sync(FULL, ld_relaxed(p.gts), 0);
         if ((++it & 255u) == 0 && __shfl_sync(FULL, (uint32_t)(lane == 0 && watchdog(p, t_begin, 4)), 0)) break;
       }
     }
-    if (commit) {  // the batch's last CTS: equal values for shared slots, race-free
-      filt_st<false>(fbase + cur.w0.x, t);
-      filt_st<false>(fbase + cur.w0.y, t);
-      filt_st<false>(fbase + cur.w0.z, t);
-      filt_st<false>(fbase + cur.w0.w, t);
-      filt_st<false>(fbase + cur.w1.x, t);
-      filt_st<false>(fbase + cur.w1.y, t);
+#pragma unroll
+    for (int k = 0; k < G; ++k) {
+      if (commit[k]) {  // the unit's last CTS: equal values for shared slots, race-free
+        filt_st<false>(fbase + cur[k].w0.x, t);
+        filt_st<false>(fbase + cur[k].w0.y, t);
+        filt_st<false>(fbase + cur[k].w0.z, t);
+        filt_st<false>(fbase + cur[k].w0.w, t);
+        filt_st<false>(fbase + cur[k].w1.x, t);
+        filt_st<false>(fbase + cur[k].w1.y, t);
+      }
     }
     if (lane == 0) {  // respond: round-tagged words, no fence (kernel.cuh Resp); slot release
-      const uint64_t tag = (uint64_t)cur.round << 32;
-      st_relaxed64x2(&p.resp[cur.cw].base, tag | base, tag | cm);
-      st_relaxed64(&p.resp[cur.cw].ovf, tag | om);
-      *(volatile uint32_t*)&c.sh->ring_done = next + 1;
+#pragma unroll
+      for (int k = 0; k < G; ++k) {
+        if (G == 1 || cur[k].msk != 0) {  // grouped: only the warps that submitted something
+          const uint64_t tag = (uint64_t)cur[k].round << 32;
+          st_relaxed64x2(&p.resp[cur[k].cw].base, tag | base[k], tag | cm[k]);
+          st_relaxed64(&p.resp[cur[k].cw].ovf, tag | om[k]);
+        }
+      }
+      *(volatile uint32_t*)&c.sh->ring_done = next + G;
     }
     if (lane == 0) *(volatile uint32_t*)&c.sh->tail = t;  // the CTS counter (read at exit)
-    __syncwarp();  // this batch's filter stores precede the next batch's loads
+    __syncwarp();  // this unit's filter stores precede the next unit's loads
     const long long t2 = clock64();
     wait += (unsigned long long)(t1 - tw);
     cs += (unsigned long long)(t2 - t1);
@@ -1500,7 +1573,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   const uint32_t rt_words = (uint32_t)kRtWays << local_log2;
   c.queue = c.rt + rt_words;
   c.evmax = reinterpret_cast<uint32_t*>(c.queue + (1u << c.qn_log2));
-  c.last_seen = c.evmax + (1u << local_log2);
+  c.last_seen = c.evmax + (1u << p.ev_log2);
   const uint32_t ls_words = (per + 31) / 32 * 32;
   c.sh = reinterpret_cast<SrvShared*>(c.last_seen + ls_words);
   CmSlot* ring = reinterpret_cast<CmSlot*>(reinterpret_cast<uint8_t*>(c.sh) + sizeof(SrvShared));
@@ -1516,10 +1589,10 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   const bool filt = KIND == CSMV_KIND_BANK ? p.atr_mode == CSMV_ATR_HASH : kv_filter_mode(p);
   const uint64_t rt_init = filt ? 0ull : 0xFFFFFFFFull;
   for (uint32_t i = threadIdx.x; i < rt_words; i += blockDim.x) c.rt[i] = rt_init;  // table: cts 0, no item; filter: 0
-  for (uint32_t i = threadIdx.x; i < (1u << local_log2); i += blockDim.x) c.evmax[i] = 0;
+  for (uint32_t i = threadIdx.x; i < (1u << p.ev_log2); i += blockDim.x) c.evmax[i] = 0;
   for (uint32_t i = threadIdx.x; i < (1u << c.qn_log2); i += blockDim.x) c.queue[i] = 0;
   for (uint32_t i = threadIdx.x; i < ls_words; i += blockDim.x) c.last_seen[i] = 0;
-  for (uint32_t i = threadIdx.x; i < (1u << kCmRingLog2); i += blockDim.x) ring[i].flag = 0;
+  for (uint32_t i = threadIdx.x; i < (1u << p.cm_ring_log2); i += blockDim.x) ring[i].flag = 0;
   if (threadIdx.x == 0) {
     const uint32_t g0 = *p.gts;
     c.sh->tail = g0;
@@ -1550,6 +1623,8 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
       else server_worker_generic<CL>(p, c, t_begin);
     }
     else if (!CL && p.commit == CSMV_COMMIT_ONLYCS) server_worker_onlycs<NS>(p, c, t_begin);
+    else if (cmring && p.group == 2) server_worker_cm<CL, 2>(p, c, t_begin);
+    else if (cmring && p.group == 4) server_worker_cm<CL, 4>(p, c, t_begin);
     else if (cmring) server_worker_cm<CL>(p, c, t_begin);
     else if (!CL && p.group == 2) server_worker<CL, false, 2>(p, c, t_begin);
     else if (!CL && p.group == 4) server_worker<CL, false, 4>(p, c, t_begin);
@@ -1558,7 +1633,9 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   } else if (warp == p.n_workers + 1 && rank == 0 && p.publish == CSMV_PUBLISH_SERVER) {
     server_publisher(p, c, t_begin);
   } else if (warp == kWarps - 1 && rank == 0 && cmring) {
-    server_committer<CL>(p, c, ring, t_begin);
+    if (p.group == 2) server_committer<CL, 2>(p, c, ring, t_begin);
+    else if (p.group == 4) server_committer<CL, 4>(p, c, ring, t_begin);
+    else server_committer<CL>(p, c, ring, t_begin);
   }
   if constexpr (CL) cg::this_cluster().sync();
   else __syncthreads();

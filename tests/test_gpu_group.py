@@ -51,9 +51,26 @@ def test_group_negative_control():
     assert not rep["ok"]
 
 
-@pytest.mark.parametrize("kw", [dict(server=csmv.SERVER_CLUSTER, cluster_size=4), dict(server_recv=csmv.RECV_SELF),
-                                dict(atr_mode=csmv.ATR_LIST), dict(commit=csmv.COMMIT_JVSTM),
-                                dict(debug_flags=csmv.DBG_ALT_COMMIT), dict(client_group=3)])
+@pytest.mark.parametrize("group", [2, 4])
+@pytest.mark.parametrize("kw", [dict(server=csmv.SERVER_CLUSTER, cluster_size=4),
+                                dict(server=csmv.SERVER_CLUSTER, cluster_size=16),
+                                dict(debug_flags=csmv.DBG_ALT_COMMIT),
+                                dict(server=csmv.SERVER_CLUSTER, cluster_size=8, debug_flags=csmv.DBG_JITTER)])
+def test_group_commit_ring(group, kw):
+    """Client groups into the commit ring (cluster server, or one CTA with
+    DBG_ALT_COMMIT): a request's G batches take G consecutive ring slots and
+    the committer commits them in one step of its chain."""
+    cfg = W.c2(n_items=1 << 16, n_tx=1 << 18, client_warps=148 * group, client_group=group,
+               publish=csmv.PUBLISH_SERVER, ro_streak=8, ro_adaptive=1, server_combine=8, **kw)
+    rep, stats, log, rings, descs = check(cfg)
+    assert (newest(rings, cfg.n_items, cfg.n_versions) == closed_form(cfg, descs, cfg.init_values())).all()
+    check(W.c3(n_tx=1 << 16, client_warps=148 * group, client_group=group, server=csmv.SERVER_CLUSTER,
+               cluster_size=4, ro_streak=4))
+
+
+@pytest.mark.parametrize("kw", [dict(server_recv=csmv.RECV_SELF), dict(atr_mode=csmv.ATR_LIST),
+                                dict(commit=csmv.COMMIT_JVSTM), dict(client_group=3),
+                                dict(server=csmv.SERVER_CLUSTER, cluster_size=4, client_group=8)])
 def test_group_rejects_other_servers(kw):
     kw = dict(kw)
     g = kw.pop("client_group", 2)
