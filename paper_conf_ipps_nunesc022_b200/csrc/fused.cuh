@@ -461,6 +461,10 @@ inline cudaError_t launch_ns(const KParams& p, uint32_t grid, size_t smem, cudaS
   auto kern = csmv_fused<NS, KIND, CL>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
+#ifdef CSMV_CARVEOUT  // A/B: the shared-memory share of the unified L1 (percent)
+  e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, CSMV_CARVEOUT);
+  if (e != cudaSuccess) return e;
+#endif
   if (CL) {
     e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     if (e != cudaSuccess) return e;

@@ -447,7 +447,24 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   const uint32_t ring_log2 = cm_ring_log2(group, cmring);
   // eviction watermarks: only the KV item-set table (server_worker_generic) uses them
   const uint32_t ev_log2 = (h->kind == CSMV_KIND_KV && !filt) ? rt_log2 - clog2 : 2u;  // 16 B keeps what follows aligned
-  size_t smem = server_smem_bytes(rt_log2 - clog2, per_srv, ring_log2, ev_log2);
+  // A/B knob (default off): keep the locked single-CTA bank server's 16-bit
+  // filter under CSMV_FILT_TRIM_KB of shared memory in all, with a
+  // non-power-of-two slot count, so that every SM's allocation (taken from
+  // its unified L1) stays below a carveout step.  Measured neutral at 132 KB
+  // (C2 527-537 vs 529-539 M tx/s, profiles/r02/raw/r02ai_ab_trim.jsonl),
+  // unlike dropping the unused commit ring (+12 %).
+#ifndef CSMV_FILT_TRIM_KB
+#define CSMV_FILT_TRIM_KB 0
+#endif
+  uint32_t filt16_n = 0;
+  const bool lock_filter = h->kind == CSMV_KIND_BANK && filt && n_srv == 1 && !cmring && w->commit == CSMV_COMMIT_CSMV;
+  if (lock_filter && CSMV_FILT_TRIM_KB) {
+    const size_t full = server_smem_bytes(rt_log2 - clog2, per_srv, ring_log2, ev_log2);
+    const size_t other = full - (size_t)8 * rt_region_words(rt_log2 - clog2, 0);
+    const size_t cap = (size_t)CSMV_FILT_TRIM_KB * 1024;
+    if (full > cap && cap > other + 32768) filt16_n = (uint32_t)(((cap - other) / 2) & ~(size_t)255);
+  }
+  size_t smem = server_smem_bytes(rt_log2 - clog2, per_srv, ring_log2, ev_log2, filt16_n);
   if (h->kind == CSMV_KIND_KV && smem < kv_client_smem_bytes()) smem = kv_client_smem_bytes();
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
 
@@ -537,6 +554,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.group = group;
   p.cm_ring_log2 = ring_log2;
   p.ev_log2 = ev_log2;
+  p.filt16_n = filt16_n;
   const bool traced = (w->debug_flags & CSMV_DBG_TRACE) != 0;
   if (traced && !h->d_trace) CK(cudaMalloc(&h->d_trace, sizeof(csmv_trace_rec) * kTraceCap));
   p.trace = h->d_trace;

@@ -172,6 +172,7 @@ struct KParams {
   uint32_t group;             // client warps per request (1 = per-warp batches; 2/4/8 = CTA-level batches)
   uint32_t cm_ring_log2;      // commit-ring slots (cm_ring_log2())
   uint32_t ev_log2;           // eviction-watermark words per server CTA (log2; 2 = four unused words)
+  uint32_t filt16_n;          // locked single-CTA bank server: 16-bit filter slots when trimmed (0 = 16 << rt_log2)
   csmv_trace_rec* trace;      // CSMV_DBG_TRACE buffer (kTraceCap records)
   uint32_t trace_item;        // bank account / KV set traced
   uint32_t* req_vals;         // ONLYCS: new values [n_cw][2][32] for the server-side write-back
@@ -205,8 +206,13 @@ __host__ __device__ inline uint32_t queue_log2(uint32_t n_cw) {
 // shared memory, and what it takes comes out of the SM's unified L1 --
 // dropping the unused 33 KB ring of the locked server took C2 from ~485 to
 // ~540 M tx/s (profiles/r02/raw/r02ae_ab_smem.jsonl).
-inline size_t server_smem_bytes(uint32_t local_log2, uint32_t n_cw, uint32_t ring_log2, uint32_t ev_log2) {
-  return ((size_t)32 << local_log2) + ((size_t)4 << ev_log2) + ((size_t)8 << queue_log2(n_cw)) +
+// bytes of the recent-commit table / filter region (u64 words * 8)
+__host__ __device__ inline uint32_t rt_region_words(uint32_t local_log2, uint32_t filt16_n) {
+  return filt16_n ? (filt16_n * 2u + 31u) / 32u * 4u : 4u << local_log2;
+}
+inline size_t server_smem_bytes(uint32_t local_log2, uint32_t n_cw, uint32_t ring_log2, uint32_t ev_log2,
+                                uint32_t filt16_n = 0) {
+  return (size_t)8 * rt_region_words(local_log2, filt16_n) + ((size_t)4 << ev_log2) + ((size_t)8 << queue_log2(n_cw)) +
          (((size_t)n_cw + 31) / 32 * 32) * 4 + 64 + (sizeof(CmSlot) << ring_log2);
 }
 

@@ -214,6 +214,11 @@ __device__ __forceinline__ uint32_t filt_slot(uint32_t x, int k, uint32_t slots_
   const uint32_t C[3] = {0x9E3779B1u, 0x85EBCA77u, 0xC2B2AE3Du};
   return (x * C[k]) >> (32 - slots_log2);
 }
+// the same hashes onto n slots (n not a power of two): the high word of h * n
+__device__ __forceinline__ uint32_t filt_slot_n(uint32_t x, int k, uint32_t n) {
+  const uint32_t C[3] = {0x9E3779B1u, 0x85EBCA77u, 0xC2B2AE3Du};
+  return __umulhi(x * C[k], n);
+}
 
 // 32-bit shared-window address of filter slot i (a shared::cluster address
 // of the owning CTA for the cluster server)
@@ -688,8 +693,8 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       chk[j] = mine[j] && (novalid || (lw0 <= sn[j] && lw1 <= sn[j]));
 #pragma unroll
       for (int k = 0; k < kFiltK; ++k) {
-        fa[j][k] = filt16_addr<CL>(c, filt_slot(id0[j], k, fl2));
-        fb[j][k] = filt16_addr<CL>(c, filt_slot(id1[j], k, fl2));
+        fa[j][k] = filt16_addr<CL>(c, p.filt16_n ? filt_slot_n(id0[j], k, p.filt16_n) : filt_slot(id0[j], k, fl2));
+        fb[j][k] = filt16_addr<CL>(c, p.filt16_n ? filt_slot_n(id1[j], k, p.filt16_n) : filt_slot(id1[j], k, fl2));
       }
       xor_all ^= lw0 ^ lw1 ^ sn[j];
     }
@@ -1570,7 +1575,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   c.qn_log2 = queue_log2(per);
   c.rt = reinterpret_cast<uint64_t*>(smem);
   c.rt32 = (uint32_t)__cvta_generic_to_shared(c.rt);
-  const uint32_t rt_words = (uint32_t)kRtWays << local_log2;
+  const uint32_t rt_words = rt_region_words(local_log2, p.filt16_n);
   c.queue = c.rt + rt_words;
   c.evmax = reinterpret_cast<uint32_t*>(c.queue + (1u << c.qn_log2));
   c.last_seen = c.evmax + (1u << p.ev_log2);
