@@ -228,7 +228,10 @@ struct NoPoll {
 template <int NS, typename Poll = NoPoll>
 __device__ __forceinline__ void rot_coop(const KParams& p, uint32_t act, uint32_t start, uint32_t len, uint32_t s,
                                          uint64_t tx, bool& ok, int64_t& sum, uint64_t& dg, Poll poll = Poll()) {
-  constexpr int U = NS <= 4 ? 8 : (NS == 8 ? 4 : 2);
+#ifndef CSMV_ROT_U
+#define CSMV_ROT_U 8
+#endif
+  constexpr int U = NS <= 4 ? CSMV_ROT_U : (NS == 8 ? 4 : 2);
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t N = p.n_items;
