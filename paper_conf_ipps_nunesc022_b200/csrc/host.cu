@@ -409,9 +409,11 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (cmring && n_workers > kWarps - 3) n_workers = kWarps - 3;
   // bank, one CTA, locked commit: self-receiving workers (no receiver warp)
   if (w->server_recv > CSMV_RECV_SELF) return set_err(CSMV_EINVAL, "csmv_run: unknown server_recv %u", w->server_recv);
-  const bool selfrecv = w->server_recv == CSMV_RECV_SELF && h->kind == CSMV_KIND_BANK && w->server == CSMV_SERVER_CTA &&
-                        w->atr_mode == CSMV_ATR_HASH && w->commit == CSMV_COMMIT_CSMV &&
-                        !(w->debug_flags & CSMV_DBG_ALT_COMMIT);
+  const bool kv_filt = h->kind == CSMV_KIND_KV && (h->kv_A > kKvFullWays || !(w->debug_flags & CSMV_DBG_KV_ITEMSETS));
+  const bool selfrecv = w->server_recv == CSMV_RECV_SELF && w->server == CSMV_SERVER_CTA &&
+                        (h->kind == CSMV_KIND_BANK ? w->atr_mode == CSMV_ATR_HASH && w->commit == CSMV_COMMIT_CSMV &&
+                                                         !(w->debug_flags & CSMV_DBG_ALT_COMMIT)
+                                                   : kv_filt);
   if (selfrecv) {  // warps 0..n_workers-1 workers, warp n_workers the publisher
     n_workers = w->server_workers ? w->server_workers : 4u;
     if (n_workers > kWarps - 1) n_workers = kWarps - 1;

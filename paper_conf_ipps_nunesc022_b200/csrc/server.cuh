@@ -484,9 +484,12 @@ __device__ __forceinline__ void atr_list_validate(const KParams& p, const SrvCtx
 
 // CSMV_RECV_SELF (bank, one CTA, ticket-locked commit): the worker warps
 // receive for themselves -- no receiver warp, no dispatch queue
+__device__ __forceinline__ bool kv_filter_mode(const KParams& p);
+
 __device__ __forceinline__ bool server_self_recv(const KParams& p) {
-  return p.server_recv == CSMV_RECV_SELF && p.kind == CSMV_KIND_BANK && p.n_server_ctas == 1 &&
-         p.atr_mode == CSMV_ATR_HASH && p.commit == CSMV_COMMIT_CSMV && !(p.debug & CSMV_DBG_ALT_COMMIT);
+  if (p.server_recv != CSMV_RECV_SELF || p.n_server_ctas != 1) return false;
+  if (p.kind == CSMV_KIND_KV) return kv_filter_mode(p);  // the KV filter worker, one batch per claim
+  return p.atr_mode == CSMV_ATR_HASH && p.commit == CSMV_COMMIT_CSMV && !(p.debug & CSMV_DBG_ALT_COMMIT);
 }
 
 // Self-receiving worker: sweep this worker's slice [lo, hi) of the client
@@ -1297,7 +1300,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
 // (as the bank worker).  Only clocks enter the filter: nothing else is ever
 // validated in this mode; lastw is written for all four written items.
 // ---------------------------------------------------------------------------
-template <bool CL>
+template <bool CL, bool SELF = false>
 __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
@@ -1307,12 +1310,24 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
   unsigned long long busy = 0, locked = 0, batches = 0;
   unsigned long long ph[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   Jitter jit(p, 8);
+  uint32_t my_lo = 0, my_hi = 0;  // SELF: this worker's slice of the doorbells
+  if constexpr (SELF) {
+    const uint32_t w = threadIdx.x >> 5, per = (c.cw_hi - c.cw_lo + p.n_workers - 1) / p.n_workers;
+    my_lo = min(c.cw_lo + w * per, c.cw_hi);
+    my_hi = min(my_lo + per, c.cw_hi);
+  }
   for (;;) {
     uint32_t cw;
     const long long tq = clock64();
-    if (!claim_request(c, cw)) break;
+    if constexpr (SELF) {  // sweep own slice; the claim's acquire fence orders the payload loads
+      uint32_t one[1], g;
+      if (!self_claim<1>(p, c, my_lo, my_hi, 1, one, t_begin, g)) break;
+      cw = one[0];
+    } else {
+      if (!claim_request(c, cw)) break;
+      fence_cta();  // after the receiver's acquire (see server_receiver)
+    }
     const long long t0 = clock64();
-    fence_cta();  // after the receiver's acquire (see server_receiver)
     const uint32_t sq = ld_relaxed(&p.req_hdr[cw].round);
     const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
     const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
@@ -1616,8 +1631,12 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   const bool serving = !(ring_cl && rank == 0);
   if (!CL && server_self_recv(p)) {
     // warps 0..n_workers-1 self-receiving workers, then the publisher
-    if (warp < p.n_workers) server_worker<CL, !CL>(p, c, t_begin);
-    else if (warp == p.n_workers && p.publish == CSMV_PUBLISH_SERVER) server_publisher(p, c, t_begin);
+    if (warp < p.n_workers) {
+      if constexpr (KIND == CSMV_KIND_KV) server_worker_kv_filter<CL, !CL>(p, c, t_begin);
+      else server_worker<CL, !CL>(p, c, t_begin);
+    } else if (warp == p.n_workers && p.publish == CSMV_PUBLISH_SERVER) {
+      server_publisher(p, c, t_begin);
+    }
   } else if (!serving && warp <= p.n_workers) {
     // CTA 0 of a ring cluster: no receiver, no workers
   } else if (warp == 0) {

@@ -174,3 +174,20 @@ def test_kv_small_atr():
     cfg = W.c4(n_items=1 << 14, n_tx=1 << 17, p_update_ppm=100_000, client_warps=256, server_workers=6,
                atr_capacity=256, dist=0)
     _check_kv(cfg)
+
+
+@pytest.mark.parametrize("workers,jitter", [(7, 0), (3, 0), (7, csmv.DBG_JITTER)])
+def test_kv_self_receiving_workers(workers, jitter):
+    """The KV filter worker with self-receiving worker warps
+    (CSMV_RECV_SELF): each sweeps its slice of the doorbells, no receiver."""
+    cfg = W.c4(n_items=1 << 14, n_tx=1 << 17, p_update_ppm=100_000, ro_streak=8, client_warps=256,
+               server_workers=workers, server_recv=csmv.RECV_SELF, publish=1, debug_flags=jitter)
+    pre, stats, log, fin = run(cfg)
+    oc = ocfg_of(cfg)
+    rep = oracle.kv_check(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), log,
+                          final=as_state(fin, cfg.n_items, cfg.workload.kv_ways),
+                          claims=dict(committed_update=stats["committed_update"],
+                                      committed_ro=stats["committed_ro"], gts_final=stats["gts_final"],
+                                      total_aborts=stats["total_aborts"]))
+    assert rep["ok"], (rep, stats)
+    assert stats["server_workers"] == workers
