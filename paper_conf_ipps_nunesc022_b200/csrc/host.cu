@@ -401,8 +401,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
     return set_err(CSMV_EINVAL, "csmv_run: unknown server kind %u", w->server);
   }
   // server CTA: warp 0 receiver, warps 1..n_workers workers, last warp publisher
+  // (the last warp hosts the publisher unless it runs on a client CTA or the
+  // clients publish: then it can be a 7th worker -- clamped below)
   uint32_t n_workers = w->server_workers ? w->server_workers : 4u;
-  if (n_workers > kWarps - 2) n_workers = kWarps - 2;
+  if (n_workers > kWarps - 1) n_workers = kWarps - 1;
   // bank + filter: the last warp of CTA 0 is the committer (server.cuh commit ring)
   const bool cmring = h->kind == CSMV_KIND_BANK && w->atr_mode == CSMV_ATR_HASH && w->commit == CSMV_COMMIT_CSMV &&
                       ((w->server == CSMV_SERVER_CLUSTER) != ((w->debug_flags & CSMV_DBG_ALT_COMMIT) != 0));
@@ -557,6 +559,18 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.cm_ring_log2 = ring_log2;
   p.ev_log2 = ev_log2;
   p.filt16_n = filt16_n;
+  p.gts_start = gts0;
+  // the publisher takes the last warp slot of the first client CTA when no
+  // client warp lives there (client warp cw runs on CTA cw % n_ctas, warp
+  // cw / n_ctas): it then does not share the server SM with the critical
+  // section.  CSMV_PUB_REMOTE=0 keeps it on the server CTA.
+#ifndef CSMV_PUB_REMOTE
+#define CSMV_PUB_REMOTE 1
+#endif
+  p.pub_remote = CSMV_PUB_REMOTE && w->publish == CSMV_PUBLISH_SERVER && !jvstm &&
+                 (uint64_t)(kWarps - 1) * n_ctas >= n_cw;
+  if (!selfrecv && !cmring && w->publish == CSMV_PUBLISH_SERVER && !p.pub_remote && p.n_workers > kWarps - 2)
+    p.n_workers = kWarps - 2;  // the publisher needs the server CTA's last warp
   const bool traced = (w->debug_flags & CSMV_DBG_TRACE) != 0;
   if (traced && !h->d_trace) CK(cudaMalloc(&h->d_trace, sizeof(csmv_trace_rec) * kTraceCap));
   p.trace = h->d_trace;
@@ -622,7 +636,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (jvstm) ctl.tail_final = ctl.jv_tail;
   s.client_warps = n_cw;
   s.server_ctas = n_srv;
-  s.server_workers = n_workers;
+  s.server_workers = p.n_workers;
   s.atr_entries = 4u << rt_log2;
   s.sm_count = (uint32_t)h->sm_count;
   s.kernel_launches = 1;

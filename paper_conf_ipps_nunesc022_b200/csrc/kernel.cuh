@@ -92,6 +92,7 @@ struct Ctl {
   uint32_t where;       // which spin loop fired the watchdog
   uint32_t jv_tail;     // CSMV_COMMIT_JVSTM: last CTS reserved (global CAS target)
   uint32_t trace_n;     // CSMV_DBG_TRACE: records claimed
+  uint32_t srv_done;    // server finished, tail_final valid (release; the remote publisher's exit)
 };
 constexpr uint32_t kTraceCap = 1u << 18;
 
@@ -173,6 +174,8 @@ struct KParams {
   uint32_t cm_ring_log2;      // commit-ring slots (cm_ring_log2())
   uint32_t ev_log2;           // eviction-watermark words per server CTA (log2; 2 = four unused words)
   uint32_t filt16_n;          // locked single-CTA bank server: 16-bit filter slots when trimmed (0 = 16 << rt_log2)
+  uint32_t pub_remote;        // CSMV_PUBLISH_SERVER: the publisher runs on an idle warp of the first client CTA
+  uint32_t gts_start;         // GTS when the run started
   csmv_trace_rec* trace;      // CSMV_DBG_TRACE buffer (kTraceCap records)
   uint32_t trace_item;        // bank account / KV set traced
   uint32_t* req_vals;         // ONLYCS: new values [n_cw][2][32] for the server-side write-back

@@ -577,7 +577,10 @@ constexpr bool kLastwOneTrip = CSMV_LASTW_ONE_TRIP;  // grouped requests: every 
 
 template <bool CL, bool SELF, int G = 1>
 __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
-  constexpr int M = kMaxCombine;
+#ifndef CSMV_G4_REQS
+#define CSMV_G4_REQS 2
+#endif
+  constexpr int M = G == 4 ? 4 * CSMV_G4_REQS : kMaxCombine;  // sub-batches held per critical section
   constexpr int MR = M / G;  // requests per critical section
   static_assert(!SELF || G == 1, "self-receiving workers take per-warp batches");
   const uint32_t FULL = 0xFFFFFFFFu;
@@ -1507,11 +1510,15 @@ __device__ void server_worker_onlycs(const KParams& p, const SrvCtx& c, uint64_t
 // are done.  Same invariant as P:116 (GTS = c only once every commit <= c
 // has written back), without a client-side serial chain.  CTA 0 only.
 // ---------------------------------------------------------------------------
-static __device__ void server_publisher(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
+// With pub_remote it runs on an idle warp of the first client CTA instead
+// (c == nullptr): its done-flag sweeps then use another SM's load pipe and
+// issue slots than the critical section's, and it stops once the server has
+// finished (ctl->srv_done, release) and GTS reached the final tail.
+static __device__ void server_publisher(const KParams& p, const SrvCtx* c, uint64_t t_begin, uint32_t g0) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t dmask = (1u << kDoneLog2) - 1;
-  uint32_t g = *(volatile uint32_t*)&c.sh->tail;
+  uint32_t g = g0;
   uint32_t spins = 0;
   Jitter jit(p, 10);
   // one sweep looks at the next 32 * 4 * W flags: W 16-byte loads per lane in
@@ -1565,7 +1572,13 @@ static __device__ void server_publisher(const KParams& p, const SrvCtx& c, uint6
       dw = __shfl_sync(FULL, dw, 0);
       er = __shfl_sync(FULL, er, 0);
       if (er) break;
-      if (dw >= p.n_cw && g == *(volatile uint32_t*)&c.sh->tail) break;
+      if (c) {
+        if (dw >= p.n_cw && g == *(volatile uint32_t*)&c->sh->tail) break;
+      } else {
+        uint32_t fin = 0;
+        if (lane == 0 && dw >= p.n_cw && ld_acquire(&p.ctl->srv_done)) fin = g == ld_relaxed(&p.ctl->tail_final);
+        if (__shfl_sync(FULL, fin, 0)) break;
+      }
     }
   }
 }
@@ -1634,8 +1647,8 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     if (warp < p.n_workers) {
       if constexpr (KIND == CSMV_KIND_KV) server_worker_kv_filter<CL, !CL>(p, c, t_begin);
       else server_worker<CL, !CL>(p, c, t_begin);
-    } else if (warp == p.n_workers && p.publish == CSMV_PUBLISH_SERVER) {
-      server_publisher(p, c, t_begin);
+    } else if (warp == p.n_workers && p.publish == CSMV_PUBLISH_SERVER && !p.pub_remote) {
+      server_publisher(p, &c, t_begin, c.sh->tail);
     }
   } else if (!serving && warp <= p.n_workers) {
     // CTA 0 of a ring cluster: no receiver, no workers
@@ -1654,8 +1667,8 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     else if (!CL && p.group == 4) server_worker<CL, false, 4>(p, c, t_begin);
     else if (!CL && p.group == 8) server_worker<CL, false, 8>(p, c, t_begin);
     else server_worker<CL, false>(p, c, t_begin);
-  } else if (warp == p.n_workers + 1 && rank == 0 && p.publish == CSMV_PUBLISH_SERVER) {
-    server_publisher(p, c, t_begin);
+  } else if (warp == p.n_workers + 1 && rank == 0 && p.publish == CSMV_PUBLISH_SERVER && !p.pub_remote) {
+    server_publisher(p, &c, t_begin, c.sh->tail);
   } else if (warp == kWarps - 1 && rank == 0 && cmring) {
     if (p.group == 2) server_committer<CL, 2>(p, c, ring, t_begin);
     else if (p.group == 4) server_committer<CL, 4>(p, c, ring, t_begin);
@@ -1663,7 +1676,10 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   }
   if constexpr (CL) cg::this_cluster().sync();
   else __syncthreads();
-  if (rank == 0 && threadIdx.x == 0) p.ctl->tail_final = c.sh->tail;
+  if (rank == 0 && threadIdx.x == 0) {
+    p.ctl->tail_final = c.sh->tail;
+    st_release(&p.ctl->srv_done, 1u);  // the remote publisher may stop once GTS reaches tail_final
+  }
 }
 
 }  // namespace csmvd

@@ -96,7 +96,8 @@ def test_bank_self_receiving_workers(workers):
         cfg = W.c2(n_items=1 << 14, n_tx=1 << 17, publish=1, ro_streak=8, server_workers=workers,
                    server_combine=8, client_warps=200, server_recv=recv)
         rep, stats, log, rings, descs = check(cfg)
-        assert stats["server_workers"] == (workers if recv == csmv.RECV_SELF else min(workers, 6))
+        # a receiver warp takes one of the 8; the publisher another unless it runs on a client CTA
+        assert stats["server_workers"] == (workers if recv == csmv.RECV_SELF else min(workers, 7))
         assert np.array_equal(newest(rings, cfg.n_items, cfg.n_versions),
                               closed_form(cfg, descs, cfg.init_values()))
 
