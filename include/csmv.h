@@ -57,6 +57,11 @@ extern "C" {
 #define CSMV_LOG_FULL 2u       /* + every value read */
 #define CSMV_SERVER_CTA 0u     /* single-SM server (the paper's) */
 #define CSMV_SERVER_CLUSTER 1u /* thread-block-cluster server (DSMEM) */
+#define CSMV_SERVER_PART 2u    /* item-partitioned servers (NEXT-3): cluster_size =
+                                  S = 2..8 independent server CTAs, server k owning the items that hash to k;
+                                  a batch prepares at every server owning one of its items (validate that
+                                  part, mark it pending), takes its CTS from one global counter once all
+                                  voted yes, then decides at each (record, unmark).  Bank, per-warp batches */
 #define CSMV_PUBLISH_CLIENT 0u /* client advances GTS when GTS == CTS-1 */
 #define CSMV_PUBLISH_SERVER 1u /* a server warp advances GTS over finished write-backs */
 #define CSMV_ATR_HASH 0u       /* item-indexed ATR (set-associative, smem) */

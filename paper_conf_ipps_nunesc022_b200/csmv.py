@@ -19,7 +19,7 @@ OK, EINVAL, ENOMEM, ECUDA, ESTATE, ETIMEOUT, EOVERFLOW = 0, -1, -2, -3, -4, -5, 
 KIND_BANK, KIND_KV = 0, 1
 DIST_UNIFORM, DIST_ZIPF = 0, 1
 LOG_NONE, LOG_DIGEST, LOG_FULL = 0, 1, 2
-SERVER_CTA, SERVER_CLUSTER = 0, 1
+SERVER_CTA, SERVER_CLUSTER, SERVER_PART = 0, 1, 2
 PUBLISH_CLIENT, PUBLISH_SERVER = 0, 1
 ATR_HASH, ATR_LIST, ATR_LIST_NOCV = 0, 1, 2
 COMMIT_CSMV, COMMIT_ONLYCS, COMMIT_JVSTM = 0, 1, 2

@@ -143,6 +143,26 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
   if (cw >= p.n_cw) return;
   const Group grp = make_group(p, smem);
   const bool grouped = grp.size > 1;
+  // CSMV_SERVER_PART (server_part.cuh): the servers this warp's last batch
+  // prepared at, whose decide acknowledgements are outstanding
+  const bool part = p.part_log2 != 0;
+  uint32_t dec_mask = 0, dec_round = 0, smask = 0;
+  auto wait_acks = [&]() {  // every server's decide of the previous batch was processed
+    if (!dec_mask) return;
+    uint32_t it = 0;
+    for (;;) {
+      uint32_t a = dec_round;
+      if (lane < 32 && ((dec_mask >> lane) & 1u)) a = ld_acquire(p.mdack + (size_t)lane * p.mstride + cw);
+      if (__all_sync(FULL, a == dec_round)) break;
+      if ((++it & 255u) == 0) {
+        uint32_t bad = 0;
+        if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 13);
+        if (__shfl_sync(FULL, bad, 0)) break;
+      }
+      __nanosleep(32);
+    }
+    dec_mask = 0;
+  };
   const uint64_t T = (uint64_t)p.n_cw * 32;
   uint64_t cu = kNoTx;                       // pending update
   uint64_t du_id = kNoTx;                    // cu's descriptor, drawn once (not every retry round)
@@ -326,6 +346,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       if (tracing) t_sub = globaltimer();
       pc.mark(PH_SUBMIT);
     } else if (kept) {
+      if (part) wait_acks();  // the servers still read this slot for the previous decide
       if (mine) {
         my_ids[lane] = d.src | kWriteBit;
         my_ids[32 + lane] = d.dst | kWriteBit;
@@ -342,7 +363,14 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       __syncwarp();
       fence_gpu();
       jit();  // payload written, doorbell not yet
-      if (lane == 0) st_relaxed(&p.req_seq[cw], round);
+      if (part) {  // the servers owning an item of the batch; prepared one at a time, lowest first
+        smask = __reduce_or_sync(FULL, mine ? (1u << part_owner(d.src, p.part_log2)) |
+                                                  (1u << part_owner(d.dst, p.part_log2))
+                                            : 0u);
+        if (lane == (uint32_t)(__ffs(smask) - 1)) st_relaxed(p.mreq_seq + (size_t)lane * p.mstride + cw, round);
+      } else if (lane == 0) {
+        st_relaxed(&p.req_seq[cw], round);
+      }
       if (tracing) t_sub = globaltimer();
       pc.mark(PH_SUBMIT);
     }
@@ -422,7 +450,61 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       pc.mark(PH_PUBLISH);
       d_done = true;
     };
-    const bool early_d = p.ro_adaptive && kept && p.commit == CSMV_COMMIT_CSMV;
+    // CSMV_SERVER_PART: prepare server by server in increasing order (the
+    // first was rung with the batch), each with only the lanes every earlier
+    // one accepted -- a transaction holding marks at lower servers never
+    // waits on one that needs them, so two spanning transactions cannot keep
+    // aborting each other (with all prepares at once, ~10^4 in-flight
+    // transfers on 4K accounts livelocked: each held the mark the other
+    // needed); then the CTS from the global counter and a decide at every
+    // server prepared.  A state machine (p_sm: servers still to prepare, the
+    // lowest one rung) that the read-only phase advances at every row group,
+    // like the early D of the other servers.
+    uint32_t p_ok = kept, p_om = 0, p_sm = smask, p_rung = smask & (0u - smask);
+    auto part_vote = [&](uint32_t& v, uint32_t& o) -> bool {  // the current server's vote, if in
+      uint64_t w = 0;
+      if (lane < 2) w = ld_relaxed64(&p.mresp[(size_t)(__ffs(p_sm) - 1) * p.mstride + cw].base + lane);
+      const uint64_t w1 = __shfl_sync(FULL, w, 1), w0 = __shfl_sync(FULL, w, 0);
+      if ((uint32_t)(w0 >> 32) != round || (uint32_t)(w1 >> 32) != round) return false;
+      v = (uint32_t)w0;
+      o = (uint32_t)w1;
+      return true;
+    };
+    auto part_advance = [&](uint32_t v, uint32_t o) {
+      p_ok &= v;
+      p_om |= o;
+      p_sm &= p_sm - 1;
+      if (p_sm && p_ok) {  // the next server, with the surviving lanes
+        const uint32_t k = __ffs(p_sm) - 1;
+        if (lane == 0) p.req_hdr[cw].mask = p_ok;
+        __syncwarp();
+        fence_gpu();
+        if (lane == k) st_relaxed(p.mreq_seq + (size_t)k * p.mstride + cw, round);
+        p_rung |= 1u << k;
+        return;
+      }
+      uint32_t base = 0;
+      if (lane == 0 && p_ok) {
+        base = atomicAdd(&p.ctl->cts_next, (uint32_t)__popc(p_ok)) + 1;  // the one global CTS sequence
+        // done-ring room (server publish): CTS c reuses flag c & mask only once GTS >= c - 2^20
+        for (uint32_t it = 0; base + __popc(p_ok) > ld_relaxed(p.gts) + (1u << kDoneLog2); ++it) {
+          if ((it & 255u) == 255u && (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 15))) break;
+          __nanosleep(64);
+        }
+      }
+      base = __shfl_sync(FULL, base, 0);
+      if (lane == 0) {
+        st_relaxed64(p.mdec + 2 * (size_t)cw, ((uint64_t)round << 32) | base);
+        st_relaxed64(p.mdec + 2 * (size_t)cw + 1, ((uint64_t)round << 32) | p_ok);
+      }
+      __syncwarp();
+      fence_gpu();
+      if ((p_rung >> lane) & 1u) st_relaxed(p.mdec_seq + (size_t)lane * p.mstride + cw, round);
+      dec_mask = p_rung;
+      dec_round = round;
+      phase_d(base, p_ok, p_om & ~p_ok);
+    };
+    const bool early_d = p.ro_adaptive && kept && p.commit == CSMV_COMMIT_CSMV && !part;
     // ro_adaptive: the watched response slot's first word is prefetched by
     // lane 0 one row group ahead (its latency hides behind the group's own
     // loads; a blocking poll would add an L2 round trip to every group);
@@ -430,14 +512,28 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
     uint64_t pf = 0;
     bool answered = false;
     const uint32_t wslot = kept ? cw : watch;
+    // the word that says the batch was answered
+    const uint64_t* wword = &p.resp[wslot].base;
     auto poll = [&]() {
       if (!p.ro_adaptive || !gkept || d_done || answered) return;
+      if (part) {  // advance the partitioned protocol by one step if its current vote is in
+        if (__shfl_sync(FULL, (uint32_t)(pf >> 32), 0) == round) {
+          uint32_t v, o;
+          if (part_vote(v, o)) {
+            part_advance(v, o);
+            pf = 0;
+          }
+        } else if (lane == 0) {
+          pf = ld_relaxed64(&p.mresp[(size_t)(__ffs(p_sm) - 1) * p.mstride + cw].base);
+        }
+        return;
+      }
       if (__shfl_sync(FULL, (uint32_t)(pf >> 32), 0) == round) {
         answered = true;
         uint32_t b0, c0, o0;
         if (early_d && try_response(p, cw, round, b0, c0, o0)) phase_d(b0, c0, o0);
       } else if (lane == 0) {
-        pf = ld_relaxed64(&p.resp[wslot].base);
+        pf = ld_relaxed64(wword);
       }
     };
 
@@ -485,7 +581,21 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
     if (!kept) continue;  // grouped: the server answers only the warps that submitted something
 
     // ---- D, unless the read-only phase already ran it
-    if (!d_done) {
+    if (!d_done && part) {
+      for (uint32_t it = 0; !d_done;) {  // the rest of the protocol, blocking
+        uint32_t v = 0, o = 0;
+        if (part_vote(v, o)) {
+          part_advance(v, o);
+          continue;
+        }
+        if ((++it & 255u) == 0) {
+          uint32_t bad = 0;
+          if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 14);
+          if (__shfl_sync(FULL, bad, 0)) break;
+        }
+        __nanosleep(CSMV_SLEEP_RESP);
+      }
+    } else if (!d_done) {
       uint32_t base = 0, cmask = 0, omask = 0;
       wait_response(p, cw, round, t_begin, base, cmask, omask, jit);
       phase_d(base, cmask, omask);
@@ -493,6 +603,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
     if (tracing && cts && (d.src == p.trace_item || d.dst == p.trace_item))
       trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer());
   }
+  if (part) wait_acks();  // the servers have processed our last decide before we count as done
   client_flush(p, cc);
   pc.flush(p);
 }

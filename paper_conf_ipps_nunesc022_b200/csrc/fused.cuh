@@ -447,6 +447,7 @@ __device__ __forceinline__ void client_flush(const KParams& p, const ClientCount
 #include "kv.cuh"
 #include "server.cuh"
 #include "client_kv.cuh"
+#include "server_part.cuh"
 
 namespace csmvd {
 
@@ -454,7 +455,15 @@ template <int NS, int KIND, bool CL>
 __global__ void __launch_bounds__(kBlock, 1) csmv_fused(const KParams p) {
   extern __shared__ __align__(16) uint8_t smem[];
   const uint64_t t_begin = globaltimer();
-  if (blockIdx.x < p.n_server_ctas) server_cta<NS, KIND, CL>(p, smem, t_begin);
+  if (blockIdx.x < p.n_server_ctas) {
+    if constexpr (KIND == CSMV_KIND_BANK && !CL) {
+      if (p.part_log2) {
+        server_part_cta<NS>(p, smem, t_begin);
+        return;
+      }
+    }
+    server_cta<NS, KIND, CL>(p, smem, t_begin);
+  }
   else if (p.pub_remote && blockIdx.x == p.n_server_ctas && (threadIdx.x >> 5) == kWarps - 1)
     server_publisher(p, nullptr, t_begin, p.gts_start);  // an idle client warp slot (host.cu)
   else if constexpr (KIND == CSMV_KIND_KV) client_warp_kv<NS>(p, t_begin, reinterpret_cast<uint32_t*>(smem));

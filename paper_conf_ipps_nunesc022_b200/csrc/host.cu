@@ -89,6 +89,10 @@ struct csmv {
   uint32_t* d_req_cnt = nullptr;
   Resp* d_resp = nullptr;
   uint32_t* d_req_vals = nullptr;  // CSMV_COMMIT_ONLYCS (bank)
+  // CSMV_SERVER_PART message slots (allocated on first use): 8 servers x max_cw
+  uint32_t *d_mreq_seq = nullptr, *d_mdec_seq = nullptr, *d_mdack = nullptr;
+  Resp* d_mresp = nullptr;
+  uint64_t* d_mdec = nullptr;
   uint64_t* d_jv_ws = nullptr;     // CSMV_COMMIT_JVSTM global ATR (allocated on first use)
   csmv_trace_rec* d_trace = nullptr;  // CSMV_DBG_TRACE (allocated on first use)
   bool last_traced = false;
@@ -112,7 +116,7 @@ static void free_all(csmv* h) {
   void* ps[] = {h->d_rings, h->d_key, h->d_val, h->d_lru, h->d_clk, h->d_lastw, h->d_gts, h->d_ctl,
                 h->d_stats, h->d_done, h->d_req_seq, h->d_req_hdr, h->d_req_ids, h->d_req_cnt,
                 h->d_resp, h->d_log, h->d_vals, h->d_zipf, h->d_req_vals, h->d_jv_ws, h->d_jv_tag, h->d_init,
-                h->d_kvstage, h->d_trace};
+                h->d_kvstage, h->d_trace, h->d_mreq_seq, h->d_mdec_seq, h->d_mdack, h->d_mresp, h->d_mdec};
   for (void* q : ps) cudaFree(q);
   if (h->ev0) cudaEventDestroy(h->ev0);
   if (h->ev1) cudaEventDestroy(h->ev1);
@@ -391,8 +395,18 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
 
   // server: one CTA, a thread-block cluster of C CTAs (DSMEM), or
   // none (JVSTM-GPU: every CTA is a client)
-  uint32_t n_srv = jvstm ? 0u : 1u, clog2 = 0;
-  if (w->server == CSMV_SERVER_CLUSTER) {
+  uint32_t n_srv = jvstm ? 0u : 1u, clog2 = 0, part_log2 = 0;
+  const bool part = w->server == CSMV_SERVER_PART;
+  if (part) {  // item-partitioned servers (server_part.cuh): S independent server CTAs
+    n_srv = w->cluster_size ? w->cluster_size : 2u;
+    if (n_srv < 2 || n_srv > 8 || (n_srv & (n_srv - 1)))
+      return set_err(CSMV_EINVAL, "csmv_run: CSMV_SERVER_PART needs cluster_size (servers) = 2, 4 or 8");
+    if (h->kind != CSMV_KIND_BANK || w->atr_mode != CSMV_ATR_HASH || w->commit != CSMV_COMMIT_CSMV ||
+        (w->client_group && w->client_group != 1) || (w->debug_flags & CSMV_DBG_ALT_COMMIT))
+      return set_err(CSMV_EINVAL, "csmv_run: CSMV_SERVER_PART is built for the bank workload with per-warp "
+                                  "batches (atr_mode HASH, CSMV commit)");
+    while ((1u << part_log2) < n_srv) ++part_log2;
+  } else if (w->server == CSMV_SERVER_CLUSTER) {
     n_srv = w->cluster_size ? w->cluster_size : 16u;
     if (n_srv < 2 || n_srv > 16 || (n_srv & (n_srv - 1)))
       return set_err(CSMV_EINVAL, "csmv_run: cluster_size must be 2, 4, 8 or 16");
@@ -468,13 +482,14 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
     const size_t cap = (size_t)CSMV_FILT_TRIM_KB * 1024;
     if (full > cap && cap > other + 32768) filt16_n = (uint32_t)(((cap - other) / 2) & ~(size_t)255);
   }
-  size_t smem = server_smem_bytes(rt_log2 - clog2, per_srv, ring_log2, ev_log2, filt16_n);
+  size_t smem = part ? part_smem_bytes(n_cw) : server_smem_bytes(rt_log2 - clog2, per_srv, ring_log2, ev_log2, filt16_n);
   if (h->kind == CSMV_KIND_KV && smem < kv_client_smem_bytes()) smem = kv_client_smem_bytes();
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
 
   // grid: server CTAs first, then client CTAs (client warps spread round-robin)
   p.kind = (uint32_t)h->kind;
   p.n_server_ctas = n_srv;
+  p.clustered = w->server == CSMV_SERVER_CLUSTER;
   int cap = 0;
   CK(fused_capacity(p, h->nslot, smem, &cap));
   if (cap < (int)n_srv + (int)n_srv)
@@ -483,8 +498,8 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (max_client_ctas > (uint32_t)h->sm_count - n_srv) max_client_ctas = (uint32_t)h->sm_count - n_srv;
   if (n_cw > max_client_ctas * kWarps) n_cw = max_client_ctas * kWarps;
   uint32_t n_ctas = n_cw < max_client_ctas ? n_cw : max_client_ctas;
-  if (n_srv > 1) n_ctas = (n_ctas + n_srv - 1) / n_srv * n_srv;  // grid a multiple of the cluster
-  if (n_srv > 1 && n_ctas > max_client_ctas) n_ctas = max_client_ctas / n_srv * n_srv;
+  if (p.clustered) n_ctas = (n_ctas + n_srv - 1) / n_srv * n_srv;  // grid a multiple of the cluster
+  if (p.clustered && n_ctas > max_client_ctas) n_ctas = max_client_ctas / n_srv * n_srv;
   if (n_ctas == 0) return set_err(CSMV_EINVAL, "csmv_run: no client CTA fits beside the server");
   // client warp cw runs on CTA cw mod n_ctas, warp cw / n_ctas: never more than the grid holds
   if (n_cw > n_ctas * kWarps) n_cw = n_ctas * kWarps;
@@ -543,6 +558,29 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.n_client_ctas = n_ctas;
   p.n_server_ctas = n_srv;
   p.clog2 = clog2;
+  p.clustered = w->server == CSMV_SERVER_CLUSTER;
+  p.part_log2 = part_log2;
+  if (part) {
+    const size_t m = (size_t)8 * h->max_cw;
+    if (!h->d_mreq_seq) {
+      CK(cudaMalloc(&h->d_mreq_seq, m * 4));
+      CK(cudaMalloc(&h->d_mdec_seq, m * 4));
+      CK(cudaMalloc(&h->d_mdack, m * 4));
+      CK(cudaMalloc(&h->d_mresp, m * sizeof(Resp)));
+      CK(cudaMalloc(&h->d_mdec, (size_t)h->max_cw * 16));
+    }
+    CK(cudaMemsetAsync(h->d_mreq_seq, 0, m * 4, h->stream));
+    CK(cudaMemsetAsync(h->d_mdec_seq, 0, m * 4, h->stream));
+    CK(cudaMemsetAsync(h->d_mdack, 0, m * 4, h->stream));
+    CK(cudaMemsetAsync(h->d_mresp, 0, m * sizeof(Resp), h->stream));
+    CK(cudaMemsetAsync(h->d_mdec, 0, (size_t)h->max_cw * 16, h->stream));
+    p.mstride = h->max_cw;
+    p.mreq_seq = h->d_mreq_seq;
+    p.mdec_seq = h->d_mdec_seq;
+    p.mdack = h->d_mdack;
+    p.mresp = h->d_mresp;
+    p.mdec = h->d_mdec;
+  }
   p.n_workers = n_workers;
   p.rt_log2 = rt_log2;
   p.lastw = h->d_lastw;
@@ -586,6 +624,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.watchdog_ns = (uint64_t)(w->watchdog_ms ? w->watchdog_ms : 20000u) * 1000000ull;
 
   CK(cudaMemsetAsync(h->d_ctl, 0, sizeof(Ctl), h->stream));
+  if (part) CK(cudaMemcpyAsync(&h->d_ctl->cts_next, &gts0, 4, cudaMemcpyHostToDevice, h->stream));
   if (jvstm) {  // the global ATR starts empty at the current GTS
     CK(cudaMemcpyAsync(&h->d_ctl->jv_tail, &gts0, 4, cudaMemcpyHostToDevice, h->stream));
     CK(cudaMemsetAsync(h->d_jv_tag, 0, sizeof(uint32_t) << kJvLog2, h->stream));
@@ -646,7 +685,8 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   h->last_traced = traced;
   if (ctl.error) {
     h->loaded = false;
-    return set_err(CSMV_ETIMEOUT, "csmv_run: device watchdog fired (loop %u); store state undefined", ctl.where);
+    return set_err(CSMV_ETIMEOUT, "csmv_run: device watchdog fired (loop %u; gts %u, cts %u); store state undefined",
+                   ctl.where, gts1, part ? ctl.cts_next : ctl.tail_final);
   }
   if (s.committed_update + s.committed_ro != n_tx || gts1 != ctl.tail_final)
     return set_err(CSMV_ECUDA, "csmv_run: protocol error (committed %llu of %llu, gts %u, tail %u)",

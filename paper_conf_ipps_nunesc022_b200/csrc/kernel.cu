@@ -36,7 +36,7 @@ __global__ void gen_descs_kernel(GenParams g, uint64_t tx0, uint64_t n, uint32_t
 
 static cudaError_t launch_any(const KParams& p, uint32_t nslot, uint32_t grid, size_t smem, cudaStream_t st,
                               int* occ) {
-  const bool cl = p.n_server_ctas > 1;
+  const bool cl = p.clustered != 0;
   if (p.kind == CSMV_KIND_KV)
     return cl ? launch_fused_kv_cl(p, nslot, grid, smem, st, occ) : launch_fused_kv_cta(p, nslot, grid, smem, st, occ);
   return cl ? launch_fused_bank_cl(p, nslot, grid, smem, st, occ) : launch_fused_bank_cta(p, nslot, grid, smem, st, occ);

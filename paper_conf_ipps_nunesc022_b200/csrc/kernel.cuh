@@ -93,6 +93,7 @@ struct Ctl {
   uint32_t jv_tail;     // CSMV_COMMIT_JVSTM: last CTS reserved (global CAS target)
   uint32_t trace_n;     // CSMV_DBG_TRACE: records claimed
   uint32_t srv_done;    // server finished, tail_final valid (release; the remote publisher's exit)
+  uint32_t cts_next;    // CSMV_SERVER_PART: last CTS handed out by the global counter
 };
 constexpr uint32_t kTraceCap = 1u << 18;
 
@@ -175,7 +176,17 @@ struct KParams {
   uint32_t ev_log2;           // eviction-watermark words per server CTA (log2; 2 = four unused words)
   uint32_t filt16_n;          // locked single-CTA bank server: 16-bit filter slots when trimmed (0 = 16 << rt_log2)
   uint32_t pub_remote;        // CSMV_PUBLISH_SERVER: the publisher runs on an idle warp of the first client CTA
+  // CSMV_SERVER_PART (item-partitioned servers, server_part.cuh): server k of
+  // 2^part_log2 owns the items with part_owner(x) == k
+  uint32_t part_log2;         // 0 = not partitioned
+  uint32_t mstride;           // per-server stride of the arrays below (client warps)
+  uint32_t* mreq_seq;         // [S][mstride] prepare doorbells
+  Resp* mresp;                // [S][mstride] prepare votes {ok mask, overflow mask}, round-tagged
+  uint32_t* mdec_seq;         // [S][mstride] decide doorbells
+  uint32_t* mdack;            // [S][mstride] decide acknowledgements (round)
+  uint64_t* mdec;             // [mstride][2] decide payload {round << 32 | first CTS, round << 32 | commit mask}
   uint32_t gts_start;         // GTS when the run started
+  uint32_t clustered;         // the server CTAs form a thread-block cluster (CSMV_SERVER_CLUSTER)
   csmv_trace_rec* trace;      // CSMV_DBG_TRACE buffer (kTraceCap records)
   uint32_t trace_item;        // bank account / KV set traced
   uint32_t* req_vals;         // ONLYCS: new values [n_cw][2][32] for the server-side write-back
@@ -188,6 +199,16 @@ constexpr uint32_t kKvMaxWays = 256;              // KV ways supported by the de
 constexpr uint32_t kKvFullWays = 16;              // up to here PUT read-sets are shipped item by item
 constexpr uint32_t kKvMaxRs = 2 * kKvFullWays + 1;  // keys + LRU stamps + clock
 constexpr uint32_t kKvMaxId = 2 * kKvFullWays + 2;  // RS u WS
+
+// CSMV_SERVER_PART: the server owning item x (a hash unrelated to the filter's)
+__host__ __device__ inline uint32_t part_owner(uint32_t x, uint32_t log2s) {
+  return log2s ? (x * 0x2545F491u) >> (32 - log2s) : 0u;
+}
+constexpr uint32_t kPartFiltLog2 = 13;  // 32-bit recent-commit filter slots per partition server
+constexpr uint32_t kPartPendLog2 = 15;  // pending-prepare set: item ids in 4-way buckets per partition server
+inline size_t part_smem_bytes(uint32_t n_cw) {
+  return ((size_t)4 << kPartFiltLog2) + ((size_t)4 << kPartPendLog2) + (((size_t)n_cw + 31) / 32 * 32) * 4 * 3 + 64;
+}
 
 // client smem scratch per warp (KV read/write sets of its update lanes)
 inline size_t kv_client_smem_bytes() { return (size_t)kWarps * 32 * (kKvMaxRs + 4 + 1) * 4; }

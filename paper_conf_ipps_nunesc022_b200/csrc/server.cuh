@@ -1576,7 +1576,10 @@ static __device__ void server_publisher(const KParams& p, const SrvCtx* c, uint6
         if (dw >= p.n_cw && g == *(volatile uint32_t*)&c->sh->tail) break;
       } else {
         uint32_t fin = 0;
-        if (lane == 0 && dw >= p.n_cw && ld_acquire(&p.ctl->srv_done)) fin = g == ld_relaxed(&p.ctl->tail_final);
+        if (lane == 0 && dw >= p.n_cw) {
+          if (p.part_log2) fin = g == ld_relaxed(&p.ctl->cts_next);  // every CTS is handed out by then
+          else if (ld_acquire(&p.ctl->srv_done)) fin = g == ld_relaxed(&p.ctl->tail_final);
+        }
         if (__shfl_sync(FULL, fin, 0)) break;
       }
     }
