@@ -482,7 +482,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
     const size_t cap = (size_t)CSMV_FILT_TRIM_KB * 1024;
     if (full > cap && cap > other + 32768) filt16_n = (uint32_t)(((cap - other) / 2) & ~(size_t)255);
   }
-  size_t smem = part ? part_smem_bytes(n_cw) : server_smem_bytes(rt_log2 - clog2, per_srv, ring_log2, ev_log2, filt16_n);
+  size_t smem = part ? part_smem_bytes(n_cw, part_bits_log2(h->n_items, part_log2)) : server_smem_bytes(rt_log2 - clog2, per_srv, ring_log2, ev_log2, filt16_n);
   if (h->kind == CSMV_KIND_KV && smem < kv_client_smem_bytes()) smem = kv_client_smem_bytes();
   if (smem > 227 * 1024) return set_err(CSMV_EINVAL, "csmv_run: ATR capacity too large for smem");
 
@@ -560,6 +560,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.clog2 = clog2;
   p.clustered = w->server == CSMV_SERVER_CLUSTER;
   p.part_log2 = part_log2;
+  p.part_bits_log2 = part ? part_bits_log2(h->n_items, part_log2) : 0u;
   if (part) {
     const size_t m = (size_t)8 * h->max_cw;
     if (!h->d_mreq_seq) {

@@ -179,6 +179,7 @@ struct KParams {
   // CSMV_SERVER_PART (item-partitioned servers, server_part.cuh): server k of
   // 2^part_log2 owns the items with part_owner(x) == k
   uint32_t part_log2;         // 0 = not partitioned
+  uint32_t part_bits_log2;    // pending bits per server (part_bits_log2())
   uint32_t mstride;           // per-server stride of the arrays below (client warps)
   uint32_t* mreq_seq;         // [S][mstride] prepare doorbells
   Resp* mresp;                // [S][mstride] prepare votes {ok mask, overflow mask}, round-tagged
@@ -202,12 +203,18 @@ constexpr uint32_t kKvMaxId = 2 * kKvFullWays + 2;  // RS u WS
 
 // CSMV_SERVER_PART: the server owning item x (a hash unrelated to the filter's)
 __host__ __device__ inline uint32_t part_owner(uint32_t x, uint32_t log2s) {
-  return log2s ? (x * 0x2545F491u) >> (32 - log2s) : 0u;
+  return x & ((1u << log2s) - 1);  // items spread evenly (bank and zipf ranks alike)
 }
-constexpr uint32_t kPartFiltLog2 = 13;  // 32-bit recent-commit filter slots per partition server
-constexpr uint32_t kPartPendLog2 = 15;  // pending-prepare set: item ids in 4-way buckets per partition server
-inline size_t part_smem_bytes(uint32_t n_cw) {
-  return ((size_t)4 << kPartFiltLog2) + ((size_t)4 << kPartPendLog2) + (((size_t)n_cw + 31) / 32 * 32) * 4 * 3 + 64;
+constexpr uint32_t kPartFiltLog2 = 13;      // 32-bit recent-commit filter slots per partition server
+constexpr uint32_t kPartBitsLog2Max = 20;   // pending bits per partition server (128 KiB); more items fold
+__host__ __device__ inline uint32_t part_pend_words(uint32_t bits_log2) { return bits_log2 > 5 ? 1u << (bits_log2 - 5) : 1u; }
+inline uint32_t part_bits_log2(uint64_t n_items, uint32_t log2s) {
+  uint32_t b = 5;
+  while (b < kPartBitsLog2Max && ((uint64_t)1 << b) < ((n_items + (1u << log2s) - 1) >> log2s)) ++b;
+  return b;
+}
+inline size_t part_smem_bytes(uint32_t n_cw, uint32_t bits_log2) {
+  return ((size_t)4 << kPartFiltLog2) + (size_t)4 * part_pend_words(bits_log2) + (((size_t)n_cw + 31) / 32 * 32) * 4 * 3;
 }
 
 // client smem scratch per warp (KV read/write sets of its update lanes)
