@@ -17,7 +17,9 @@ code, on a small abstract machine in the style of test_oracle_bruteforce
    in-flight prepares, then mark its items pending), takes its CTS from one
    global counter only once every server voted yes, and RECORDs its
    write-set at each server.  Every interleaving of those steps is accepted
-   by the oracle; without the pending marks some history is not.
+   by the oracle; without the pending marks some history is not.  The
+   same holds with the GPU's finer lock-free steps (a claim per item, then
+   the check; record, then release) -- and not with release before record.
 
 Test infrastructure only: the machine is test-side Python, the checker is
 oracle/ (bank_check) plus an independent commit-order replay.
@@ -68,9 +70,10 @@ class Machine:
     servers = 2: PREPARE at every owning server, DECIDE (global CTS),
     RECORD at every owning server (`pending` = in-flight prepares block)."""
 
-    def __init__(self, k, init, descs, ww=True, servers=1, pending=True, max_att=2):
+    def __init__(self, k, init, descs, ww=True, servers=1, pending=True, max_att=2, claims=False):
         self.K, self.init, self.d = k, init, descs
         self.ww, self.S, self.pending, self.max_att = ww, servers, pending, max_att
+        self.claims = claims  # the GPU's lock-free PREPARE: per-item CLAIM steps, then CHECK; REC then REL
         self.ops = []
         for t, d in enumerate(descs):
             rs, ws = rs_ws(d)
@@ -79,6 +82,12 @@ class Machine:
                 owners = sorted({x % servers for x in rs + ws})
                 if servers == 1:
                     ops.append(("COMMIT",))
+                elif claims:
+                    for o in owners:
+                        ops += [("CLAIM", o, x) for x in self.items_at(t, o)] + [("CHECK", o)]
+                    ops += [("DECIDE",)]
+                    for o in owners:
+                        ops += [("REC", o), ("REL", o)]
                 else:
                     ops += [("PREP", o) for o in owners] + [("DECIDE",)] + [("REC", o) for o in owners]
                 ops += [("WB", x) for x in ws] + [("PUBLISH",)]
@@ -139,6 +148,26 @@ class Machine:
                 else:
                     votes = votes + (srv,)
                     pend = pend[:srv] + (pend[srv] + ((t, wsx),),) + pend[srv + 1:]
+        elif kind == "CLAIM":  # atomicOr of one pending bit; a taken bit fails the lane here
+            srv, x = op[1], op[2]
+            if stat == "run":
+                if any(x in w for u, w in pend[srv] if u != t):
+                    stat = "fail"
+                    pend = pend[:srv] + (tuple(e for e in pend[srv] if e[0] != t),) + pend[srv + 1:]
+                else:
+                    pend = pend[:srv] + (pend[srv] + ((t, (x,)),),) + pend[srv + 1:]
+        elif kind == "CHECK":  # after the claims: the records after the snapshot
+            srv = op[1]
+            if stat == "run":
+                mine = set(self.items_at(t, srv))
+                if any(c > s and set(w) & mine for c, w in atr[srv]):
+                    stat = "fail"
+                    pend = pend[:srv] + (tuple(e for e in pend[srv] if e[0] != t),) + pend[srv + 1:]
+                else:
+                    votes = votes + (srv,)
+        elif kind == "REL":
+            srv = op[1]
+            pend = pend[:srv] + (tuple(e for e in pend[srv] if e[0] != t),) + pend[srv + 1:]
         elif kind == "DECIDE":
             if stat == "run":
                 tail += 1
@@ -150,7 +179,8 @@ class Machine:
             if stat == "ok":
                 wsx = tuple(sorted(x for x in ws if x % self.S == srv))
                 atr = atr[:srv] + (atr[srv] + ((cts, wsx),),) + atr[srv + 1:]
-                pend = pend[:srv] + (tuple(e for e in pend[srv] if e[0] != t),) + pend[srv + 1:]
+                if not self.claims:  # (claims: released by the REL step after the record)
+                    pend = pend[:srv] + (tuple(e for e in pend[srv] if e[0] != t),) + pend[srv + 1:]
         elif kind == "WB":
             if stat == "ok":
                 x = op[1]
@@ -304,6 +334,40 @@ def test_two_server_commit_is_opaque(name, k):
     C = sum(d["is_update"] for d in SPANNING[name])
     for st in finals:
         assert sorted(x[4] for x in st[5] if x[4]) == list(range(1, C + 1))
+
+
+@pytest.mark.parametrize("k", [1, 2])
+@pytest.mark.parametrize("name", sorted(SPANNING))
+def test_two_server_lockfree_claims_are_opaque(name, k):
+    """The GPU's server_part.cuh prepares without a lock: one atomic claim
+    per item (increasing order), then the record check; a decide records
+    first and releases after.  Every interleaving of those finer steps is
+    accepted too, with CTS 1..C."""
+    m = Machine(k, [1000] * 4, SPANNING[name], servers=2, claims=True)
+    finals = m.explore()
+    assert finals
+    C = sum(d["is_update"] for d in SPANNING[name])
+    for st in finals:
+        assert replay_ok(m, st), (name, k)
+        assert oracle_accepts(m, st), (name, k)
+        assert sorted(x[4] for x in st[5] if x[4]) == list(range(1, C + 1))
+
+
+def test_lockfree_release_before_record_is_caught():
+    """Negative control for the decide's order: releasing the bits before
+    recording the write-set lets a conflicting prepare slip in between."""
+    class Early(Machine):
+        def __init__(self, *a, **kw):
+            super().__init__(*a, **kw)
+            for ops in self.ops:  # swap every (REC o, REL o) pair
+                for i in range(len(ops) - 1):
+                    if ops[i][0] == "REC" and ops[i + 1][0] == "REL":
+                        ops[i], ops[i + 1] = ops[i + 1], ops[i]
+    bad = False
+    for name in ("chain", "same_pair"):
+        m = Early(1, [1000] * 4, SPANNING[name], servers=2, claims=True)
+        bad = bad or any(not oracle_accepts(m, st) for st in m.explore())
+    assert bad
 
 
 def test_two_server_commit_needs_pending_marks():
