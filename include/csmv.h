@@ -145,7 +145,17 @@ typedef struct csmv_workload {
                                   write-write check; allowed only for workloads without blind writes: the
                                   bank (every transfer reads what it writes: RS = WS, so validating RS is
                                   the whole check); EINVAL for KV, whose PUTs write the value blindly */
+    uint32_t retry_order;      /* CSMV_RETRY_*: client-side contention management of update retries
+                                  (the paper leaves retry scheduling open) */
 } csmv_workload;
+
+#define CSMV_RETRY_FREE 0u     /* every pending update attempts each round (optionally backoff_max) */
+#define CSMV_RETRY_FIFO 1u     /* KV: PUTs on one cache set attempt in FIFO ticket order -- a PUT takes a
+                                  ticket of its set when its lane adopts it and reads/submits only once the
+                                  set's previous ticket committed and GTS covers that commit.  All PUTs on a
+                                  set conflict (each reads and writes the set clock), so this only removes
+                                  attempts that were certain to abort; validation is unchanged.  The schedule
+                                  is timing-dependent (not for the 1-warp determinism tests) */
 
 /* ---- statistics ---- */
 #define CSMV_AB_PREVAL 0u      /* lost client pre-validation */
@@ -198,6 +208,8 @@ typedef struct csmv_log_rec {
 typedef struct csmv_trace_rec {
     uint32_t cts, snapshot;
     uint64_t t_begin, t_submit, t_response, t_publish;
+    uint64_t t_claim, t_served; /* server side: the worker took the request / stored the response
+                                   (0 where the commit path does not stamp them) */
 } csmv_trace_rec;
 
 typedef struct csmv csmv_t;

@@ -21,6 +21,7 @@ DIST_UNIFORM, DIST_ZIPF = 0, 1
 LOG_NONE, LOG_DIGEST, LOG_FULL = 0, 1, 2
 SERVER_CTA, SERVER_CLUSTER, SERVER_PART = 0, 1, 2
 PUBLISH_CLIENT, PUBLISH_SERVER = 0, 1
+RETRY_FREE, RETRY_FIFO = 0, 1
 ATR_HASH, ATR_LIST, ATR_LIST_NOCV = 0, 1, 2
 COMMIT_CSMV, COMMIT_ONLYCS, COMMIT_JVSTM = 0, 1, 2
 DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER, DBG_PHASES, DBG_KV_ITEMSETS, DBG_ALT_COMMIT, DBG_TRACE = 1, 2, 4, 8, 16, 32, 64
@@ -29,7 +30,7 @@ CLIENT_PHASES = ("read", "preval", "submit", "rot", "wait_server", "writeback", 
 ABORT_REASONS = ("preval", "conflict", "early", "overflow", "version")
 
 TRACE_DTYPE = np.dtype([("cts", "<u4"), ("snapshot", "<u4"), ("t_begin", "<u8"), ("t_submit", "<u8"),
-                        ("t_response", "<u8"), ("t_publish", "<u8")])
+                        ("t_response", "<u8"), ("t_publish", "<u8"), ("t_claim", "<u8"), ("t_served", "<u8")])
 LOG_DTYPE = np.dtype([("tx", "<u4"), ("snapshot", "<u4"), ("cts", "<u4"),
                       ("attempts", "<u4"), ("read_digest", "<u8"), ("aux", "<u8")])
 
@@ -45,7 +46,7 @@ class _Workload(C.Structure):
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
         "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers", "server_combine",
         "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms", "commit",
-        "ro_adaptive", "server_recv", "client_group", "trace_item", "elide_ww")]
+        "ro_adaptive", "server_recv", "client_group", "trace_item", "elide_ww", "retry_order")]
 
 
 class _Stats(C.Structure):
@@ -94,6 +95,7 @@ class Workload:
     client_group: int = 0
     trace_item: int = 0xFFFFFFFF
     elide_ww: int = 0
+    retry_order: int = 0
 
     def to_c(self) -> _Workload:
         return _Workload(*[getattr(self, f.name) for f in fields(self)])

@@ -600,8 +600,11 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       wait_response(p, cw, round, t_begin, base, cmask, omask, jit);
       phase_d(base, cmask, omask);
     }
-    if (tracing && cts && (d.src == p.trace_item || d.dst == p.trace_item))
-      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer());
+    if (tracing && cts && (d.src == p.trace_item || d.dst == p.trace_item)) {
+      uint64_t tc, tv;
+      trace_srv_times(p, cw, round, t_sub, tc, tv);
+      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv);
+    }
   }
   if (part) wait_acks();  // the servers have processed our last decide before we count as done
   client_flush(p, cc);

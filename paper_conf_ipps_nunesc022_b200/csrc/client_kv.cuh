@@ -1,13 +1,5 @@
 // client_kv.cuh -- the client warp of the MemcachedGPU workload.
 //
-// CSMV_KV_POLL_PREFETCH (A/B, default 0): poll the response with a load
-// issued one GET step ahead instead of a blocking load per step.  It
-// answers ~5 us sooner, yet C4 loses ~20 %: warps whose batch returns early
-// start their next round (and re-scan the hot sets) sooner, and the herd on
-// a hot set grows (tools/chain.py: restart 6.6 -> 16.9 us per link).
-#ifndef CSMV_KV_POLL_PREFETCH
-#define CSMV_KV_POLL_PREFETCH 0
-#endif
 // Same lane state machine and round phases as client_bank.cuh; GET is the
 // read-only transaction, PUT the update transaction (docs/GENERATOR.md 4).
 //
@@ -28,48 +20,113 @@ namespace csmvd {
 
 // GET(k) at snapshot s: scan set(k), stop at the matching key (then read
 // its value) or at the first empty way; never touches LRU.
-template <int NS>
-__device__ __forceinline__ int kv_get(const KParams& p, uint32_t key, uint32_t s, uint64_t& dg, uint32_t& hit) {
-  const uint32_t K = p.K, S = p.kv_S, A = p.kv_A;
+// Resumable, one memory round trip per call, so that the warp can poll its
+// response / GTS / ticket between trips (phase C): a GET in progress is
+//   vslot == 0: the key scan, next way w0 (U ways in flight per call; the
+//               over-read of at most U-1 ways past the stop is not read)
+//   vslot != 0: the value of the matching slot vslot - 1 is next.
+struct KvGet {
   uint32_t gk[4];
-  kv_key16(key, gk);
-  const uint32_t gset = kv_set(key, p.kv_T);
-  dg = 0;
-  hit = 0;
-  // U ways in flight per lane (the scan stops at a match or an empty way;
-  // the over-read of at most U-1 ways is the price of U x fewer round trips)
-  constexpr int U = NS <= 4 ? 4 : (NS == 8 ? 2 : 1);
-  for (uint32_t w0 = 0; w0 < A; w0 += U) {
-    Ring<4> r[U][NS];
+  uint32_t gset, w0, vslot, hit;
+  uint64_t dg;
+};
+
+template <int NS>
+__device__ __forceinline__ void kv_get_start(const KParams& p, uint32_t key, KvGet& g) {
+  kv_key16(key, g.gk);
+  g.gset = kv_set(key, p.kv_T);
+  g.w0 = g.vslot = g.hit = 0;
+  g.dg = 0;
+}
+
+// One step of a GET, split in two so that the warp can look at its polls
+// (issued before the step's loads) while the loads are in flight:
+// kv_get_issue puts the step's loads in flight into rb, kv_get_finish
+// evaluates them; fin = the GET is complete (g.dg, g.hit final).
+template <int NS>
+struct KvStep {
+  static constexpr int U = NS <= 4 ? 4 : (NS == 8 ? 2 : 1);  // key ways per step
+  static constexpr int R = U * NS;                           // Ring<4> registers per step
+  static constexpr bool kValOne = 2 * NS <= R;               // the value ring fits: one trip
+};
+
+template <int NS>
+__device__ __forceinline__ void kv_get_issue(const KParams& p, const KvGet& g, Ring<4> (&rb)[KvStep<NS>::R]) {
+  constexpr int U = KvStep<NS>::U;
+  const uint32_t A = p.kv_A;
+  if (g.vslot) {  // the whole value ring (8-word versions as two 4-word halves)
+    if constexpr (KvStep<NS>::kValOne) {
+      const uint64_t* ring = p.kv_val + (size_t)(g.vslot - 1) * NS * 8;
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      if (w0 + u < A) {
-        const uint64_t* ring = p.kv_key + (size_t)(gset * A + w0 + u) * NS * 4;
-#pragma unroll
-        for (int j = 0; j < NS; ++j) r[u][j] = ld_ring<4>(ring + j * 4);
-      }
+      for (int j = 0; j < 2 * NS; ++j) rb[j] = ld_ring<4>(ring + j * 4);
     }
+    return;
+  }
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      if (w0 + u >= A) break;
-      const uint32_t slot = gset * A + w0 + u;
-      uint32_t k4[4];
-      int rr = kv_key_pick<NS>(p.kv_key + (size_t)slot * NS * 4, r[u], K, s, true, k4);
-      if (rr != RD_OK) return rr;
+  for (int u = 0; u < U; ++u) {
+    if (g.w0 + u < A) {
+      const uint64_t* ring = p.kv_key + (size_t)(g.gset * A + g.w0 + u) * NS * 4;
 #pragma unroll
-      for (int j = 0; j < 4; ++j) dg += dig_word(slot, j, k4[j]);
-      if (k4[0] == gk[0] && k4[1] == gk[1] && k4[2] == gk[2] && k4[3] == gk[3]) {
-        uint32_t val[8];
-        rr = kv_read_mw<NS, 8>(p.kv_val + (size_t)slot * NS * 8, K, s, true, val);
-        if (rr != RD_OK) return rr;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) dg += dig_word(S + slot, j, val[j]);
-        hit = w0 + u + 1;
-        return RD_OK;
-      }
-      if (!(k4[0] | k4[1] | k4[2] | k4[3])) return RD_OK;
+      for (int j = 0; j < NS; ++j) rb[u * NS + j] = ld_ring<4>(ring + j * 4);
     }
   }
+}
+
+template <int NS>
+__device__ __forceinline__ int kv_get_finish(const KParams& p, uint32_t s, KvGet& g,
+                                             const Ring<4> (&rb)[KvStep<NS>::R], bool& fin) {
+  constexpr int U = KvStep<NS>::U;
+  const uint32_t K = p.K, S = p.kv_S, A = p.kv_A;
+  fin = false;
+  if (g.vslot) {  // + a re-read of the chosen version if a newer one is present (kv_key_pick)
+    const uint32_t slot = g.vslot - 1;
+    const uint64_t* ring = p.kv_val + (size_t)slot * NS * 8;
+    uint32_t val[8];
+    int rr;
+    if constexpr (KvStep<NS>::kValOne) {
+      Ring<8> rv[NS];
+#pragma unroll
+      for (int j = 0; j < NS; ++j)
+#pragma unroll
+        for (int w = 0; w < 4; ++w) {
+          rv[j].s[w] = rb[2 * j].s[w];
+          rv[j].s[4 + w] = rb[2 * j + 1].s[w];
+        }
+      rr = kv_key_pick<NS, 8>(ring, rv, K, s, true, val);
+    } else {
+      rr = kv_read_mw<NS, 8>(ring, K, s, true, val);
+    }
+    if (rr != RD_OK) return rr;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) g.dg += dig_word(S + slot, j, val[j]);
+    fin = true;
+    return RD_OK;
+  }
+  const uint32_t w0 = g.w0;
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    if (w0 + u >= A) break;
+    const uint32_t slot = g.gset * A + w0 + u;
+    Ring<4> ru[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) ru[j] = rb[u * NS + j];
+    uint32_t k4[4];
+    const int rr = kv_key_pick<NS>(p.kv_key + (size_t)slot * NS * 4, ru, K, s, true, k4);
+    if (rr != RD_OK) return rr;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) g.dg += dig_word(slot, j, k4[j]);
+    if (k4[0] == g.gk[0] && k4[1] == g.gk[1] && k4[2] == g.gk[2] && k4[3] == g.gk[3]) {
+      g.hit = w0 + u + 1;
+      g.vslot = slot + 1;  // the value next
+      return RD_OK;
+    }
+    if (!(k4[0] | k4[1] | k4[2] | k4[3])) {
+      fin = true;
+      return RD_OK;
+    }
+  }
+  g.w0 = w0 + U;
+  fin = g.w0 >= A;
   return RD_OK;
 }
 
@@ -85,6 +142,9 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
   uint32_t dk_key = 0;
   uint64_t cr = (uint64_t)cw * 32 + lane;
   uint32_t att_u = 0, att_r = 0, hold = 0, n_srv_ab = 0;
+  // CSMV_RETRY_FIFO: the pending PUT's ticket of its set (taken at adoption)
+  const bool tickets = p.kv_tk_next != nullptr;
+  uint32_t tk = 0;
   ClientCounters cc;
   uint32_t round = 0;
   const uint32_t K = p.K, S = p.kv_S, A = p.kv_A, Tn = p.kv_T;
@@ -120,13 +180,36 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     KvTx d{};
     uint32_t kk[4] = {0, 0, 0, 0};
     uint32_t victim = 0, tset = 0, clk = 0, nrs = 0;
+    int iv = 0, ic = 0;  // ring slots the PUT's versions replace: key/value/LRU rings, clock ring
     uint64_t rdig = 0;
     uint32_t need = 0;  // a PUT that met a version newer than s retries once GTS >= need
+    bool adopted = false;
     if (cu == kNoTx && cr < p.n_tx && gen_is_update(p.gen, cr)) {
       cu = cr;
       cr += T;
+      adopted = true;
+    }
+    if (tickets) {
+      // CSMV_RETRY_FIFO: a PUT takes its set's next ticket when adopted; the
+      // lanes of the warp adopting PUTs on one set take consecutive tickets
+      // in lane order with one atomic (the set's lowest such lane adds)
+      const uint32_t am = __ballot_sync(FULL, adopted);
+      if (am) {
+        if (adopted) {
+          dk_key = gen_kv_key(p.gen, cu);
+          dk_id = cu;
+        }
+        const uint32_t ts = adopted ? kv_set(dk_key, Tn) : 0xFFFFFFFFu;
+        const uint32_t peers = __match_any_sync(FULL, ts) & am;
+        const uint32_t leader = adopted ? (uint32_t)__ffs(peers) - 1 : lane;
+        uint32_t b = 0;
+        if (adopted && lane == leader) b = atomicAdd(p.kv_tk_next + ts, (uint32_t)__popc(peers));
+        b = __shfl_sync(FULL, b, leader);
+        if (adopted) tk = b + __popc(peers & lt);
+      }
     }
     bool pending = false;  // a PUT to read this round
+    bool tkwait = false;   // CSMV_RETRY_FIFO: an earlier ticket of the set is still being served
     if (cu != kNoTx) {
       if (hold) {
         --hold;
@@ -137,10 +220,24 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           dk_id = cu;
         }
         d = gen_kv_k(p.gen, cu, dk_key);
-        kv_key16(d.key, kk);
         tset = kv_set(d.key, Tn);
-        ++att_u;
-        pending = true;
+        if (tickets) {
+          // the turn of this ticket: the previous one committed (its CTS in
+          // the low word) -- read only once the snapshot covers that commit
+          const uint64_t sv = ld_relaxed64(p.kv_tk_serv + tset);
+          if ((uint32_t)(sv >> 32) != tk) {
+            tkwait = true;
+            status = ST_WAIT;
+          } else if ((uint32_t)sv > s) {
+            need = (uint32_t)sv;
+            status = ST_WAIT;
+          }
+        }
+        if (status != ST_WAIT) {
+          kv_key16(d.key, kk);
+          ++att_u;
+          pending = true;
+        }
       }
     }
     // Pre-validation before the reads ({set clock} u WS requests): two PUTs
@@ -166,13 +263,13 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         int r = RD_OK;
         uint32_t seen = 0;  // newest version timestamp the reads met
         victim = 0xFFFFFFFFu;
-        // the set clock first: every PUT on the set writes it, so a PUT
-        // committed after s on this set shows here after one load and the
-        // scans are skipped (the abort is the same: the clock is in RS)
-        if (compact) {
-          r = kv_read_1<NS>(p.kv_clk + (size_t)tset * NS, K, s, clk, &seen);
-          if (r == RD_OK) rdig += dig1(3 * S + tset, clk);
-        }
+        // The set clock's whole ring (one 64-bit word per version: one
+        // load, no re-read) travels with the first group of key ways.  It
+        // is evaluated first: every PUT on the set writes it, so a PUT
+        // committed after s on this set shows there and the rest of the
+        // scan is skipped (the abort is the same: the clock is in RS).
+        const Ring<NS> rcl = ld_ring<NS>(p.kv_clk + (size_t)tset * NS);
+        bool clk_done = false;
         // key scan, U ways in flight (as in kv_get), stop at match or empty;
         // the ways loaded past the stop are not read (not in RS)
         constexpr int U = NS <= 4 ? 4 : (NS == 8 ? 2 : 1);
@@ -186,6 +283,12 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
               for (int j = 0; j < NS; ++j) rk[u][j] = ld_ring<4>(ring + j * 4);
             }
           }
+          if (compact && !clk_done) {
+            clk_done = true;
+            r = kv_read_clk<NS>(rcl, K, s, clk, seen, ic);
+            if (r != RD_OK) break;
+            rdig += dig1(3 * S + tset, clk);
+          }
 #pragma unroll
           for (int u = 0; u < U; ++u) {
             if (w0 + u >= A || victim != 0xFFFFFFFFu || r != RD_OK) break;
@@ -197,8 +300,17 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
 #pragma unroll
             for (int j = 0; j < 4; ++j) rdig += dig_word(slot, j, key[j]);
             if ((key[0] == kk[0] && key[1] == kk[1] && key[2] == kk[2] && key[3] == kk[3]) ||
-                !(key[0] | key[1] | key[2] | key[3]))
+                !(key[0] | key[1] | key[2] | key[3])) {
               victim = slot;
+              // the key, value and LRU rings of a slot are written together by
+              // every PUT (same CTS, same replacement rule) from identical
+              // initial rings, so their slot timestamps are identical and the
+              // key ring read here fixes the slot all three versions replace
+              uint32_t ts[NS];
+#pragma unroll
+              for (int j = 0; j < NS; ++j) ts[j] = (uint32_t)(rk[u][j].s[0] >> 32);
+              iv = kv_install_slot<NS>(ts, K);
+            }
           }
         }
         if (r == RD_OK && victim == 0xFFFFFFFFu) {
@@ -231,12 +343,16 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
               if (w0 + u == 0 || l < best) {
                 best = l;
                 victim = slot;
+                uint32_t ts[NS];  // the LRU ring's slot timestamps = the key and value rings' (above)
+#pragma unroll
+                for (int j = 0; j < NS; ++j) ts[j] = (uint32_t)(rl[u].s[j] >> 32);
+                iv = kv_install_slot<NS>(ts, K);
               }
             }
           }
         }
         if (r == RD_OK && !compact) {
-          r = kv_read_1<NS>(p.kv_clk + (size_t)tset * NS, K, s, clk, &seen);
+          r = kv_read_clk<NS>(rcl, K, s, clk, seen, ic);
           if (r == RD_OK) {
             RS[nrs++ * 32 + lane] = 3 * S + tset;
             rdig += dig1(3 * S + tset, clk);
@@ -246,7 +362,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           need = seen;  // retry once GTS covers the newer version (its commit is then visible)
           cc.abort(CSMV_AB_EARLY, true);
           status = ST_ABORT;
-          if (p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
+          if (p.backoff_max && !tickets) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
         } else if (r == RD_MISS) {
           need = s + 1;  // every version <= s is recycled: only a newer snapshot can read it
           cc.abort(CSMV_AB_VERSION, true);
@@ -344,59 +460,97 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       pc.mark(PH_SUBMIT);
     }
 
-    // ---- C: GETs at s while the batch is at the server, one
-    // per active lane per step.  ro_adaptive ends the run early, warp-wide:
-    // once the server has answered the warp's batch; with ro_adaptive = 2
-    // also -- when the warp submitted nothing because its PUTs read versions
-    // newer than s -- as soon as GTS covers the newest of those versions (a
-    // retry can then read them).
+    bool have_resp = false;
+    uint32_t base = 0, cmask = 0, omask = 0;
+    // ---- C: GETs at s while the batch is at the server: each
+    // active lane runs up to lim GETs, one after another, ending its run at
+    // its next update or a VERSION miss (the same GETs per round as one GET
+    // per lane per step).  The lanes advance one memory round trip per
+    // iteration, each on its own GET, and the warp polls between trips: with
+    // ro_adaptive the run ends early, warp-wide, once the server has
+    // answered the warp's batch; with ro_adaptive = 2 also -- when the warp
+    // submitted nothing because its PUTs read versions newer than s -- as
+    // soon as GTS covers the newest of those versions (a retry can then read
+    // them); and (CSMV_RETRY_FIFO) when a waiting PUT's turn comes.  A GET
+    // cut short is not an attempt: it runs again in a later round.
     {
-      const bool blocked = cu != kNoTx && status == ST_ABORT && need != 0;
+      const bool blocked = cu != kNoTx && (status == ST_ABORT || status == ST_WAIT) && need != 0;
       uint32_t need_min = blocked ? need : 0xFFFFFFFFu;
       need_min = __reduce_min_sync(FULL, need_min);
+      const bool any_tkwait = __any_sync(FULL, tkwait);
+      const bool poll_gts = p.ro_adaptive >= 2 && !kept && need_min != 0xFFFFFFFFu;
       bool run = streak || cu == kNoTx;
       const uint32_t lim = streak ? streak : 1u;
-      uint64_t pf = 0;  // CSMV_KV_POLL_PREFETCH: the response's first word, prefetched one GET step ahead
-      (void)pf;
-      for (uint32_t n_ro = 0; n_ro < lim; ++n_ro) {
-        bool has = run && cr < p.n_tx && !gen_kv_is_update(p.gen, cr);  // an update: the next round adopts it
-        if (!__any_sync(FULL, has)) break;
-        if (has) {
-          const KvTx g = gen_kv(p.gen, cr);
+      uint32_t n_ro = 0;  // GETs this lane completed this round
+      bool act = false;   // a GET in progress
+      bool idle = true;   // no GET ran this round
+      KvGet g;
+      for (;;) {
+        if (!act && run && n_ro < lim && cr < p.n_tx && !gen_kv_is_update(p.gen, cr)) {
+          kv_get_start<NS>(p, gen_kv_key(p.gen, cr), g);  // an update: the next round adopts it
           ++att_r;
-          uint64_t dg;
-          uint32_t hit;
-          if (kv_get<NS>(p, g.key, s, dg, hit) != RD_OK) {
-            cc.abort(CSMV_AB_VERSION, false);  // retried next round (P:291)
-            run = false;
-          } else {
-            if (p.log_mode) log_commit(p, cr, s, 0, att_r, dg, hit);
-            ++cc.c_ro;
-            cc.ro_ck ^= dg;
-            cr += T;
-            att_r = 0;
-          }
+          act = true;
         }
+        if (!__any_sync(FULL, act)) break;
+        idle = false;
+        // this trip's polls, issued before its loads and looked at while
+        // they are in flight: lanes 0-2 the three response words (the
+        // answer is then complete: no further load), lane 0 GTS, waiting
+        // PUTs their set's ticket word
+        uint64_t pv = 0, sv = 0;
         if (p.ro_adaptive) {
           if (kept) {
-#if CSMV_KV_POLL_PREFETCH
-            if (__shfl_sync(FULL, (uint32_t)(pf >> 32), 0) == round) break;
-            if (lane == 0) pf = ld_relaxed64(&p.resp[cw].base);
-#else
-            if ((uint32_t)(warp_ld_relaxed64(&p.resp[cw].base) >> 32) == round) break;
-#endif
+            if (lane < 3) pv = ld_relaxed64(&p.resp[cw].base + lane);
+          } else if (poll_gts && lane == 0) {
+            pv = ld_relaxed(p.gts);
           }
-          if (p.ro_adaptive >= 2 && !kept && need_min != 0xFFFFFFFFu && warp_ld_relaxed(p.gts) >= need_min) break;
+        }
+        if (tkwait) sv = ld_relaxed64(p.kv_tk_serv + tset);
+        Ring<4> rb[KvStep<NS>::R];
+        if (act) kv_get_issue<NS>(p, g, rb);
+        if (p.ro_adaptive) {
+          if (kept) {
+            const uint64_t b = __shfl_sync(FULL, pv, 0), c = __shfl_sync(FULL, pv, 1), o = __shfl_sync(FULL, pv, 2);
+            if ((uint32_t)(b >> 32) == round && (uint32_t)(c >> 32) == round && (uint32_t)(o >> 32) == round) {
+              have_resp = true;
+              base = (uint32_t)b;
+              cmask = (uint32_t)c;
+              omask = (uint32_t)o;
+              break;
+            }
+          } else if (poll_gts && (uint32_t)__shfl_sync(FULL, pv, 0) >= need_min) {
+            break;
+          }
+        }
+        if (any_tkwait && __any_sync(FULL, tkwait && (uint32_t)(sv >> 32) == tk)) break;  // a turn came
+        if (act) {
+          bool fin;
+          if (kv_get_finish<NS>(p, s, g, rb, fin) != RD_OK) {
+            cc.abort(CSMV_AB_VERSION, false);  // retried next round (P:291)
+            run = false;
+            act = false;
+          } else if (fin) {
+            if (p.log_mode) log_commit(p, cr, s, 0, att_r, g.dg, g.hit);
+            ++cc.c_ro;
+            cc.ro_ck ^= g.dg;
+            cr += T;
+            att_r = 0;
+            act = false;
+            ++n_ro;
+          }
         }
       }
+      if (act) --att_r;  // cut short: not an attempt
+      // nothing to submit, read or wait on the server for: back off before
+      // the next round's polls (CSMV_RETRY_FIFO lanes waiting for a turn)
+      if (tickets && !kept && idle) __nanosleep(256);
     }
     __syncwarp();
     pc.mark(PH_ROT);
     if (!kept) continue;
 
-    // ---- D: response, write-back, GTS
-    uint32_t base = 0, cmask = 0, omask = 0;
-    wait_response(p, cw, round, t_begin, base, cmask, omask, jit);
+    // ---- D: response (unless phase C's poll already has it), write-back, GTS
+    if (!have_resp) wait_response(p, cw, round, t_begin, base, cmask, omask, jit);
     const uint64_t t_resp = tracing ? globaltimer() : 0;
     if (p.commit == CSMV_COMMIT_ONLYCS) fence_gpu();  // acquire: the server's write-backs
     pc.mark(PH_WAIT);
@@ -406,22 +560,20 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       if ((cmask >> lane) & 1u) {
         // Client-side write-back: the paper's 4 writes.
         cts = base + __popc(cmask & lt);
+        // CSMV_RETRY_FIFO: hand the set to the next ticket, which reads once GTS covers cts
+        if (tickets) st_relaxed64(p.kv_tk_serv + tset, ((uint64_t)(tk + 1) << 32) | cts);
         const uint32_t cn = clk + 1;
-        // the four rings' slot timestamps in one round trip, then the stores
+        // stores only: the slots were fixed by the read (the rings are as
+        // read -- nothing wrote the set after s: this commit validated)
         uint64_t* rk = p.kv_key + (size_t)victim * NS * 4;
         uint64_t* rv = p.kv_val + (size_t)victim * NS * 8;
         uint64_t* rl = p.kv_lru + (size_t)victim * NS;
         uint64_t* rc = p.kv_clk + (size_t)tset * NS;
-        uint32_t tk[NS], tv[NS], tl[NS], tc[NS];
-        kv_ring_ts<NS, 4>(rk, K, tk);
-        kv_ring_ts<NS, 8>(rv, K, tv);
-        kv_ring_ts<NS, 1>(rl, K, tl);
-        kv_ring_ts<NS, 1>(rc, K, tc);
         const uint32_t cn1[1] = {cn};
-        kv_install<NS, 4>(rk, tk, K, cts, kk);
-        kv_install<NS, 8>(rv, tv, K, cts, d.val);
-        kv_install<NS, 1>(rl, tl, K, cts, cn1);
-        kv_install<NS, 1>(rc, tc, K, cts, cn1);
+        kv_install_at<4>(rk, iv, cts, kk);
+        kv_install_at<8>(rv, iv, cts, d.val);
+        kv_install_at<1>(rl, iv, cts, cn1);
+        kv_install_at<1>(rc, ic, cts, cn1);
         if (p.log_mode) {
           uint64_t wd = dig1(2 * S + victim, cn) + dig1(3 * S + tset, cn);
 #pragma unroll
@@ -437,7 +589,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       } else {
         const bool ovf = (omask >> lane) & 1u;
         cc.abort(ovf ? CSMV_AB_OVERFLOW : CSMV_AB_CONFLICT, true);
-        if (!ovf && p.backoff_max) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
+        if (!ovf && p.backoff_max && !tickets) hold = min(p.backoff_max, 1u << min(n_srv_ab++, 8u));
       }
     }
     __syncwarp();
@@ -463,8 +615,11 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       }
     }
     pc.mark(PH_PUBLISH);
-    if (tracing && cts && tset == p.trace_item)
-      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer());
+    if (tracing && cts && tset == p.trace_item) {
+      uint64_t tc, tv;
+      trace_srv_times(p, cw, round, t_sub, tc, tv);
+      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv);
+    }
   }
   client_flush(p, cc);
   pc.flush(p);

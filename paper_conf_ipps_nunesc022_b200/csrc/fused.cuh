@@ -35,7 +35,7 @@
 
 namespace csmvd {
 
-enum : int { ST_NONE = 0, ST_RO_OK, ST_CAND, ST_UPD_OK, ST_ABORT };
+enum : int { ST_NONE = 0, ST_RO_OK, ST_CAND, ST_UPD_OK, ST_ABORT, ST_WAIT };
 
 // --------------------------------------------------------------------------
 // VBox read (TXRead) and write-back
@@ -383,8 +383,38 @@ struct PhaseClock {
 };
 
 // CSMV_DBG_TRACE: one record per committed writer of the traced item
+// CSMV_DBG_TRACE, server side: the worker stamps when it claimed a request
+// and when it stores the response into the response's spare word -- 16 bits
+// of the round, then the low 24 bits of each globaltimer value (ns; the
+// client rebuilds them next to its own submit time).  Stored before the
+// round-tagged words; the client reads it after them, so a stale stamp is
+// possible (diagnostics only) and shows as a round mismatch or an odd delta.
+__device__ __forceinline__ uint64_t trace_now(const KParams& p) {
+  return (p.debug & CSMV_DBG_TRACE) ? globaltimer() : 0ull;
+}
+__device__ __forceinline__ void trace_served(const KParams& p, uint32_t cw, uint32_t round, uint64_t t_claim) {
+  if (p.debug & CSMV_DBG_TRACE)
+    st_relaxed64(&p.resp[cw].pad, ((uint64_t)(round & 0xFFFFu) << 48) | ((t_claim & 0xFFFFFFull) << 24) |
+                                      (globaltimer() & 0xFFFFFFull));
+}
+// the server stamps of warp cw's answered request `round` (0, 0 if absent)
+__device__ __forceinline__ void trace_srv_times(const KParams& p, uint32_t cw, uint32_t round, uint64_t t_sub,
+                                                uint64_t& tc, uint64_t& tv) {
+  const uint64_t v = ld_relaxed64(&p.resp[cw].pad);
+  tc = tv = 0;
+  if ((uint32_t)(v >> 48) != (round & 0xFFFFu)) return;
+  const uint64_t ref = t_sub - (1ull << 22);  // the claim may be stamped a little before t_sub is read
+  auto rebuild = [&](uint64_t lo) {
+    uint64_t t = (ref & ~0xFFFFFFull) | lo;
+    if (t < ref) t += 1ull << 24;
+    return t;
+  };
+  tc = rebuild((v >> 24) & 0xFFFFFFull);
+  tv = rebuild(v & 0xFFFFFFull);
+}
+
 __device__ __forceinline__ void trace_commit(const KParams& p, uint32_t cts, uint32_t s, uint64_t tb, uint64_t ts,
-                                             uint64_t tr, uint64_t tp) {
+                                             uint64_t tr, uint64_t tp, uint64_t tc = 0, uint64_t tv = 0) {
   const uint32_t i = atomicAdd(&p.ctl->trace_n, 1u);
   if (i < kTraceCap) {
     csmv_trace_rec r;
@@ -394,6 +424,8 @@ __device__ __forceinline__ void trace_commit(const KParams& p, uint32_t cts, uin
     r.t_submit = ts;
     r.t_response = tr;
     r.t_publish = tp;
+    r.t_claim = tc;
+    r.t_served = tv;
     p.trace[i] = r;
   }
 }

@@ -97,6 +97,7 @@ struct csmv {
   csmv_trace_rec* d_trace = nullptr;  // CSMV_DBG_TRACE (allocated on first use)
   bool last_traced = false;
   uint32_t* d_jv_tag = nullptr;
+  uint32_t* d_tk = nullptr;  // CSMV_RETRY_FIFO: u32 next[T] + u64 serving[T] (allocated on first use)
   // logs
   csmv_log_rec* d_log = nullptr;
   uint64_t log_cap = 0;
@@ -116,7 +117,7 @@ static void free_all(csmv* h) {
   void* ps[] = {h->d_rings, h->d_key, h->d_val, h->d_lru, h->d_clk, h->d_lastw, h->d_gts, h->d_ctl,
                 h->d_stats, h->d_done, h->d_req_seq, h->d_req_hdr, h->d_req_ids, h->d_req_cnt,
                 h->d_resp, h->d_log, h->d_vals, h->d_zipf, h->d_req_vals, h->d_jv_ws, h->d_jv_tag, h->d_init,
-                h->d_kvstage, h->d_trace, h->d_mreq_seq, h->d_mdec_seq, h->d_mdack, h->d_mresp, h->d_mdec};
+                h->d_kvstage, h->d_trace, h->d_mreq_seq, h->d_mdec_seq, h->d_mdack, h->d_mresp, h->d_mdec, h->d_tk};
   for (void* q : ps) cudaFree(q);
   if (h->ev0) cudaEventDestroy(h->ev0);
   if (h->ev1) cudaEventDestroy(h->ev1);
@@ -372,6 +373,9 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (w->elide_ww && h->kind == CSMV_KIND_KV)
     return set_err(CSMV_EINVAL, "csmv_run: elide_ww refused: KV PUTs write blindly (value, LRU), so the "
                                 "write-write check of P:115 cannot be omitted");
+  if (w->retry_order > CSMV_RETRY_FIFO) return set_err(CSMV_EINVAL, "csmv_run: unknown retry_order %u", w->retry_order);
+  if (w->retry_order == CSMV_RETRY_FIFO && h->kind != CSMV_KIND_KV)
+    return set_err(CSMV_EINVAL, "csmv_run: CSMV_RETRY_FIFO is built for the KV workload (one set per PUT)");
   if (w->commit > CSMV_COMMIT_JVSTM) return set_err(CSMV_EINVAL, "csmv_run: unknown commit %u", w->commit);
   const bool jvstm = w->commit == CSMV_COMMIT_JVSTM;
   if (w->commit != CSMV_COMMIT_CSMV && (h->kind != CSMV_KIND_BANK || w->server != CSMV_SERVER_CTA))
@@ -629,6 +633,13 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   if (jvstm) {  // the global ATR starts empty at the current GTS
     CK(cudaMemcpyAsync(&h->d_ctl->jv_tail, &gts0, 4, cudaMemcpyHostToDevice, h->stream));
     CK(cudaMemsetAsync(h->d_jv_tag, 0, sizeof(uint32_t) << kJvLog2, h->stream));
+  }
+  if (w->retry_order == CSMV_RETRY_FIFO) {  // tickets restart at 0 every run (every one taken is served by its end)
+    const size_t tkb = (size_t)h->kv_T * 12;
+    if (!h->d_tk) CK(cudaMalloc(&h->d_tk, tkb));
+    CK(cudaMemsetAsync(h->d_tk, 0, tkb, h->stream));
+    p.kv_tk_serv = reinterpret_cast<uint64_t*>(h->d_tk);
+    p.kv_tk_next = h->d_tk + 2 * (size_t)h->kv_T;
   }
   CK(cudaMemsetAsync(h->d_stats, 0, sizeof(DevStats), h->stream));
   CK(cudaMemsetAsync(h->d_req_seq, 0, n_cw * sizeof(uint32_t), h->stream));

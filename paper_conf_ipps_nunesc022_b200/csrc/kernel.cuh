@@ -194,6 +194,10 @@ struct KParams {
   uint64_t* jv_ws;            // JVSTM: global ATR, write-set of CTS c at c & (2^jv_log2 - 1)
   uint32_t* jv_tag;           //        entry tag = c once the record of c is written
   uint32_t jv_log2;
+  // CSMV_RETRY_FIFO (KV): per-set PUT tickets -- next ticket to hand out,
+  // and {ticket now served << 32 | CTS of the previous ticket's commit}
+  uint32_t* kv_tk_next;       // u32[T], nullptr = CSMV_RETRY_FREE
+  uint64_t* kv_tk_serv;       // u64[T]
 };
 
 constexpr uint32_t kKvMaxWays = 256;              // KV ways supported by the device path

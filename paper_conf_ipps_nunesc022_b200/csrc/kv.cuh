@@ -102,7 +102,7 @@ __device__ __forceinline__ int kv_read_mw(const uint64_t* ring, uint32_t K, uint
   return RD_OK;
 }
 
-// GET-side read of a key item (W = 4) at snapshot s from its whole ring,
+// GET-side read of a key (W = 4) or value (W = 8) item at snapshot s from its whole ring,
 // loaded in one pass (NS x 32 B, independent 256-bit loads) -- one memory
 // round trip per way instead of kv_read_mw's two.  A slot counts only if
 // all its words carry the same ts; a torn slot (a write-back in flight: its
@@ -113,9 +113,9 @@ __device__ __forceinline__ int kv_read_mw(const uint64_t* ring, uint32_t K, uint
 // first recycling) -- the argument of rot_coop (kernel.cu).
 // rot = false (a PUT's read): any version newer than s -> RD_NEWER, as in
 // kv_read_mw (a torn slot carries a newer ts, so it is covered too).
-template <int NS>
-__device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (&r)[NS], uint32_t K, uint32_t s,
-                                           bool rot, uint32_t (&out)[4], uint32_t* seen = nullptr) {
+template <int NS, int W = 4>
+__device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<W> (&r)[NS], uint32_t K, uint32_t s,
+                                           bool rot, uint32_t (&out)[W], uint32_t* seen = nullptr) {
   int cand = -1;
   uint32_t cts = 0, newest = 0, torn_max = 0;
   bool torn = false;
@@ -125,7 +125,7 @@ __device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (
     const uint32_t t0 = (uint32_t)(r[j].s[0] >> 32);
     bool intact = true;
 #pragma unroll
-    for (int w = 0; w < 4; ++w) {
+    for (int w = 0; w < W; ++w) {
       const uint32_t tw = (uint32_t)(r[j].s[w] >> 32);
       intact &= tw == t0;
       if (tw != kEmptyTs) newest = max(newest, tw);
@@ -144,9 +144,9 @@ __device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (
   if (!rot && newest > s) return RD_NEWER;
   if (cand < 0 || (torn && torn_max > cts)) return RD_MISS;
   if (newest > s) {
-    const Ring<4> q = ld_ring<4>(ring + cand * 4);
+    const Ring<W> q = ld_ring<W>(ring + cand * W);
 #pragma unroll
-    for (int w = 0; w < 4; ++w) {
+    for (int w = 0; w < W; ++w) {
       if ((uint32_t)(q.s[w] >> 32) != cts) return RD_MISS;
       out[w] = (uint32_t)q.s[w];
     }
@@ -156,7 +156,7 @@ __device__ __forceinline__ int kv_key_pick(const uint64_t* ring, const Ring<4> (
   for (int j = 0; j < NS; ++j)
     if (j == cand) {
 #pragma unroll
-      for (int w = 0; w < 4; ++w) out[w] = (uint32_t)r[j].s[w];
+      for (int w = 0; w < W; ++w) out[w] = (uint32_t)r[j].s[w];
     }
   return RD_OK;
 }
@@ -168,12 +168,10 @@ __device__ __forceinline__ void kv_ring_ts(const uint64_t* ring, uint32_t K, uin
   for (int j = 0; j < NS; ++j) ts[j] = ((uint32_t)j < K) ? (uint32_t)(ld_relaxed64(ring + j * W) >> 32) : 0u;
 }
 
-// Install version (cts, data) over the first unused slot, else the oldest
-// (P:291), given the ring's slot timestamps.  The writer owns the item (WW
-// check): nothing else writes it between those loads and the store.
-template <int NS, int W>
-__device__ __forceinline__ void kv_install(uint64_t* ring, const uint32_t (&ts)[NS], uint32_t K, uint32_t cts,
-                                           const uint32_t (&data)[W]) {
+// The slot a new version replaces: the first unused slot, else the oldest
+// (P:291), given the ring's slot timestamps.
+template <int NS>
+__device__ __forceinline__ int kv_install_slot(const uint32_t (&ts)[NS], uint32_t K) {
   int victim = -1;
 #pragma unroll
   for (int j = 0; j < NS; ++j)
@@ -188,6 +186,12 @@ __device__ __forceinline__ void kv_install(uint64_t* ring, const uint32_t (&ts)[
         vts = ts[j];
       }
   }
+  return victim;
+}
+
+// Store version (cts, data) into slot `victim` of a W-word ring.
+template <int W>
+__device__ __forceinline__ void kv_install_at(uint64_t* ring, int victim, uint32_t cts, const uint32_t (&data)[W]) {
   uint64_t* dst = ring + victim * W;
 #pragma unroll
   for (int w = 0; w < W; w += 4) {
@@ -200,6 +204,44 @@ __device__ __forceinline__ void kv_install(uint64_t* ring, const uint32_t (&ts)[
       st_relaxed64(dst + w, ((uint64_t)cts << 32) | data[w]);
     }
   }
+}
+
+// Install version (cts, data) over kv_install_slot's slot.  The writer owns
+// the item (WW check): nothing else writes it between the loads of
+// ts and the store.
+template <int NS, int W>
+__device__ __forceinline__ void kv_install(uint64_t* ring, const uint32_t (&ts)[NS], uint32_t K, uint32_t cts,
+                                           const uint32_t (&data)[W]) {
+  kv_install_at<W>(ring, kv_install_slot<NS>(ts, K), cts, data);
+}
+
+// The set clock (or any one-word item) read by a PUT at snapshot s from its
+// whole ring in one load: a slot's (ts, word) is one 64-bit word, so no
+// re-read is needed; any version newer than s -> RD_NEWER (the PUT cannot
+// commit).  *slot = the slot the PUT's own version will replace.
+template <int NS>
+__device__ __forceinline__ int kv_read_clk(const Ring<NS>& r, uint32_t K, uint32_t s, uint32_t& out, uint32_t& seen,
+                                           int& slot) {
+  uint32_t ts[NS];
+#pragma unroll
+  for (int j = 0; j < NS; ++j) ts[j] = (uint32_t)j < K ? (uint32_t)(r.s[j] >> 32) : kEmptyTs;
+  int cand = -1;
+  uint32_t cts = 0, newest = 0;
+#pragma unroll
+  for (int j = 0; j < NS; ++j) {
+    if (ts[j] == kEmptyTs) continue;
+    newest = max(newest, ts[j]);
+    if (ts[j] <= s && (cand < 0 || ts[j] > cts)) {
+      cand = j;
+      cts = ts[j];
+    }
+  }
+  seen = max(seen, newest);
+  if (newest > s) return RD_NEWER;
+  if (cand < 0) return RD_MISS;
+  out = (uint32_t)slot_at<NS>(r, cand);
+  slot = kv_install_slot<NS>(ts, K);
+  return RD_OK;
 }
 
 template <int NS, int W>

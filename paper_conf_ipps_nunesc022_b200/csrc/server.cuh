@@ -610,6 +610,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     } else {
       if (!claim_request(c, cwv[0])) break;
     }
+    const uint64_t t_claim = trace_now(p);
     // ---- combine: grab further requests that are already queued
 #pragma unroll
     for (int j = 1; j < MR; ++j) {
@@ -810,6 +811,7 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
 #pragma unroll
       for (int j = 0; j < M; ++j) {
         if ((uint32_t)j == lane && msk[j] != 0) {
+          trace_served(p, cwv[j], sq[j], t_claim);
           const uint64_t tag = (uint64_t)sq[j] << 32;
           st_relaxed64(&p.resp[cwv[j]].base, tag | base[j]);
           st_relaxed64(&p.resp[cwv[j]].commit, tag | cm[j]);
@@ -1193,6 +1195,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     uint32_t cw;
     const long long tq = clock64();
     if (!claim_request(c, cw)) break;
+    const uint64_t t_claim = trace_now(p);
     const long long t0 = clock64();
     fence_cta();  // after the receiver's acquire (see server_receiver)
     const uint32_t sq = ld_relaxed(&p.req_hdr[cw].round);
@@ -1267,6 +1270,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
     cs_leave<CL>(c, ticket, t0c + n);
     const long long t2 = clock64();
     if (lane == 0) {  // round-tagged words, no fence (kernel.cuh Resp)
+      trace_served(p, cw, sq, t_claim);
       const uint64_t tag = (uint64_t)sq << 32;
       st_relaxed64(&p.resp[cw].base, tag | (t0c + 1));
       st_relaxed64(&p.resp[cw].commit, tag | cm);
@@ -1330,6 +1334,7 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
       if (!claim_request(c, cw)) break;
       fence_cta();  // after the receiver's acquire (see server_receiver)
     }
+    const uint64_t t_claim = trace_now(p);
     const long long t0 = clock64();
     const uint32_t sq = ld_relaxed(&p.req_hdr[cw].round);
     const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
@@ -1377,6 +1382,7 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
     cs_leave<CL>(c, ticket, t0c + n);
     const long long t2 = clock64();
     if (lane == 0) {  // round-tagged words, no fence (kernel.cuh Resp)
+      trace_served(p, cw, sq, t_claim);
       const uint64_t tag = (uint64_t)sq << 32;
       st_relaxed64(&p.resp[cw].base, tag | (t0c + 1));
       st_relaxed64(&p.resp[cw].commit, tag | cm);

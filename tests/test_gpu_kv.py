@@ -191,3 +191,48 @@ def test_kv_self_receiving_workers(workers, jitter):
                                       total_aborts=stats["total_aborts"]))
     assert rep["ok"], (rep, stats)
     assert stats["server_workers"] == workers
+
+
+# ---- CSMV_RETRY_FIFO: per-set PUT tickets (client-side contention management) ----
+@pytest.mark.parametrize("kw", [
+    dict(p_update_ppm=10_000, ro_streak=32, ro_adaptive=2),                          # C4-shaped, zipf
+    dict(p_update_ppm=300_000, ro_streak=4, ro_adaptive=1),                          # many PUTs per set
+    dict(p_update_ppm=100_000, ro_streak=8, ro_adaptive=2, publish=1),               # server publisher
+    dict(p_update_ppm=100_000, ro_streak=8, ro_adaptive=2, debug_flags=csmv.DBG_JITTER),
+    dict(p_update_ppm=100_000, ro_streak=8, server_recv=csmv.RECV_SELF, server_workers=7, publish=1),
+    dict(p_update_ppm=50_000, ro_streak=8, ro_adaptive=2, debug_flags=csmv.DBG_KV_ITEMSETS),
+    dict(p_update_ppm=50_000, ro_streak=8, ro_adaptive=2, server=csmv.SERVER_CLUSTER, cluster_size=4),
+])
+def test_kv_retry_fifo_parity(kw):
+    """PUTs on a set attempt in ticket order: the history is still the one
+    the replaying oracle accepts (validation is unchanged), every PUT commits
+    once, and no PUT loses to another PUT of its set (no PREVAL, no EARLY)."""
+    kw = dict(dict(server_workers=6), **kw)
+    cfg = W.c4(n_items=1 << 14, n_tx=1 << 17, client_warps=256, retry_order=csmv.RETRY_FIFO, **kw)
+    stats = _check_kv(cfg)
+    ab = stats["aborts"]
+    assert ab["preval"]["update"] == 0 and ab["early"]["update"] == 0 and ab["conflict"]["update"] == 0, ab
+
+
+def test_kv_retry_fifo_one_set():
+    """Every PUT on one cache set (T = 1): a single ticket queue of 64 warps."""
+    cfg = W.c4(n_items=16, kv_ways=16, kv_keys=64, n_tx=1 << 14, p_update_ppm=200_000, client_warps=64,
+               ro_streak=4, ro_adaptive=2, retry_order=csmv.RETRY_FIFO)
+    stats = _check_kv(cfg)
+    assert stats["aborts"]["preval"]["update"] == 0
+
+
+def test_kv_retry_fifo_orders_each_set():
+    """The tickets alone serialise the PUTs of a set (each reads at a
+    snapshot covering the previous ticket's commit, and nothing else writes
+    the set): even with the server's validation and the clients'
+    pre-validation switched off the history is one the oracle accepts --
+    whereas the same run without tickets is rejected
+    (test_kv_no_validate_is_caught)."""
+    cfg = W.c4(n_items=1 << 8, kv_ways=4, n_tx=1 << 14, p_update_ppm=600_000, client_warps=64, dist=0,
+               retry_order=csmv.RETRY_FIFO, debug_flags=csmv.DBG_NO_VALIDATE | csmv.DBG_NO_PREVAL)
+    pre, stats, log, fin = run(cfg)
+    oc = ocfg_of(cfg)
+    rep = oracle.kv_check(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), log,
+                          final=as_state(fin, cfg.n_items, cfg.workload.kv_ways))
+    assert rep["ok"], rep

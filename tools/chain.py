@@ -8,7 +8,9 @@ the median of
   publish   t_publish(i) - t_response(i)          write-back + publish of i
   restart   t_begin(i+1) - t_publish(i)           until the next winner's round starts
   read      t_submit(i+1) - t_begin(i+1)          its snapshot + reads + pre-validation
-  server    t_response(i+1) - t_submit(i+1)       request -> response
+  server    t_response(i+1) - t_submit(i+1)       request -> response, split by the
+            server's stamps into to_claim (doorbell -> a worker took it),
+            worker (claim -> response stored), to_client (-> client saw it)
 (restart can be negative: the winner's round began before i was
 published, e.g. when GTS was advanced by the server publisher meanwhile).
 
@@ -46,11 +48,15 @@ def main(argv):
         tr = st.trace()
     tr = np.sort(tr, order="cts")
     f = lambda a: float(np.median(a)) / 1e3 if len(a) else None  # noqa: E731
-    r, p, b, sub = (tr[k].astype(np.int64) for k in ("t_response", "t_publish", "t_begin", "t_submit"))
+    r, p, b, sub, tc, tv = (tr[k].astype(np.int64) for k in ("t_response", "t_publish", "t_begin", "t_submit",
+                                                             "t_claim", "t_served"))
+    ok = (tc > 0) & (tv >= tc) & (tc >= sub - 1000) & (tv <= r)  # server stamps present and consistent
     out = {"cfg": argv, "tx_per_s_M": round(s["tx_per_s"] / 1e6, 2), "kernel_ms": s["elapsed_ns"] / 1e6,
            "hot_commits": int(len(tr)), "span_ms": float((r[-1] - r[0]) / 1e6) if len(tr) > 1 else None,
            "median_us": {"link": f(np.diff(r)), "publish": f(p - r), "restart": f(b[1:] - p[:-1]),
                          "read": f(sub - b), "server": f(r - sub)},
+           "server_us": {"stamped": int(ok.sum()), "to_claim": f((tc - sub)[ok]), "worker": f((tv - tc)[ok]),
+                         "to_client": f((r - tv)[ok])},
            "mean_link_us": float(np.mean(np.diff(r))) / 1e3 if len(tr) > 1 else None,
            "snapshot_lag_median": float(np.median(tr["cts"][1:].astype(np.int64) - tr["snapshot"][1:]))
            if len(tr) > 1 else None}
