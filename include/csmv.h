@@ -91,6 +91,8 @@ extern "C" {
                                    ticket-locked critical section, the cluster server the other way
                                    round; A/B only */
 
+#define CSMV_DBG_KV_SEQREAD 128u /* KV: a PUT lane scans its set itself, way group by way group (A/B and
+                                    parity cross-check of the default warp-cooperative one-trip read) */
 #define CSMV_DBG_TRACE 64u     /* hot-chain trace: every committed update that writes csmv_workload.
                                    trace_item (bank: an account; KV: a set) logs a csmv_trace_rec with
                                    device-wide timestamps (globaltimer) -- csmv_get_trace */
@@ -210,6 +212,10 @@ typedef struct csmv_trace_rec {
     uint64_t t_begin, t_submit, t_response, t_publish;
     uint64_t t_claim, t_served; /* server side: the worker took the request / stored the response
                                    (0 where the commit path does not stamp them) */
+    uint64_t t_snap, t_read;    /* client: snapshot taken (GTS read) / read-set read, before
+                                   pre-validation and submit (0 where not stamped) */
+    uint32_t n_readers;         /* KV: PUT lanes of the warp that read their set in that round */
+    uint32_t n_kept;            /* transactions of the request that carried this commit */
 } csmv_trace_rec;
 
 typedef struct csmv csmv_t;

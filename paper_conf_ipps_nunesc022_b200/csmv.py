@@ -25,12 +25,14 @@ RETRY_FREE, RETRY_FIFO = 0, 1
 ATR_HASH, ATR_LIST, ATR_LIST_NOCV = 0, 1, 2
 COMMIT_CSMV, COMMIT_ONLYCS, COMMIT_JVSTM = 0, 1, 2
 DBG_NO_PREVAL, DBG_NO_VALIDATE, DBG_JITTER, DBG_PHASES, DBG_KV_ITEMSETS, DBG_ALT_COMMIT, DBG_TRACE = 1, 2, 4, 8, 16, 32, 64
+DBG_KV_SEQREAD = 128
 RECV_WARP, RECV_SELF = 0, 1
 CLIENT_PHASES = ("read", "preval", "submit", "rot", "wait_server", "writeback", "publish", "divergence")
 ABORT_REASONS = ("preval", "conflict", "early", "overflow", "version")
 
 TRACE_DTYPE = np.dtype([("cts", "<u4"), ("snapshot", "<u4"), ("t_begin", "<u8"), ("t_submit", "<u8"),
-                        ("t_response", "<u8"), ("t_publish", "<u8"), ("t_claim", "<u8"), ("t_served", "<u8")])
+                        ("t_response", "<u8"), ("t_publish", "<u8"), ("t_claim", "<u8"), ("t_served", "<u8"),
+                        ("t_snap", "<u8"), ("t_read", "<u8"), ("n_readers", "<u4"), ("n_kept", "<u4")])
 LOG_DTYPE = np.dtype([("tx", "<u4"), ("snapshot", "<u4"), ("cts", "<u4"),
                       ("attempts", "<u4"), ("read_digest", "<u8"), ("aux", "<u8")])
 

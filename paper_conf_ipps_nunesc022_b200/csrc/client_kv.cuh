@@ -43,9 +43,12 @@ __device__ __forceinline__ void kv_get_start(const KParams& p, uint32_t key, KvG
 // (issued before the step's loads) while the loads are in flight:
 // kv_get_issue puts the step's loads in flight into rb, kv_get_finish
 // evaluates them; fin = the GET is complete (g.dg, g.hit final).
+#ifndef CSMV_KV_GET_U
+#define CSMV_KV_GET_U 2  // key ways per GET step at NS <= 4 (build knob for A/B: 2 beats 4 by ~12 % on C4, fewer spills)
+#endif
 template <int NS>
 struct KvStep {
-  static constexpr int U = NS <= 4 ? 4 : (NS == 8 ? 2 : 1);  // key ways per step
+  static constexpr int U = NS <= 4 ? CSMV_KV_GET_U : (NS == 8 ? 2 : 1);  // key ways per step
   static constexpr int R = U * NS;                           // Ring<4> registers per step
   static constexpr bool kValOne = 2 * NS <= R;               // the value ring fits: one trip
 };
@@ -130,6 +133,166 @@ __device__ __forceinline__ int kv_get_finish(const KParams& p, uint32_t s, KvGet
   return RD_OK;
 }
 
+// A PUT's read of its set t at snapshot s by the whole warp (compact
+// requests, A <= 16 ways; every lane calls it with the same t, kk), split in
+// an issue and an evaluation half so that the reads of several PUTs are in
+// flight together: lanes 2w and 2w+1 load the two halves of way w's key
+// ring, lane 31 the set clock's ring; the LRU stamps cost a second trip,
+// only when no way stops the scan.  It decides exactly as the sequential
+// scan (the reader's own loop in client_warp_kv): the clock first, then ways
+// in order up to the first one that matches the key, is empty, or cannot be
+// read at s (NEWER / MISS: the PUT aborts with that reason); ways past the
+// stop are not read (not in the digest); with no stop, the LRU stamps of
+// all ways, the victim being the first least recently used way.  Results
+// are warp-uniform.
+template <int NS>
+struct KvCoopLd {
+  static constexpr int H = NS / 2;  // versions per lane
+  Ring<4> kr[H];
+  Ring<NS> cr;
+};
+
+template <int NS>
+__device__ __forceinline__ void kv_put_read_issue(const KParams& p, uint32_t t, KvCoopLd<NS>& ld) {
+  constexpr int H = KvCoopLd<NS>::H;
+  const uint32_t lane = threadIdx.x & 31, A = p.kv_A;
+  const uint32_t w = lane >> 1, h = lane & 1;
+  if (w < A) {
+    const uint32_t slot = t * A + w;
+#pragma unroll
+    for (int q = 0; q < H; ++q) ld.kr[q] = ld_ring<4>(p.kv_key + ((size_t)slot * NS + h * H + q) * 4);
+  }
+  if (lane == 31) ld.cr = ld_ring<NS>(p.kv_clk + (size_t)t * NS);
+}
+
+template <int NS>
+__device__ __forceinline__ void kv_put_read_eval(const KParams& p, uint32_t s, uint32_t t, const uint32_t (&kk)[4],
+                                                 const KvCoopLd<NS>& ld, int& st, uint32_t& seen, uint32_t& victim,
+                                                 int& iv, int& ic, uint32_t& clk, uint64_t& rdig) {
+  const uint32_t FULL = 0xFFFFFFFFu;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t K = p.K, S = p.kv_S, A = p.kv_A;
+  constexpr int H = KvCoopLd<NS>::H;
+  const uint32_t w = lane >> 1, h = lane & 1;
+  const bool wl = w < A;
+  const uint32_t slot = t * A + w;
+  // the clock (lane 31)
+  int cst = RD_OK, cic = 0;
+  uint32_t cval = 0, cseen = 0;
+  if (lane == 31) cst = kv_read_clk<NS>(ld.cr, K, s, cval, cseen, cic);
+  cst = __shfl_sync(FULL, cst, 31);
+  cval = __shfl_sync(FULL, cval, 31);
+  cseen = __shfl_sync(FULL, cseen, 31);
+  ic = __shfl_sync(FULL, cic, 31);
+  seen = cseen;
+  st = cst;
+  clk = cval;
+  victim = 0xFFFFFFFFu;
+  iv = 0;
+  rdig = 0;
+  // this lane's versions of way w (kv_key_pick with rot = false, per half)
+  int cand = -1;
+  uint32_t cts = 0, newest = 0, torn_max = 0, key[4] = {0u, 0u, 0u, 0u}, lts[H];
+  bool torn = false;
+#pragma unroll
+  for (int q = 0; q < H; ++q) {
+    const uint32_t jg = h * H + q;
+    lts[q] = kEmptyTs;
+    if (!wl || jg >= K) continue;
+    const uint32_t t0 = (uint32_t)(ld.kr[q].s[0] >> 32);
+    lts[q] = t0;
+    bool intact = true;
+#pragma unroll
+    for (int x = 0; x < 4; ++x) {
+      const uint32_t tw = (uint32_t)(ld.kr[q].s[x] >> 32);
+      intact &= tw == t0;
+      if (tw != kEmptyTs) newest = max(newest, tw);
+      if (tw <= s) torn_max = max(torn_max, tw);
+    }
+    if (!intact) {
+      torn = true;
+      continue;
+    }
+    if (t0 != kEmptyTs && t0 <= s && (cand < 0 || t0 > cts)) {
+      cand = (int)jg;
+      cts = t0;
+#pragma unroll
+      for (int x = 0; x < 4; ++x) key[x] = (uint32_t)ld.kr[q].s[x];
+    }
+  }
+  // combine the two halves of the way (lanes 2w, 2w+1)
+  {
+    const int ocand = __shfl_xor_sync(FULL, cand, 1);
+    const uint32_t octs = __shfl_xor_sync(FULL, cts, 1);
+    uint32_t okey[4];
+#pragma unroll
+    for (int x = 0; x < 4; ++x) okey[x] = __shfl_xor_sync(FULL, key[x], 1);
+    newest = max(newest, __shfl_xor_sync(FULL, newest, 1));
+    torn_max = max(torn_max, __shfl_xor_sync(FULL, torn_max, 1));
+    torn = __shfl_xor_sync(FULL, (uint32_t)torn, 1) || torn;
+    if (ocand >= 0 && (cand < 0 || octs > cts)) {
+      cand = ocand;
+      cts = octs;
+#pragma unroll
+      for (int x = 0; x < 4; ++x) key[x] = okey[x];
+    }
+  }
+  const int wst = newest > s ? RD_NEWER : ((cand < 0 || (torn && torn_max > cts)) ? RD_MISS : RD_OK);
+  const bool match = key[0] == kk[0] && key[1] == kk[1] && key[2] == kk[2] && key[3] == kk[3];
+  const bool empty = !(key[0] | key[1] | key[2] | key[3]);
+  const bool lead = wl && h == 0;  // one lane per way
+  if (cst != RD_OK) return;
+  const uint32_t stops = __ballot_sync(FULL, lead && (wst != RD_OK || match || empty));
+  const uint32_t ws = stops ? (uint32_t)(__ffs(stops) - 1) >> 1 : A;  // the scan's last way (A: none)
+  // the ways read: 0..ws (all of them when nothing stopped the scan)
+  const bool rd = lead && w <= ws;
+  seen = max(seen, __reduce_max_sync(FULL, rd ? newest : 0u));
+  if (stops) {
+    const int sst = __shfl_sync(FULL, wst, 2 * ws);
+    if (sst != RD_OK) {
+      st = sst;
+      return;
+    }
+  }
+  uint64_t dg = 0;
+  if (rd) {
+#pragma unroll
+    for (int x = 0; x < 4; ++x) dg += dig_word(slot, x, key[x]);
+  }
+  uint32_t vw = ws;  // victim way
+  if (!stops) {  // LRU stamps of every way; the first least recently used way is the victim
+    int lst = RD_OK;
+    uint32_t l = 0xFFFFFFFFu, ln = 0;
+    if (lead) {
+      const Ring<NS> lr = ld_ring<NS>(p.kv_lru + (size_t)slot * NS);
+      const Sel q = select_version<NS>(lr, s);
+      ln = q.newest;
+      if (q.newest > s) lst = RD_NEWER;
+      else if (q.best < 0 || (uint32_t)q.best >= K) lst = RD_MISS;
+      else l = (uint32_t)slot_at<NS>(lr, q.best);
+    }
+    seen = max(seen, __reduce_max_sync(FULL, ln));
+    const uint32_t bad = __ballot_sync(FULL, lead && lst != RD_OK);
+    if (bad) {
+      st = __shfl_sync(FULL, lst, __ffs(bad) - 1);
+      return;
+    }
+    if (lead) dg += dig1(2 * S + slot, l);
+    const uint32_t lmin = __reduce_min_sync(FULL, l);
+    vw = (uint32_t)(__ffs(__ballot_sync(FULL, lead && l == lmin)) - 1) >> 1;
+  }
+  // the digest of everything read, summed over the warp
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) dg += __shfl_xor_sync(FULL, dg, o);
+  rdig = dg + dig1(3 * S + t, clk);
+  victim = t * A + vw;
+  // the victim's key ring timestamps (= its value and LRU rings'): the slot all three replace
+  uint32_t ts[NS];
+#pragma unroll
+  for (int j = 0; j < NS; ++j) ts[j] = __shfl_sync(FULL, lts[j % H], 2 * vw + j / H);
+  iv = kv_install_slot<NS>(ts, K);
+}
+
 template <int NS>
 __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scratch) {
   const uint32_t FULL = 0xFFFFFFFFu;
@@ -174,6 +337,11 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     }
     s = __shfl_sync(FULL, s, 0);
     if (__shfl_sync(FULL, err, 0)) break;
+#ifndef CSMV_TRACE_SNAP_LATE
+    const uint64_t t_snap = tracing ? globaltimer() : 0;
+#else
+    uint64_t t_snap = 0;
+#endif
 
     // ---- A: the pending PUT reads at s (read-set tracked)
     int status = ST_NONE;
@@ -195,7 +363,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       // in lane order with one atomic (the set's lowest such lane adds)
       const uint32_t am = __ballot_sync(FULL, adopted);
       if (am) {
-        if (adopted) {
+        if (adopted && dk_id != cu) {
           dk_key = gen_kv_key(p.gen, cu);
           dk_id = cu;
         }
@@ -258,10 +426,63 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       cc.abort(CSMV_AB_PREVAL, true);
       status = ST_ABORT;
     }
+    // compact requests on sets of up to 16 ways: the warp reads each
+    // reader's set together, one memory round trip per reader
+    const bool coop = compact && A <= 16 && !(p.debug & CSMV_DBG_KV_SEQREAD);
+    int r_c = RD_OK;
+    uint32_t seen_c = 0;
+    const uint32_t n_readers = __popc(__ballot_sync(FULL, reader));
+#ifdef CSMV_TRACE_SNAP_LATE
+    t_snap = tracing ? globaltimer() : 0;
+#endif
+    if (coop) {
+      // up to kCoopMax readers' sets in flight together, then evaluated one by one
+#ifndef CSMV_KV_COOP_MAX
+#define CSMV_KV_COOP_MAX 2
+#endif
+      constexpr int kCoopMax = CSMV_KV_COOP_MAX;
+      uint32_t rem = __ballot_sync(FULL, reader);
+      while (rem) {
+        int rls[kCoopMax];
+        uint32_t tss[kCoopMax];
+        KvCoopLd<NS> ld[kCoopMax];
+#pragma unroll
+        for (int i = 0; i < kCoopMax; ++i) {
+          rls[i] = rem ? __ffs(rem) - 1 : -1;
+          rem &= rem - 1;
+          tss[i] = rls[i] >= 0 ? __shfl_sync(FULL, tset, rls[i]) : 0u;
+          if (rls[i] >= 0) kv_put_read_issue<NS>(p, tss[i], ld[i]);
+        }
+#pragma unroll
+        for (int i = 0; i < kCoopMax; ++i) {
+          if (rls[i] < 0) break;
+          uint32_t k4[4];
+#pragma unroll
+          for (int x = 0; x < 4; ++x) k4[x] = __shfl_sync(FULL, kk[x], rls[i]);
+          int st_, iv_, ic_;
+          uint32_t seen_, vic_, clk_;
+          uint64_t dg_;
+          kv_put_read_eval<NS>(p, s, tss[i], k4, ld[i], st_, seen_, vic_, iv_, ic_, clk_, dg_);
+          if (lane == (uint32_t)rls[i]) {
+            r_c = st_;
+            seen_c = seen_;
+            victim = vic_;
+            iv = iv_;
+            ic = ic_;
+            clk = clk_;
+            rdig = dg_;
+          }
+        }
+      }
+    }
     if (reader) {
       {
         int r = RD_OK;
         uint32_t seen = 0;  // newest version timestamp the reads met
+        if (coop) {
+          r = r_c;
+          seen = seen_c;
+        } else {
         victim = 0xFFFFFFFFu;
         // The set clock's whole ring (one 64-bit word per version: one
         // load, no re-read) travels with the first group of key ways.  It
@@ -358,6 +579,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
             rdig += dig1(3 * S + tset, clk);
           }
         }
+        }  // sequential read
         if (r == RD_NEWER) {
           need = seen;  // retry once GTS covers the newer version (its commit is then visible)
           cc.abort(CSMV_AB_EARLY, true);
@@ -380,6 +602,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       }
     }
     __syncwarp();
+    const uint64_t t_read = tracing ? globaltimer() : 0;
     pc.mark(PH_READ);
     jit();  // versions read, not yet validated
 
@@ -615,10 +838,16 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       }
     }
     pc.mark(PH_PUBLISH);
+    // the key of the lane's next update, drawn now (a zipf pick: a few
+    // dependent loads) rather than when the next round adopts it
+    if (cu == kNoTx && cr < p.n_tx && dk_id != cr && gen_is_update(p.gen, cr)) {
+      dk_key = gen_kv_key(p.gen, cr);
+      dk_id = cr;
+    }
     if (tracing && cts && tset == p.trace_item) {
       uint64_t tc, tv;
       trace_srv_times(p, cw, round, t_sub, tc, tv);
-      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv);
+      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv, t_snap, t_read, n_readers, __popc(kept));
     }
   }
   client_flush(p, cc);

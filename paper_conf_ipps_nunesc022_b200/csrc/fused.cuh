@@ -414,7 +414,9 @@ __device__ __forceinline__ void trace_srv_times(const KParams& p, uint32_t cw, u
 }
 
 __device__ __forceinline__ void trace_commit(const KParams& p, uint32_t cts, uint32_t s, uint64_t tb, uint64_t ts,
-                                             uint64_t tr, uint64_t tp, uint64_t tc = 0, uint64_t tv = 0) {
+                                             uint64_t tr, uint64_t tp, uint64_t tc = 0, uint64_t tv = 0,
+                                             uint64_t tsn = 0, uint64_t trd = 0, uint32_t nrd = 0,
+                                             uint32_t nkept = 0) {
   const uint32_t i = atomicAdd(&p.ctl->trace_n, 1u);
   if (i < kTraceCap) {
     csmv_trace_rec r;
@@ -426,6 +428,10 @@ __device__ __forceinline__ void trace_commit(const KParams& p, uint32_t cts, uin
     r.t_publish = tp;
     r.t_claim = tc;
     r.t_served = tv;
+    r.t_snap = tsn;
+    r.t_read = trd;
+    r.n_readers = nrd;
+    r.n_kept = nkept;
     p.trace[i] = r;
   }
 }

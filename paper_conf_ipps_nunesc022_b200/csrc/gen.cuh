@@ -20,11 +20,18 @@ __host__ __device__ __forceinline__ uint64_t draw(uint64_t seed, uint64_t tx, ui
 
 __device__ __forceinline__ uint64_t uniform(uint64_t u, uint64_t n) { return __umul64hi(u, n); }
 
-// first i with cdf[i] > u, clamped to n-1 (the table's last entry is 2^64-1)
-__device__ __forceinline__ uint32_t zipf_pick(const uint64_t* __restrict__ cdf, uint32_t n, uint64_t u) {
-  uint32_t lo = 0, hi = n;
-  while (lo < hi) {
-    uint32_t mid = (lo + hi) >> 1;
+// first i with cdf[i] > u, clamped to n-1 (the table's last entry is
+// 2^64-1).  The guide table narrows the search: with 2^m buckets of u,
+// guide[b] = the pick at the start of bucket b and guide[2^m] = n-1, so the
+// pick of any u in bucket b lies in [guide[b], guide[b+1]] (picks are
+// monotone in u) -- the upper_bound over that range is the same as over
+// the whole table (a couple of dependent loads instead of log2 n).
+__device__ __forceinline__ uint32_t zipf_pick(const uint64_t* __restrict__ cdf, const uint32_t* __restrict__ guide,
+                                              uint32_t m, uint32_t n, uint64_t u) {
+  const uint32_t b = m ? (uint32_t)(u >> (64 - m)) : 0u;
+  uint32_t lo = __ldg(guide + b), hi = __ldg(guide + b + 1);
+  while (lo < hi) {  // the answer is in [lo, hi]: hi itself needs no test
+    const uint32_t mid = (lo + hi) >> 1;
     if (__ldg(cdf + mid) > u) hi = mid; else lo = mid + 1;
   }
   return lo < n ? lo : n - 1;
@@ -34,6 +41,8 @@ struct GenParams {
   uint64_t seed;
   uint64_t upd_thresh;       // update iff (draw(.,0) >> 32) < upd_thresh
   const uint64_t* zipf_cdf;  // non-null iff zipf
+  const uint32_t* zipf_guide;  // [2^guide_log2 + 1] (zipf_pick)
+  uint32_t guide_log2;
   uint32_t n_items;          // bank: accounts; KV: key space
   uint32_t ro_period;
   uint32_t ro_reads;
@@ -48,7 +57,7 @@ struct BankTx {
 };
 
 __device__ __forceinline__ uint32_t gen_pick(const GenParams& g, uint64_t u) {
-  return g.zipf_cdf ? zipf_pick(g.zipf_cdf, g.n_items, u) : (uint32_t)uniform(u, g.n_items);
+  return g.zipf_cdf ? zipf_pick(g.zipf_cdf, g.zipf_guide, g.guide_log2, g.n_items, u) : (uint32_t)uniform(u, g.n_items);
 }
 
 __device__ __forceinline__ bool gen_is_update(const GenParams& g, uint64_t tx) {

@@ -314,13 +314,35 @@ int csmv_load_kv(csmv_t* h, uint64_t n_keys) {
   return CSMV_OK;
 }
 
+// guide buckets of the zipf search: 2^log2 with 2^log2 >= n, at most 2^22
+static uint32_t zipf_guide_log2(uint32_t n) {
+  uint32_t l = 0;
+  while ((1u << l) < n && l < 22) ++l;
+  return l;
+}
+
 static int prepare_zipf(csmv* h, uint32_t n, uint32_t theta) {
   if (h->d_zipf && h->zipf_n == n && h->zipf_theta == theta) return CSMV_OK;
   cudaFree(h->d_zipf);
   h->d_zipf = nullptr;
   std::vector<uint64_t> cdf = build_zipf(n, theta);
-  CK(cudaMalloc(&h->d_zipf, n * sizeof(uint64_t)));
-  CK(cudaMemcpy(h->d_zipf, cdf.data(), n * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  // guide table (the cutpoint method): g[b] = pick(b * 2^(64-m)) for the
+  // 2^m buckets of u plus g[2^m] = n-1, so that a pick in bucket b lies in
+  // [g[b], g[b+1]] -- the same upper_bound, over a few entries instead of
+  // all n (gen.cuh zipf_pick)
+  const uint32_t m = zipf_guide_log2(n);
+  std::vector<uint32_t> guide(((size_t)1 << m) + 1);
+  uint32_t i = 0;
+  for (uint64_t b = 0; b < ((uint64_t)1 << m); ++b) {
+    const uint64_t u = m ? b << (64 - m) : 0;
+    while (i < n - 1 && cdf[i] <= u) ++i;
+    guide[b] = i;
+  }
+  guide[(size_t)1 << m] = n - 1;
+  const size_t cb = (size_t)n * sizeof(uint64_t), gb = guide.size() * sizeof(uint32_t);
+  CK(cudaMalloc(&h->d_zipf, cb + gb));
+  CK(cudaMemcpy(h->d_zipf, cdf.data(), cb, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(reinterpret_cast<uint8_t*>(h->d_zipf) + cb, guide.data(), gb, cudaMemcpyHostToDevice));
   h->zipf_n = n;
   h->zipf_theta = theta;
   return CSMV_OK;
@@ -343,6 +365,8 @@ static int make_gen(csmv* h, const csmv_workload* w, uint64_t seed, GenParams* g
     int rc = prepare_zipf(h, g->n_items, w->zipf_theta_milli);
     if (rc) return rc;
     g->zipf_cdf = h->d_zipf;
+    g->zipf_guide = reinterpret_cast<const uint32_t*>(h->d_zipf + g->n_items);
+    g->guide_log2 = zipf_guide_log2(g->n_items);
   } else if (w->dist != CSMV_DIST_UNIFORM) {
     return set_err(CSMV_EINVAL, "unknown dist %u", w->dist);
   }

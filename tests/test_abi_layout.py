@@ -54,4 +54,4 @@ def test_log_record_is_32_bytes():
 def test_trace_record_mirror():
     c = c_struct_fields("csmv_trace_rec")
     assert [n for n, _, _ in c] == list(csmv.TRACE_DTYPE.names)
-    assert sum(s * n for _, s, n in c) == csmv.TRACE_DTYPE.itemsize == 56
+    assert sum(s * n for _, s, n in c) == csmv.TRACE_DTYPE.itemsize == 80

@@ -236,3 +236,30 @@ def test_kv_retry_fifo_orders_each_set():
     rep = oracle.kv_check(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), log,
                           final=as_state(fin, cfg.n_items, cfg.workload.kv_ways))
     assert rep["ok"], rep
+
+
+# ---- the warp-cooperative PUT read (default) against the lane's own scan ----
+@pytest.mark.parametrize("ways,k", [(16, 4), (8, 2), (4, 8), (16, 16), (2, 4)])
+def test_kv_coop_read_one_warp_matches_predictor(ways, k):
+    """The one-trip cooperative read decides every PUT as the oracle's
+    item-level predictor does (same victims, digests, aborts), at several
+    associativities and version counts, with and without the lane's own scan."""
+    for flags in (0, csmv.DBG_KV_SEQREAD):
+        cfg = W.c4(n_items=ways * 128, kv_ways=ways, n_versions=k, n_tx=3000, p_update_ppm=300_000,
+                   client_warps=1, ro_streak=4, debug_flags=flags)
+        pre, stats, log, fin = run(cfg)
+        oc = ocfg_of(cfg)
+        plog, pfin, ps = oracle.kv_predict(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), 32)
+        assert np.array_equal(log, plog), flags
+        for a, b in zip(fin, (pfin.keys, pfin.vals, pfin.lru, pfin.clocks)):
+            assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("kw", [dict(kv_keys=3 << 12), dict(kv_keys=1000), dict(n_versions=2), dict(n_versions=8),
+                                dict(debug_flags=csmv.DBG_JITTER)])
+def test_kv_coop_read_parity(kw):
+    """Contended runs with the cooperative read: misses (more keys than
+    slots: LRU victims), fewer keys than slots (empty ways), K = 2/8, jitter."""
+    kw = dict(dict(n_items=1 << 12, n_tx=1 << 16, p_update_ppm=100_000, ro_streak=8, ro_adaptive=2,
+                   client_warps=256, server_workers=6), **kw)
+    _check_kv(W.c4(**kw))

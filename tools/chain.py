@@ -48,8 +48,9 @@ def main(argv):
         tr = st.trace()
     tr = np.sort(tr, order="cts")
     f = lambda a: float(np.median(a)) / 1e3 if len(a) else None  # noqa: E731
-    r, p, b, sub, tc, tv = (tr[k].astype(np.int64) for k in ("t_response", "t_publish", "t_begin", "t_submit",
-                                                             "t_claim", "t_served"))
+    r, p, b, sub, tc, tv, tsn, trd = (tr[k].astype(np.int64) for k in (
+        "t_response", "t_publish", "t_begin", "t_submit", "t_claim", "t_served", "t_snap", "t_read"))
+    okc = (tsn >= b) & (trd >= tsn) & (sub >= trd)  # client stamps present
     ok = (tc > 0) & (tv >= tc) & (tc >= sub - 1000) & (tv <= r)  # server stamps present and consistent
     out = {"cfg": argv, "tx_per_s_M": round(s["tx_per_s"] / 1e6, 2), "kernel_ms": s["elapsed_ns"] / 1e6,
            "hot_commits": int(len(tr)), "span_ms": float((r[-1] - r[0]) / 1e6) if len(tr) > 1 else None,
@@ -57,6 +58,10 @@ def main(argv):
                          "read": f(sub - b), "server": f(r - sub)},
            "server_us": {"stamped": int(ok.sum()), "to_claim": f((tc - sub)[ok]), "worker": f((tv - tc)[ok]),
                          "to_client": f((r - tv)[ok])},
+           "read_us": {"stamped": int(okc.sum()), "snapshot": f((tsn - b)[okc]), "reads": f((trd - tsn)[okc]),
+                       "submit": f((sub - trd)[okc])},
+           "readers_mean": float(np.mean(tr["n_readers"])) if len(tr) else None,
+           "kept_mean": float(np.mean(tr["n_kept"])) if len(tr) else None,
            "mean_link_us": float(np.mean(np.diff(r))) / 1e3 if len(tr) > 1 else None,
            "snapshot_lag_median": float(np.median(tr["cts"][1:].astype(np.int64) - tr["snapshot"][1:]))
            if len(tr) > 1 else None}
