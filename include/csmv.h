@@ -149,6 +149,14 @@ typedef struct csmv_workload {
                                   the whole check); EINVAL for KV, whose PUTs write the value blindly */
     uint32_t retry_order;      /* CSMV_RETRY_*: client-side contention management of update retries
                                   (the paper leaves retry scheduling open) */
+    uint32_t req_tagged;       /* 0: a client fences its request's payload before ringing the doorbell
+                                  and the server's receiver fences after seeing it (acquire); 1: no
+                                  fences -- every payload word carries the request's round and the
+                                  server re-reads the payload until all of it does (as the client does
+                                  with the response).  Shorter request path (hot-item chains, C3/C4);
+                                  costs server time when payloads arrive after their doorbell (C2).
+                                  Taken by the bank's self-receiving workers (CSMV_RECV_SELF) and the
+                                  KV filter workers, with item ids < 2^24; elsewhere ignored (fenced) */
 } csmv_workload;
 
 #define CSMV_RETRY_FREE 0u     /* every pending update attempts each round (optionally backoff_max) */

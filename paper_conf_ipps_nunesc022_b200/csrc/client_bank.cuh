@@ -202,6 +202,14 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
     }
     s = __shfl_sync(FULL, s, 0);
     if (!grouped && __shfl_sync(FULL, err, 0)) break;
+    // the trace's snapshot/read stamps are a build option for the bank
+    // client (CSMV_BANK_STAMPS): two more 64-bit values live across the
+    // round cost C2 ~1-2 % (profiles/r02/raw/r02bc_ab_load_stamps.txt)
+#ifdef CSMV_BANK_STAMPS
+    const uint64_t t_snap = tracing ? globaltimer() : 0;
+#else
+    const uint64_t t_snap = 0;
+#endif
 
     // ---- A: the pending update reads at s
     int status = ST_NONE;
@@ -241,6 +249,11 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       }
     }
 
+#ifdef CSMV_BANK_STAMPS
+    const uint64_t t_read = tracing ? globaltimer() : 0;
+#else
+    const uint64_t t_read = 0;
+#endif
     pc.mark(PH_READ);
     jit();  // versions read, not yet validated
     if (p.commit == CSMV_COMMIT_JVSTM) {
@@ -323,16 +336,12 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       // slots of a group); the first warp rings the group's doorbell after
       // every payload is fenced
       if (mine) {
-        my_ids[lane] = d.src | kWriteBit;
-        my_ids[32 + lane] = d.dst | kWriteBit;
+        put_req_id(p, my_ids + lane, d.src | kWriteBit, round);
+        put_req_id(p, my_ids + 32 + lane, d.dst | kWriteBit, round);
       }
-      if (lane == 0) {
-        p.req_hdr[cw].snapshot = s;
-        p.req_hdr[cw].mask = kept;
-        p.req_hdr[cw].round = round;
-      }
+      if (lane == 0) put_req_hdr(p, cw, s, kept, round);
       __syncwarp();
-      fence_gpu();
+      if (!p.req_tagged) fence_gpu();  // tagged: the server checks the round in every word instead
       gkept = grp.vote_or(kept, 2);
       // the server answers the warps that submitted something; all warps of
       // the group watch the first of them, so their rounds stay aligned
@@ -348,20 +357,16 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
     } else if (kept) {
       if (part) wait_acks();  // the servers still read this slot for the previous decide
       if (mine) {
-        my_ids[lane] = d.src | kWriteBit;
-        my_ids[32 + lane] = d.dst | kWriteBit;
+        put_req_id(p, my_ids + lane, d.src | kWriteBit, round);
+        put_req_id(p, my_ids + 32 + lane, d.dst | kWriteBit, round);
         if (p.commit == CSMV_COMMIT_ONLYCS) {  // the server writes back
           p.req_vals[(size_t)cw * 64 + lane] = vs - (uint32_t)d.amt;
           p.req_vals[(size_t)cw * 64 + 32 + lane] = vd + (uint32_t)d.amt;
         }
       }
-      if (lane == 0) {
-        p.req_hdr[cw].snapshot = s;
-        p.req_hdr[cw].mask = kept;
-        p.req_hdr[cw].round = round;
-      }
+      if (lane == 0) put_req_hdr(p, cw, s, kept, round);
       __syncwarp();
-      fence_gpu();
+      if (!p.req_tagged) fence_gpu();  // tagged: the server checks the round in every word instead
       jit();  // payload written, doorbell not yet
       if (part) {  // the servers owning an item of the batch; prepared one at a time, lowest first
         smask = __reduce_or_sync(FULL, mine ? (1u << part_owner(d.src, p.part_log2)) |
@@ -603,7 +608,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
     if (tracing && cts && (d.src == p.trace_item || d.dst == p.trace_item)) {
       uint64_t tc, tv;
       trace_srv_times(p, cw, round, t_sub, tc, tv);
-      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv);
+      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv, t_snap, t_read, 0, __popc(kept));
     }
   }
   if (part) wait_acks();  // the servers have processed our last decide before we count as done

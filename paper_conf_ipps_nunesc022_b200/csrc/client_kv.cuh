@@ -645,10 +645,10 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     if (status == ST_CAND && !mine) cc.abort(CSMV_AB_PREVAL, true);
     pc.mark(PH_PREVAL);
     if (kept && mine && compact) {
-      my_ids[0 * 32 + lane] = (3 * S + tset) | kWriteBit;  // read and written: stands for the set
-      my_ids[1 * 32 + lane] = victim | kWriteBit;
-      my_ids[2 * 32 + lane] = (S + victim) | kWriteBit;
-      my_ids[3 * 32 + lane] = (2 * S + victim) | kWriteBit;
+      put_req_id(p, my_ids + 0 * 32 + lane, (3 * S + tset) | kWriteBit, round);  // read and written: the set
+      put_req_id(p, my_ids + 1 * 32 + lane, victim | kWriteBit, round);
+      put_req_id(p, my_ids + 2 * 32 + lane, (S + victim) | kWriteBit, round);
+      put_req_id(p, my_ids + 3 * 32 + lane, (2 * S + victim) | kWriteBit, round);
       p.req_cnt[(size_t)cw * 32 + lane] = 4;
     } else if (kept && mine) {
       // request ids: RS u WS (bit 31: in WS)
@@ -670,13 +670,9 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       p.req_cnt[(size_t)cw * 32 + lane] = n;
     }
     if (kept) {
-      if (lane == 0) {
-        p.req_hdr[cw].snapshot = s;
-        p.req_hdr[cw].mask = kept;
-        p.req_hdr[cw].round = round;
-      }
+      if (lane == 0) put_req_hdr(p, cw, s, kept, round);
       __syncwarp();
-      fence_gpu();
+      if (!p.req_tagged) fence_gpu();  // tagged: the server checks the round in every word instead
       jit();  // payload written, doorbell not yet
       if (lane == 0) st_relaxed(&p.req_seq[cw], round);
       if (tracing) t_sub = globaltimer();

@@ -137,6 +137,24 @@ struct Jitter {
 
 // Non-blocking: the server's answer to request `round` of client warp cw,
 // if all three words carry the round's tag yet.
+// A request's header (ReqHdr): tagged, two 64-bit relaxed stores; else
+// plain stores of the fields (a fence follows before the doorbell).
+__device__ __forceinline__ void put_req_hdr(const KParams& p, uint32_t cw, uint32_t s, uint32_t mask, uint32_t round) {
+  if (p.req_tagged) {
+    st_relaxed64x2(reinterpret_cast<uint64_t*>(&p.req_hdr[cw]), ((uint64_t)round << 32) | s,
+                   ((uint64_t)round << 32) | mask);
+  } else {
+    p.req_hdr[cw].snapshot = s;
+    p.req_hdr[cw].mask = mask;
+    p.req_hdr[cw].round = p.req_hdr[cw].round2 = round;
+  }
+}
+// one id of a request: tagged, a relaxed store carrying the round; else a plain store
+__device__ __forceinline__ void put_req_id(const KParams& p, uint32_t* a, uint32_t id, uint32_t round) {
+  if (p.req_tagged) st_relaxed(a, id | id_tag(round));
+  else *a = id;
+}
+
 // The three words of a response, loaded by lanes 0-2 at once (one L2 round
 // trip, not three) and broadcast.
 __device__ __forceinline__ void ld_response(const KParams& p, uint32_t cw, uint64_t& b, uint64_t& c, uint64_t& o) {

@@ -627,6 +627,16 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
   p.ev_log2 = ev_log2;
   p.filt16_n = filt16_n;
   p.gts_start = gts0;
+  // round-tagged requests (ReqHdr, no client fence before the doorbell) on
+  // the commit paths that check the tags: the self-receiving bank worker
+  // (ticket-locked single CTA) and the KV filter workers
+  {
+    const uint64_t max_id = h->kind == CSMV_KIND_KV ? 3ull * h->kv_S + h->kv_T : h->n_items;
+    const bool bank_lock = h->kind == CSMV_KIND_BANK && selfrecv;  // the self-receiving bank worker
+    if (w->req_tagged > 1) return set_err(CSMV_EINVAL, "csmv_run: req_tagged must be 0 or 1");
+    p.req_tagged = w->req_tagged && (max_id <= (1ull << kIdItemBits)) &&
+                   (bank_lock || (h->kind == CSMV_KIND_KV && kv_filt));
+  }
   // the publisher takes the last warp slot of the first client CTA when no
   // client warp lives there (client warp cw runs on CTA cw % n_ctas, warp
   // cw / n_ctas): it then does not share the server SM with the critical

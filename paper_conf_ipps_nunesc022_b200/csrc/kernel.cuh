@@ -97,12 +97,23 @@ struct Ctl {
 };
 constexpr uint32_t kTraceCap = 1u << 18;
 
-struct ReqHdr {        // written before the doorbell
+// A request's header.  Untagged requests: the three fields, written before
+// a fence and the doorbell.  Tagged requests (KParams.req_tagged): two
+// 64-bit words {round << 32 | snapshot}, {round << 32 | mask} and every id
+// carrying the round's low kIdTagBits bits above the item (kIdItemBits):
+// no fence between payload and doorbell -- the server re-reads the payload
+// until every word carries the round of the doorbell it saw (as the client
+// does with the response, Resp).
+struct ReqHdr {
   uint32_t snapshot;
-  uint32_t mask;
   uint32_t round;      // = the doorbell value; tags the response
-  uint32_t pad;
+  uint32_t mask;
+  uint32_t round2;     // tagged requests: the round again (the mask's word)
 };
+constexpr uint32_t kIdItemBits = 24;                       // tagged requests: item ids < 2^24
+constexpr uint32_t kIdItemMask = (1u << kIdItemBits) - 1;
+constexpr uint32_t kIdTagMask = 0x7Fu;                     // bits 24..30: round & 0x7F (bit 31: in WS)
+__host__ __device__ inline uint32_t id_tag(uint32_t round) { return (round & kIdTagMask) << kIdItemBits; }
 
 // The response: every word carries the request's round in its upper half,
 // so the client accepts it word by word -- no release/acquire pair and no
@@ -198,6 +209,7 @@ struct KParams {
   // and {ticket now served << 32 | CTS of the previous ticket's commit}
   uint32_t* kv_tk_next;       // u32[T], nullptr = CSMV_RETRY_FREE
   uint64_t* kv_tk_serv;       // u64[T]
+  uint32_t req_tagged;        // requests are round-tagged (ReqHdr): no client fence before the doorbell
 };
 
 constexpr uint32_t kKvMaxWays = 256;              // KV ways supported by the device path

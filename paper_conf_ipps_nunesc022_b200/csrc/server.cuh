@@ -318,15 +318,16 @@ static __device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64
         const uint32_t pm = __ballot_sync(FULL, pend);
         if (pm) {
           found = true;
-          if (!fenced) {  // acquire: the payloads of this group's doorbells precede
-            fence_gpu();  // every worker's reads of them (queue -> fence.cta -> loads)
-            fenced = true;
+          if (!fenced && !p.req_tagged) {  // acquire: the payloads of this group's doorbells
+            fence_gpu();  // precede every worker's reads of them (queue -> fence.cta -> loads);
+            fenced = true;  // tagged requests: the worker checks the round in every word instead
           }
           if (pend) {
             const uint32_t pos = tail + __popc(pm & lt);
             c.last_seen[i] = seq[k];
+            // {slot tag, request round (low 16 bits) << 16 | client warp}
             *(volatile uint64_t*)&c.queue[pos & qmask] =
-                ((uint64_t)((pos >> c.qn_log2) + 1) << 32) | (c.cw_lo + i);
+                ((uint64_t)((pos >> c.qn_log2) + 1) << 32) | ((seq[k] & 0xFFFFu) << 16) | (c.cw_lo + i);
           }
           tail += __popc(pm);
         }
@@ -356,9 +357,10 @@ static __device__ void server_receiver(const KParams& p, const SrvCtx& c, uint64
   }
 }
 
-// Claim the next dispatched request of this CTA's queue (blocking).
-// Returns false when the receiver has finished.
-__device__ __forceinline__ bool claim_request(const SrvCtx& c, uint32_t& cw) {
+// Claim the next dispatched request of this CTA's queue (blocking): its
+// client warp and (rq) the low 16 bits of its round.  Returns false when the
+// receiver has finished.
+__device__ __forceinline__ bool claim_request(const SrvCtx& c, uint32_t& cw, uint32_t* rq = nullptr) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t qmask = (1u << c.qn_log2) - 1;
   uint32_t slot = 0;
@@ -367,7 +369,8 @@ __device__ __forceinline__ bool claim_request(const SrvCtx& c, uint32_t& cw) {
   for (;;) {  // convergent wait: every lane polls the same word (broadcast LDS)
     const uint64_t ent = *(volatile uint64_t*)&c.queue[slot & qmask];
     if ((uint32_t)(ent >> 32) == (slot >> c.qn_log2) + 1) {
-      cw = (uint32_t)ent;
+      cw = (uint32_t)ent & 0xFFFFu;
+      if (rq) *rq = ((uint32_t)ent >> 16) & 0xFFFFu;
       return true;
     }
     if (*(volatile uint32_t*)&c.sh->exit) return false;
@@ -503,14 +506,17 @@ __device__ __forceinline__ bool server_self_recv(const KParams& p) {
 // trip (ld.relaxed; fence.acq_rel.gpu = acquire).
 template <int M>
 __device__ __forceinline__ uint32_t self_claim(const KParams& p, const SrvCtx& c, uint32_t lo, uint32_t hi,
-                                               uint32_t m_max, uint32_t (&cwv)[M], uint64_t t_begin, uint32_t& gts) {
+                                               uint32_t m_max, uint32_t (&cwv)[M], uint32_t (&rqv)[M], uint64_t t_begin,
+                                               uint32_t& gts) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t n = hi - lo, rows = (n + 31) / 32;
   for (uint32_t idle = 1;; ++idle) {
     uint32_t m = 0;
     uint32_t g = 0;
-    if (lane == 0) g = ld_relaxed(p.gts);
+    // tagged requests: no fence after the sweep, so GTS is read with
+    // acquire semantics here (the lastw prefetch is ordered after it)
+    if (lane == 0) g = p.req_tagged ? ld_acquire(p.gts) : ld_relaxed(p.gts);
     for (uint32_t r0 = 0; r0 < rows && m < m_max; r0 += 4) {
       // the doorbells of up to 4 rows in flight at once: one L2 round trip
       uint32_t sqv[4];
@@ -531,13 +537,14 @@ __device__ __forceinline__ uint32_t self_claim(const KParams& p, const SrvCtx& c
             pm &= pm - 1;
             if (lane == l) c.last_seen[lo - c.cw_lo + i] = sqv[k];
             cwv[j] = lo + r * 32 + l;
+            rqv[j] = __shfl_sync(FULL, sqv[k], l) & 0xFFFFu;
             m = j + 1;
           }
         }
       }
     }
     if (m) {
-      fence_gpu();  // acquire: the payloads of the doorbells just seen precede our loads of them
+      if (!p.req_tagged) fence_gpu();  // acquire: the payloads of the doorbells just seen precede our loads of them
       gts = __shfl_sync(FULL, g, 0);
       return m;
     }
@@ -602,13 +609,13 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
   uint32_t gts_claim = 0;  // SELF: GTS read with the doorbells (acquired by the claim's fence)
   for (;;) {
     const long long tq = clock64();
-    uint32_t cwv[M];
+    uint32_t cwv[M], rqv[M];  // client warps, their rounds (low 16 bits: tagged requests)
     uint32_t m = 1;
     if constexpr (SELF) {
-      m = self_claim<M>(p, c, my_lo, my_hi, m_max, cwv, t_begin, gts_claim);
+      m = self_claim<M>(p, c, my_lo, my_hi, m_max, cwv, rqv, t_begin, gts_claim);
       if (!m) break;
     } else {
-      if (!claim_request(c, cwv[0])) break;
+      if (!claim_request(c, cwv[0], &rqv[0])) break;
     }
     const uint64_t t_claim = trace_now(p);
     // ---- combine: grab further requests that are already queued
@@ -622,7 +629,8 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       }
       if (self) continue;
       got = __shfl_sync(FULL, got, 0);
-      cwv[j] = got;
+      cwv[j] = got == 0xFFFFFFFFu ? got : got & 0xFFFFu;
+      rqv[j] = got >> 16;
       if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
     }
     const uint32_t m_req = m;
@@ -631,12 +639,14 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       // the group's warps lead + k * n_client_ctas, as many as the CTA has
 #pragma unroll
       for (int r = MR - 1; r >= 0; --r) {
-        const uint32_t lead = cwv[r], cta = lead % p.n_client_ctas, w0 = lead / p.n_client_ctas;
+        const uint32_t lead = cwv[r], cta = lead % p.n_client_ctas, w0 = lead / p.n_client_ctas, lq = rqv[r];
         const uint32_t n_act = min((uint32_t)kWarps, (p.n_cw - cta + p.n_client_ctas - 1) / p.n_client_ctas);
         const uint32_t gs = min((uint32_t)G, n_act - w0);
 #pragma unroll
-        for (int k = 0; k < G; ++k)
+        for (int k = 0; k < G; ++k) {
           cwv[r * G + k] = ((uint32_t)r < m_req && (uint32_t)k < gs) ? lead + k * p.n_client_ctas : 0xFFFFFFFFu;
+          rqv[r * G + k] = lq;  // a group's warps run their rounds in lock-step: one round for all
+        }
       }
       m = m_req * G;
     }
@@ -646,6 +656,12 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     // ordered them after the doorbells; ours orders them after the queue)
     if (!self) fence_cta();
     uint32_t sq[M], sn[M], msk[M], id0[M], id1[M];
+    // fenced requests: every load in flight at once, no checks (the
+    // receiver's or the claim's fence ordered them after the doorbells).
+    // Tagged requests are taken by the self-receiving worker only (the
+    // receiver-fed worker of C2 is server-bound: the check costs it ~2 %
+    // even when off, so it is not compiled there)
+    if (!SELF || !p.req_tagged) {
 #pragma unroll
     for (int j = 0; j < M; ++j) {
       sq[j] = sn[j] = msk[j] = id0[j] = id1[j] = 0;
@@ -655,6 +671,48 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
         sq[j] = ld_relaxed(&p.req_hdr[cwv[j]].round);
         id0[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + lane) & ~kWriteBit;
         id1[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + 32 + lane) & ~kWriteBit;
+      }
+    }
+    } else
+    // tagged requests: loaded again until every word carries the round of
+    // the doorbell (the client did not fence the payload before it).  All
+    // loads are issued before any is looked at (one round trip).
+    for (uint32_t pass = 0;; ++pass) {
+      uint64_t w0[M], w1[M];
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        w0[j] = w1[j] = 0;
+        id0[j] = id1[j] = 0;
+        if (j < (int)m && (G == 1 || cwv[j] != 0xFFFFFFFFu)) {
+          const uint64_t* hw = reinterpret_cast<const uint64_t*>(&p.req_hdr[cwv[j]]);
+          w0[j] = ld_relaxed64(hw);
+          w1[j] = ld_relaxed64(hw + 1);
+          id0[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + lane);
+          id1[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + 32 + lane);
+        }
+      }
+      bool stale = false;
+      const uint32_t keep = p.req_tagged ? kIdItemMask : ~kWriteBit, tm = kIdTagMask << kIdItemBits;
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        sn[j] = (uint32_t)w0[j];
+        sq[j] = (uint32_t)(w0[j] >> 32);
+        msk[j] = (uint32_t)w1[j];
+        const bool live = j < (int)m && (G == 1 || cwv[j] != 0xFFFFFFFFu);
+        if (p.req_tagged && live) {
+          const uint32_t tg = id_tag(rqv[j]);
+          const bool mj = (msk[j] >> lane) & 1u;
+          stale |= (sq[j] & 0xFFFFu) != rqv[j] || (uint32_t)(w1[j] >> 32) != sq[j] ||
+                   (mj && ((id0[j] & tm) != tg || (id1[j] & tm) != tg));
+        }
+        id0[j] &= keep;
+        id1[j] &= keep;
+      }
+      if (!__any_sync(FULL, stale)) break;
+      if ((pass & 1023u) == 1023u) {  // a lost payload would be a protocol error: let the watchdog see it
+        uint32_t bad = 0;
+        if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 5);
+        if (__shfl_sync(FULL, bad, 0)) break;
       }
     }
     bool mine[M];
@@ -895,7 +953,7 @@ __device__ void server_worker_cm(const KParams& p, const SrvCtx& c, uint64_t t_b
         if ((uint32_t)(e >> 32) == (h >> c.qn_log2) + 1 && atomicCAS(&c.sh->q_head, h, h + 1) == h) got = (uint32_t)e;
       }
       got = __shfl_sync(FULL, got, 0);
-      cwv[j] = got;
+      cwv[j] = got == 0xFFFFFFFFu ? got : got & 0xFFFFu;  // the entry's client warp (server_receiver)
       if (got != 0xFFFFFFFFu && m == (uint32_t)j) m = j + 1;
     }
     const uint32_t m_req = m;
@@ -1324,24 +1382,50 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
     my_hi = min(my_lo + per, c.cw_hi);
   }
   for (;;) {
-    uint32_t cw;
+    uint32_t cw, rq = 0;
     const long long tq = clock64();
     if constexpr (SELF) {  // sweep own slice; the claim's acquire fence orders the payload loads
-      uint32_t one[1], g;
-      if (!self_claim<1>(p, c, my_lo, my_hi, 1, one, t_begin, g)) break;
+      uint32_t one[1], r1[1], g;
+      if (!self_claim<1>(p, c, my_lo, my_hi, 1, one, r1, t_begin, g)) break;
       cw = one[0];
+      rq = r1[0];
     } else {
-      if (!claim_request(c, cw)) break;
+      if (!claim_request(c, cw, &rq)) break;
       fence_cta();  // after the receiver's acquire (see server_receiver)
     }
     const uint64_t t_claim = trace_now(p);
     const long long t0 = clock64();
-    const uint32_t sq = ld_relaxed(&p.req_hdr[cw].round);
-    const uint32_t s = ld_relaxed(&p.req_hdr[cw].snapshot);
-    const uint32_t mask = ld_relaxed(&p.req_hdr[cw].mask);
-    uint32_t ids[4];
+    uint32_t sq, s, mask, ids[4];
+    // tagged requests: loaded again until every word carries the round of
+    // the doorbell (the client did not fence the payload before it)
+    for (uint32_t pass = 0;; ++pass) {
+      const uint64_t* hw = reinterpret_cast<const uint64_t*>(&p.req_hdr[cw]);
+      const uint64_t w0 = ld_relaxed64(hw), w1 = ld_relaxed64(hw + 1);
+      s = (uint32_t)w0;
+      sq = (uint32_t)(w0 >> 32);
+      mask = (uint32_t)w1;
 #pragma unroll
-    for (int k = 0; k < 4; ++k) ids[k] = ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + k) * 32 + lane) & ~kWriteBit;
+      for (int k = 0; k < 4; ++k) ids[k] = ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + k) * 32 + lane);
+      if (!p.req_tagged) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) ids[k] &= ~kWriteBit;
+        break;
+      }
+      const uint32_t tg = id_tag(rq), tm = kIdTagMask << kIdItemBits;
+      bool stale = (sq & 0xFFFFu) != rq || (uint32_t)(w1 >> 32) != sq;
+      if ((mask >> lane) & 1u) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) stale |= (ids[k] & tm) != tg;
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k) ids[k] &= kIdItemMask;
+      if (!__any_sync(FULL, stale)) break;
+      if ((pass & 1023u) == 1023u) {  // a lost payload would be a protocol error: let the watchdog see it
+        uint32_t bad = 0;
+        if (lane == 0) bad = ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 5);
+        if (__shfl_sync(FULL, bad, 0)) break;
+      }
+    }
     const bool mine = (mask >> lane) & 1u;
     const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
     srv_fence<CL>();

@@ -34,6 +34,12 @@ J = csmv.DBG_JITTER
                             debug_flags=csmv.DBG_ALT_COMMIT)),
     ("list ATR", dict(atr_mode=csmv.ATR_LIST, server_combine=2)),
     ("list ATR NoCV", dict(atr_mode=csmv.ATR_LIST_NOCV)),
+    ("grouped G=4", dict(publish=csmv.PUBLISH_SERVER, client_group=4, ro_streak=8, server_workers=6,
+                         server_combine=8, ro_adaptive=1)),
+    ("self-receiving tagged requests", dict(publish=csmv.PUBLISH_CLIENT, server_recv=csmv.RECV_SELF,
+                                            server_workers=7, server_combine=2, req_tagged=1)),
+    ("self-receiving tagged, publisher", dict(publish=csmv.PUBLISH_SERVER, server_recv=csmv.RECV_SELF,
+                                              server_workers=6, server_combine=4, ro_adaptive=1, req_tagged=1)),
     ("onlyCS", dict(commit=csmv.COMMIT_ONLYCS)),
     ("JVSTM-GPU", dict(commit=csmv.COMMIT_JVSTM)),
 ])
@@ -59,13 +65,15 @@ def test_bank_c1_full_log_under_jitter():
 
 
 @pytest.mark.parametrize("server,flags", [(csmv.SERVER_CTA, 0), (csmv.SERVER_CTA, csmv.DBG_KV_ITEMSETS),
-                                          (csmv.SERVER_CLUSTER, 0), (csmv.SERVER_CLUSTER, csmv.DBG_KV_ITEMSETS)])
+                                          (csmv.SERVER_CLUSTER, 0), (csmv.SERVER_CLUSTER, csmv.DBG_KV_ITEMSETS),
+                                          (csmv.SERVER_CTA, csmv.DBG_KV_SEQREAD)])
+@pytest.mark.parametrize("tagged", [0, 1])
 @pytest.mark.parametrize("p_update", [10_000, 300_000])
-def test_kv_c4_shrunk_under_jitter(server, flags, p_update):
+def test_kv_c4_shrunk_under_jitter(server, flags, p_update, tagged):
     """KV workers read e_pre = tail outside the lock and then load lastw: the
     jitter sits exactly in that window (cs_leave's fence covers it)."""
     cfg = W.c4(n_items=1 << 12, n_tx=1 << 15, p_update_ppm=p_update, ro_streak=4, client_warps=192,
-               server_workers=6, server=server, cluster_size=4, debug_flags=flags | J)
+               server_workers=6, server=server, cluster_size=4, debug_flags=flags | J, req_tagged=tagged)
     pre, stats, log, fin = run_kv(cfg)
     oc = ocfg_of(cfg)
     d = oracle.kv_gen(oc, cfg.seed, cfg.n_tx)
