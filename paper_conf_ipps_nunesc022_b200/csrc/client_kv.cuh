@@ -345,7 +345,6 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
 
     // ---- A: the pending PUT reads at s (read-set tracked)
     int status = ST_NONE;
-    KvTx d{};
     uint32_t kk[4] = {0, 0, 0, 0};
     uint32_t victim = 0, tset = 0, clk = 0, nrs = 0;
     int iv = 0, ic = 0;  // ring slots the PUT's versions replace: key/value/LRU rings, clock ring
@@ -387,8 +386,8 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           dk_key = gen_kv_key(p.gen, cu);
           dk_id = cu;
         }
-        d = gen_kv_k(p.gen, cu, dk_key);
-        tset = kv_set(d.key, Tn);
+        // only the key now: the value's draws wait for the write-back
+        tset = kv_set(dk_key, Tn);
         if (tickets) {
           // the turn of this ticket: the previous one committed (its CTS in
           // the low word) -- read only once the snapshot covers that commit
@@ -402,7 +401,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           }
         }
         if (status != ST_WAIT) {
-          kv_key16(d.key, kk);
+          kv_key16(dk_key, kk);
           ++att_u;
           pending = true;
         }
@@ -778,6 +777,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     if (mine) {
       if ((cmask >> lane) & 1u) {
         // Client-side write-back: the paper's 4 writes.
+        const KvTx d = gen_kv_k(p.gen, cu, dk_key);  // the PUT's value
         cts = base + __popc(cmask & lt);
         // CSMV_RETRY_FIFO: hand the set to the next ticket, which reads once GTS covers cts
         if (tickets) st_relaxed64(p.kv_tk_serv + tset, ((uint64_t)(tk + 1) << 32) | cts);

@@ -25,15 +25,16 @@ import numpy as np
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
 
-BASE = {"C3": dict(client_warps=294, server_recv=1, server_workers=7, server_combine=2, publish=0, ro_streak=8,
-                   ro_adaptive=1),
-        "C4": dict(client_warps=294, server_workers=6, server_combine=8, publish=1, ro_streak=32, ro_adaptive=1),
-        "C2": dict(client_warps=588, client_group=4, server_workers=6, server_combine=8, publish=1, ro_streak=8,
-                   ro_adaptive=1)}
+def base(name: str) -> dict:
+    """bench.py's tuned launch of the config (so a trace describes the benchmarked run)."""
+    import bench
+    t = dict(bench.tuned(name))
+    return dict({k: v for k, v in t.items() if k != "client_warps_per_sm"},
+                client_warps=t["client_warps_per_sm"] * 147)
 
 
 def main(argv):
-    kw = dict(BASE.get(argv[0], {}))
+    kw = base(argv[0])
     kw.update({k: int(v) for k, v in (a.split("=") for a in argv[1:])})
     kw["debug_flags"] = kw.get("debug_flags", 0) | csmv.DBG_TRACE
     cfg = workloads.PRESETS[argv[0]](**kw)
