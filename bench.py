@@ -490,7 +490,7 @@ def bench_ours(args):
         "kernel_ms_per_step": statistics.mean(kern_ns) / 1e6,
         "aborts": last["aborts"],
     }
-    if args.config == "C3" and rf.get("xsm_roundtrip_ns"):
+    if args.config in ("C3", "C4") and rf.get("xsm_roundtrip_ns"):
         line["hot_chain"] = hot_chain(last, lcfg, rf, statistics.mean(kern_ns))
     if cpu:
         line["cpu_baseline"] = cpu
@@ -501,19 +501,39 @@ def bench_ours(args):
 
 
 def hot_chain(st, lcfg, rf, kern_ns):
-    """C3: every committed transfer touching the hottest account must see the
-    previous one in its snapshot, so those commits form a chain
-    whose link is at least publish -> snapshot -> read -> request -> server
-    -> response: two cross-SM round trips (client->server->client, and the
-    GTS publish -> next client's acquire) plus the ring read.  Floor per link
-    = 2 x xsm_roundtrip + l2_load (tools/ubench/roofs.cu)."""
+    """C3 / C4: every committed transfer touching the hottest account (C4:
+    every PUT on the hottest cache set) must see the previous one in its
+    snapshot, so those commits form a chain whose link is at
+    least publish -> snapshot -> read -> request -> server -> response: two
+    cross-SM round trips (client->server->client, and the GTS publish -> next
+    client's acquire) plus the read (one L2 round trip: the bank's two rings,
+    the KV set read by the warp together).  Floor per link = 2 x
+    xsm_roundtrip + l2_load (tools/ubench/roofs.cu)."""
     import numpy as np
-    n = lcfg.n_items
-    theta = lcfg.workload.zipf_theta_milli / 1000.0
-    r = np.arange(1, n + 1, dtype=np.float64) ** -theta
-    p0 = r[0] / r.sum()
-    # a transfer touches account 0 if src or dst is 0 (dst = src+1 on a collision)
-    p_touch = 1 - (1 - p0) ** 2
+    w = lcfg.workload
+    theta = w.zipf_theta_milli / 1000.0
+    if w.kind == 1:
+        # C4: every PUT on the hottest cache set (the set of key 0, zipf rank
+        # 0) reads and writes its clock, so those PUTs form the chain; the
+        # set of key k is uniform(mix64(k ^ 0xA5..A5), T) (docs/GENERATOR.md)
+        n = w.kv_keys
+        r = np.arange(1, n + 1, dtype=np.float64) ** -theta
+        k = np.arange(n, dtype=np.uint64) ^ np.uint64(0xA5A5A5A5A5A5A5A5)
+        with np.errstate(over="ignore"):
+            z = k + np.uint64(0x9E3779B97F4A7C15)
+            z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+            z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+            z = z ^ (z >> np.uint64(31))
+        T = lcfg.n_items // w.kv_ways
+        sets = ((z >> np.uint64(32)) * np.uint64(T) + (((z & np.uint64(0xFFFFFFFF)) * np.uint64(T)) >> np.uint64(32))) \
+            >> np.uint64(32)
+        p_touch = float(r[sets == sets[0]].sum() / r.sum())
+    else:
+        n = lcfg.n_items
+        r = np.arange(1, n + 1, dtype=np.float64) ** -theta
+        p0 = r[0] / r.sum()
+        # a transfer touches account 0 if src or dst is 0 (dst = src+1 on a collision)
+        p_touch = 1 - (1 - p0) ** 2
     links = st["committed_update"] * p_touch
     floor_ns = 2 * rf["xsm_roundtrip_ns"] + rf["l2_load_ns"]
     link_ns = kern_ns / links if links else None

@@ -452,6 +452,13 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           tss[i] = rls[i] >= 0 ? __shfl_sync(FULL, tset, rls[i]) : 0u;
           if (rls[i] >= 0) kv_put_read_issue<NS>(p, tss[i], ld[i]);
         }
+#ifdef CSMV_TRACE_COOP_SPLIT  // diagnostics: t_snap = the loads have arrived (t_read - t_snap = evaluation)
+        if (tracing) {
+          uint64_t x = ld[0].kr[0].s[0] ^ ld[0].cr.s[0];
+          x = __reduce_or_sync(FULL, (uint32_t)x) ;
+          t_snap = globaltimer() + (x == 0x9u ? 1 : 0);
+        }
+#endif
 #pragma unroll
         for (int i = 0; i < kCoopMax; ++i) {
           if (rls[i] < 0) break;
