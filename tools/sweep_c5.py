@@ -5,10 +5,10 @@ For every point (SURVEY 8(d) protocol): one DIGEST-logged run (seed 1)
 checked element by element against the CPU oracle (--check), then timed runs
 without logging for seeds 1..--seeds (mean, min, max of tx/s).  The launch
 is bench.py's tuned one scaled to the point: client warps = max(16,
-min(W, N/64)) so that in-flight updates stay well below the item count
-(Q29), W = 588 in CTA-level groups of 4 for the single-CTA server (when a
-CTA hosts at least two client warps), 294 per-warp batches for the cluster
-server.  Writes one JSON line per point.
+min(588, N/64)) so that in-flight updates stay well below the item count
+(Q29), in CTA-level groups of 4 when a CTA hosts at least two client warps
+(both servers: the cluster's commit ring takes grouped requests).  Writes
+one JSON line per point.
 
 usage: python tools/sweep_c5.py [--n-tx N] [--check] [--seeds 3] [--out FILE] [--servers 0,1]
 """
@@ -77,8 +77,8 @@ def main():
     f = open(args.out, "w") if args.out else None
     for cfg in workloads.c5_points(args.n_tx, servers=servers):
         single = cfg.workload.server == csmv.SERVER_CTA
-        cw = max(16, min(588 if single else 294, cfg.n_items // 64))  # in-flight updates << items (Q29)
-        group = 4 if single and cw >= 296 else 1
+        cw = max(16, min(588, cfg.n_items // 64))  # in-flight updates << items (Q29)
+        group = 4 if cw >= 296 else 1  # CTA-level batches (the commit ring takes them too)
         cfg = cfg.with_(cluster_size=args.cluster_size, watchdog_ms=60_000, client_group=group,
                         **dict(TUNED, client_warps=cw))
         try:
