@@ -101,7 +101,8 @@ __device__ __forceinline__ int kv_get_finish(const KParams& p, uint32_t s, KvGet
     }
     if (rr != RD_OK) return rr;
 #pragma unroll
-    for (int j = 0; j < 8; ++j) g.dg += dig_word(S + slot, j, val[j]);
+    for (int j = 0; j < 8; ++j)  // the log's digest; unlogged: the value folded into the checksum
+      g.dg = p.log_mode ? g.dg + dig_word(S + slot, j, val[j]) : g.dg ^ ((uint64_t)val[j] << (32 * (j & 1)));
     fin = true;
     return RD_OK;
   }
@@ -116,8 +117,10 @@ __device__ __forceinline__ int kv_get_finish(const KParams& p, uint32_t s, KvGet
     uint32_t k4[4];
     const int rr = kv_key_pick<NS>(p.kv_key + (size_t)slot * NS * 4, ru, K, s, true, k4);
     if (rr != RD_OK) return rr;
+    if (p.log_mode) {  // the log's digest of every key read (S14)
 #pragma unroll
-    for (int j = 0; j < 4; ++j) g.dg += dig_word(slot, j, k4[j]);
+      for (int j = 0; j < 4; ++j) g.dg += dig_word(slot, j, k4[j]);
+    }
     if (k4[0] == g.gk[0] && k4[1] == g.gk[1] && k4[2] == g.gk[2] && k4[3] == g.gk[3]) {
       g.hit = w0 + u + 1;
       g.vslot = slot + 1;  // the value next
@@ -134,33 +137,38 @@ __device__ __forceinline__ int kv_get_finish(const KParams& p, uint32_t s, KvGet
 }
 
 // A PUT's read of its set t at snapshot s by the whole warp (compact
-// requests, A <= 16 ways; every lane calls it with the same t, kk), split in
-// an issue and an evaluation half so that the reads of several PUTs are in
-// flight together: lanes 2w and 2w+1 load the two halves of way w's key
-// ring, lane 31 the set clock's ring; the LRU stamps cost a second trip,
-// only when no way stops the scan.  It decides exactly as the sequential
-// scan (the reader's own loop in client_warp_kv): the clock first, then ways
-// in order up to the first one that matches the key, is empty, or cannot be
-// read at s (NEWER / MISS: the PUT aborts with that reason); ways past the
-// stop are not read (not in the digest); with no stop, the LRU stamps of
-// all ways, the victim being the first least recently used way.  Results
-// are warp-uniform.
+// requests, A <= 16 ways, NS <= 8; every lane calls it with the same t, kk),
+// split in an issue and an evaluation half so that the reads of several PUTs
+// can be in flight together: lane w < A loads way w's whole key ring, lane
+// 31 the set clock's ring; the LRU stamps cost a second trip, only when no
+// way stops the scan.  It decides exactly as the sequential scan (the
+// reader's own loop in client_warp_kv): the clock first, then ways in order
+// up to the first one that matches the key, is empty, or cannot be read at s
+// (NEWER / MISS: the PUT aborts with that reason); ways past the stop are
+// not read (not in the digest); with no stop, the LRU stamps of all ways,
+// the victim being the first least recently used way.  One lane per way
+// keeps the evaluation to a handful of warp-wide operations (its latency is
+// on the hot set's commit chain).  Results are warp-uniform.
+#ifdef CSMV_TRACE_EVAL_END
+__device__ uint32_t g_dbg_lru_dummy;
+#define g_dbg_lru dbg_lru_local
+static __device__ __forceinline__ uint32_t& dbg_lru_ref() { static __shared__ uint32_t x[256]; return x[threadIdx.x]; }
+#undef g_dbg_lru
+#define g_dbg_lru dbg_lru_ref()
+#endif
 template <int NS>
 struct KvCoopLd {
-  static constexpr int H = NS / 2;  // versions per lane
-  Ring<4> kr[H];
+  Ring<4> kr[NS];
   Ring<NS> cr;
 };
 
 template <int NS>
 __device__ __forceinline__ void kv_put_read_issue(const KParams& p, uint32_t t, KvCoopLd<NS>& ld) {
-  constexpr int H = KvCoopLd<NS>::H;
   const uint32_t lane = threadIdx.x & 31, A = p.kv_A;
-  const uint32_t w = lane >> 1, h = lane & 1;
-  if (w < A) {
-    const uint32_t slot = t * A + w;
+  if (lane < A) {
+    const uint64_t* ring = p.kv_key + (size_t)(t * A + lane) * NS * 4;
 #pragma unroll
-    for (int q = 0; q < H; ++q) ld.kr[q] = ld_ring<4>(p.kv_key + ((size_t)slot * NS + h * H + q) * 4);
+    for (int j = 0; j < NS; ++j) ld.kr[j] = ld_ring<4>(ring + j * 4);
   }
   if (lane == 31) ld.cr = ld_ring<NS>(p.kv_clk + (size_t)t * NS);
 }
@@ -172,39 +180,34 @@ __device__ __forceinline__ void kv_put_read_eval(const KParams& p, uint32_t s, u
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t K = p.K, S = p.kv_S, A = p.kv_A;
-  constexpr int H = KvCoopLd<NS>::H;
-  const uint32_t w = lane >> 1, h = lane & 1;
-  const bool wl = w < A;
-  const uint32_t slot = t * A + w;
-  // the clock (lane 31)
+  const bool lead = lane < A;  // this lane's way
+  const uint32_t slot = t * A + lane;
+  // the clock (lane 31): status and replacement slot in one word
   int cst = RD_OK, cic = 0;
   uint32_t cval = 0, cseen = 0;
   if (lane == 31) cst = kv_read_clk<NS>(ld.cr, K, s, cval, cseen, cic);
-  cst = __shfl_sync(FULL, cst, 31);
-  cval = __shfl_sync(FULL, cval, 31);
-  cseen = __shfl_sync(FULL, cseen, 31);
-  ic = __shfl_sync(FULL, cic, 31);
-  seen = cseen;
-  st = cst;
-  clk = cval;
+  const uint32_t cw = __shfl_sync(FULL, ((uint32_t)cst << 8) | (uint32_t)cic, 31);
+  cst = (int)(cw >> 8);
+  ic = (int)(cw & 0xFFu);
+  clk = __shfl_sync(FULL, cval, 31);
   victim = 0xFFFFFFFFu;
   iv = 0;
   rdig = 0;
-  // this lane's versions of way w (kv_key_pick with rot = false, per half)
+  // this lane's way: kv_key_pick with rot = false, and the slot a new
+  // version would replace (the key, value and LRU rings' timestamps agree)
   int cand = -1;
-  uint32_t cts = 0, newest = 0, torn_max = 0, key[4] = {0u, 0u, 0u, 0u}, lts[H];
+  uint32_t cts = 0, newest = 0, torn_max = 0, key[4] = {0u, 0u, 0u, 0u}, lts[NS];
   bool torn = false;
 #pragma unroll
-  for (int q = 0; q < H; ++q) {
-    const uint32_t jg = h * H + q;
-    lts[q] = kEmptyTs;
-    if (!wl || jg >= K) continue;
-    const uint32_t t0 = (uint32_t)(ld.kr[q].s[0] >> 32);
-    lts[q] = t0;
+  for (int j = 0; j < NS; ++j) {
+    lts[j] = kEmptyTs;
+    if (!lead || (uint32_t)j >= K) continue;
+    const uint32_t t0 = (uint32_t)(ld.kr[j].s[0] >> 32);
+    lts[j] = t0;
     bool intact = true;
 #pragma unroll
     for (int x = 0; x < 4; ++x) {
-      const uint32_t tw = (uint32_t)(ld.kr[q].s[x] >> 32);
+      const uint32_t tw = (uint32_t)(ld.kr[j].s[x] >> 32);
       intact &= tw == t0;
       if (tw != kEmptyTs) newest = max(newest, tw);
       if (tw <= s) torn_max = max(torn_max, tw);
@@ -214,52 +217,39 @@ __device__ __forceinline__ void kv_put_read_eval(const KParams& p, uint32_t s, u
       continue;
     }
     if (t0 != kEmptyTs && t0 <= s && (cand < 0 || t0 > cts)) {
-      cand = (int)jg;
+      cand = j;
       cts = t0;
 #pragma unroll
-      for (int x = 0; x < 4; ++x) key[x] = (uint32_t)ld.kr[q].s[x];
-    }
-  }
-  // combine the two halves of the way (lanes 2w, 2w+1)
-  {
-    const int ocand = __shfl_xor_sync(FULL, cand, 1);
-    const uint32_t octs = __shfl_xor_sync(FULL, cts, 1);
-    uint32_t okey[4];
-#pragma unroll
-    for (int x = 0; x < 4; ++x) okey[x] = __shfl_xor_sync(FULL, key[x], 1);
-    newest = max(newest, __shfl_xor_sync(FULL, newest, 1));
-    torn_max = max(torn_max, __shfl_xor_sync(FULL, torn_max, 1));
-    torn = __shfl_xor_sync(FULL, (uint32_t)torn, 1) || torn;
-    if (ocand >= 0 && (cand < 0 || octs > cts)) {
-      cand = ocand;
-      cts = octs;
-#pragma unroll
-      for (int x = 0; x < 4; ++x) key[x] = okey[x];
+      for (int x = 0; x < 4; ++x) key[x] = (uint32_t)ld.kr[j].s[x];
     }
   }
   const int wst = newest > s ? RD_NEWER : ((cand < 0 || (torn && torn_max > cts)) ? RD_MISS : RD_OK);
   const bool match = key[0] == kk[0] && key[1] == kk[1] && key[2] == kk[2] && key[3] == kk[3];
   const bool empty = !(key[0] | key[1] | key[2] | key[3]);
-  const bool lead = wl && h == 0;  // one lane per way
-  if (cst != RD_OK) return;
+  const int my_iv = kv_install_slot<NS>(lts, K);
   const uint32_t stops = __ballot_sync(FULL, lead && (wst != RD_OK || match || empty));
-  const uint32_t ws = stops ? (uint32_t)(__ffs(stops) - 1) >> 1 : A;  // the scan's last way (A: none)
-  // the ways read: 0..ws (all of them when nothing stopped the scan)
-  const bool rd = lead && w <= ws;
-  seen = max(seen, __reduce_max_sync(FULL, rd ? newest : 0u));
-  if (stops) {
-    const int sst = __shfl_sync(FULL, wst, 2 * ws);
-    if (sst != RD_OK) {
-      st = sst;
-      return;
-    }
+  const uint32_t ws = stops ? (uint32_t)__ffs(stops) - 1 : A;  // the scan's last way (A: none)
+  const bool rd = lead && lane <= ws;  // the ways read: 0..ws (all of them when nothing stopped the scan)
+  seen = max(__shfl_sync(FULL, cseen, 31), __reduce_max_sync(FULL, rd ? newest : 0u));
+  st = cst;
+  if (cst != RD_OK) return;
+  // the stopping way's status and replacement slot
+  const uint32_t sw = __shfl_sync(FULL, ((uint32_t)wst << 8) | (uint32_t)my_iv, stops ? ws : 0);
+  if (stops && (sw >> 8) != RD_OK) {
+    st = (int)(sw >> 8);
+    return;
   }
+  const bool lg = p.log_mode != 0;  // the read digest exists for the log (S14) only
   uint64_t dg = 0;
-  if (rd) {
+  if (rd && lg) {
 #pragma unroll
     for (int x = 0; x < 4; ++x) dg += dig_word(slot, x, key[x]);
   }
   uint32_t vw = ws;  // victim way
+  iv = (int)(sw & 0xFFu);
+#ifdef CSMV_TRACE_EVAL_END
+  g_dbg_lru = !stops;
+#endif
   if (!stops) {  // LRU stamps of every way; the first least recently used way is the victim
     int lst = RD_OK;
     uint32_t l = 0xFFFFFFFFu, ln = 0;
@@ -277,20 +267,17 @@ __device__ __forceinline__ void kv_put_read_eval(const KParams& p, uint32_t s, u
       st = __shfl_sync(FULL, lst, __ffs(bad) - 1);
       return;
     }
-    if (lead) dg += dig1(2 * S + slot, l);
+    if (lead && lg) dg += dig1(2 * S + slot, l);
     const uint32_t lmin = __reduce_min_sync(FULL, l);
-    vw = (uint32_t)(__ffs(__ballot_sync(FULL, lead && l == lmin)) - 1) >> 1;
+    vw = (uint32_t)__ffs(__ballot_sync(FULL, lead && l == lmin)) - 1;
+    iv = __shfl_sync(FULL, my_iv, vw);
   }
-  // the digest of everything read, summed over the warp
+  if (lg) {  // the digest of everything read, summed over the warp
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) dg += __shfl_xor_sync(FULL, dg, o);
-  rdig = dg + dig1(3 * S + t, clk);
+    for (int o = 16; o > 0; o >>= 1) dg += __shfl_xor_sync(FULL, dg, o);
+    rdig = dg + dig1(3 * S + t, clk);
+  }
   victim = t * A + vw;
-  // the victim's key ring timestamps (= its value and LRU rings'): the slot all three replace
-  uint32_t ts[NS];
-#pragma unroll
-  for (int j = 0; j < NS; ++j) ts[j] = __shfl_sync(FULL, lts[j % H], 2 * vw + j / H);
-  iv = kv_install_slot<NS>(ts, K);
 }
 
 template <int NS>
@@ -427,17 +414,21 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     }
     // compact requests on sets of up to 16 ways: the warp reads each
     // reader's set together, one memory round trip per reader
-    const bool coop = compact && A <= 16 && !(p.debug & CSMV_DBG_KV_SEQREAD);
+    const bool coop = NS <= 8 && compact && A <= 16 && !(p.debug & CSMV_DBG_KV_SEQREAD);
     int r_c = RD_OK;
     uint32_t seen_c = 0;
     const uint32_t n_readers = __popc(__ballot_sync(FULL, reader));
+#ifdef CSMV_TRACE_EVAL_END
+    uint64_t t_eval_end = 0;
+    uint32_t n_lru = 0;
+#endif
 #ifdef CSMV_TRACE_SNAP_LATE
     t_snap = tracing ? globaltimer() : 0;
 #endif
     if (coop) {
       // up to kCoopMax readers' sets in flight together, then evaluated one by one
 #ifndef CSMV_KV_COOP_MAX
-#define CSMV_KV_COOP_MAX 2
+#define CSMV_KV_COOP_MAX 1
 #endif
       constexpr int kCoopMax = CSMV_KV_COOP_MAX;
       uint32_t rem = __ballot_sync(FULL, reader);
@@ -454,7 +445,9 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         }
 #ifdef CSMV_TRACE_COOP_SPLIT  // diagnostics: t_snap = the loads have arrived (t_read - t_snap = evaluation)
         if (tracing) {
-          uint64_t x = ld[0].kr[0].s[0] ^ ld[0].cr.s[0];
+          uint64_t x = ld[0].cr.s[0];
+#pragma unroll
+          for (int j = 0; j < NS; ++j) x ^= ld[0].kr[j].s[0] ^ ld[0].kr[j].s[1] ^ ld[0].kr[j].s[2] ^ ld[0].kr[j].s[3];
           x = __reduce_or_sync(FULL, (uint32_t)x) ;
           t_snap = globaltimer() + (x == 0x9u ? 1 : 0);
         }
@@ -469,6 +462,12 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           uint32_t seen_, vic_, clk_;
           uint64_t dg_;
           kv_put_read_eval<NS>(p, s, tss[i], k4, ld[i], st_, seen_, vic_, iv_, ic_, clk_, dg_);
+#ifdef CSMV_TRACE_EVAL_END  // diagnostics: t_read - t_snap = the first reader's evaluation
+          if (tracing && i == 0) {
+            t_eval_end = globaltimer() + (vic_ == 0x12345u ? 1 : 0);
+            n_lru = g_dbg_lru;  // the eval's LRU path was taken
+          }
+#endif
           if (lane == (uint32_t)rls[i]) {
             r_c = st_;
             seen_c = seen_;
@@ -608,7 +607,11 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       }
     }
     __syncwarp();
+#ifdef CSMV_TRACE_EVAL_END
+    const uint64_t t_read = t_eval_end;
+#else
     const uint64_t t_read = tracing ? globaltimer() : 0;
+#endif
     pc.mark(PH_READ);
     jit();  // versions read, not yet validated
 
@@ -850,7 +853,12 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     if (tracing && cts && tset == p.trace_item) {
       uint64_t tc, tv;
       trace_srv_times(p, cw, round, t_sub, tc, tv);
+#ifdef CSMV_TRACE_EVAL_END
+      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv, t_snap, t_read, n_readers + 100 * n_lru,
+                   __popc(kept));
+#else
       trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv, t_snap, t_read, n_readers, __popc(kept));
+#endif
     }
   }
   client_flush(p, cc);
