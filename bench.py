@@ -49,8 +49,11 @@ UNIT = "tx/s"
 # tuned launch configuration of the C2 workload: 4 client warps
 # per SM submitting CTA-level batches of 4 warps (client_group, 355 -> 490 M
 # tx/s with the 2-hash filter, profiles/r02/tune_group.md)
-TUNED = dict(client_warps_per_sm=4, client_group=4, server_workers=6, server_combine=8, ro_streak=8, publish=1,
-             ro_adaptive=1, server_recv=0)
+# (round-2 retune at 801ce07: a read-only run of 2 per round (was 8), the
+# fixed-length rounds (ro_adaptive 0) and a 7th worker: 501 -> 555 M in tune
+# runs, profiles/r02/raw/r02bf_c2_retune.txt)
+TUNED = dict(client_warps_per_sm=4, client_group=4, server_workers=7, server_combine=8, ro_streak=2, publish=1,
+             ro_adaptive=0, server_recv=0)
 # per-workload overrides of the tuned launch (tools/tune.py on B200): the hot-item
 # chains of C3 want the lower-latency self-receiving server combining at most 2
 # batches per critical section (3.3M -> 4.5M tx/s against 8) and the clients'
@@ -63,9 +66,9 @@ TUNED = dict(client_warps_per_sm=4, client_group=4, server_workers=6, server_com
 # payload and doorbell: a shorter link; C4 103 -> 113 M tx/s, while C2's
 # server-bound step prefers fenced payloads, 494 vs 505 M)
 TUNED_PER_CONFIG = {"C3": dict(server_recv=1, server_workers=7, server_combine=2, publish=0, client_warps_per_sm=2,
-                               client_group=1, req_tagged=1),
+                               client_group=1, req_tagged=1, ro_streak=8, ro_adaptive=1),
                     "C4": dict(ro_streak=32, client_warps_per_sm=2, client_group=1, ro_adaptive=2, backoff_max=16,
-                               req_tagged=1)}
+                               req_tagged=1, server_workers=6)}
 
 
 def tuned(config: str) -> dict:
