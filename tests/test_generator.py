@@ -103,3 +103,44 @@ def test_tx_offset_is_counter_based():
     a = oracle.bank_gen(cfg, 9, 500)
     b = oracle.bank_gen(cfg, 9, 100, tx0=400)
     assert np.array_equal(a[400:], b)
+
+
+# ---- the KV generator (or_kv_gen, docs/GENERATOR.md 4): pinned by the
+# statistics the workload is defined by (zipf keys, a GET/PUT mix),
+# not by re-typing its formulas ----
+def test_kv_gen_mix_and_zipf_frequencies():
+    n_keys, n = 1024, 400_000
+    cfg = oracle.kv_cfg(4096, 16, n_keys=n_keys, p_update_ppm=200_000, zipf_theta_milli=990)
+    d = oracle.kv_gen(cfg, 7, n)
+    # PUT fraction 20 %: binomial, 5 sigma
+    f = d["is_update"].mean()
+    assert abs(f - 0.2) < 5 * np.sqrt(0.2 * 0.8 / n), f
+    # key frequencies against the zipf pmf r^-0.99 / H (numpy, independent of the oracle's CDF)
+    r = np.arange(1, n_keys + 1, dtype=np.float64) ** -0.99
+    pmf = r / r.sum()
+    cnt = np.bincount(d["key"], minlength=n_keys)
+    assert cnt.shape[0] == n_keys  # every key < n_keys
+    for k in (0, 1, 2, 9, 99):
+        sd = np.sqrt(n * pmf[k] * (1 - pmf[k]))
+        assert abs(cnt[k] - n * pmf[k]) < 5 * sd, (k, cnt[k], n * pmf[k])
+    # GETs carry no value; PUT values are 32 uniformly random bytes
+    assert not d["val"][d["is_update"] == 0].any()
+    bits = np.unpackbits(d["val"][d["is_update"] == 1].view(np.uint8))
+    assert abs(bits.mean() - 0.5) < 0.005
+
+
+def test_kv_gen_is_counter_based():
+    cfg = oracle.kv_cfg(1 << 12, 16, p_update_ppm=300_000)
+    whole = oracle.kv_gen(cfg, 11, 5000)
+    part = oracle.kv_gen(cfg, 11, 1000, tx0=3000)
+    assert np.array_equal(whole[3000:4000], part)
+    other = oracle.kv_gen(cfg, 12, 5000)
+    assert (whole["key"] != other["key"]).mean() > 0.5
+
+
+def test_kv_gen_uniform_keys():
+    n_keys, n = 64, 200_000
+    cfg = oracle.kv_cfg(1 << 10, 16, n_keys=n_keys, dist=oracle.DIST_UNIFORM, p_update_ppm=500_000)
+    cnt = np.bincount(oracle.kv_gen(cfg, 3, n)["key"], minlength=n_keys)
+    chi2 = ((cnt - n / n_keys) ** 2 / (n / n_keys)).sum()
+    assert chi2 < 63 + 5 * np.sqrt(2 * 63), chi2  # 63 degrees of freedom
