@@ -3,6 +3,12 @@
 // Same lane state machine and round phases as client_bank.cuh; GET is the
 // read-only transaction, PUT the update transaction (docs/GENERATOR.md 4).
 //
+// Trace diagnostics (build knobs, CSMV_NVCC_EXTRA; CSMV_DBG_TRACE runs):
+// CSMV_TRACE_SNAP_LATE stamps t_snap when the PUT read starts instead of
+// after the snapshot; CSMV_TRACE_COOP_SPLIT when the cooperative read's
+// loads have arrived; CSMV_TRACE_EVAL_END makes t_read the end of the first
+// reader's evaluation (profiles/r02/raw/r02be_c4_chain_eval_split.txt).
+//
 // Read-set representation.  By default (and always above kKvFullWays ways,
 // up to 256) a PUT's read/write set is shipped as {set clock} u WS;
 // with CSMV_DBG_KV_ITEMSETS (A <= 16) it is tracked item by item (smem
@@ -149,13 +155,6 @@ __device__ __forceinline__ int kv_get_finish(const KParams& p, uint32_t s, KvGet
 // the victim being the first least recently used way.  One lane per way
 // keeps the evaluation to a handful of warp-wide operations (its latency is
 // on the hot set's commit chain).  Results are warp-uniform.
-#ifdef CSMV_TRACE_EVAL_END
-__device__ uint32_t g_dbg_lru_dummy;
-#define g_dbg_lru dbg_lru_local
-static __device__ __forceinline__ uint32_t& dbg_lru_ref() { static __shared__ uint32_t x[256]; return x[threadIdx.x]; }
-#undef g_dbg_lru
-#define g_dbg_lru dbg_lru_ref()
-#endif
 template <int NS>
 struct KvCoopLd {
   Ring<4> kr[NS];
@@ -247,9 +246,6 @@ __device__ __forceinline__ void kv_put_read_eval(const KParams& p, uint32_t s, u
   }
   uint32_t vw = ws;  // victim way
   iv = (int)(sw & 0xFFu);
-#ifdef CSMV_TRACE_EVAL_END
-  g_dbg_lru = !stops;
-#endif
   if (!stops) {  // LRU stamps of every way; the first least recently used way is the victim
     int lst = RD_OK;
     uint32_t l = 0xFFFFFFFFu, ln = 0;
@@ -420,7 +416,6 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     const uint32_t n_readers = __popc(__ballot_sync(FULL, reader));
 #ifdef CSMV_TRACE_EVAL_END
     uint64_t t_eval_end = 0;
-    uint32_t n_lru = 0;
 #endif
 #ifdef CSMV_TRACE_SNAP_LATE
     t_snap = tracing ? globaltimer() : 0;
@@ -463,10 +458,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
           uint64_t dg_;
           kv_put_read_eval<NS>(p, s, tss[i], k4, ld[i], st_, seen_, vic_, iv_, ic_, clk_, dg_);
 #ifdef CSMV_TRACE_EVAL_END  // diagnostics: t_read - t_snap = the first reader's evaluation
-          if (tracing && i == 0) {
-            t_eval_end = globaltimer() + (vic_ == 0x12345u ? 1 : 0);
-            n_lru = g_dbg_lru;  // the eval's LRU path was taken
-          }
+          if (tracing && i == 0) t_eval_end = globaltimer() + (vic_ == 0x12345u ? 1 : 0);
 #endif
           if (lane == (uint32_t)rls[i]) {
             r_c = st_;
@@ -853,12 +845,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     if (tracing && cts && tset == p.trace_item) {
       uint64_t tc, tv;
       trace_srv_times(p, cw, round, t_sub, tc, tv);
-#ifdef CSMV_TRACE_EVAL_END
-      trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv, t_snap, t_read, n_readers + 100 * n_lru,
-                   __popc(kept));
-#else
       trace_commit(p, cts, s, t_rb, t_sub, t_resp, globaltimer(), tc, tv, t_snap, t_read, n_readers, __popc(kept));
-#endif
     }
   }
   client_flush(p, cc);
