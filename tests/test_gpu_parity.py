@@ -276,3 +276,14 @@ def test_blind_write_elision():
         with pytest.raises(csmv.CsmvError) as e:
             st.run(kv.workload, kv.n_tx, kv.seed)
         assert e.value.code == csmv.EINVAL
+
+
+def test_tagged_requests_fall_back_above_24_bit_items():
+    """Round-tagged requests carry the round in id bits 24-30, so a store
+    with item ids >= 2^24 must run fenced requests instead -- and still pass
+    the oracle (the self-receiving worker, where tags are otherwise taken)."""
+    n = (1 << 24) + 4096
+    cfg = W.c2(n_items=n, n_tx=1 << 15, client_warps=128, ro_reads=64, server_recv=csmv.RECV_SELF,
+               server_workers=7, server_combine=2, publish=csmv.PUBLISH_CLIENT, req_tagged=1)
+    rep, stats, *_ = check(cfg)
+    assert stats["committed"] == cfg.n_tx
