@@ -28,8 +28,8 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
 
 VARIANTS = {
-    "csmv-b200": dict(atr_mode=csmv.ATR_HASH, server_combine=4, server_workers=6, ro_streak=8, ro_adaptive=1,
-                      publish=csmv.PUBLISH_SERVER),
+    "csmv-b200": dict(atr_mode=csmv.ATR_HASH, server_combine=8, server_workers=7, ro_streak=2, ro_adaptive=0,
+                      publish=csmv.PUBLISH_SERVER),  # bench.py's C2 launch (per-warp batches)
     "csmv": dict(atr_mode=csmv.ATR_LIST, server_combine=1, ro_streak=0, publish=csmv.PUBLISH_CLIENT),
     "nocv": dict(atr_mode=csmv.ATR_LIST_NOCV, server_combine=1, ro_streak=0, publish=csmv.PUBLISH_CLIENT),
     "onlycs": dict(commit=csmv.COMMIT_ONLYCS, ro_streak=0, publish=csmv.PUBLISH_CLIENT),

@@ -17,7 +17,8 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
 
 WAYS = (4, 8, 16, 32, 64, 128, 256)
-TUNED = dict(server_workers=6, ro_streak=8, ro_adaptive=1, publish=csmv.PUBLISH_SERVER)
+TUNED = dict(server_workers=6, ro_streak=32, ro_adaptive=2, backoff_max=16, req_tagged=1, client_warps=294,
+             publish=csmv.PUBLISH_SERVER)  # bench.py's C4 launch
 
 
 def cfg_for(ways: int, n_tx: int, slots: int, **kw):
