@@ -48,7 +48,7 @@ class _Workload(C.Structure):
         "kind", "dist", "zipf_theta_milli", "p_update_ppm", "ro_period", "ro_reads",
         "amount_max", "kv_ways", "kv_keys", "client_warps", "server", "cluster_size", "server_workers", "server_combine",
         "atr_capacity", "atr_mode", "publish", "ro_streak", "backoff_max", "log_mode", "debug_flags", "watchdog_ms", "commit",
-        "ro_adaptive", "server_recv", "client_group", "trace_item", "elide_ww", "retry_order", "req_tagged")]
+        "ro_adaptive", "server_recv", "client_group", "trace_item", "elide_ww", "retry_order", "server_writeback", "req_tagged")]
 
 
 class _Stats(C.Structure):
@@ -98,6 +98,7 @@ class Workload:
     trace_item: int = 0xFFFFFFFF
     elide_ww: int = 0
     retry_order: int = 0
+    server_writeback: int = 0
     req_tagged: int = 0
 
     def to_c(self) -> _Workload:

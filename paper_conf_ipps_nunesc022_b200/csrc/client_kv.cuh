@@ -651,6 +651,16 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
       put_req_id(p, my_ids + 2 * 32 + lane, (S + victim) | kWriteBit, round);
       put_req_id(p, my_ids + 3 * 32 + lane, (2 * S + victim) | kWriteBit, round);
       p.req_cnt[(size_t)cw * 32 + lane] = 4;
+      if (p.kv_swb) {  // what the server needs to write the four versions back
+        const KvTx d = gen_kv_k(p.gen, cu, dk_key);
+        uint32_t* r = my_ids + kSwbRow * 32 + lane;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) r[j * 32] = kk[j];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) r[(4 + j) * 32] = d.val[j];
+        r[12 * 32] = clk + 1;
+        r[13 * 32] = (uint32_t)iv | ((uint32_t)ic << 8);
+      }
     } else if (kept && mine) {
       // request ids: RS u WS (bit 31: in WS)
       uint32_t n = 0;
@@ -784,17 +794,19 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         // CSMV_RETRY_FIFO: hand the set to the next ticket, which reads once GTS covers cts
         if (tickets) st_relaxed64(p.kv_tk_serv + tset, ((uint64_t)(tk + 1) << 32) | cts);
         const uint32_t cn = clk + 1;
-        // stores only: the slots were fixed by the read (the rings are as
-        // read -- nothing wrote the set after s: this commit validated)
-        uint64_t* rk = p.kv_key + (size_t)victim * NS * 4;
-        uint64_t* rv = p.kv_val + (size_t)victim * NS * 8;
-        uint64_t* rl = p.kv_lru + (size_t)victim * NS;
-        uint64_t* rc = p.kv_clk + (size_t)tset * NS;
-        const uint32_t cn1[1] = {cn};
-        kv_install_at<4>(rk, iv, cts, kk);
-        kv_install_at<8>(rv, iv, cts, d.val);
-        kv_install_at<1>(rl, iv, cts, cn1);
-        kv_install_at<1>(rc, ic, cts, cn1);
+        if (!p.kv_swb) {  // (server write-back: the worker has written them and published)
+          // stores only: the slots were fixed by the read (the rings are as
+          // read -- nothing wrote the set after s: this commit validated)
+          uint64_t* rk = p.kv_key + (size_t)victim * NS * 4;
+          uint64_t* rv = p.kv_val + (size_t)victim * NS * 8;
+          uint64_t* rl = p.kv_lru + (size_t)victim * NS;
+          uint64_t* rc = p.kv_clk + (size_t)tset * NS;
+          const uint32_t cn1[1] = {cn};
+          kv_install_at<4>(rk, iv, cts, kk);
+          kv_install_at<8>(rv, iv, cts, d.val);
+          kv_install_at<1>(rl, iv, cts, cn1);
+          kv_install_at<1>(rc, ic, cts, cn1);
+        }
         if (p.log_mode) {
           uint64_t wd = dig1(2 * S + victim, cn) + dig1(3 * S + tset, cn);
 #pragma unroll
@@ -815,7 +827,7 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
     }
     __syncwarp();
     pc.mark(PH_WRITEBACK);
-    const uint32_t n = __popc(cmask);
+    const uint32_t n = p.kv_swb ? 0u : __popc(cmask);  // server write-back: published by the server
     if (n) {
       jit();  // write-backs done, commit not yet published
       if (p.publish == CSMV_PUBLISH_CLIENT) {

@@ -634,8 +634,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
     const uint64_t max_id = h->kind == CSMV_KIND_KV ? 3ull * h->kv_S + h->kv_T : h->n_items;
     const bool bank_lock = h->kind == CSMV_KIND_BANK && selfrecv;  // the self-receiving bank worker
     if (w->req_tagged > 1) return set_err(CSMV_EINVAL, "csmv_run: req_tagged must be 0 or 1");
+    if (w->server_writeback > 1) return set_err(CSMV_EINVAL, "csmv_run: server_writeback must be 0 or 1");
+    p.kv_swb = w->server_writeback && h->kind == CSMV_KIND_KV && kv_filt && h->maxid >= kSwbRow + kSwbRows;
     p.req_tagged = w->req_tagged && (max_id <= (1ull << kIdItemBits)) &&
-                   (bank_lock || (h->kind == CSMV_KIND_KV && kv_filt));
+                   (bank_lock || (h->kind == CSMV_KIND_KV && kv_filt)) && !p.kv_swb;
   }
   // the publisher takes the last warp slot of the first client CTA when no
   // client warp lives there (client warp cw runs on CTA cw % n_ctas, warp

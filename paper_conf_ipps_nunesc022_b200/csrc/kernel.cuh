@@ -210,7 +210,11 @@ struct KParams {
   uint32_t* kv_tk_next;       // u32[T], nullptr = CSMV_RETRY_FREE
   uint64_t* kv_tk_serv;       // u64[T]
   uint32_t req_tagged;        // requests are round-tagged (ReqHdr): no client fence before the doorbell
+  uint32_t kv_swb;            // KV: the server writes committed PUTs back and publishes (rows kSwbRow.. of a request)
 };
+// KV server write-back: request rows 4-7 the key, 8-15 the value, 16 the new
+// LRU / clock value, 17 the replacement slots (key/value/LRU | clock << 8)
+constexpr uint32_t kSwbRow = 4, kSwbRows = 14;
 
 constexpr uint32_t kKvMaxWays = 256;              // KV ways supported by the device path
 constexpr uint32_t kKvFullWays = 16;              // up to here PUT read-sets are shipped item by item

@@ -1365,7 +1365,7 @@ __device__ void server_worker_generic(const KParams& p, const SrvCtx& c, uint64_
 // (as the bank worker).  Only clocks enter the filter: nothing else is ever
 // validated in this mode; lastw is written for all four written items.
 // ---------------------------------------------------------------------------
-template <bool CL, bool SELF = false>
+template <int NS, bool CL, bool SELF = false>
 __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint64_t t_begin) {
   const uint32_t FULL = 0xFFFFFFFFu;
   const uint32_t lane = threadIdx.x & 31;
@@ -1427,6 +1427,14 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
       }
     }
     const bool mine = (mask >> lane) & 1u;
+    // server write-back: the PUT's key, value, new LRU / clock value and
+    // replacement slots, loaded with the payload (fenced requests)
+    uint32_t wb[kSwbRows];
+    if (p.kv_swb) {
+#pragma unroll
+      for (int k = 0; k < (int)kSwbRows; ++k)
+        wb[k] = mine ? ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + kSwbRow + k) * 32 + lane) : 0u;
+    }
     const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
     srv_fence<CL>();
     jit();  // e_pre read, lastw not yet (the window cs_leave's fence covers)
@@ -1465,6 +1473,40 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
     const long long tr = clock64();
     cs_leave<CL>(c, ticket, t0c + n);
     const long long t2 = clock64();
+    if (p.kv_swb && n) {
+      // Server write-back (csmv_workload.server_writeback): the four
+      // versions of each committed PUT, then GTS advanced in CTS order
+      // -- by this worker once GTS reaches its first CTS - 1, or through the
+      // done flags and the publisher.  No lock is held: a later range's
+      // worker waits for this one's publish, never the other way round.
+      jit();
+      if (commit) {
+        const uint32_t cts = t0c + 1 + __popc(cm & lt);
+        const uint32_t S = p.kv_S, victim = ids[1], tset = ids[0] - 3 * S;
+        const int iv = (int)(wb[13] & 0xFFu), ic = (int)((wb[13] >> 8) & 0xFFu);
+        const uint32_t kk[4] = {wb[0], wb[1], wb[2], wb[3]};
+        const uint32_t vv[8] = {wb[4], wb[5], wb[6], wb[7], wb[8], wb[9], wb[10], wb[11]};
+        const uint32_t cn1[1] = {wb[12]};
+        kv_install_at<4>(p.kv_key + (size_t)victim * NS * 4, iv, cts, kk);
+        kv_install_at<8>(p.kv_val + (size_t)victim * NS * 8, iv, cts, vv);
+        kv_install_at<1>(p.kv_lru + (size_t)victim * NS, iv, cts, cn1);
+        kv_install_at<1>(p.kv_clk + (size_t)tset * NS, ic, cts, cn1);
+        if (p.publish == CSMV_PUBLISH_SERVER) st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
+      }
+      if (p.publish == CSMV_PUBLISH_CLIENT) {
+        __syncwarp();
+        fence_gpu();
+        if (lane == 0) {
+          uint32_t it = 0;
+          while (ld_relaxed(p.gts) != t0c) {
+            if ((++it & 255u) == 0 && (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 6))) break;
+            __nanosleep(32);
+          }
+          st_release(p.gts, t0c + n);
+        }
+      }
+      __syncwarp();
+    }
     if (lane == 0) {  // round-tagged words, no fence (kernel.cuh Resp)
       trace_served(p, cw, sq, t_claim);
       const uint64_t tag = (uint64_t)sq << 32;
@@ -1738,7 +1780,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
   if (!CL && server_self_recv(p)) {
     // warps 0..n_workers-1 self-receiving workers, then the publisher
     if (warp < p.n_workers) {
-      if constexpr (KIND == CSMV_KIND_KV) server_worker_kv_filter<CL, !CL>(p, c, t_begin);
+      if constexpr (KIND == CSMV_KIND_KV) server_worker_kv_filter<NS, CL, !CL>(p, c, t_begin);
       else server_worker<CL, !CL>(p, c, t_begin);
     } else if (warp == p.n_workers && p.publish == CSMV_PUBLISH_SERVER && !p.pub_remote) {
       server_publisher(p, &c, t_begin, c.sh->tail);
@@ -1749,7 +1791,7 @@ __device__ void server_cta(const KParams& p, uint8_t* smem, uint64_t t_begin) {
     server_receiver(p, c, t_begin);
   } else if (warp <= p.n_workers) {
     if constexpr (KIND == CSMV_KIND_KV) {
-      if (kv_filter_mode(p)) server_worker_kv_filter<CL>(p, c, t_begin);
+      if (kv_filter_mode(p)) server_worker_kv_filter<NS, CL>(p, c, t_begin);
       else server_worker_generic<CL>(p, c, t_begin);
     }
     else if (!CL && p.commit == CSMV_COMMIT_ONLYCS) server_worker_onlycs<NS>(p, c, t_begin);

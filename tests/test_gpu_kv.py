@@ -263,3 +263,33 @@ def test_kv_coop_read_parity(kw):
     kw = dict(dict(n_items=1 << 12, n_tx=1 << 16, p_update_ppm=100_000, ro_streak=8, ro_adaptive=2,
                    client_warps=256, server_workers=6), **kw)
     _check_kv(W.c4(**kw))
+
+
+# ---- server write-back (csmv_workload.server_writeback): the worker writes the PUT's versions and publishes ----
+@pytest.mark.parametrize("kw", [
+    dict(p_update_ppm=10_000, ro_streak=32, ro_adaptive=2, backoff_max=16, publish=1),
+    dict(p_update_ppm=300_000, ro_streak=4, ro_adaptive=1, publish=0),
+    dict(p_update_ppm=100_000, ro_streak=8, ro_adaptive=2, publish=1, debug_flags=csmv.DBG_JITTER),
+    dict(p_update_ppm=100_000, ro_streak=8, ro_adaptive=2, publish=0, debug_flags=csmv.DBG_JITTER),
+    dict(p_update_ppm=100_000, ro_streak=8, server_recv=csmv.RECV_SELF, server_workers=7, publish=1, req_tagged=1),
+    dict(p_update_ppm=50_000, ro_streak=8, ro_adaptive=2, server=csmv.SERVER_CLUSTER, cluster_size=4, publish=1),
+    dict(p_update_ppm=50_000, ro_streak=8, ro_adaptive=2, n_versions=2, publish=0),
+])
+def test_kv_server_writeback_parity(kw):
+    kw = dict(dict(server_workers=6), **kw)
+    cfg = W.c4(n_items=1 << 14, n_tx=1 << 17, client_warps=256, server_writeback=1, **kw)
+    _check_kv(cfg)
+
+
+def test_kv_server_writeback_one_warp():
+    """With one client warp the schedule is the client's own: the server
+    writing the versions back changes no snapshot, CTS or ring slot."""
+    for swb in (0, 1):
+        cfg = W.c4(n_items=1 << 11, kv_ways=8, n_tx=4000, p_update_ppm=300_000, client_warps=1, ro_streak=4,
+                   server_writeback=swb)
+        pre, stats, log, fin = run(cfg)
+        oc = ocfg_of(cfg)
+        plog, pfin, ps = oracle.kv_predict(oc, oracle.kv_preload(oc), oracle.kv_gen(oc, cfg.seed, cfg.n_tx), 32)
+        assert np.array_equal(log, plog), swb
+        for a, b in zip(fin, (pfin.keys, pfin.vals, pfin.lru, pfin.clocks)):
+            assert np.array_equal(a, b)
