@@ -149,11 +149,13 @@ typedef struct csmv_workload {
                                   the whole check); EINVAL for KV, whose PUTs write the value blindly */
     uint32_t retry_order;      /* CSMV_RETRY_*: client-side contention management of update retries
                                   (the paper leaves retry scheduling open) */
-    uint32_t server_writeback; /* KV (compact requests): 1 = the server worker writes a committed PUT's
-                                  four versions back and publishes GTS itself right after the critical
-                                  section (the PUT's key, value and replacement slots travel with the
-                                  request), as CSMV-onlyCS does for the bank; 0 = the client
-                                  writes back.  Takes fenced requests (req_tagged ignored) */
+    uint32_t server_writeback; /* 1 = the server worker writes a committed update's versions back right
+                                  after the critical section and publishes it (done flags; KV with
+                                  publish CLIENT: the worker advances GTS itself), the new values and
+                                  replacement slots travelling with the request -- as CSMV-onlyCS does
+                                  (P:266); 0 = the client writes back.  KV: compact requests;
+                                  bank: self-receiving workers with publish SERVER; elsewhere ignored.
+                                  Takes fenced requests (req_tagged ignored) */
     uint32_t req_tagged;       /* 0: a client fences its request's payload before ringing the doorbell
                                   and the server's receiver fences after seeing it (acquire); 1: no
                                   fences -- every payload word carries the request's round and the

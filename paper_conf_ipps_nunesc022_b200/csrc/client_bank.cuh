@@ -359,9 +359,12 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       if (mine) {
         put_req_id(p, my_ids + lane, d.src | kWriteBit, round);
         put_req_id(p, my_ids + 32 + lane, d.dst | kWriteBit, round);
-        if (p.commit == CSMV_COMMIT_ONLYCS) {  // the server writes back
-          p.req_vals[(size_t)cw * 64 + lane] = vs - (uint32_t)d.amt;
-          p.req_vals[(size_t)cw * 64 + 32 + lane] = vd + (uint32_t)d.amt;
+        if (p.commit == CSMV_COMMIT_ONLYCS || p.bank_swb) {  // the server writes back
+          p.req_vals[(size_t)cw * 96 + lane] = vs - (uint32_t)d.amt;
+          p.req_vals[(size_t)cw * 96 + 32 + lane] = vd + (uint32_t)d.amt;
+          // the slots the versions replace, fixed by this read (nothing writes
+          // either account before this commit: it validated)
+          if (p.bank_swb) p.req_vals[(size_t)cw * 96 + 64 + lane] = ring_victim<NS>(rs, K) | (ring_victim<NS>(rd, K) << 8);
         }
       }
       if (lane == 0) put_req_hdr(p, cw, s, kept, round);
@@ -400,7 +403,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
           // Client-side write-back with CTS = base + rank.
           cts = base + __popc(cmask & lt);
           const uint32_t ns = vs - (uint32_t)d.amt, nd = vd + (uint32_t)d.amt;
-          if (p.commit != CSMV_COMMIT_ONLYCS) {
+          if (p.commit != CSMV_COMMIT_ONLYCS && !p.bank_swb) {
             write_back<NS>(p.rings + (size_t)d.src * NS, rs, K, cts, ns);
             write_back<NS>(p.rings + (size_t)d.dst * NS, rd, K, cts, nd);
             // lastw (the item-indexed ATR's exact level, server.cuh): written
@@ -430,7 +433,7 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
       }
       __syncwarp();
       pc.mark(PH_WRITEBACK);
-      const uint32_t n = __popc(cmask);
+      const uint32_t n = p.bank_swb ? 0u : __popc(cmask);  // server write-back: published by the server
       if (n) {
         jit();  // write-backs done, commit not yet published
         if (p.publish == CSMV_PUBLISH_CLIENT) {

@@ -74,6 +74,30 @@ __device__ __forceinline__ uint64_t slot_at(const Ring<NS>& r, int j) {
 // Replace the first unused slot, else the oldest version.  The
 // writer owns the item: the WW check orders all writers of an item
 // and the ring is unchanged since this transaction read it.
+// the slot a new version of ring r replaces: the first unused, else the oldest
+template <int NS>
+__device__ __forceinline__ int ring_victim(const Ring<NS>& r, uint32_t K) {
+  int victim = -1;
+#pragma unroll
+  for (int j = 0; j < NS; ++j) {
+    uint32_t ts = (uint32_t)(r.s[j] >> 32);
+    if ((uint32_t)j < K && victim < 0 && ts == kEmptyTs) victim = j;
+  }
+  if (victim < 0) {
+    victim = 0;
+    uint32_t vts = (uint32_t)(r.s[0] >> 32);
+#pragma unroll
+    for (int j = 1; j < NS; ++j) {
+      uint32_t ts = (uint32_t)(r.s[j] >> 32);
+      if ((uint32_t)j < K && ts < vts) {
+        victim = j;
+        vts = ts;
+      }
+    }
+  }
+  return victim;
+}
+
 template <int NS>
 __device__ __forceinline__ void write_back(uint64_t* ring, const Ring<NS>& r, uint32_t K,
                                            uint32_t cts, uint32_t val) {

@@ -211,6 +211,7 @@ struct KParams {
   uint64_t* kv_tk_serv;       // u64[T]
   uint32_t req_tagged;        // requests are round-tagged (ReqHdr): no client fence before the doorbell
   uint32_t kv_swb;            // KV: the server writes committed PUTs back and publishes (rows kSwbRow.. of a request)
+  uint32_t bank_swb;          // bank, self-receiving workers: the server writes committed transfers back (req_vals)
 };
 // KV server write-back: request rows 4-7 the key, 8-15 the value, 16 the new
 // LRU / clock value, 17 the replacement slots (key/value/LRU | clock << 8)

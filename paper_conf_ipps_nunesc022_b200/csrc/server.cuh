@@ -656,6 +656,21 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     // ordered them after the doorbells; ours orders them after the queue)
     if (!self) fence_cta();
     uint32_t sq[M], sn[M], msk[M], id0[M], id1[M];
+    // server write-back (self-receiving workers, csmv_workload.server_writeback):
+    // the new balances and replacement slots, with the payload
+    uint32_t wv0[SELF ? M : 1], wv1[SELF ? M : 1], wvi[SELF ? M : 1];
+    if constexpr (SELF) {
+#pragma unroll
+      for (int j = 0; j < M; ++j) {
+        wv0[j] = wv1[j] = wvi[j] = 0;
+        if (p.bank_swb && j < (int)m) {
+          const uint32_t* rv = p.req_vals + (size_t)cwv[j] * 96 + lane;
+          wv0[j] = ld_relaxed(rv);
+          wv1[j] = ld_relaxed(rv + 32);
+          wvi[j] = ld_relaxed(rv + 64);
+        }
+      }
+    }
     // fenced requests: every load in flight at once, no checks (the
     // receiver's or the claim's fence ordered them after the doorbells).
     // Tagged requests are taken by the self-receiving worker only (the
@@ -858,6 +873,27 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
     if (p.publish == CSMV_PUBLISH_SERVER && t != t0c) done_ring_room(p, c, t, t_begin);
     cs_leave<CL>(c, ticket, t);
     const long long t2 = clock64();
+    if constexpr (SELF) {
+      // Server write-back (csmv_workload.server_writeback): each committed
+      // transfer's two versions and lastw, then its done flag -- the
+      // publisher advances GTS over them (the clients' invariant: GTS = g
+      // implies lastw and the rings hold every commit <= g)
+      if (p.bank_swb && t != t0c) {
+        const uint32_t NS = p.K <= 2 ? 2u : p.K <= 4 ? 4u : p.K <= 8 ? 8u : 16u;  // ring slots (host nslot_for)
+        jit();
+#pragma unroll
+        for (int j = 0; j < M; ++j) {
+          if (j < (int)m && ((cm[j] >> lane) & 1u)) {
+            const uint32_t cts = base[j] + __popc(cm[j] & lt);
+            st_relaxed64(p.rings + (size_t)id0[j] * NS + (wvi[j] & 0xFFu), ((uint64_t)cts << 32) | wv0[j]);
+            st_relaxed64(p.rings + (size_t)id1[j] * NS + ((wvi[j] >> 8) & 0xFFu), ((uint64_t)cts << 32) | wv1[j]);
+            st_relaxed(p.lastw + id0[j], cts);
+            st_relaxed(p.lastw + id1[j], cts);
+            st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
+          }
+        }
+      }
+    }
     if (hash) {
 #pragma unroll
       for (int j = 0; j < M; ++j) om[j] = __ballot_sync(FULL, ovfl[j]);
@@ -1569,8 +1605,8 @@ __device__ void server_worker_onlycs(const KParams& p, const SrvCtx& c, uint64_t
     if (mine) {
       a = ld_relaxed(p.req_ids + (size_t)cw * 64 + lane) & ~kWriteBit;
       b = ld_relaxed(p.req_ids + (size_t)cw * 64 + 32 + lane) & ~kWriteBit;
-      na = ld_relaxed(p.req_vals + (size_t)cw * 64 + lane);
-      nb = ld_relaxed(p.req_vals + (size_t)cw * 64 + 32 + lane);
+      na = ld_relaxed(p.req_vals + (size_t)cw * 96 + lane);
+      nb = ld_relaxed(p.req_vals + (size_t)cw * 96 + 32 + lane);
     }
     if (__ballot_sync(FULL, (a ^ b ^ na ^ nb ^ s) == 0x12345679u) == FULL) __nanosleep(1);
     jit();
