@@ -155,7 +155,8 @@ typedef struct csmv_workload {
                                   replacement slots travelling with the request -- as CSMV-onlyCS does
                                   (P:266); 0 = the client writes back.  KV: compact requests;
                                   bank: self-receiving workers with publish SERVER; elsewhere ignored.
-                                  Takes fenced requests (req_tagged ignored) */
+                                  With req_tagged (KV) the written words carry a check word of the
+                                  round that the server verifies; the bank's take fenced requests */
     uint32_t req_tagged;       /* 0: a client fences its request's payload before ringing the doorbell
                                   and the server's receiver fences after seeing it (acquire); 1: no
                                   fences -- every payload word carries the request's round and the

@@ -660,6 +660,16 @@ __device__ void client_warp_kv(const KParams& p, uint64_t t_begin, uint32_t* scr
         for (int j = 0; j < 8; ++j) r[(4 + j) * 32] = d.val[j];
         r[12 * 32] = clk + 1;
         r[13 * 32] = (uint32_t)iv | ((uint32_t)ic << 8);
+        if (p.req_tagged) {  // no fence before the doorbell: the server checks this word instead
+          uint32_t w[kSwbRows];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) w[j] = kk[j];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) w[4 + j] = d.val[j];
+          w[12] = clk + 1;
+          w[13] = (uint32_t)iv | ((uint32_t)ic << 8);
+          st_relaxed(r + kSwbRows * 32, swb_check(round, w, 1));
+        }
       }
     } else if (kept && mine) {
       // request ids: RS u WS (bit 31: in WS)

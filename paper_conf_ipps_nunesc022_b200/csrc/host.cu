@@ -635,10 +635,10 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
     const bool bank_lock = h->kind == CSMV_KIND_BANK && selfrecv;  // the self-receiving bank worker
     if (w->req_tagged > 1) return set_err(CSMV_EINVAL, "csmv_run: req_tagged must be 0 or 1");
     if (w->server_writeback > 1) return set_err(CSMV_EINVAL, "csmv_run: server_writeback must be 0 or 1");
-    p.kv_swb = w->server_writeback && h->kind == CSMV_KIND_KV && kv_filt && h->maxid >= kSwbRow + kSwbRows;
+    p.kv_swb = w->server_writeback && h->kind == CSMV_KIND_KV && kv_filt && h->maxid >= kSwbRow + kSwbRows + 1;
     p.bank_swb = w->server_writeback && h->kind == CSMV_KIND_BANK && selfrecv && w->publish == CSMV_PUBLISH_SERVER;
     p.req_tagged = w->req_tagged && (max_id <= (1ull << kIdItemBits)) &&
-                   (bank_lock || (h->kind == CSMV_KIND_KV && kv_filt)) && !p.kv_swb && !p.bank_swb;
+                   (bank_lock || (h->kind == CSMV_KIND_KV && kv_filt)) && !p.bank_swb;
   }
   // the publisher takes the last warp slot of the first client CTA when no
   // client warp lives there (client warp cw runs on CTA cw % n_ctas, warp

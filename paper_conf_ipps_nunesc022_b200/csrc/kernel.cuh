@@ -214,8 +214,14 @@ struct KParams {
   uint32_t bank_swb;          // bank, self-receiving workers: the server writes committed transfers back (req_vals)
 };
 // KV server write-back: request rows 4-7 the key, 8-15 the value, 16 the new
-// LRU / clock value, 17 the replacement slots (key/value/LRU | clock << 8)
+// LRU / clock value, 17 the replacement slots (key/value/LRU | clock << 8),
+// 18 (tagged requests) a check word of the round and rows 4-17
 constexpr uint32_t kSwbRow = 4, kSwbRows = 14;
+__host__ __device__ inline uint32_t swb_check(uint32_t round, const uint32_t* w, uint32_t stride) {
+  uint32_t h = round * 0x9E3779B1u + 0x7F4A7C15u;
+  for (uint32_t k = 0; k < kSwbRows; ++k) h = ((h ^ w[k * stride]) * 0x85EBCA77u) ^ (h >> 15);
+  return h;
+}
 
 constexpr uint32_t kKvMaxWays = 256;              // KV ways supported by the device path
 constexpr uint32_t kKvFullWays = 16;              // up to here PUT read-sets are shipped item by item

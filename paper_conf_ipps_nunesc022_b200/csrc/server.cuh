@@ -1432,6 +1432,9 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
     const uint64_t t_claim = trace_now(p);
     const long long t0 = clock64();
     uint32_t sq, s, mask, ids[4];
+    // server write-back: the PUT's key, value, new LRU / clock value and
+    // replacement slots, loaded with the payload (+ the check word when tagged)
+    uint32_t wb[kSwbRows];
     // tagged requests: loaded again until every word carries the round of
     // the doorbell (the client did not fence the payload before it)
     for (uint32_t pass = 0;; ++pass) {
@@ -1442,6 +1445,13 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
       mask = (uint32_t)w1;
 #pragma unroll
       for (int k = 0; k < 4; ++k) ids[k] = ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + k) * 32 + lane);
+      uint32_t wck = 0;
+      if (p.kv_swb) {
+#pragma unroll
+        for (int k = 0; k < (int)kSwbRows; ++k)
+          wb[k] = ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + kSwbRow + k) * 32 + lane);
+        if (p.req_tagged) wck = ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + kSwbRow + kSwbRows) * 32 + lane);
+      }
       if (!p.req_tagged) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) ids[k] &= ~kWriteBit;
@@ -1452,6 +1462,7 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
       if ((mask >> lane) & 1u) {
 #pragma unroll
         for (int k = 0; k < 4; ++k) stale |= (ids[k] & tm) != tg;
+        if (p.kv_swb) stale |= swb_check(sq, wb, 1) != wck;  // the write-back words of this round
       }
 #pragma unroll
       for (int k = 0; k < 4; ++k) ids[k] &= kIdItemMask;
@@ -1463,14 +1474,6 @@ __device__ void server_worker_kv_filter(const KParams& p, const SrvCtx& c, uint6
       }
     }
     const bool mine = (mask >> lane) & 1u;
-    // server write-back: the PUT's key, value, new LRU / clock value and
-    // replacement slots, loaded with the payload (fenced requests)
-    uint32_t wb[kSwbRows];
-    if (p.kv_swb) {
-#pragma unroll
-      for (int k = 0; k < (int)kSwbRows; ++k)
-        wb[k] = mine ? ld_relaxed(p.req_ids + ((size_t)cw * p.maxid + kSwbRow + k) * 32 + lane) : 0u;
-    }
     const uint32_t e_pre = *(volatile uint32_t*)&c.sh0->tail;  // lastw covers every CTS <= e_pre
     srv_fence<CL>();
     jit();  // e_pre read, lastw not yet (the window cs_leave's fence covers)

@@ -274,6 +274,9 @@ def test_kv_coop_read_parity(kw):
     dict(p_update_ppm=100_000, ro_streak=8, server_recv=csmv.RECV_SELF, server_workers=7, publish=1, req_tagged=1),
     dict(p_update_ppm=50_000, ro_streak=8, ro_adaptive=2, server=csmv.SERVER_CLUSTER, cluster_size=4, publish=1),
     dict(p_update_ppm=50_000, ro_streak=8, ro_adaptive=2, n_versions=2, publish=0),
+    dict(p_update_ppm=10_000, ro_streak=32, ro_adaptive=2, backoff_max=16, publish=1, req_tagged=1),
+    dict(p_update_ppm=200_000, ro_streak=8, ro_adaptive=2, publish=1, req_tagged=1, debug_flags=csmv.DBG_JITTER),
+    dict(p_update_ppm=200_000, ro_streak=8, ro_adaptive=2, publish=0, req_tagged=1, debug_flags=csmv.DBG_JITTER),
 ])
 def test_kv_server_writeback_parity(kw):
     kw = dict(dict(server_workers=6), **kw)
