@@ -154,7 +154,7 @@ typedef struct csmv_workload {
                                   publish CLIENT: the worker advances GTS itself), the new values and
                                   replacement slots travelling with the request -- as CSMV-onlyCS does
                                   (P:266); 0 = the client writes back.  KV: compact requests;
-                                  bank: self-receiving workers with publish SERVER; elsewhere ignored.
+                                  bank: self-receiving workers (either publish mode); elsewhere ignored.
                                   With req_tagged (KV) the written words carry a check word of the
                                   round that the server verifies; the bank's take fenced requests */
     uint32_t req_tagged;       /* 0: a client fences its request's payload before ringing the doorbell

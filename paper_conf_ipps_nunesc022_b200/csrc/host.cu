@@ -636,7 +636,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
     if (w->req_tagged > 1) return set_err(CSMV_EINVAL, "csmv_run: req_tagged must be 0 or 1");
     if (w->server_writeback > 1) return set_err(CSMV_EINVAL, "csmv_run: server_writeback must be 0 or 1");
     p.kv_swb = w->server_writeback && h->kind == CSMV_KIND_KV && kv_filt && h->maxid >= kSwbRow + kSwbRows + 1;
-    p.bank_swb = w->server_writeback && h->kind == CSMV_KIND_BANK && selfrecv && w->publish == CSMV_PUBLISH_SERVER;
+    p.bank_swb = w->server_writeback && h->kind == CSMV_KIND_BANK && selfrecv;
     p.req_tagged = w->req_tagged && (max_id <= (1ull << kIdItemBits)) &&
                    (bank_lock || (h->kind == CSMV_KIND_KV && kv_filt)) && !p.bank_swb;
   }

@@ -889,8 +889,21 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
             st_relaxed64(p.rings + (size_t)id1[j] * NS + ((wvi[j] >> 8) & 0xFFu), ((uint64_t)cts << 32) | wv1[j]);
             st_relaxed(p.lastw + id0[j], cts);
             st_relaxed(p.lastw + id1[j], cts);
-            st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
+            if (p.publish == CSMV_PUBLISH_SERVER) st_release(p.done_ring + (cts & ((1u << kDoneLog2) - 1)), cts);
           }
+        }
+        if (p.publish == CSMV_PUBLISH_CLIENT) {  // this worker advances GTS over its range, in CTS order
+          __syncwarp();
+          fence_gpu();
+          if (lane == 0) {
+            uint32_t it = 0;
+            while (ld_relaxed(p.gts) != t0c) {
+              if ((++it & 255u) == 0 && (ld_relaxed(&p.ctl->error) || watchdog(p, t_begin, 6))) break;
+              __nanosleep(32);
+            }
+            st_release(p.gts, t);
+          }
+          __syncwarp();
         }
       }
     }

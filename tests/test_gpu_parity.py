@@ -289,16 +289,18 @@ def test_tagged_requests_fall_back_above_24_bit_items():
     assert stats["committed"] == cfg.n_tx
 
 
-@pytest.mark.parametrize("kw", [dict(), dict(debug_flags=csmv.DBG_JITTER), dict(n_versions=2), dict(n_versions=8)])
+@pytest.mark.parametrize("kw", [dict(), dict(debug_flags=csmv.DBG_JITTER), dict(n_versions=2), dict(n_versions=8),
+                                dict(publish=csmv.PUBLISH_CLIENT), dict(publish=csmv.PUBLISH_CLIENT, debug_flags=csmv.DBG_JITTER)])
 def test_bank_server_writeback(kw):
     """Bank, self-receiving workers with server_writeback: the worker writes
     each committed transfer's versions and lastw and sets its done flag; the
     oracle replays the history and the final rings match the closed form."""
+    kw = dict(dict(publish=csmv.PUBLISH_SERVER), **kw)
     cfg = W.c3(n_tx=1 << 16, client_warps=128, server_recv=csmv.RECV_SELF, server_workers=7, server_combine=2,
-               publish=csmv.PUBLISH_SERVER, ro_streak=4, ro_adaptive=1, server_writeback=1, **kw)
+               ro_streak=4, ro_adaptive=1, server_writeback=1, **kw)
     rep, stats, log, rings, descs = check(cfg)
     assert stats["committed"] == cfg.n_tx
     c2 = W.c2(n_items=1 << 14, n_tx=1 << 16, client_warps=256, server_recv=csmv.RECV_SELF, server_workers=7,
-              publish=csmv.PUBLISH_SERVER, server_writeback=1, **kw)
+              server_writeback=1, **kw)
     rep, stats, log, rings, descs = check(c2)
     assert np.array_equal(newest(rings, c2.n_items, c2.n_versions), closed_form(c2, descs, c2.init_values()))
