@@ -66,10 +66,12 @@ TUNED = dict(client_warps_per_sm=4, client_group=4, server_workers=7, server_com
 # payload and doorbell: a shorter link; C4 103 -> 113 M tx/s, while C2's
 # server-bound step prefers fenced payloads, 494 vs 505 M); C4's server
 # worker writes the committed PUTs back itself and the publisher advances
-# GTS (server_writeback, fenced payloads: 115 -> 125 M, the client's answer
-# and write-back off the hot set's chain)
+# GTS (server_writeback: 115 -> 125 M fenced, 135 M tagged, the client's
+# answer and write-back off the hot set's chain); C3's self-receiving workers
+# write back too and advance GTS themselves in CTS order (4.9 -> 5.3 M on one
+# box)
 TUNED_PER_CONFIG = {"C3": dict(server_recv=1, server_workers=7, server_combine=2, publish=0, client_warps_per_sm=2,
-                               client_group=1, req_tagged=1, ro_streak=8, ro_adaptive=1),
+                               client_group=1, req_tagged=1, ro_streak=8, ro_adaptive=1, server_writeback=1),
                     "C4": dict(ro_streak=32, client_warps_per_sm=2, client_group=1, ro_adaptive=2, backoff_max=16,
                                req_tagged=1, server_workers=7, server_writeback=1)}
 

@@ -360,11 +360,17 @@ __device__ void client_warp(const KParams& p, uint64_t t_begin, uint8_t* smem) {
         put_req_id(p, my_ids + lane, d.src | kWriteBit, round);
         put_req_id(p, my_ids + 32 + lane, d.dst | kWriteBit, round);
         if (p.commit == CSMV_COMMIT_ONLYCS || p.bank_swb) {  // the server writes back
-          p.req_vals[(size_t)cw * 96 + lane] = vs - (uint32_t)d.amt;
-          p.req_vals[(size_t)cw * 96 + 32 + lane] = vd + (uint32_t)d.amt;
+          uint32_t* rv = p.req_vals + (size_t)cw * 128 + lane;
+          const uint32_t na = vs - (uint32_t)d.amt, nb = vd + (uint32_t)d.amt;
+          rv[0] = na;
+          rv[32] = nb;
           // the slots the versions replace, fixed by this read (nothing writes
           // either account before this commit: it validated)
-          if (p.bank_swb) p.req_vals[(size_t)cw * 96 + 64 + lane] = ring_victim<NS>(rs, K) | (ring_victim<NS>(rd, K) << 8);
+          if (p.bank_swb) {
+            const uint32_t sl = ring_victim<NS>(rs, K) | (ring_victim<NS>(rd, K) << 8);
+            rv[64] = sl;
+            if (p.req_tagged) rv[96] = bank_swb_check(round, na, nb, sl);  // no fence: the server checks it
+          }
         }
       }
       if (lane == 0) put_req_hdr(p, cw, s, kept, round);

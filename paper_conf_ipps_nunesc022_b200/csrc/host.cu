@@ -193,7 +193,7 @@ csmv_t* csmv_create(uint64_t n_items, uint32_t n_versions) {
   if (cudaMalloc(&h->d_rings, n_items * h->nslot * sizeof(uint64_t)) != cudaSuccess) return create_fail(h, "rings");
   if (cudaMalloc(&h->d_init, n_items * sizeof(int32_t)) != cudaSuccess) return create_fail(h, "init staging");
   if (!alloc_common(h)) return create_fail(h, "control buffers");
-  if (cudaMalloc(&h->d_req_vals, (size_t)h->max_cw * 96 * sizeof(uint32_t)) != cudaSuccess)
+  if (cudaMalloc(&h->d_req_vals, (size_t)h->max_cw * 128 * sizeof(uint32_t)) != cudaSuccess)
     return create_fail(h, "request values");
   return h;
 }
@@ -638,7 +638,7 @@ int csmv_run(csmv_t* h, const csmv_workload* w, uint64_t n_tx, uint64_t seed) {
     p.kv_swb = w->server_writeback && h->kind == CSMV_KIND_KV && kv_filt && h->maxid >= kSwbRow + kSwbRows + 1;
     p.bank_swb = w->server_writeback && h->kind == CSMV_KIND_BANK && selfrecv;
     p.req_tagged = w->req_tagged && (max_id <= (1ull << kIdItemBits)) &&
-                   (bank_lock || (h->kind == CSMV_KIND_KV && kv_filt)) && !p.bank_swb;
+                   (bank_lock || (h->kind == CSMV_KIND_KV && kv_filt));
   }
   // the publisher takes the last warp slot of the first client CTA when no
   // client warp lives there (client warp cw runs on CTA cw % n_ctas, warp

@@ -217,6 +217,13 @@ struct KParams {
 // LRU / clock value, 17 the replacement slots (key/value/LRU | clock << 8),
 // 18 (tagged requests) a check word of the round and rows 4-17
 constexpr uint32_t kSwbRow = 4, kSwbRows = 14;
+// bank server write-back (req_vals rows 0-2: new balances, slots; row 3 the check word)
+__host__ __device__ inline uint32_t bank_swb_check(uint32_t round, uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t h = round * 0x9E3779B1u + 0x7F4A7C15u;
+  h = ((h ^ a) * 0x85EBCA77u) ^ (h >> 15);
+  h = ((h ^ b) * 0x85EBCA77u) ^ (h >> 15);
+  return ((h ^ c) * 0x85EBCA77u) ^ (h >> 15);
+}
 __host__ __device__ inline uint32_t swb_check(uint32_t round, const uint32_t* w, uint32_t stride) {
   uint32_t h = round * 0x9E3779B1u + 0x7F4A7C15u;
   for (uint32_t k = 0; k < kSwbRows; ++k) h = ((h ^ w[k * stride]) * 0x85EBCA77u) ^ (h >> 15);

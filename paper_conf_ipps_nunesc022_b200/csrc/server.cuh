@@ -664,10 +664,12 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
       for (int j = 0; j < M; ++j) {
         wv0[j] = wv1[j] = wvi[j] = 0;
         if (p.bank_swb && j < (int)m) {
-          const uint32_t* rv = p.req_vals + (size_t)cwv[j] * 96 + lane;
-          wv0[j] = ld_relaxed(rv);
-          wv1[j] = ld_relaxed(rv + 32);
-          wvi[j] = ld_relaxed(rv + 64);
+          const uint32_t* rv = p.req_vals + (size_t)cwv[j] * 128 + lane;
+          if (!p.req_tagged) {  // tagged: loaded (and checked) with the payload below
+            wv0[j] = ld_relaxed(rv);
+            wv1[j] = ld_relaxed(rv + 32);
+            wvi[j] = ld_relaxed(rv + 64);
+          }
         }
       }
     }
@@ -706,6 +708,21 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
           id1[j] = ld_relaxed(p.req_ids + (size_t)cwv[j] * 64 + 32 + lane);
         }
       }
+      // server write-back words: re-read with the payload, checked against the round
+      uint32_t wck[SELF ? M : 1];
+      if constexpr (SELF) {
+#pragma unroll
+        for (int j = 0; j < M; ++j) {
+          wck[j] = 0;
+          if (p.bank_swb && j < (int)m) {
+            const uint32_t* rv = p.req_vals + (size_t)cwv[j] * 128 + lane;
+            wv0[j] = ld_relaxed(rv);
+            wv1[j] = ld_relaxed(rv + 32);
+            wvi[j] = ld_relaxed(rv + 64);
+            wck[j] = ld_relaxed(rv + 96);
+          }
+        }
+      }
       bool stale = false;
       const uint32_t keep = p.req_tagged ? kIdItemMask : ~kWriteBit, tm = kIdTagMask << kIdItemBits;
 #pragma unroll
@@ -719,6 +736,9 @@ __device__ void server_worker(const KParams& p, const SrvCtx& c, uint64_t t_begi
           const bool mj = (msk[j] >> lane) & 1u;
           stale |= (sq[j] & 0xFFFFu) != rqv[j] || (uint32_t)(w1[j] >> 32) != sq[j] ||
                    (mj && ((id0[j] & tm) != tg || (id1[j] & tm) != tg));
+          if constexpr (SELF) {
+            if (p.bank_swb && mj) stale |= bank_swb_check(sq[j], wv0[j], wv1[j], wvi[j]) != wck[j];
+          }
         }
         id0[j] &= keep;
         id1[j] &= keep;
@@ -1621,8 +1641,8 @@ __device__ void server_worker_onlycs(const KParams& p, const SrvCtx& c, uint64_t
     if (mine) {
       a = ld_relaxed(p.req_ids + (size_t)cw * 64 + lane) & ~kWriteBit;
       b = ld_relaxed(p.req_ids + (size_t)cw * 64 + 32 + lane) & ~kWriteBit;
-      na = ld_relaxed(p.req_vals + (size_t)cw * 96 + lane);
-      nb = ld_relaxed(p.req_vals + (size_t)cw * 96 + 32 + lane);
+      na = ld_relaxed(p.req_vals + (size_t)cw * 128 + lane);
+      nb = ld_relaxed(p.req_vals + (size_t)cw * 128 + 32 + lane);
     }
     if (__ballot_sync(FULL, (a ^ b ^ na ^ nb ^ s) == 0x12345679u) == FULL) __nanosleep(1);
     jit();

@@ -290,7 +290,8 @@ def test_tagged_requests_fall_back_above_24_bit_items():
 
 
 @pytest.mark.parametrize("kw", [dict(), dict(debug_flags=csmv.DBG_JITTER), dict(n_versions=2), dict(n_versions=8),
-                                dict(publish=csmv.PUBLISH_CLIENT), dict(publish=csmv.PUBLISH_CLIENT, debug_flags=csmv.DBG_JITTER)])
+                                dict(publish=csmv.PUBLISH_CLIENT), dict(publish=csmv.PUBLISH_CLIENT, debug_flags=csmv.DBG_JITTER),
+                                dict(req_tagged=1), dict(req_tagged=1, publish=csmv.PUBLISH_CLIENT, debug_flags=csmv.DBG_JITTER)])
 def test_bank_server_writeback(kw):
     """Bank, self-receiving workers with server_writeback: the worker writes
     each committed transfer's versions and lastw and sets its done flag; the
