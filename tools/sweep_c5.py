@@ -22,7 +22,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 from paper_conf_ipps_nunesc022_b200 import csmv, workloads  # noqa: E402
 
-TUNED = dict(server_workers=6, server_combine=8, ro_streak=8, ro_adaptive=1, publish=csmv.PUBLISH_SERVER)
+TUNED = dict(server_workers=7, server_combine=8, ro_streak=2, ro_adaptive=0, publish=csmv.PUBLISH_SERVER)  # bench.py's C2 launch
 
 
 def run_point(cfg, check: bool, seeds: int):
